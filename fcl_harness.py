@@ -1,0 +1,70 @@
+"""Glue between ``workloads.Problem`` (seeded inputs) and the fcl C-ABI binding.
+
+Used by tests/, bench.py and __graft_entry__.smoke(); never by the oracle.  It only
+creates buffers, forwards arguments in the kernel's signature order and reads results
+back -- every step of the method runs inside libfcl.so.
+"""
+from __future__ import annotations
+
+from typing import Dict, List, Optional, Tuple
+
+import numpy as np
+
+from paper_conf_cgo_panditg14_b200 import fcl
+import workloads as W
+
+
+def kernel_name(P: W.Problem) -> str:
+    return f"{P.kernel}_{'i32' if P.integer else 'f32'}"
+
+
+def make_args(ctx: fcl.Context, P: W.Problem, bufs: List[fcl.Buffer]) -> list:
+    k = ctx.kernel(kernel_name(P))
+    args, nb, ni = [], 0, 0
+    for pname, pkind in k.params:
+        if pkind in ("in", "out", "inout"):
+            args.append(bufs[nb]); nb += 1
+        elif pname == "alpha":
+            args.append(P.ialpha if P.integer else P.alpha)
+        elif pname == "beta":
+            args.append(P.ibeta if P.integer else P.beta)
+        elif pname == "eps":
+            args.append(P.eps)
+        else:
+            args.append(P.n0 if ni == 0 else P.n1); ni += 1
+    return args
+
+
+def create_buffers(ctx: fcl.Context, P: W.Problem) -> List[fcl.Buffer]:
+    return [ctx.buffer_from_array(b) for b in P.bufs]
+
+
+def run(ctx: fcl.Context, P: W.Problem, mode: str = "coop", bufs: Optional[List[fcl.Buffer]] = None,
+        read_all: bool = False, **opts) -> Tuple[Dict[int, np.ndarray], dict]:
+    """Launch P through the C-ABI, wait, and return ({buffer index: host array}, launch info)."""
+    own = bufs is None
+    if own:
+        bufs = create_buffers(ctx, P)
+    info = ctx.enqueue_ndrange(kernel_name(P), P.gws, P.lws, make_args(ctx, P, bufs), mode=mode, **opts)
+    ctx.finish()
+    info = ctx.launch_info()
+    dt = np.int32 if P.integer else np.float32
+    idx = range(len(P.bufs)) if read_all else P.out_indices
+    outs = {k: bufs[k].read_array(dt) for k in idx}
+    if own:
+        for b in bufs:
+            b.release()
+    return outs, info
+
+
+def device_array(buf: fcl.Buffer, dtype) -> np.ndarray:
+    """Copy a buffer's DEVICE copy to a numpy array (bypassing the host mirror), via torch."""
+    import torch
+    n = buf.nbytes // np.dtype(dtype).itemsize
+    t = torch.empty(n, dtype=torch.int32 if np.dtype(dtype) == np.int32 else torch.float32, device="cuda")
+    torch.cuda.synchronize()
+    import ctypes
+    cudart = torch.cuda.cudart()
+    res = cudart.cudaMemcpy(t.data_ptr(), buf.device_ptr, buf.nbytes, 3)  # device-to-device
+    torch.cuda.synchronize()
+    return t.cpu().numpy().view(dtype)

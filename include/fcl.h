@@ -1,0 +1,251 @@
+/*
+ * fcl.h -- C-ABI of the B200-native FluidiCL hot path.
+ *
+ * FluidiCL (Pandit & Govindarajan, CGO 2014; /root/reference/PAPER.md, cited
+ * as L<line>.s<sentence>) takes a kernel written for one
+ * device and executes its flattened work-group range cooperatively: the GPU
+ * claims work-groups from the bottom (ascending flattened id), host threads
+ * execute chunks from the top (descending) and publish a completed-from
+ * watermark; a GPU work-group exits early once the host covers it; a
+ * diff-merge then restores one coherent buffer (L14.s32-44, L16.s5-22,
+ * L16.s28-35, Fig 9).
+ *
+ * Conventions shared by every entry point:
+ *  - Plain C types only; no torch/CUDA types.  "device pointer" arguments are
+ *    CUDA device addresses; "stream" arguments are cudaStream_t passed as
+ *    void* (NULL = the context's own stream).
+ *  - Every function returns an fcl_status (FCL_SUCCESS = 0; errors < 0 use
+ *    OpenCL-style codes).  No C++ exception crosses this boundary.
+ *  - Asynchronous CUDA / host-thread failures are reported by the next call
+ *    that synchronises (fcl_finish) and make the context sticky-failed
+ *    (FCL_CONTEXT_LOST), mirroring CUDA's sticky errors.
+ *  - A context is NOT thread-safe: one in-order queue, as an OpenCL command
+ *    queue (L22.s14: kernel calls block).  One context per GPU per process.
+ *  - Kernels must not use atomics (L14.s50 footnote): work-groups are
+ *    independent (L14.s22-23), which is what makes the split legal.
+ */
+#ifndef FCL_H
+#define FCL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t fcl_status;
+
+/* Status codes (values follow OpenCL where an equivalent exists). */
+#define FCL_SUCCESS                   0
+#define FCL_DEVICE_NOT_AVAILABLE     -2
+#define FCL_OUT_OF_RESOURCES         -5
+#define FCL_INVALID_VALUE           -30
+#define FCL_INVALID_CONTEXT         -34
+#define FCL_INVALID_MEM_OBJECT      -38
+#define FCL_INVALID_KERNEL_NAME     -46
+#define FCL_INVALID_KERNEL          -48
+#define FCL_INVALID_KERNEL_ARGS     -52
+#define FCL_INVALID_WORK_DIMENSION  -53
+#define FCL_INVALID_WORK_GROUP_SIZE -54
+#define FCL_INVALID_GLOBAL_WORK_SIZE -63
+#define FCL_CONTEXT_LOST          -1000  /* sticky: a prior asynchronous failure */
+#define FCL_CUDA_ERROR            -1001  /* a CUDA runtime call failed (see fcl_last_error) */
+#define FCL_NOT_SUPPORTED         -1002
+
+typedef struct fcl_context_st *fcl_context;
+typedef struct fcl_buffer_st  *fcl_buffer;
+typedef struct fcl_kernel_st  *fcl_kernel;
+
+/* Where the GPU reads the host's watermark from.
+ * HOST_MAPPED: a 64-bit word in pinned, mapped host memory (north_star);
+ * DEVICE: a 64-bit word in device memory.  In both cases the word is written
+ * by a stream memory operation on the `hd` stream right after the chunk's
+ * data copy, so status always follows data on an in-order queue (L16.s15). */
+#define FCL_STATUS_HOST_MAPPED 0
+#define FCL_STATUS_DEVICE      1
+
+typedef struct {
+    int32_t device;          /* CUDA device ordinal */
+    int32_t n_host_threads;  /* host executor threads; 0 = (cores in affinity mask) - 1 */
+    int32_t pin_threads;     /* 1 = pin executor threads to cores of the affinity mask */
+    int32_t status_location; /* FCL_STATUS_HOST_MAPPED (default) | FCL_STATUS_DEVICE */
+    void   *main_stream;     /* optional cudaStream_t for kernels/merge; NULL = own stream */
+    void   *hd_stream;       /* optional cudaStream_t for CPU->GPU staging (L20.s10-12) */
+    void   *dh_stream;       /* optional cudaStream_t for GPU->CPU results   (L20.s10-12) */
+} fcl_context_desc;
+
+/* Create a context on desc->device (desc may be NULL: device 0, defaults).
+ * Owns: streams it creates, the pinned status words, device counters, the
+ * twin/stage pool and the host executor threads.  Errors: FCL_INVALID_VALUE,
+ * FCL_DEVICE_NOT_AVAILABLE, FCL_OUT_OF_RESOURCES, FCL_CUDA_ERROR. */
+fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out);
+fcl_status fcl_release_context(fcl_context ctx);
+
+/* ---- Buffers (C3, L14.s49-50; L16.s1): every buffer exists on both the
+ * host (a pinned mirror) and the device; writes go to both. ---- */
+#define FCL_MEM_READ_WRITE     (1u << 0)
+#define FCL_MEM_WRITE_ONLY     (1u << 1)
+#define FCL_MEM_READ_ONLY      (1u << 2)
+#define FCL_MEM_USE_HOST_PTR   (1u << 3)  /* host mirror = caller's memory (must be pinned) */
+#define FCL_MEM_USE_DEVICE_PTR (1u << 4)  /* device copy = caller's device allocation */
+
+/* Create a dual-resident buffer of `bytes` bytes whose merge granularity is
+ * `elem_size` bytes (the buffer's base type, L16.s32-35; must be 1, 2, 4 or
+ * 8 and divide `bytes`).  host_init (nullable) is copied to both copies.
+ * Errors: FCL_INVALID_VALUE (size/elem_size), FCL_OUT_OF_RESOURCES. */
+fcl_status fcl_create_buffer(fcl_context ctx, uint32_t flags, size_t bytes, uint32_t elem_size,
+                             const void *host_init, fcl_buffer *out);
+
+/* As fcl_create_buffer, but adopt caller-owned memory: with
+ * FCL_MEM_USE_HOST_PTR, host_ptr (pinned, >= bytes) becomes the host mirror;
+ * with FCL_MEM_USE_DEVICE_PTR, device_ptr (>= bytes, 16-byte aligned)
+ * becomes the device copy.  The caller keeps ownership and must keep the
+ * memory alive until fcl_release_buffer.  Both copies are assumed coherent
+ * on entry unless only one pointer is given, in which case the other copy is
+ * initialised from it. */
+fcl_status fcl_create_buffer_ext(fcl_context ctx, uint32_t flags, size_t bytes, uint32_t elem_size,
+                                 void *host_ptr, void *device_ptr, fcl_buffer *out);
+fcl_status fcl_release_buffer(fcl_buffer buf);
+
+/* Write [offset, offset+n) of buf from host memory src to both copies
+ * (clEnqueueWriteBuffer -> writes to both devices, L16.s1).  src may be the
+ * buffer's own host mirror (then only the device copy is updated).  With
+ * blocking == 0 the host->device copy is asynchronous on the main stream;
+ * src may be reused as soon as the call returns (it is copied to the pinned
+ * mirror first).  Errors: FCL_INVALID_VALUE (range), FCL_CONTEXT_LOST. */
+fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer buf, size_t offset, size_t n,
+                            const void *src, int32_t blocking);
+
+/* Read [offset, offset+n) of buf into dst.  Uses the host mirror when it is
+ * current (data location tracking, L20.s31-33), else copies device->host.
+ * Always blocking for the returned bytes. */
+fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer buf, size_t offset, size_t n,
+                           void *dst, int32_t blocking);
+
+/* Query a buffer's pointers and sizes (any out pointer may be NULL). */
+fcl_status fcl_buffer_info(fcl_buffer buf, void **host_ptr, void **device_ptr, size_t *bytes,
+                           uint32_t *elem_size);
+
+/* ---- Kernels.  Built in: each is a GPU body (instantiated in the
+ * persistent dispatcher) plus a host work-group body with the same
+ * arithmetic.  Names: atax_tmp, atax_y, bicg_s, bicg_q,
+ * gesummv, syrk, syr2k, conv2d (suffix _f32 or _i32) and corr_mean,
+ * corr_std, corr_reduce, corr_corr (suffix _f32).  Argument signatures are
+ * listed in DESIGN.md §5 and returned by fcl_kernel_signature. ---- */
+fcl_status fcl_get_kernel(fcl_context ctx, const char *name, fcl_kernel *out);
+/* Writes a '\0'-terminated signature such as "A:in x:in tmp:out n0:i n1:i"
+ * into buf (at most len bytes). */
+fcl_status fcl_kernel_signature(fcl_kernel k, char *buf, size_t len);
+
+#define FCL_ARG_BUFFER 0
+#define FCL_ARG_INT    1
+#define FCL_ARG_FLOAT  2
+
+#define FCL_ACCESS_IN    1
+#define FCL_ACCESS_OUT   2
+#define FCL_ACCESS_INOUT 3   /* IN | OUT (C4: out/inout identification, L16.s2) */
+
+typedef struct {
+    int32_t    kind;    /* FCL_ARG_BUFFER | FCL_ARG_INT | FCL_ARG_FLOAT */
+    int32_t    access;  /* for buffers: FCL_ACCESS_*; must cover what the kernel writes */
+    fcl_buffer buffer;
+    int64_t    i;       /* FCL_ARG_INT value */
+    double     f;       /* FCL_ARG_FLOAT value (rounded to the kernel's float type) */
+} fcl_arg;
+
+#define FCL_MODE_COOP     0  /* FluidiCL cooperative execution (the method) */
+#define FCL_MODE_GPU_ONLY 1  /* the same GPU bodies as a plain grid, + D2H of outputs */
+#define FCL_MODE_CPU_ONLY 2  /* the host executor runs every work-group */
+
+typedef struct {
+    int32_t mode;            /* FCL_MODE_* (default COOP) */
+    int64_t forced_split;    /* >= 0: test hook -- the host executes exactly [s, hi) and the GPU
+                                is told so before it starts (deterministic split); -1 = race */
+    int32_t init_chunk_pct;  /* C11 initial chunk, % of work-groups (default 2; L26.s28) */
+    int32_t step_pct;        /* C11 growth step, % of work-groups (default 2) */
+    int32_t cpu_wg_split;    /* C23 work-group splitting across host threads (default 1) */
+    int32_t abort_period;    /* in-loop abort check every K inner iterations (C24/C25); 0 = default,
+                                < 0 = checks at work-group start only (NoAbortUnroll analog) */
+    int32_t defer_merge;     /* 1 = leave staged results unmerged until fcl_merge (test hook) */
+    int32_t n_host_threads;  /* 0 = context default; else use at most this many */
+    int32_t host_delay_us;   /* fault injection: sleep before each host chunk */
+    int32_t drop_publish;    /* fault injection: stage chunks but never publish the watermark */
+    int64_t wg_lo, wg_hi;    /* execute only flattened ids [wg_lo, wg_hi) (multi-GPU slice);
+                                wg_hi <= 0 means the whole NDRange */
+} fcl_launch_opts;
+
+/* Fill *opts with the defaults above. */
+fcl_status fcl_default_launch_opts(fcl_launch_opts *opts);
+
+typedef struct {
+    int64_t n_wg;                /* work-groups in the executed range */
+    int64_t wg_lo, wg_hi;
+    int64_t gpu_watermark;       /* lowest watermark the GPU acted on (hi if it never skipped) */
+    int64_t published_watermark; /* last watermark the host published (hi if none) */
+    int64_t gpu_tasks, gpu_tasks_total;  /* GPU tasks executed / in the range */
+    int64_t cpu_wgs;             /* work-groups the host executed (incl. abandoned partial chunks) */
+    int32_t n_chunks;            /* host chunks started */
+    int32_t cpu_did_all;         /* the host covered the whole range first (L16.s21) */
+    int32_t merged;              /* a diff-merge was enqueued */
+    int32_t gpu_launches;        /* kernels of ours launched for this call */
+    int64_t merge_bytes;         /* bytes of each stream covered by the merge(s) */
+    int64_t h2d_bytes, d2h_bytes;
+    double  t_call_ms;           /* host wall time of fcl_enqueue_ndrange */
+    double  t_gpu_kernel_ms;     /* CUDA-event time of the dispatcher / plain grid on the main stream */
+    double  t_merge_ms;          /* CUDA-event time of the merge kernel(s) */
+    double  t_host_ms;           /* host executor busy time */
+    int32_t chunk_sizes[64];     /* first chunk sizes (C11 trace) */
+} fcl_launch_info;
+
+/* Launch `kernel` over the NDRange (work_dim in 1..3, gws[k] % lws[k] == 0,
+ * prod(lws) <= 1024) with args in the kernel's signature order.
+ * COOP: the GPU dispatcher and the host executor race over the range; on
+ * return every output buffer is current on the host (or will be once the
+ * queued device->host copy completes -- see fcl_finish) and, once the queued
+ * device work completes, on the device.  opts / info may be NULL.
+ * Errors: FCL_INVALID_WORK_DIMENSION, FCL_INVALID_WORK_GROUP_SIZE,
+ * FCL_INVALID_GLOBAL_WORK_SIZE, FCL_INVALID_KERNEL_ARGS, FCL_INVALID_VALUE,
+ * FCL_OUT_OF_RESOURCES, FCL_CONTEXT_LOST. */
+fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work_dim,
+                               const size_t gws[3], const size_t lws[3],
+                               const fcl_arg *args, uint32_t n_args,
+                               const fcl_launch_opts *opts, fcl_launch_info *info);
+
+/* Merge the staged host results of the last kernel into buf's device copy
+ * (only needed with opts.defer_merge = 1; otherwise a no-op).  Fig 9. */
+fcl_status fcl_merge(fcl_context ctx, fcl_buffer buf);
+
+/* The diff-merge kernel on raw device memory (microbench / test entry):
+ * for every elem_size-byte element e of [0, bytes):
+ *     if (cpu[e] != twin[e]) gpu[e] = cpu[e]        (bitwise compare)
+ * gpu, cpu, twin: device pointers, equal alignment mod 16 for the vector
+ * path; bytes % elem_size == 0; elem_size in {1,2,4,8}.  Asynchronous on
+ * `stream` (cudaStream_t; NULL = legacy default stream). */
+fcl_status fcl_merge_raw(void *gpu, const void *cpu, const void *twin, size_t bytes,
+                         uint32_t elem_size, void *stream);
+
+/* Wait until every launch, merge and copy of the context has completed;
+ * outputs are then coherent on host and device.  Reports deferred errors. */
+fcl_status fcl_finish(fcl_context ctx);
+
+/* Info of the most recent fcl_enqueue_ndrange, with event timings resolved
+ * (call after fcl_finish). */
+fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info);
+
+/* Multi-GPU slicing helper: a contiguous flattened-id range for
+ * rank `rank` of `nranks`, balanced and aligned to the kernel's GPU task
+ * granularity so slices never split a task. */
+fcl_status fcl_slice_range(fcl_kernel kernel, uint32_t work_dim, const size_t gws[3],
+                           const size_t lws[3], int32_t rank, int32_t nranks,
+                           int64_t *wg_lo, int64_t *wg_hi);
+
+const char *fcl_status_string(fcl_status s);
+const char *fcl_last_error(fcl_context ctx);
+/* Library version string, e.g. "fcl-b200 0.1 sm_100a". */
+const char *fcl_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FCL_H */

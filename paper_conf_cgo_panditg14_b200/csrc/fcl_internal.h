@@ -1,0 +1,99 @@
+// fcl_internal.h -- internal interfaces of the FluidiCL B200 runtime (not part of the C-ABI).
+//
+// Three translation units share these declarations:
+//   runtime.cpp      context, buffers, twin/stage pool, host executor, launch orchestration, C-ABI
+//   host_bodies.cpp  host work-group bodies (the CPU side of every kernel)
+//   kernels.cu       sm_100a persistent dispatcher, GPU task bodies, diff-merge kernel
+//
+// Bit-identity contract: for every fp32 kernel the host body
+// and the GPU body perform the same IEEE-754 operations on the same operands in the same
+// order (explicit fma / add / mul / div / sqrt, no contraction: host code is compiled with
+// -ffp-contract=off, device code uses __f*_rn intrinsics).  Hence a word computed by the
+// host is bit-identical to the word the GPU would have computed, for any split.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+
+typedef struct CUstream_st *cudaStream_t_fwd;
+
+namespace fcl {
+
+enum KernelId : int {
+    K_ATAX_TMP = 0, K_ATAX_Y, K_BICG_S, K_BICG_Q, K_GESUMMV, K_SYRK, K_SYR2K,
+    K_CORR_MEAN, K_CORR_STD, K_CORR_REDUCE, K_CORR_CORR, K_CONV2D, K_NUM
+};
+
+// Canonical reduction shapes shared by host and device bodies (they define the
+// fp32 operation order, not a thread mapping).
+constexpr int kRowPartitions = 128;  // row-dot: partial q sums columns j with j % 128 == q
+constexpr int kColPartitions = 32;   // col-dot: partial q sums rows i with i % 32 == q
+
+// NDRange geometry.  fgid = g0 + ng0 * (g1 + ng1 * g2) (Fig 5, dimension 0 fastest).
+struct Geom {
+    int work_dim;
+    int64_t gws[3], lws[3], ng[3];
+    int64_t n_wg;
+};
+
+// Resolved kernel arguments (device and host addresses of every buffer argument).
+struct KArgs {
+    int kernel;
+    bool integer;
+    int nbuf;
+    void *dev[6];
+    void *host[6];
+    int64_t n0, n1;        // rows / columns of the row-major input (SYRK/SYR2K: N, M)
+    float alpha, beta, eps;
+    int32_t ialpha, ibeta;
+};
+
+// Parameters of one cooperative (FluidiCL) dispatcher launch.
+struct CoopCtl {
+    const unsigned long long *status;   // {epoch:32 | W:32}; device-visible address
+    unsigned int epoch;                 // this launch's kernel id (C14)
+    unsigned int w_default;             // watermark when the status is stale: the range end
+    unsigned long long *claim;          // device claim counter (0 on entry, reset by last CTA)
+    unsigned int *done;                 // CTA exit counter (0 on entry, reset by last CTA)
+    unsigned int *wmin;                 // lowest watermark acted on (0xFFFFFFFF on entry)
+    unsigned long long *tasks;          // tasks executed (0 on entry)
+    unsigned long long *exit_rec;       // device-visible address of the mapped host exit record
+    long long task_lo, task_hi;         // task index range of this launch
+    int abort_period;                   // in-task poll period (body-specific units); 0 = none
+};
+
+// ---- GPU side (kernels.cu) ----
+struct TaskSpace {
+    int64_t ntasks;      // tasks covering the whole NDRange, keys ascending
+    int threads;         // CTA size of the body
+};
+TaskSpace gpu_task_space(const KArgs &a, const Geom &g);
+int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t);   // min fgid of task t
+bool gpu_geometry_ok(const KArgs &a, const Geom &g, const char **why);
+int gpu_default_abort_period(const KArgs &a);
+// Slice boundaries (multi-GPU / wg_lo, wg_hi) must be multiples of this many work-groups
+// so that no GPU task straddles a boundary.
+int64_t gpu_slice_align(const KArgs &a, const Geom &g);
+// Launch the persistent cooperative dispatcher; returns the grid size used (<= 0 on error).
+int gpu_launch_coop(const KArgs &a, const Geom &g, const CoopCtl &c, int num_sms, void *stream);
+// Plain grid over tasks [task_lo, task_hi) with no status reads (GPU-only baseline).
+int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream);
+// Fig 9 diff-merge on [0, bytes) of three device buffers.
+int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes, int elem_size,
+                     int num_sms, void *stream);
+// One-thread kernel that stores `value` to `addr` (status publication fallback).
+int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream);
+const char *gpu_last_error_string();
+
+// ---- Host side (host_bodies.cpp) ----
+// Execute part `part` of `nparts` of work-group `fgid` on host memory (C9 / C23).
+// `abort_flag` is polled inside long bodies; a body that sees it set stops before
+// storing an incomplete value (write-once).
+void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts,
+                  const volatile int *abort_flag);
+
+// Conservative contiguous byte span [*b0, *b1) of output buffer `buf_index` written by
+// work-groups [lo, hi) (superset of the exact footprint; the diff-merge tolerates it).
+void out_span(const KArgs &a, const Geom &g, int buf_index, int64_t lo, int64_t hi,
+              size_t *b0, size_t *b1);
+
+}  // namespace fcl

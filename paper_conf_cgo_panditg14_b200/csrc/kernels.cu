@@ -1,0 +1,1045 @@
+// kernels.cu -- sm_100a kernels of the B200 FluidiCL hot path.
+//
+//  * coop_kernel<Body>: the persistent work-group dispatcher (C8, Fig 8, L16.s12/s.26-27,
+//    Figs 11-12 / L22.s1-4).  CTAs claim GPU tasks in ascending key order (key = lowest
+//    flattened work-group id a task covers, so the GPU "starts executing from the other end",
+//    L16.s8) and read the host's watermark word {epoch, W} with an ld.relaxed.sys load.  A task
+//    runs iff epoch matches and key < W; otherwise the CTA exits -- every later task is covered
+//    too because W only decreases and keys only increase.  Long tasks poll the word again every
+//    `abort_period` inner iterations (C24/C25, L20.s44-51) and abort before storing (write-once).
+//  * plain_kernel<Body>: the same bodies as an ordinary grid with no status reads (GPU-only).
+//  * merge_kernel<ES>: the Fig 9 diff-merge (L18.s1-5), 128-bit vectorised, bitwise compare at
+//    element granularity (L16.s32-35), predicated stores, warp ballot to skip unchanged runs.
+//
+// A "task" is the GPU's unit of claiming: a sub-range of one work-group (row/col dot kernels)
+// or a tile of several work-groups (GEMM-like, stencil and elementwise kernels).  Work-group
+// independence (L14.s22-23) makes both legal; the merge absorbs any duplicated work.
+//
+// Arithmetic follows the canonical operation order shared with host_bodies.cpp (see
+// fcl_internal.h): __fmaf_rn / __fadd_rn / __fmul_rn / __fdiv_rn / __fsqrt_rn only.
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstdio>
+
+#include "fcl_internal.h"
+
+namespace fcl {
+
+// ------------------------------------------------------------------------------------------
+// Arithmetic (canonical IEEE operations; integer variants wrap mod 2^32)
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ float op_fma(float a, float b, float c) { return __fmaf_rn(a, b, c); }
+__device__ __forceinline__ int32_t op_fma(int32_t a, int32_t b, int32_t c) {
+    return (int32_t)((uint32_t)a * (uint32_t)b + (uint32_t)c);
+}
+__device__ __forceinline__ float op_add(float a, float b) { return __fadd_rn(a, b); }
+__device__ __forceinline__ int32_t op_add(int32_t a, int32_t b) { return (int32_t)((uint32_t)a + (uint32_t)b); }
+__device__ __forceinline__ float op_mul(float a, float b) { return __fmul_rn(a, b); }
+__device__ __forceinline__ int32_t op_mul(int32_t a, int32_t b) { return (int32_t)((uint32_t)a * (uint32_t)b); }
+
+template <typename T> struct V4;
+template <> struct V4<float> { typedef float4 type; };
+template <> struct V4<int32_t> { typedef int4 type; };
+
+// Streaming 128-bit load that does not allocate in L1 (data read exactly once).
+template <typename T>
+__device__ __forceinline__ typename V4<T>::type ld_stream4(const T *p) {
+    typename V4<T>::type v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(*reinterpret_cast<uint32_t *>(&v.x)), "=r"(*reinterpret_cast<uint32_t *>(&v.y)),
+                   "=r"(*reinterpret_cast<uint32_t *>(&v.z)), "=r"(*reinterpret_cast<uint32_t *>(&v.w))
+                 : "l"(p));
+    return v;
+}
+template <typename T>
+__device__ __forceinline__ typename V4<T>::type ld_cached4(const T *p) {
+    return __ldg(reinterpret_cast<const typename V4<T>::type *>(p));
+}
+
+// ------------------------------------------------------------------------------------------
+// Watermark access (D1/D2, Fig 8)
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ unsigned long long ld_status(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned int decode_w(unsigned long long st, const CoopCtl &c) {
+    // A status word from another kernel (stale epoch) means "nothing covered" (C14, L20.s9).
+    return ((unsigned int)(st >> 32) == c.epoch) ? (unsigned int)st : c.w_default;
+}
+
+// Per-task view of the status for in-task polling (abort checks in loops, Fig 12).
+struct TaskCtx {
+    const CoopCtl *c;          // nullptr for plain launches
+    long long key;
+    unsigned long long pending;  // thread 0: status word loaded at the previous poll
+    int *s_flag;                 // shared memory broadcast slot (D2: the local 'completedatcpu')
+    unsigned int abort_w;
+
+    // Called by ALL threads at a CTA-uniform point with a CTA-uniform iteration count.
+    __device__ __forceinline__ bool poll(int it) {
+        if (c == nullptr || c->abort_period <= 0 || it == 0 || (it % c->abort_period) != 0) return false;
+        if (threadIdx.x == 0) {
+            unsigned int w = decode_w(pending, *c);
+            pending = ld_status(c->status);   // prefetch: consumed at the next poll
+            *s_flag = ((unsigned long long)key >= (unsigned long long)w) ? (int)(w + 1u) : 0;
+        }
+        __syncthreads();
+        int f = *s_flag;
+        __syncthreads();
+        if (f) { abort_w = (unsigned int)(f - 1); return true; }
+        return false;
+    }
+};
+
+// ------------------------------------------------------------------------------------------
+// Dispatcher (persistent, ascending claim) and plain grid
+// ------------------------------------------------------------------------------------------
+template <class Body>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+coop_kernel(const CoopCtl c, const typename Body::Params bp) {
+    __shared__ long long s_task;
+    __shared__ unsigned int s_w;
+    __shared__ int s_flag;
+    __shared__ __align__(16) typename Body::Smem smem;
+
+    long long t_next = 0;
+    unsigned long long st_next = 0;
+    unsigned long long executed = 0;
+    if (threadIdx.x == 0) {
+        t_next = c.task_lo + (long long)atomicAdd(c.claim, 1ull);
+        st_next = ld_status(c.status);
+    }
+    for (;;) {
+        if (threadIdx.x == 0) { s_task = t_next; s_w = decode_w(st_next, c); }
+        __syncthreads();
+        const long long t = s_task;
+        const unsigned int w = s_w;
+        if (t >= c.task_hi) break;
+        const long long key = Body::key(bp, t);
+        if ((unsigned long long)key >= (unsigned long long)w) {   // covered by the host (Fig 8)
+            if (threadIdx.x == 0) atomicMin(c.wmin, w);
+            break;
+        }
+        TaskCtx tc;
+        tc.c = &c; tc.key = key; tc.s_flag = &s_flag; tc.abort_w = 0; tc.pending = 0;
+        if (threadIdx.x == 0) {
+            // claim the next task and prefetch the status while this one runs
+            t_next = c.task_lo + (long long)atomicAdd(c.claim, 1ull);
+            st_next = ld_status(c.status);
+            tc.pending = st_next;
+        }
+        const bool aborted = Body::run(bp, t, tc, smem);
+        if (aborted) {
+            if (threadIdx.x == 0) atomicMin(c.wmin, tc.abort_w);
+            break;
+        }
+        ++executed;
+        __syncthreads();
+    }
+    // Exit protocol: the last CTA out publishes the exit record to mapped host memory and
+    // resets the device counters for the next launch (stream order serialises launches).
+    if (threadIdx.x == 0) {
+        if (executed) atomicAdd(c.tasks, executed);
+        __threadfence();
+        const unsigned int prev = atomicAdd(c.done, 1u);
+        if (prev == gridDim.x - 1) {
+            __threadfence();
+            const unsigned int wm = atomicExch(c.wmin, 0xFFFFFFFFu);
+            const unsigned long long nt = atomicExch(c.tasks, 0ull);
+            atomicExch(c.claim, 0ull);
+            atomicExch(c.done, 0u);
+            __threadfence_system();
+            asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(c.exit_rec + 1), "l"(nt) : "memory");
+            __threadfence_system();
+            const unsigned long long rec = ((unsigned long long)c.epoch << 32) | wm;
+            asm volatile("st.release.sys.global.b64 [%0], %1;" ::"l"(c.exit_rec), "l"(rec) : "memory");
+        }
+    }
+}
+
+template <class Body>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+plain_kernel(const typename Body::Params bp, long long task_lo) {
+    __shared__ int s_flag;
+    __shared__ __align__(16) typename Body::Smem smem;
+    TaskCtx tc;
+    tc.c = nullptr; tc.key = 0; tc.pending = 0; tc.s_flag = &s_flag; tc.abort_w = 0;
+    Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
+}
+
+__global__ void store64_kernel(unsigned long long *addr, unsigned long long v) {
+    asm volatile("st.release.sys.global.b64 [%0], %1;" ::"l"(addr), "l"(v) : "memory");
+}
+
+// ------------------------------------------------------------------------------------------
+// Row-dot bodies: ATAX kernel 1 (tmp = A x), BICG kernel 2 (q = A p), GESUMMV.
+// A work-group is lws consecutive rows; a task is R <= 8 of them, one warp per row.
+// Canonical order: partial q (q = j % 128) accumulates A[i][j]*x[j] for ascending j; lane l
+// owns partials 4l..4l+3, folds them ((p0+p1)+p2)+p3, then a xor-butterfly over lanes
+// (offsets 16, 8, 4, 2, 1) -- host_bodies.cpp replays exactly this.
+// ------------------------------------------------------------------------------------------
+struct EmptySmem { int dummy; };
+
+template <typename T, int NMAT>
+struct RowDotBody {
+    static constexpr int kThreads = 256;
+    static constexpr int kMinBlocks = 2;
+    struct Params {
+        const T *A; const T *B; const T *x; T *out0; T *out1;
+        long long nrows, ncols, lws; int R; T alpha, beta; int vec4;
+    };
+    typedef EmptySmem Smem;
+
+    __device__ static long long key(const Params &p, long long t) { return (t * p.R) / p.lws; }
+
+    __device__ static T warp_fold(T p0, T p1, T p2, T p3) {
+        T v = op_add(op_add(op_add(p0, p1), p2), p3);
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) v = op_add(v, __shfl_xor_sync(0xffffffffu, v, off));
+        return v;
+    }
+
+    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
+        const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+        if (warp >= p.R) return false;
+        const long long i = t * p.R + warp;
+        if (i >= p.nrows) return false;
+        const T *Ar = p.A + i * p.ncols;
+        const T *Br = (NMAT == 2) ? p.B + i * p.ncols : nullptr;
+        T a0 = 0, a1 = 0, a2 = 0, a3 = 0, b0 = 0, b1 = 0, b2 = 0, b3 = 0;
+        const long long nfull = p.ncols / 128;
+        long long k = 0;
+        if (p.vec4) {
+            // main loop: loads of 4 blocks issued before their FMAs (memory-level parallelism)
+            for (; k + 4 <= nfull; k += 4) {
+                typename V4<T>::type av[4], bv[4], xv[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const long long j = (k + u) * 128 + 4 * lane;
+                    av[u] = ld_stream4(Ar + j);
+                    if (NMAT == 2) bv[u] = ld_stream4(Br + j);
+                    xv[u] = ld_cached4(p.x + j);
+                }
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    a0 = op_fma(av[u].x, xv[u].x, a0); a1 = op_fma(av[u].y, xv[u].y, a1);
+                    a2 = op_fma(av[u].z, xv[u].z, a2); a3 = op_fma(av[u].w, xv[u].w, a3);
+                    if (NMAT == 2) {
+                        b0 = op_fma(bv[u].x, xv[u].x, b0); b1 = op_fma(bv[u].y, xv[u].y, b1);
+                        b2 = op_fma(bv[u].z, xv[u].z, b2); b3 = op_fma(bv[u].w, xv[u].w, b3);
+                    }
+                }
+            }
+            for (; k < nfull; ++k) {
+                const long long j = k * 128 + 4 * lane;
+                typename V4<T>::type av = ld_stream4(Ar + j), xv = ld_cached4(p.x + j);
+                a0 = op_fma(av.x, xv.x, a0); a1 = op_fma(av.y, xv.y, a1);
+                a2 = op_fma(av.z, xv.z, a2); a3 = op_fma(av.w, xv.w, a3);
+                if (NMAT == 2) {
+                    typename V4<T>::type bv = ld_stream4(Br + j);
+                    b0 = op_fma(bv.x, xv.x, b0); b1 = op_fma(bv.y, xv.y, b1);
+                    b2 = op_fma(bv.z, xv.z, b2); b3 = op_fma(bv.w, xv.w, b3);
+                }
+            }
+        }
+        // scalar path (unaligned rows) and the ragged tail, same partition order
+        for (; k * 128 < p.ncols; ++k) {
+            const long long j = k * 128 + 4 * lane;
+#define FCL_ROWDOT_TAIL(C, AC, BC)                                             \
+            if (j + C < p.ncols) {                                             \
+                const T xv = p.x[j + C];                                       \
+                AC = op_fma(Ar[j + C], xv, AC);                                \
+                if (NMAT == 2) BC = op_fma(Br[j + C], xv, BC);                 \
+            }
+            FCL_ROWDOT_TAIL(0, a0, b0)
+            FCL_ROWDOT_TAIL(1, a1, b1)
+            FCL_ROWDOT_TAIL(2, a2, b2)
+            FCL_ROWDOT_TAIL(3, a3, b3)
+#undef FCL_ROWDOT_TAIL
+        }
+        const T va = warp_fold(a0, a1, a2, a3);
+        if (NMAT == 1) {
+            if (lane == 0) p.out0[i] = va;
+        } else {
+            const T vb = warp_fold(b0, b1, b2, b3);
+            if (lane == 0) {
+                p.out0[i] = va;                                           // tmp[i]
+                p.out1[i] = op_add(op_mul(p.alpha, va), op_mul(p.beta, vb)); // y[i]
+            }
+        }
+        return false;
+    }
+};
+
+// ------------------------------------------------------------------------------------------
+// Column-dot bodies: ATAX kernel 2 (y = A^T tmp), BICG kernel 1 (s = A^T r), CORR mean / std.
+// A work-group is lws consecutive columns; a task is CB <= 32 of them, all rows.
+// Canonical order: partial q (q = i % 32) accumulates rows i = q, q+32, ... ascending; the 32
+// partials are then added sequentially q = 0..31.  Warp w of the CTA owns partial w.
+// ------------------------------------------------------------------------------------------
+enum { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
+
+template <typename T, int MODE>
+struct ColDotBody {
+    static constexpr int kThreads = 1024;
+    static constexpr int kMinBlocks = 1;
+    struct Params {
+        const T *A; const T *v; const T *mean; T *out;
+        long long nrows, ncols, lws; int CB; float nf, eps;
+    };
+    struct Smem { T red[32][33]; };
+
+    __device__ static long long key(const Params &p, long long t) { return (t * p.CB) / p.lws; }
+
+    __device__ static T term(const Params &p, T a, long long i, T mj, T acc) {
+        if (MODE == COL_DOT) return op_fma(a, p.v[i], acc);
+        if (MODE == COL_SUM) return op_add(acc, a);
+        const T c = op_add(a, -mj);   // a - mean (exact negation, then one rounding)
+        return op_fma(c, c, acc);
+    }
+
+    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &sm) {
+        const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+        const long long j = t * p.CB + lane;
+        const bool active = (lane < p.CB) && (j < p.ncols);
+        T acc = 0;
+        if (active) {
+            const T mj = (MODE == COL_SQDEV) ? p.mean[j] : T(0);
+            const T *col = p.A + j;
+            long long i = w;
+            for (; i + 7 * 32 < p.nrows; i += 8 * 32) {
+                T a[8];
+#pragma unroll
+                for (int u = 0; u < 8; ++u) a[u] = __ldcs(col + (i + 32 * u) * p.ncols);
+#pragma unroll
+                for (int u = 0; u < 8; ++u) acc = term(p, a[u], i + 32 * u, mj, acc);
+            }
+            for (; i < p.nrows; i += 32) acc = term(p, __ldcs(col + i * p.ncols), i, mj, acc);
+        }
+        sm.red[w][lane] = acc;
+        __syncthreads();
+        if (w == 0 && active) {
+            T tot = sm.red[0][lane];
+#pragma unroll 8
+            for (int q = 1; q < 32; ++q) tot = op_add(tot, sm.red[q][lane]);
+            if (MODE == COL_DOT) {
+                p.out[j] = tot;
+            } else if (MODE == COL_SUM) {
+                p.out[j] = (T)__fdiv_rn((float)tot, p.nf);
+            } else {
+                float s = __fsqrt_rn(__fdiv_rn((float)tot, p.nf));
+                p.out[j] = (T)((s <= p.eps) ? 1.0f : s);
+            }
+        }
+        __syncthreads();
+        return false;
+    }
+};
+
+// ------------------------------------------------------------------------------------------
+// 2-D tiled bodies over a row-major output: a task is a tile of th x tw work-groups, tiles
+// enumerated row-major so that keys ascend.  key = gx0 + ngx * gy0.
+// ------------------------------------------------------------------------------------------
+struct Tile2D {
+    long long nrows, ncols;  // output extent
+    long long ngx, lws0, lws1;
+    int tw, th;              // tile size in work-groups
+    long long ntx;           // tiles per tile-row
+    __device__ __host__ long long key(long long t) const {
+        const long long tx = t % ntx, ty = t / ntx;
+        return tx * tw + ngx * (ty * th);
+    }
+};
+
+// CORR reduce (in place): d[i][j] = (d[i][j] - mean[j]) / (sqrt(n) * std[j]).
+struct CorrReduceBody {
+    static constexpr int kThreads = 256;
+    static constexpr int kMinBlocks = 4;
+    struct Params { float *data; const float *mean; const float *std_; Tile2D tl; float sqrtn; };
+    typedef EmptySmem Smem;
+    __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
+    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
+        const Tile2D &tl = p.tl;
+        const long long tx = t % tl.ntx, ty = t / tl.ntx;
+        const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
+        const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
+        for (int e = threadIdx.x; e < tcols * trows; e += kThreads) {
+            const long long i = r0 + e / tcols, j = c0 + e % tcols;
+            if (i < tl.nrows && j < tl.ncols) {
+                float *q = p.data + i * tl.ncols + j;
+                const float den = __fmul_rn(p.sqrtn, p.std_[j]);
+                *q = __fdiv_rn(__fadd_rn(*q, -p.mean[j]), den);
+            }
+        }
+        return false;
+    }
+};
+
+// 2DCONV (PolyBench/GPU): interior B[i][j] = sum of 9 taps, canonical PolyBench term order
+// (column j-1 rows i-1..i+1, then column j, then column j+1): first tap a product, the other
+// eight fused multiply-adds.  Border untouched.
+template <typename T>
+struct Conv2DBody {
+    static constexpr int kThreads = 256;
+    static constexpr int kMinBlocks = 4;
+    struct Params { const T *A; T *B; Tile2D tl; T c[9]; };   // c[a*3+b]: row offset a-1, col offset b-1
+    typedef EmptySmem Smem;
+    __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
+    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
+        const Tile2D &tl = p.tl;
+        const long long tx = t % tl.ntx, ty = t / tl.ntx;
+        const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
+        const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
+        const long long ni = tl.nrows, nj = tl.ncols;
+        for (int cc = threadIdx.x; cc < tcols; cc += kThreads) {
+            const long long j = c0 + cc;
+            if (j < 1 || j >= nj - 1) continue;
+            long long i = r0 < 1 ? 1 : r0;
+            const long long iend = (r0 + trows < ni - 1) ? r0 + trows : ni - 1;
+            if (i >= iend) continue;
+            const T *a = p.A + j;
+            // sliding window: w[a][b] = A[i + a - 1][j + b - 1]
+            T w0[3], w1[3], w2[3];
+#pragma unroll
+            for (int b = 0; b < 3; ++b) { w0[b] = __ldg(a + (i - 1) * nj + b - 1); w1[b] = __ldg(a + i * nj + b - 1); }
+            for (; i < iend; ++i) {
+#pragma unroll
+                for (int b = 0; b < 3; ++b) w2[b] = __ldg(a + (i + 1) * nj + b - 1);
+                T s = op_mul(p.c[0], w0[0]);
+                s = op_fma(p.c[3], w1[0], s);
+                s = op_fma(p.c[6], w2[0], s);
+                s = op_fma(p.c[1], w0[1], s);
+                s = op_fma(p.c[4], w1[1], s);
+                s = op_fma(p.c[7], w2[1], s);
+                s = op_fma(p.c[2], w0[2], s);
+                s = op_fma(p.c[5], w1[2], s);
+                s = op_fma(p.c[8], w2[2], s);
+                __stcs(p.B + i * nj + j, s);
+#pragma unroll
+                for (int b = 0; b < 3; ++b) { w0[b] = w1[b]; w1[b] = w2[b]; }
+            }
+        }
+        return false;
+    }
+};
+
+// ------------------------------------------------------------------------------------------
+// GEMM-like bodies on CUDA cores (fp32 FFMA / int32 IMAD; no tensor cores: fp32 parity, see
+// DESIGN.md §6): SYRK, SYR2K and CORR's symmat.  Output tile 128 x 128, 256 threads, 8 x 8
+// outputs per thread, k-tile 8, double-buffered shared memory.  Every output accumulates its
+// k-chain in ascending k with one fma per term (SYR2K: A_i*B_j then B_i*A_j per k).
+// ------------------------------------------------------------------------------------------
+enum { G_SYRK = 0, G_SYR2K = 1, G_CORR = 2 };
+constexpr int GBM = 128, GBK = 8, GPAD = 4;
+
+template <typename T, int OP>
+struct GemmBody {
+    static constexpr int kThreads = 256;
+    static constexpr int kMinBlocks = 2;
+    static constexpr int kOps = (OP == G_SYR2K) ? 4 : 2;   // operand tiles per stage
+    struct Params {
+        const T *A; const T *B; T *C;
+        long long n;      // output is n x n (CORR: M x M)
+        long long m;      // contraction length (CORR: number of data rows N)
+        long long ld;     // row length of the operand matrix (SYRK/SYR2K: m; CORR: n)
+        T alpha, beta;
+        long long ntile;  // tiles per dimension
+        long long ngx, lws0, lws1, lws;  // work-group geometry for keys
+        int vec4;
+    };
+    struct Smem { T s[2][kOps][GBK][GBM + GPAD]; };
+
+    __device__ static void tile_of(const Params &p, long long t, long long &bi, long long &bj) {
+        if (OP == G_CORR) {  // upper triangle, row-major over (b1 <= b2)
+            long long b1 = 0, rem = t;
+            while (rem >= p.ntile - b1) { rem -= p.ntile - b1; ++b1; }
+            bi = b1; bj = b1 + rem;
+        } else {
+            bi = t / p.ntile; bj = t % p.ntile;
+        }
+    }
+    __device__ static long long key(const Params &p, long long t) {
+        long long bi, bj;
+        tile_of(p, t, bi, bj);
+        if (OP == G_CORR) return (bi * GBM) / p.lws;
+        return (bj * GBM) / p.lws0 + p.ngx * ((bi * GBM) / p.lws1);
+    }
+
+    // Load one k-tile of operand `which` into registers (4 elements per thread).
+    // K-contiguous operands (SYRK/SYR2K): element (row r, k) at X[(row0 + r) * ld + k].
+    // MN-contiguous operands (CORR): element (k, col c) at X[k * ld + col0 + c].
+    __device__ static void gload(const Params &p, const T *X, long long base, long long k0, T r[4]) {
+        const int tid = threadIdx.x;
+        if (OP == G_CORR) {
+            const int kk = tid >> 5, c = (tid & 31) * 4;
+            const long long k = k0 + kk, col = base + c;
+            if (k < p.m && p.vec4 && col + 3 < p.n) {
+                typename V4<T>::type v = ld_cached4(X + k * p.ld + col);
+                r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) r[q] = (k < p.m && col + q < p.n) ? X[k * p.ld + col + q] : T(0);
+            }
+        } else {
+            const int row = tid >> 1, kq = (tid & 1) * 4;
+            const long long gr = base + row, k = k0 + kq;
+            if (gr < p.n && p.vec4 && k + 3 < p.m) {
+                typename V4<T>::type v = ld_cached4(X + gr * p.ld + k);
+                r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) r[q] = (gr < p.n && k + q < p.m) ? X[gr * p.ld + k + q] : T(0);
+            }
+        }
+    }
+    __device__ static void sstore(T (*S)[GBM + GPAD], const T r[4]) {
+        const int tid = threadIdx.x;
+        if (OP == G_CORR) {
+            const int kk = tid >> 5, c = (tid & 31) * 4;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) S[kk][c + q] = r[q];
+        } else {
+            const int row = tid >> 1, kq = (tid & 1) * 4;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) S[kq + q][row] = r[q];
+        }
+    }
+
+    __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &sm) {
+        long long bi, bj;
+        tile_of(p, t, bi, bj);
+        const long long i0 = bi * GBM, j0 = bj * GBM;
+        const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+        // operand sources: SYRK: (A rows i, A rows j); SYR2K: (A_i, B_j, B_i, A_j); CORR: (D cols i, D cols j)
+        const T *src[4];
+        long long base[4];
+        if (OP == G_SYR2K) {
+            src[0] = p.A; base[0] = i0; src[1] = p.B; base[1] = j0;
+            src[2] = p.B; base[2] = i0; src[3] = p.A; base[3] = j0;
+        } else {
+            src[0] = p.A; base[0] = i0; src[1] = p.A; base[1] = j0;
+            src[2] = src[3] = nullptr; base[2] = base[3] = 0;
+        }
+        T acc[8][8];
+#pragma unroll
+        for (int r = 0; r < 8; ++r)
+#pragma unroll
+            for (int c = 0; c < 8; ++c) acc[r][c] = 0;
+
+        const long long nkt = (p.m + GBK - 1) / GBK;
+        T reg[kOps][4];
+#pragma unroll
+        for (int o = 0; o < kOps; ++o) gload(p, src[o], base[o], 0, reg[o]);
+#pragma unroll
+        for (int o = 0; o < kOps; ++o) sstore(sm.s[0][o], reg[o]);
+        __syncthreads();
+        for (long long kt = 0; kt < nkt; ++kt) {
+            const int st = (int)(kt & 1);
+            if (kt + 1 < nkt) {
+#pragma unroll
+                for (int o = 0; o < kOps; ++o) gload(p, src[o], base[o], (kt + 1) * GBK, reg[o]);
+            }
+#pragma unroll
+            for (int kk = 0; kk < GBK; ++kk) {
+                T a[8], b[8];
+                const typename V4<T>::type a0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][0][kk][ty * 4]);
+                const typename V4<T>::type a1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][0][kk][64 + ty * 4]);
+                const typename V4<T>::type b0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][1][kk][tx * 4]);
+                const typename V4<T>::type b1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][1][kk][64 + tx * 4]);
+                a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w; a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
+                b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w; b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
+                if (OP == G_SYR2K) {
+                    T a2[8], b2[8];
+                    const typename V4<T>::type c0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][2][kk][ty * 4]);
+                    const typename V4<T>::type c1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][2][kk][64 + ty * 4]);
+                    const typename V4<T>::type d0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][3][kk][tx * 4]);
+                    const typename V4<T>::type d1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][3][kk][64 + tx * 4]);
+                    a2[0] = c0.x; a2[1] = c0.y; a2[2] = c0.z; a2[3] = c0.w; a2[4] = c1.x; a2[5] = c1.y; a2[6] = c1.z; a2[7] = c1.w;
+                    b2[0] = d0.x; b2[1] = d0.y; b2[2] = d0.z; b2[3] = d0.w; b2[4] = d1.x; b2[5] = d1.y; b2[6] = d1.z; b2[7] = d1.w;
+#pragma unroll
+                    for (int r = 0; r < 8; ++r)
+#pragma unroll
+                        for (int c = 0; c < 8; ++c) {
+                            acc[r][c] = op_fma(a[r], b[c], acc[r][c]);     // alpha*A[i][k]*B[j][k]
+                            acc[r][c] = op_fma(a2[r], b2[c], acc[r][c]);   // alpha*B[i][k]*A[j][k]
+                        }
+                } else {
+#pragma unroll
+                    for (int r = 0; r < 8; ++r)
+#pragma unroll
+                        for (int c = 0; c < 8; ++c) acc[r][c] = op_fma(a[r], b[c], acc[r][c]);
+                }
+            }
+            if (kt + 1 < nkt) {
+#pragma unroll
+                for (int o = 0; o < kOps; ++o) sstore(sm.s[st ^ 1][o], reg[o]);
+            }
+            __syncthreads();
+            if (tc.poll((int)(kt + 1))) return true;   // abort check every abort_period k-tiles (Fig 12)
+        }
+        // epilogue: write-once stores
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            const long long i = i0 + ((r < 4) ? ty * 4 + r : 64 + ty * 4 + (r - 4));
+#pragma unroll
+            for (int half = 0; half < 2; ++half) {
+                const long long jb = j0 + half * 64 + tx * 4;
+                if (OP == G_CORR) {
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) {
+                        const long long j = jb + c;
+                        if (i < p.n && j < p.n) {
+                            if (j > i) { p.C[i * p.n + j] = acc[r][half * 4 + c]; p.C[j * p.n + i] = acc[r][half * 4 + c]; }
+                            else if (j == i) p.C[i * p.n + i] = T(1);
+                        }
+                    }
+                } else {
+                    if (i >= p.n) continue;
+                    T *crow = p.C + i * p.n;
+                    if (p.vec4 && jb + 3 < p.n) {
+                        typename V4<T>::type cv = *reinterpret_cast<typename V4<T>::type *>(crow + jb);
+                        cv.x = op_fma(p.alpha, acc[r][half * 4 + 0], op_mul(p.beta, cv.x));
+                        cv.y = op_fma(p.alpha, acc[r][half * 4 + 1], op_mul(p.beta, cv.y));
+                        cv.z = op_fma(p.alpha, acc[r][half * 4 + 2], op_mul(p.beta, cv.z));
+                        cv.w = op_fma(p.alpha, acc[r][half * 4 + 3], op_mul(p.beta, cv.w));
+                        *reinterpret_cast<typename V4<T>::type *>(crow + jb) = cv;
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) {
+                            const long long j = jb + c;
+                            if (j < p.n) crow[j] = op_fma(p.alpha, acc[r][half * 4 + c], op_mul(p.beta, crow[j]));
+                        }
+                    }
+                }
+            }
+        }
+        return false;
+    }
+};
+
+// ------------------------------------------------------------------------------------------
+// Diff-merge (Fig 9): gpu[e] = (cpu[e] != twin[e]) ? cpu[e] : gpu[e], bitwise, per element.
+// cpu/twin are streamed once with 128-bit no-L1-allocate loads (4 vectors in flight per
+// thread); changed elements are stored with predicated element stores (a fully changed vector
+// with one 128-bit store), so the GPU copy is never read: traffic = 8 B/word read + 4 B per
+// changed word written.  Byte/half-word element sizes blend within the 32-bit lane.
+// ------------------------------------------------------------------------------------------
+template <int ES>
+__device__ __forceinline__ void merge_vec(uint8_t *g, const uint4 c, const uint4 t) {
+    const uint32_t cw[4] = {c.x, c.y, c.z, c.w}, tw[4] = {t.x, t.y, t.z, t.w};
+    if (ES == 4) {
+        const bool ch0 = cw[0] != tw[0], ch1 = cw[1] != tw[1], ch2 = cw[2] != tw[2], ch3 = cw[3] != tw[3];
+        if (ch0 && ch1 && ch2 && ch3) { *reinterpret_cast<uint4 *>(g) = c; return; }
+        uint32_t *gw = reinterpret_cast<uint32_t *>(g);
+        if (ch0) gw[0] = cw[0];
+        if (ch1) gw[1] = cw[1];
+        if (ch2) gw[2] = cw[2];
+        if (ch3) gw[3] = cw[3];
+    } else if (ES == 8) {
+        const bool ch0 = (cw[0] != tw[0]) || (cw[1] != tw[1]);
+        const bool ch1 = (cw[2] != tw[2]) || (cw[3] != tw[3]);
+        if (ch0 && ch1) { *reinterpret_cast<uint4 *>(g) = c; return; }
+        unsigned long long *gd = reinterpret_cast<unsigned long long *>(g);
+        if (ch0) gd[0] = ((unsigned long long)cw[1] << 32) | cw[0];
+        if (ch1) gd[1] = ((unsigned long long)cw[3] << 32) | cw[2];
+    } else {
+        uint32_t m[4];
+        bool all = true, any = false;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            if (ES == 1) m[q] = __vcmpne4(cw[q], tw[q]);
+            else m[q] = __vcmpne2(cw[q], tw[q]);
+            all &= (m[q] == 0xFFFFFFFFu);
+            any |= (m[q] != 0u);
+        }
+        if (all) { *reinterpret_cast<uint4 *>(g) = c; return; }
+        if (!any) return;
+        uint32_t *gw = reinterpret_cast<uint32_t *>(g);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            if (m[q] == 0xFFFFFFFFu) gw[q] = cw[q];
+            else if (m[q]) gw[q] = (cw[q] & m[q]) | (gw[q] & ~m[q]);
+        }
+    }
+}
+
+template <int ES>
+__device__ __forceinline__ void merge_scalar(uint8_t *g, const uint8_t *c, const uint8_t *t, size_t nbytes) {
+    for (size_t e = 0; e + ES <= nbytes; e += ES) {
+        bool ch = false;
+#pragma unroll
+        for (int b = 0; b < ES; ++b) ch |= (c[e + b] != t[e + b]);
+        if (ch) {
+#pragma unroll
+            for (int b = 0; b < ES; ++b) g[e + b] = c[e + b];
+        }
+    }
+}
+
+__device__ __forceinline__ uint4 ld_nc_v4(const uint8_t *p) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+
+template <int ES>
+__global__ void __launch_bounds__(256)
+merge_kernel(uint8_t *__restrict__ gpu, const uint8_t *__restrict__ cpu, const uint8_t *__restrict__ twin,
+             size_t head, size_t nvec, size_t tail) {
+    // bytes: [0, head) scalar, [head, head + 16*nvec) vector, then `tail` scalar bytes
+    const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const size_t nthreads = (size_t)gridDim.x * blockDim.x;
+    if (tid == 0 && head) merge_scalar<ES>(gpu, cpu, twin, head);
+    if (tid == 1 % nthreads && tail) {
+        const size_t off = head + 16 * nvec;
+        merge_scalar<ES>(gpu + off, cpu + off, twin + off, tail);
+    }
+    uint8_t *g = gpu + head;
+    const uint8_t *c = cpu + head, *t = twin + head;
+    constexpr int U = 4;
+    size_t v = tid;
+    for (; v + (U - 1) * nthreads < nvec; v += U * nthreads) {
+        uint4 cv[U], tv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) { cv[u] = ld_nc_v4(c + 16 * (v + u * nthreads)); tv[u] = ld_nc_v4(t + 16 * (v + u * nthreads)); }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const bool diff = (cv[u].x != tv[u].x) | (cv[u].y != tv[u].y) | (cv[u].z != tv[u].z) | (cv[u].w != tv[u].w);
+            // warp vote: a warp whose 512-byte segment is unchanged skips the store path
+            if (__ballot_sync(__activemask(), diff) && diff) merge_vec<ES>(g + 16 * (v + u * nthreads), cv[u], tv[u]);
+        }
+    }
+    for (; v < nvec; v += nthreads) {
+        const uint4 cv = ld_nc_v4(c + 16 * v), tv = ld_nc_v4(t + 16 * v);
+        if ((cv.x != tv.x) | (cv.y != tv.y) | (cv.z != tv.z) | (cv.w != tv.w)) merge_vec<ES>(g + 16 * v, cv, tv);
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// Host-side launch plumbing
+// ------------------------------------------------------------------------------------------
+static thread_local char g_err[256];
+const char *gpu_last_error_string() { return g_err; }
+static int seterr(cudaError_t e, const char *what) {
+    snprintf(g_err, sizeof g_err, "%s: %s", what, cudaGetErrorString(e));
+    return -1;
+}
+
+static bool is_aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+static int largest_pow2_divisor_le(long long v, int cap) {
+    int r = 1;
+    while (r * 2 <= cap && v % (r * 2) == 0) r *= 2;
+    return r;
+}
+
+template <class Body>
+static int occupancy_grid(int num_sms) {
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, coop_kernel<Body>, Body::kThreads, 0) != cudaSuccess ||
+        per_sm < 1)
+        per_sm = 1;
+    return per_sm * num_sms;
+}
+
+template <class Body>
+static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long long task_lo, long long task_hi,
+                       int num_sms, cudaStream_t s) {
+    const long long n = task_hi - task_lo;
+    if (n <= 0) return 0;
+    if (c) {
+        long long grid = occupancy_grid<Body>(num_sms);
+        if (grid > n) grid = n;
+        coop_kernel<Body><<<(unsigned)grid, Body::kThreads, 0, s>>>(*c, bp);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return seterr(e, "coop_kernel launch");
+        return (int)grid;
+    }
+    plain_kernel<Body><<<(unsigned)n, Body::kThreads, 0, s>>>(bp, task_lo);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return seterr(e, "plain_kernel launch");
+    return (int)n;
+}
+
+// ---- per-kernel parameter construction ----
+static Tile2D make_tile(const Geom &g, long long nrows, long long ncols, int tw, int th) {
+    Tile2D tl;
+    tl.nrows = nrows; tl.ncols = ncols;
+    tl.ngx = g.ng[0]; tl.lws0 = g.lws[0]; tl.lws1 = g.lws[1];
+    tl.tw = tw; tl.th = th;
+    tl.ntx = (g.ng[0] + tw - 1) / tw;
+    return tl;
+}
+static void tile_shape(const Geom &g, int want_cols, int want_rows, int &tw, int &th) {
+    tw = (int)(want_cols / g.lws[0]); if (tw < 1) tw = 1;
+    th = (int)(want_rows / g.lws[1]); if (th < 1) th = 1;
+}
+
+template <typename T, int NMAT>
+static typename RowDotBody<T, NMAT>::Params rowdot_params(const KArgs &a, const Geom &g) {
+    typename RowDotBody<T, NMAT>::Params p;
+    p.A = (const T *)a.dev[0];
+    if (a.kernel == K_GESUMMV) {
+        p.B = (const T *)a.dev[1]; p.x = (const T *)a.dev[2]; p.out0 = (T *)a.dev[3]; p.out1 = (T *)a.dev[4];
+        p.nrows = a.n0; p.ncols = a.n0;
+    } else {
+        p.B = nullptr; p.x = (const T *)a.dev[1]; p.out0 = (T *)a.dev[2]; p.out1 = nullptr;
+        p.nrows = a.n0; p.ncols = a.n1;
+    }
+    p.lws = g.lws[0];
+    p.R = largest_pow2_divisor_le(g.lws[0], 8);
+    if (a.integer) { p.alpha = (T)a.ialpha; p.beta = (T)a.ibeta; }
+    else { p.alpha = (T)a.alpha; p.beta = (T)a.beta; }
+    p.vec4 = (p.ncols % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.x) && (NMAT == 1 || is_aligned16(p.B));
+    return p;
+}
+
+template <typename T, int MODE>
+static typename ColDotBody<T, MODE>::Params coldot_params(const KArgs &a, const Geom &g) {
+    typename ColDotBody<T, MODE>::Params p;
+    p.A = (const T *)a.dev[0];
+    p.v = (MODE == COL_DOT) ? (const T *)a.dev[1] : nullptr;
+    p.mean = (MODE == COL_SQDEV) ? (const T *)a.dev[1] : nullptr;
+    p.out = (T *)a.dev[(MODE == COL_SQDEV) ? 2 : (MODE == COL_SUM ? 1 : 2)];
+    p.nrows = a.n0; p.ncols = a.n1; p.lws = g.lws[0];
+    p.CB = largest_pow2_divisor_le(g.lws[0], 32);
+    p.nf = (float)a.n0; p.eps = a.eps;
+    return p;
+}
+
+template <typename T, int OP>
+static typename GemmBody<T, OP>::Params gemm_params(const KArgs &a, const Geom &g) {
+    typename GemmBody<T, OP>::Params p;
+    p.A = (const T *)a.dev[0];
+    if (OP == G_SYR2K) { p.B = (const T *)a.dev[1]; p.C = (T *)a.dev[2]; }
+    else { p.B = nullptr; p.C = (T *)a.dev[1]; }
+    if (OP == G_CORR) { p.n = a.n1; p.m = a.n0; p.ld = a.n1; }
+    else { p.n = a.n0; p.m = a.n1; p.ld = a.n1; }
+    if (a.integer) { p.alpha = (T)a.ialpha; p.beta = (T)a.ibeta; }
+    else { p.alpha = (T)a.alpha; p.beta = (T)a.beta; }
+    p.ntile = (p.n + GBM - 1) / GBM;
+    p.ngx = g.ng[0]; p.lws0 = g.lws[0]; p.lws1 = g.work_dim > 1 ? g.lws[1] : 1; p.lws = g.lws[0];
+    p.vec4 = (p.ld % 4 == 0) && (p.n % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.C) &&
+             (OP != G_SYR2K || is_aligned16(p.B));
+    return p;
+}
+
+// Dispatch on the kernel id: F is a generic functor called with a Body type and its Params.
+template <typename F>
+static int with_body(const KArgs &a, const Geom &g, F &&f) {
+    switch (a.kernel) {
+    case K_ATAX_TMP:
+    case K_BICG_Q:
+        if (a.integer) return f.template go<RowDotBody<int32_t, 1>>(rowdot_params<int32_t, 1>(a, g));
+        return f.template go<RowDotBody<float, 1>>(rowdot_params<float, 1>(a, g));
+    case K_GESUMMV:
+        if (a.integer) return f.template go<RowDotBody<int32_t, 2>>(rowdot_params<int32_t, 2>(a, g));
+        return f.template go<RowDotBody<float, 2>>(rowdot_params<float, 2>(a, g));
+    case K_ATAX_Y:
+    case K_BICG_S:
+        if (a.integer) return f.template go<ColDotBody<int32_t, COL_DOT>>(coldot_params<int32_t, COL_DOT>(a, g));
+        return f.template go<ColDotBody<float, COL_DOT>>(coldot_params<float, COL_DOT>(a, g));
+    case K_CORR_MEAN: return f.template go<ColDotBody<float, COL_SUM>>(coldot_params<float, COL_SUM>(a, g));
+    case K_CORR_STD: return f.template go<ColDotBody<float, COL_SQDEV>>(coldot_params<float, COL_SQDEV>(a, g));
+    case K_CORR_REDUCE: {
+        CorrReduceBody::Params p;
+        p.data = (float *)a.dev[0]; p.mean = (const float *)a.dev[1]; p.std_ = (const float *)a.dev[2];
+        int tw, th; tile_shape(g, 256, 32, tw, th);
+        p.tl = make_tile(g, a.n0, a.n1, tw, th);
+        p.sqrtn = __builtin_sqrtf((float)a.n0);
+        return f.template go<CorrReduceBody>(p);
+    }
+    case K_CONV2D: {
+        int tw, th; tile_shape(g, 256, 32, tw, th);
+        if (a.integer) {
+            Conv2DBody<int32_t>::Params p;
+            p.A = (const int32_t *)a.dev[0]; p.B = (int32_t *)a.dev[1];
+            p.tl = make_tile(g, a.n0, a.n1, tw, th);
+            const int32_t c[9] = {2, 5, -8, -3, 6, -9, 4, 7, 1};
+            for (int q = 0; q < 9; ++q) p.c[q] = c[q];
+            return f.template go<Conv2DBody<int32_t>>(p);
+        }
+        Conv2DBody<float>::Params p;
+        p.A = (const float *)a.dev[0]; p.B = (float *)a.dev[1];
+        p.tl = make_tile(g, a.n0, a.n1, tw, th);
+        const float c[9] = {0.2f, 0.5f, -0.8f, -0.3f, 0.6f, -0.9f, 0.4f, 0.7f, 0.10f};
+        for (int q = 0; q < 9; ++q) p.c[q] = c[q];
+        return f.template go<Conv2DBody<float>>(p);
+    }
+    case K_SYRK:
+        if (a.integer) return f.template go<GemmBody<int32_t, G_SYRK>>(gemm_params<int32_t, G_SYRK>(a, g));
+        return f.template go<GemmBody<float, G_SYRK>>(gemm_params<float, G_SYRK>(a, g));
+    case K_SYR2K:
+        if (a.integer) return f.template go<GemmBody<int32_t, G_SYR2K>>(gemm_params<int32_t, G_SYR2K>(a, g));
+        return f.template go<GemmBody<float, G_SYR2K>>(gemm_params<float, G_SYR2K>(a, g));
+    case K_CORR_CORR: return f.template go<GemmBody<float, G_CORR>>(gemm_params<float, G_CORR>(a, g));
+    default: return -1;
+    }
+}
+
+// Host mirror of each body's task enumeration (must match Body::key exactly).
+static int64_t host_rowdot_key(const Geom &g, int64_t t) {
+    const int R = largest_pow2_divisor_le(g.lws[0], 8);
+    return (t * R) / g.lws[0];
+}
+
+TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
+    TaskSpace ts{0, 256};
+    switch (a.kernel) {
+    case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV: {
+        const int R = largest_pow2_divisor_le(g.lws[0], 8);
+        ts.ntasks = (g.ng[0] * g.lws[0] + R - 1) / R;   // covers every row of every work-group
+        ts.threads = 256; break;
+    }
+    case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD: {
+        const int CB = largest_pow2_divisor_le(g.lws[0], 32);
+        ts.ntasks = (g.ng[0] * g.lws[0] + CB - 1) / CB;
+        ts.threads = 1024; break;
+    }
+    case K_CORR_REDUCE: case K_CONV2D: {
+        int tw, th; tile_shape(g, 256, 32, tw, th);
+        const long long ntx = (g.ng[0] + tw - 1) / tw, nty = (g.ng[1] + th - 1) / th;
+        ts.ntasks = ntx * nty; ts.threads = 256; break;
+    }
+    case K_SYRK: case K_SYR2K: {
+        const long long nt = (a.n0 + GBM - 1) / GBM;
+        ts.ntasks = nt * nt; ts.threads = 256; break;
+    }
+    case K_CORR_CORR: {
+        const long long nt = (a.n1 + GBM - 1) / GBM;
+        ts.ntasks = nt * (nt + 1) / 2; ts.threads = 256; break;
+    }
+    default: break;
+    }
+    return ts;
+}
+
+int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t) {
+    switch (a.kernel) {
+    case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV: return host_rowdot_key(g, t);
+    case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD: {
+        const int CB = largest_pow2_divisor_le(g.lws[0], 32);
+        return (t * CB) / g.lws[0];
+    }
+    case K_CORR_REDUCE: case K_CONV2D: {
+        int tw, th; tile_shape(g, 256, 32, tw, th);
+        const long long ntx = (g.ng[0] + tw - 1) / tw;
+        return (t % ntx) * tw + g.ng[0] * ((t / ntx) * th);
+    }
+    case K_SYRK: case K_SYR2K: {
+        const long long nt = (a.n0 + GBM - 1) / GBM;
+        const long long bi = t / nt, bj = t % nt;
+        return (bj * GBM) / g.lws[0] + g.ng[0] * ((bi * GBM) / g.lws[1]);
+    }
+    case K_CORR_CORR: {
+        const long long nt = (a.n1 + GBM - 1) / GBM;
+        long long b1 = 0, rem = t;
+        while (rem >= nt - b1) { rem -= nt - b1; ++b1; }
+        return (b1 * GBM) / g.lws[0];
+    }
+    default: return 0;
+    }
+}
+
+bool gpu_geometry_ok(const KArgs &a, const Geom &g, const char **why) {
+    switch (a.kernel) {
+    case K_SYRK: case K_SYR2K:
+        if (g.work_dim != 2 || GBM % g.lws[0] || GBM % g.lws[1]) { *why = "lws must divide 128 in both dims"; return false; }
+        break;
+    case K_CORR_CORR:
+        if (g.work_dim != 1) { *why = "1-D NDRange expected"; return false; }
+        break;
+    case K_CORR_REDUCE: case K_CONV2D:
+        if (g.work_dim != 2) { *why = "2-D NDRange expected"; return false; }
+        break;
+    default:
+        if (g.work_dim != 1) { *why = "1-D NDRange expected"; return false; }
+    }
+    return true;
+}
+
+int64_t gpu_slice_align(const KArgs &a, const Geom &g) {
+    switch (a.kernel) {
+    case K_CORR_REDUCE: case K_CONV2D: {
+        int tw, th; tile_shape(g, 256, 32, tw, th);
+        return g.ng[0] * th;                       // whole tile rows
+    }
+    case K_SYRK: case K_SYR2K: return g.ng[0] * (GBM / g.lws[1]);
+    case K_CORR_CORR: return g.lws[0] >= GBM ? 1 : GBM / g.lws[0];
+    default: return 1;                             // tasks never span work-groups
+    }
+}
+
+int gpu_default_abort_period(const KArgs &a) {
+    switch (a.kernel) {
+    case K_SYRK: case K_SYR2K: case K_CORR_CORR: return 16;   // every 16 k-tiles (128 k)
+    default: return 0;
+    }
+}
+
+struct CoopLauncher {
+    const CoopCtl *c; int num_sms; cudaStream_t s;
+    template <class Body> int go(const typename Body::Params &bp) {
+        return launch_body<Body>(bp, c, c->task_lo, c->task_hi, num_sms, s);
+    }
+};
+struct PlainLauncher {
+    long long lo, hi; cudaStream_t s;
+    template <class Body> int go(const typename Body::Params &bp) {
+        return launch_body<Body>(bp, nullptr, lo, hi, 0, s);
+    }
+};
+
+int gpu_launch_coop(const KArgs &a, const Geom &g, const CoopCtl &c, int num_sms, void *stream) {
+    CoopLauncher L{&c, num_sms, (cudaStream_t)stream};
+    return with_body(a, g, L);
+}
+
+int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream) {
+    PlainLauncher L{task_lo, task_hi, (cudaStream_t)stream};
+    return with_body(a, g, L);
+}
+
+int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes, int elem_size, int num_sms,
+                     void *stream) {
+    if (bytes == 0) return 0;
+    uint8_t *g = (uint8_t *)gpu;
+    const uint8_t *c = (const uint8_t *)cpu, *t = (const uint8_t *)twin;
+    size_t head = 0, nvec = 0, tail = bytes;
+    const uintptr_t ag = reinterpret_cast<uintptr_t>(g) & 15u;
+    if (ag == (reinterpret_cast<uintptr_t>(c) & 15u) && ag == (reinterpret_cast<uintptr_t>(t) & 15u)) {
+        head = ag ? 16 - ag : 0;
+        if (head > bytes) head = bytes;
+        // head must hold whole elements: alignment of the buffers is a multiple of elem_size
+        nvec = (bytes - head) / 16;
+        tail = bytes - head - 16 * nvec;
+    }
+    size_t threads_needed = (nvec + 3) / 4;
+    long long grid = (long long)((threads_needed + 255) / 256);
+    const long long cap = (long long)num_sms * 8;
+    if (grid > cap) grid = cap;
+    if (grid < 1) grid = 1;
+    cudaStream_t s = (cudaStream_t)stream;
+    switch (elem_size) {
+    case 1: merge_kernel<1><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
+    case 2: merge_kernel<2><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
+    case 4: merge_kernel<4><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
+    case 8: merge_kernel<8><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
+    default: return -1;
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return seterr(e, "merge_kernel launch");
+    return 1;
+}
+
+int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream) {
+    store64_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(addr, value);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return seterr(e, "store64_kernel launch");
+    return 1;
+}
+
+}  // namespace fcl

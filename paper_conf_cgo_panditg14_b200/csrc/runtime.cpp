@@ -1,0 +1,1286 @@
+// runtime.cpp -- the FluidiCL runtime for one B200 + its host cores, behind the C-ABI fcl.h.
+//
+// Components:
+//   * context: CUDA device, streams main / hd / dh (L20.s10-13), the 64-bit watermark word
+//     {epoch, W} (D1, C14) in pinned mapped host memory (or device memory), the mapped exit
+//     record written by the dispatcher's last CTA, device claim counters, kernel-id epoch;
+//   * dual-resident buffers (C3, L14.s49-50 / L16.s1) with element-size metadata (C16, D6) and
+//     host/device validity flags (minimal data-location tracking, C22 / L20.s31-33);
+//   * twin + stage buffer pool (C5/C6, L16.s2-3, L20.s23-29);
+//   * host executor: a pinned, spinning thread pool that runs descending chunks of work-groups
+//     (C9/C10, L16.s6-10, L18.s18-21) sized by the adaptive heuristic (C11, L18.s23-32), with
+//     work-group splitting (C23, L20.s34-39);
+//   * stager/publisher: after each chunk, its output span goes host->device on `hd` and a stream
+//     memory operation then stores {epoch, lo} -- status follows data (C13, L16.s11/s.15-18);
+//   * merge launcher (C15, Fig 9) and the device->host return of the GPU's part (C17, L16.s36-38).
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <immintrin.h>
+#include <sched.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/fcl.h"
+#include "fcl_internal.h"
+
+using namespace fcl;
+
+namespace {
+
+using Clock = std::chrono::steady_clock;
+inline double now_ms() {
+    return std::chrono::duration<double, std::milli>(Clock::now().time_since_epoch()).count();
+}
+
+// ------------------------------------------------------------------------------------------
+// Kernel table (built-in kernels; C27's source transformation is replaced by templates)
+// ------------------------------------------------------------------------------------------
+struct ArgSpec {
+    const char *name;
+    char kind;      // 'b' buffer, 'i' int, 'f' float
+    uint8_t acc;    // buffers: 1 read, 2 written, 3 read+written
+};
+struct KernelDef {
+    const char *name;
+    int id;
+    bool integer;
+    int nargs;
+    ArgSpec args[9];
+};
+
+#define B_IN(n) {n, 'b', 1}
+#define B_OUT(n) {n, 'b', 2}
+#define B_INOUT(n) {n, 'b', 3}
+#define I_(n) {n, 'i', 0}
+#define F_(n) {n, 'f', 0}
+
+const KernelDef kKernels[] = {
+    {"atax_tmp_f32", K_ATAX_TMP, false, 5, {B_IN("A"), B_IN("x"), B_OUT("tmp"), I_("nx"), I_("ny")}},
+    {"atax_tmp_i32", K_ATAX_TMP, true, 5, {B_IN("A"), B_IN("x"), B_OUT("tmp"), I_("nx"), I_("ny")}},
+    {"atax_y_f32", K_ATAX_Y, false, 5, {B_IN("A"), B_IN("tmp"), B_OUT("y"), I_("nx"), I_("ny")}},
+    {"atax_y_i32", K_ATAX_Y, true, 5, {B_IN("A"), B_IN("tmp"), B_OUT("y"), I_("nx"), I_("ny")}},
+    {"bicg_s_f32", K_BICG_S, false, 5, {B_IN("A"), B_IN("r"), B_OUT("s"), I_("nx"), I_("ny")}},
+    {"bicg_s_i32", K_BICG_S, true, 5, {B_IN("A"), B_IN("r"), B_OUT("s"), I_("nx"), I_("ny")}},
+    {"bicg_q_f32", K_BICG_Q, false, 5, {B_IN("A"), B_IN("p"), B_OUT("q"), I_("nx"), I_("ny")}},
+    {"bicg_q_i32", K_BICG_Q, true, 5, {B_IN("A"), B_IN("p"), B_OUT("q"), I_("nx"), I_("ny")}},
+    {"gesummv_f32", K_GESUMMV, false, 8,
+     {B_IN("A"), B_IN("B"), B_IN("x"), B_OUT("tmp"), B_OUT("y"), I_("n"), F_("alpha"), F_("beta")}},
+    {"gesummv_i32", K_GESUMMV, true, 8,
+     {B_IN("A"), B_IN("B"), B_IN("x"), B_OUT("tmp"), B_OUT("y"), I_("n"), I_("alpha"), I_("beta")}},
+    {"syrk_f32", K_SYRK, false, 6, {B_IN("A"), B_INOUT("C"), I_("n"), I_("m"), F_("alpha"), F_("beta")}},
+    {"syrk_i32", K_SYRK, true, 6, {B_IN("A"), B_INOUT("C"), I_("n"), I_("m"), I_("alpha"), I_("beta")}},
+    {"syr2k_f32", K_SYR2K, false, 7,
+     {B_IN("A"), B_IN("B"), B_INOUT("C"), I_("n"), I_("m"), F_("alpha"), F_("beta")}},
+    {"syr2k_i32", K_SYR2K, true, 7,
+     {B_IN("A"), B_IN("B"), B_INOUT("C"), I_("n"), I_("m"), I_("alpha"), I_("beta")}},
+    {"corr_mean_f32", K_CORR_MEAN, false, 4, {B_IN("data"), B_OUT("mean"), I_("n"), I_("m")}},
+    {"corr_std_f32", K_CORR_STD, false, 6,
+     {B_IN("data"), B_IN("mean"), B_OUT("std"), I_("n"), I_("m"), F_("eps")}},
+    {"corr_reduce_f32", K_CORR_REDUCE, false, 5, {B_INOUT("data"), B_IN("mean"), B_IN("std"), I_("n"), I_("m")}},
+    {"corr_corr_f32", K_CORR_CORR, false, 4, {B_IN("data"), B_OUT("symmat"), I_("n"), I_("m")}},
+    {"conv2d_f32", K_CONV2D, false, 4, {B_IN("A"), B_OUT("B"), I_("ni"), I_("nj")}},
+    {"conv2d_i32", K_CONV2D, true, 4, {B_IN("A"), B_OUT("B"), I_("ni"), I_("nj")}},
+};
+constexpr int kNumKernels = sizeof(kKernels) / sizeof(kKernels[0]);
+
+// Elements each buffer argument must hold, given the problem extents (n0, n1).
+int64_t required_elems(int kid, int b, int64_t n0, int64_t n1) {
+    switch (kid) {
+    case K_ATAX_TMP: { const int64_t r[] = {n0 * n1, n1, n0}; return r[b]; }
+    case K_ATAX_Y: { const int64_t r[] = {n0 * n1, n0, n1}; return r[b]; }
+    case K_BICG_S: { const int64_t r[] = {n0 * n1, n0, n1}; return r[b]; }
+    case K_BICG_Q: { const int64_t r[] = {n0 * n1, n1, n0}; return r[b]; }
+    case K_GESUMMV: { const int64_t r[] = {n0 * n0, n0 * n0, n0, n0, n0}; return r[b]; }
+    case K_SYRK: { const int64_t r[] = {n0 * n1, n0 * n0}; return r[b]; }
+    case K_SYR2K: { const int64_t r[] = {n0 * n1, n0 * n1, n0 * n0}; return r[b]; }
+    case K_CORR_MEAN: { const int64_t r[] = {n0 * n1, n1}; return r[b]; }
+    case K_CORR_STD: { const int64_t r[] = {n0 * n1, n1, n1}; return r[b]; }
+    case K_CORR_REDUCE: { const int64_t r[] = {n0 * n1, n1, n1}; return r[b]; }
+    case K_CORR_CORR: { const int64_t r[] = {n0 * n1, n1 * n1}; return r[b]; }
+    case K_CONV2D: { const int64_t r[] = {n0 * n1, n0 * n1}; return r[b]; }
+    default: return 0;
+    }
+}
+
+// NDRange extent each dimension must cover (PolyBench pads gws up to a multiple of lws).
+void required_extent(int kid, int64_t n0, int64_t n1, int64_t ext[3]) {
+    ext[0] = ext[1] = ext[2] = 1;
+    switch (kid) {
+    case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV: ext[0] = n0; break;
+    case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD: case K_CORR_CORR: ext[0] = n1; break;
+    case K_SYRK: case K_SYR2K: ext[0] = n0; ext[1] = n0; break;
+    case K_CORR_REDUCE: case K_CONV2D: ext[0] = n1; ext[1] = n0; break;
+    default: break;
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// Host executor (C9/C10/C23): T pinned worker threads, spinning while hot.
+// ------------------------------------------------------------------------------------------
+struct Executor {
+    std::vector<std::thread> threads;
+    std::vector<int> cores;
+    int T = 0;
+    std::atomic<uint64_t> gen{0};
+    std::atomic<int> stop{0};
+    std::mutex mu;
+    std::condition_variable cv;
+    std::atomic<int> sleepers{0};
+    // current job (written before `next` is released)
+    KArgs a{};
+    Geom g{};
+    int64_t lo = 0, hi = 0;
+    int nparts = 1;
+    int64_t total = 0;
+    int active = 0;
+    // claim word: (job generation << 40) | next item.  Claims use compare-and-swap so a
+    // worker still looping on a finished job can never consume an item of the next one.
+    std::atomic<uint64_t> next{0};
+    std::atomic<int64_t> done{0};
+    std::atomic<int64_t> executed{0};
+    volatile int abort_flag = 0;
+    int64_t spin_ns = 20 * 1000 * 1000;   // spin 20 ms after a job before sleeping
+
+    void start(int nthreads, bool pin) {
+        cpu_set_t set;
+        CPU_ZERO(&set);
+        if (sched_getaffinity(0, sizeof set, &set) == 0) {
+            for (int c = 0; c < CPU_SETSIZE; ++c)
+                if (CPU_ISSET(c, &set)) cores.push_back(c);
+        }
+        if (cores.empty()) cores.push_back(0);
+        T = nthreads > 0 ? nthreads : std::max<int>(1, (int)cores.size() - 1);
+        active = T;
+        for (int k = 0; k < T; ++k) threads.emplace_back([this, k, pin] { worker(k, pin); });
+    }
+    void shutdown() {
+        stop.store(1);
+        {
+            std::lock_guard<std::mutex> lk(mu);
+            cv.notify_all();
+        }
+        for (auto &t : threads) t.join();
+        threads.clear();
+    }
+    void worker(int idx, bool pin) {
+        if (pin && cores.size() > 1) {
+            cpu_set_t s;
+            CPU_ZERO(&s);
+            CPU_SET(cores[(size_t)(idx + 1) % cores.size()], &s);   // leave cores[0] to the coordinator
+            sched_setaffinity(0, sizeof s, &s);
+        }
+        uint64_t seen = 0;
+        for (;;) {
+            auto t0 = Clock::now();
+            while (gen.load(std::memory_order_acquire) == seen && !stop.load(std::memory_order_relaxed)) {
+                _mm_pause();
+                if (std::chrono::duration_cast<std::chrono::nanoseconds>(Clock::now() - t0).count() > spin_ns) {
+                    std::unique_lock<std::mutex> lk(mu);
+                    sleepers.fetch_add(1);
+                    cv.wait(lk, [&] { return gen.load() != seen || stop.load(); });
+                    sleepers.fetch_sub(1);
+                    t0 = Clock::now();
+                }
+            }
+            if (stop.load()) return;
+            seen = gen.load(std::memory_order_acquire);
+            if (idx >= active) continue;
+            for (;;) {
+                uint64_t v = next.load(std::memory_order_acquire);
+                if ((v >> 40) != (seen & 0xFFFFFFu)) break;
+                const int64_t it = (int64_t)(v & ((1ull << 40) - 1));
+                if (it >= total) break;
+                if (!next.compare_exchange_weak(v, v + 1, std::memory_order_acq_rel)) continue;
+                if (!abort_flag) {
+                    const int64_t fgid = hi - 1 - it / nparts;   // descending (L14.s36)
+                    host_exec_wg(a, g, fgid, (int)(it % nparts), nparts, &abort_flag);
+                    if (!abort_flag) executed.fetch_add(1, std::memory_order_relaxed);
+                }
+                done.fetch_add(1, std::memory_order_acq_rel);
+            }
+        }
+    }
+    // Submit work-groups [lo_, hi_) split `parts` ways; returns immediately.
+    void submit(const KArgs &a_, const Geom &g_, int64_t lo_, int64_t hi_, int parts, int nact) {
+        a = a_; g = g_; lo = lo_; hi = hi_; nparts = parts;
+        total = (hi_ - lo_) * parts;
+        active = std::max(1, std::min(nact, T));
+        done.store(0, std::memory_order_relaxed);
+        const uint64_t g1 = gen.load(std::memory_order_relaxed) + 1;
+        next.store((g1 & 0xFFFFFFu) << 40, std::memory_order_release);
+        gen.store(g1, std::memory_order_release);
+        if (sleepers.load() > 0) {
+            std::lock_guard<std::mutex> lk(mu);
+            cv.notify_all();
+        }
+    }
+    bool finished() const { return done.load(std::memory_order_acquire) >= total; }
+    void wait() {
+        while (!finished()) _mm_pause();
+    }
+};
+
+struct PoolEnt {
+    void *p;
+    size_t bytes;
+    bool used;
+    uint32_t last_epoch;
+};
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------
+// Opaque handle types
+// ------------------------------------------------------------------------------------------
+struct fcl_kernel_st {
+    const KernelDef *def;
+};
+
+struct fcl_buffer_st {
+    fcl_context ctx;
+    size_t bytes;
+    uint32_t elem_size;
+    uint32_t flags;
+    void *dev;
+    void *host;
+    bool own_dev, own_host;
+    bool host_valid, dev_valid;
+    bool d2h_pending;
+    cudaEvent_t d2h_ev;
+    // deferred merge state (opts.defer_merge)
+    bool merge_pending;
+    void *twin, *stage;
+    size_t m_b0, m_b1, r_b0, r_b1;   // merge span, return (D2H) span
+};
+
+typedef CUresult (*PFN_writeValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+
+struct fcl_context_st {
+    int device = 0;
+    int num_sms = 148;
+    cudaStream_t main = nullptr, hd = nullptr, dh = nullptr;
+    bool own_main = false, own_hd = false, own_dh = false;
+    int status_location = FCL_STATUS_HOST_MAPPED;
+    // One 64-bit status word per launch slot (epoch % kSlots): a dispatcher that is still
+    // running after its host side returned never sees a later launch's watermark.
+    static constexpr int kSlots = 16;
+    unsigned long long *status_host = nullptr;   // mapped host words (HOST_MAPPED)
+    unsigned long long *status_dptr = nullptr;   // device-visible address of slot 0
+    uint32_t slot_epoch[kSlots] = {0};           // epoch of the dispatcher that last used a slot
+    unsigned long long *exit_host = nullptr;     // mapped exit record [2]
+    unsigned long long *exit_dptr = nullptr;
+    unsigned long long *dclaim = nullptr, *dtasks = nullptr;
+    unsigned int *ddone = nullptr, *dwmin = nullptr;
+    uint32_t epoch = 0;
+    PFN_writeValue64 write64 = nullptr;
+    std::vector<PoolEnt> pool;
+    Executor ex;
+    std::string err;
+    fcl_status sticky = FCL_SUCCESS;
+    std::vector<cudaEvent_t> evpool;   // timing-disabled events for chunk publication
+    cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr, ev_m0 = nullptr, ev_m1 = nullptr, ev_hd_last = nullptr;
+    cudaEvent_t ev_mark = nullptr;   // main-stream progress marker for the dh stream
+    bool have_k = false, have_m = false;
+    fcl_launch_info info{};
+    std::vector<fcl_buffer> defer_list;
+};
+
+namespace {
+
+fcl_status set_err(fcl_context ctx, fcl_status s, const char *fmt, ...) {
+    if (ctx) {
+        char b[512];
+        va_list ap;
+        va_start(ap, fmt);
+        vsnprintf(b, sizeof b, fmt, ap);
+        va_end(ap);
+        ctx->err = b;
+    }
+    return s;
+}
+
+fcl_status cuda_fail(fcl_context ctx, cudaError_t e, const char *what) {
+    set_err(ctx, FCL_CUDA_ERROR, "%s: %s", what, cudaGetErrorString(e));
+    if (ctx) ctx->sticky = FCL_CONTEXT_LOST;
+    return FCL_CUDA_ERROR;
+}
+
+#define CK(ctx, call)                                                   \
+    do {                                                                \
+        cudaError_t _e = (call);                                        \
+        if (_e != cudaSuccess) return cuda_fail((ctx), _e, #call);      \
+    } while (0)
+
+void *pool_get(fcl_context ctx, size_t bytes) {
+    int best = -1;
+    for (size_t k = 0; k < ctx->pool.size(); ++k) {
+        const PoolEnt &e = ctx->pool[k];
+        if (!e.used && e.bytes >= bytes && (best < 0 || e.bytes < ctx->pool[(size_t)best].bytes)) best = (int)k;
+    }
+    if (best >= 0) {
+        ctx->pool[(size_t)best].used = true;
+        ctx->pool[(size_t)best].last_epoch = ctx->epoch;
+        return ctx->pool[(size_t)best].p;
+    }
+    void *p = nullptr;
+    if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) {
+        cudaGetLastError();
+        // free every unused entry and retry once (L20.s29: reclaim older unused buffers)
+        for (auto it = ctx->pool.begin(); it != ctx->pool.end();) {
+            if (!it->used) { cudaFree(it->p); it = ctx->pool.erase(it); }
+            else ++it;
+        }
+        if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+    }
+    ctx->pool.push_back({p, bytes, true, ctx->epoch});
+    return p;
+}
+
+void pool_put(fcl_context ctx, void *p) {
+    for (auto &e : ctx->pool)
+        if (e.p == p) { e.used = false; e.last_epoch = ctx->epoch; }
+}
+
+// "At the end of each kernel execution, older unused buffers are freed" (L20.s29).
+void pool_trim(fcl_context ctx) {
+    for (auto it = ctx->pool.begin(); it != ctx->pool.end();) {
+        if (!it->used && it->last_epoch + 16 < ctx->epoch) {
+            cudaFree(it->p);
+            it = ctx->pool.erase(it);
+        } else {
+            ++it;
+        }
+    }
+}
+
+cudaEvent_t ev_get(fcl_context ctx, size_t k) {
+    while (ctx->evpool.size() <= k) {
+        cudaEvent_t e;
+        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+        ctx->evpool.push_back(e);
+    }
+    return ctx->evpool[k];
+}
+
+// Store {epoch, W} after everything already queued on `s` (status follows data, L16.s15).
+unsigned long long *status_slot(fcl_context ctx) {
+    return ctx->status_dptr + (ctx->epoch % fcl_context_st::kSlots);
+}
+
+fcl_status publish(fcl_context ctx, uint32_t w, cudaStream_t s) {
+    const unsigned long long v = ((unsigned long long)ctx->epoch << 32) | w;
+    unsigned long long *dst = status_slot(ctx);
+    if (ctx->write64) {
+        CUresult r = ctx->write64((CUstream)s, (CUdeviceptr)dst, v, 0);
+        if (r == CUDA_SUCCESS) return FCL_SUCCESS;
+        ctx->write64 = nullptr;   // fall back to the kernel store from now on
+    }
+    if (gpu_launch_store64(dst, v, s) < 0)
+        return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    return FCL_SUCCESS;
+}
+
+bool poll_exit(fcl_context ctx, uint32_t *wmin, uint64_t *tasks) {
+    const unsigned long long r = __atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE);
+    if ((uint32_t)(r >> 32) != ctx->epoch) return false;
+    *wmin = (uint32_t)r;
+    *tasks = __atomic_load_n(ctx->exit_host + 1, __ATOMIC_ACQUIRE);
+    return true;
+}
+
+// Bring a buffer's copies to the validity a launch needs.
+fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_dev) {
+    if (b->d2h_pending) {
+        CK(ctx, cudaEventSynchronize(b->d2h_ev));
+        b->d2h_pending = false;
+    }
+    if (need_dev && !b->dev_valid) {
+        CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
+        b->dev_valid = true;
+        ctx->info.h2d_bytes += (int64_t)b->bytes;
+    }
+    if (need_host && !b->host_valid) {
+        CK(ctx, cudaMemcpyAsync(b->host, b->dev, b->bytes, cudaMemcpyDeviceToHost, ctx->main));
+        CK(ctx, cudaStreamSynchronize(ctx->main));
+        b->host_valid = true;
+        ctx->info.d2h_bytes += (int64_t)b->bytes;
+    }
+    return FCL_SUCCESS;
+}
+
+int64_t ceil_pct(int64_t pct, int64_t n) { return (pct * n + 99) / 100; }
+
+// First task index whose key is >= f (keys are non-decreasing in the task index).
+int64_t first_task_at(const KArgs &a, const Geom &g, int64_t ntasks, int64_t f) {
+    int64_t lo = 0, hi = ntasks;
+    while (lo < hi) {
+        const int64_t mid = lo + (hi - lo) / 2;
+        if (gpu_task_key(a, g, mid) < f) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+struct Launch {
+    fcl_context ctx;
+    const KernelDef *kd;
+    KArgs a;
+    Geom g;
+    fcl_buffer bufs[6];
+    int out_idx[6];
+    int nout;
+    int64_t lo, hi;
+    fcl_launch_opts o;
+};
+
+fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, bool after_merge) {
+    if (whi <= wlo) return FCL_SUCCESS;
+    (void)after_merge;
+    CK(ctx, cudaEventRecord(ctx->ev_mark, ctx->main));   // after the kernel (and merge) on main
+    CK(ctx, cudaStreamWaitEvent(ctx->dh, ctx->ev_mark, 0));
+    for (int q = 0; q < L.nout; ++q) {
+        fcl_buffer b = L.bufs[L.out_idx[q]];
+        size_t b0, b1;
+        out_span(L.a, L.g, L.out_idx[q], wlo, whi, &b0, &b1);
+        if (b1 <= b0) continue;
+        CK(ctx, cudaMemcpyAsync((char *)b->host + b0, (char *)b->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
+        ctx->info.d2h_bytes += (int64_t)(b1 - b0);
+        CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
+        b->d2h_pending = true;
+    }
+    return FCL_SUCCESS;
+}
+
+fcl_status enqueue_merges(fcl_context ctx, Launch &L, void **twin, void **stage, int64_t mlo, int64_t mhi) {
+    if (mhi <= mlo) return FCL_SUCCESS;
+    if (!ctx->have_m) CK(ctx, cudaEventRecord(ctx->ev_m0, ctx->main));
+    for (int q = 0; q < L.nout; ++q) {
+        fcl_buffer b = L.bufs[L.out_idx[q]];
+        size_t b0, b1;
+        out_span(L.a, L.g, L.out_idx[q], mlo, mhi, &b0, &b1);
+        if (b1 <= b0) continue;
+        if (L.o.defer_merge) {
+            b->merge_pending = true;
+            b->twin = twin[q]; b->stage = stage[q];
+            b->m_b0 = b0; b->m_b1 = b1;
+            twin[q] = stage[q] = nullptr;   // ownership moves to the buffer until fcl_merge
+            ctx->defer_list.push_back(b);
+            continue;
+        }
+        if (gpu_launch_merge((char *)b->dev + b0, (char *)stage[q] + b0, (char *)twin[q] + b0, b1 - b0,
+                             (int)b->elem_size, ctx->num_sms, ctx->main) < 0)
+            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        ctx->info.gpu_launches += 1;
+        ctx->info.merge_bytes += (int64_t)(b1 - b0);
+        ctx->info.merged = 1;
+    }
+    if (!L.o.defer_merge) {
+        CK(ctx, cudaEventRecord(ctx->ev_m1, ctx->main));
+        ctx->have_m = true;
+    }
+    return FCL_SUCCESS;
+}
+
+// ---- the three modes ----
+fcl_status run_gpu_only(Launch &L) {
+    fcl_context ctx = L.ctx;
+    const TaskSpace ts = gpu_task_space(L.a, L.g);
+    const int64_t t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo), t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
+    CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
+    if (gpu_launch_plain(L.a, L.g, t0, t1, ctx->main) < 0)
+        return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
+    ctx->have_k = true;
+    ctx->info.gpu_launches += 1;
+    ctx->info.gpu_tasks = ctx->info.gpu_tasks_total = t1 - t0;
+    return enqueue_d2h(ctx, L, L.lo, L.hi, false);
+}
+
+fcl_status run_cpu_only(Launch &L) {
+    fcl_context ctx = L.ctx;
+    Executor &ex = ctx->ex;
+    const int nact = L.o.n_host_threads > 0 ? L.o.n_host_threads : ex.T;
+    const int64_t nwg = L.hi - L.lo;
+    const int parts = (L.o.cpu_wg_split && nwg < nact) ? (int)((nact + nwg - 1) / nwg) : 1;
+    const double t0 = now_ms();
+    ex.abort_flag = 0;
+    ex.executed.store(0);
+    ex.submit(L.a, L.g, L.lo, L.hi, parts, nact);
+    ex.wait();
+    ctx->info.t_host_ms = now_ms() - t0;
+    ctx->info.cpu_wgs = nwg;
+    ctx->info.n_chunks = 1;
+    ctx->info.chunk_sizes[0] = (int32_t)nwg;
+    ctx->info.cpu_did_all = 1;
+    ctx->info.published_watermark = L.lo;
+    for (int q = 0; q < L.nout; ++q) L.bufs[L.out_idx[q]]->dev_valid = false;   // lazy H2D on next GPU use
+    return FCL_SUCCESS;
+}
+
+fcl_status run_coop(Launch &L) {
+    fcl_context ctx = L.ctx;
+    Executor &ex = ctx->ex;
+    fcl_launch_info &info = ctx->info;
+    const TaskSpace ts = gpu_task_space(L.a, L.g);
+    const int64_t t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo), t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
+    info.gpu_tasks_total = t1 - t0;
+    const int64_t nwg = L.hi - L.lo;
+    const bool forced = L.o.forced_split >= 0;
+    const int64_t s_forced = forced ? std::min<int64_t>(std::max<int64_t>(L.o.forced_split, L.lo), L.hi) : -1;
+
+    // a new kernel id (C14); stale status words are ignored by the dispatcher
+    ctx->epoch += 1;
+    {
+        // the dispatcher that last used this launch's status slot must have exited
+        const uint32_t prev = ctx->slot_epoch[ctx->epoch % fcl_context_st::kSlots];
+        if (prev) {
+            const double tw = now_ms();
+            while ((uint32_t)(__atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE) >> 32) < prev) {
+                if (cudaStreamQuery(ctx->main) == cudaSuccess) break;
+                if (now_ms() - tw > 60000.0) return set_err(ctx, FCL_CONTEXT_LOST, "dispatcher %u never exited", prev);
+                _mm_pause();
+            }
+        }
+    }
+    // previous staging copies on hd must be done before the pool hands their stages out again
+    CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
+    CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_last, 0));
+
+    // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
+    void *twin[6] = {nullptr}, *stage[6] = {nullptr};
+    for (int q = 0; q < L.nout; ++q) {
+        fcl_buffer b = L.bufs[L.out_idx[q]];
+        twin[q] = pool_get(ctx, b->bytes);
+        stage[q] = pool_get(ctx, b->bytes);
+        if (!twin[q] || !stage[q]) return set_err(ctx, FCL_OUT_OF_RESOURCES, "twin/stage allocation of %zu bytes failed", b->bytes);
+        CK(ctx, cudaMemcpyAsync(twin[q], b->dev, b->bytes, cudaMemcpyDeviceToDevice, ctx->main));
+    }
+    auto release = [&]() {
+        for (int q = 0; q < L.nout; ++q) {
+            if (twin[q]) pool_put(ctx, twin[q]);
+            if (stage[q]) pool_put(ctx, stage[q]);
+        }
+    };
+
+    if (forced) {
+        // test hook: the GPU is told the split before it starts
+        fcl_status st = publish(ctx, (uint32_t)s_forced, ctx->hd);
+        if (st != FCL_SUCCESS) { release(); return st; }
+        CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
+        CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_last, 0));
+    }
+
+    // GPU: the whole range, persistent dispatcher (C8)
+    CoopCtl c;
+    c.status = status_slot(ctx);
+    c.epoch = ctx->epoch;
+    c.w_default = (unsigned int)L.hi;
+    c.claim = ctx->dclaim; c.done = ctx->ddone; c.wmin = ctx->dwmin; c.tasks = ctx->dtasks;
+    c.exit_rec = ctx->exit_dptr;
+    c.task_lo = t0; c.task_hi = t1;
+    c.abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
+    bool gpu_launched = false;
+    if (t1 > t0) {
+        CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
+        if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0) {
+            release();
+            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        }
+        CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
+        ctx->have_k = true;
+        info.gpu_launches += 1;
+        gpu_launched = true;
+        ctx->slot_epoch[ctx->epoch % fcl_context_st::kSlots] = ctx->epoch;
+    }
+
+    // CPU: descending adaptive chunks (C9-C11), staged and published after each (C13)
+    const int nact = L.o.n_host_threads > 0 ? std::min(L.o.n_host_threads, ex.T) : ex.T;
+    const int64_t hi_cpu = L.hi, lo_cpu = forced ? s_forced : L.lo;
+    int64_t hi_cur = hi_cpu;
+    int pct = std::max(1, L.o.init_chunk_pct);
+    double prev_avg = -1.0, t_start = 0.0, busy = 0.0;
+    int nch = 0;
+    bool in_flight = false, gpu_done = !gpu_launched, cpu_all = false;
+    uint32_t wmin = 0xFFFFFFFFu;
+    uint64_t gtasks = 0;
+    int64_t cur_lo = 0, cur_hi = 0, cur_size = 0, cpu_done_wgs = 0;
+    std::vector<std::pair<int64_t, size_t>> published;   // (watermark, event index)
+    size_t nev = 0;
+    ex.abort_flag = 0;
+    ex.executed.store(0);
+
+    auto start_chunk = [&]() {
+        int64_t size = ceil_pct(pct, nwg);
+        const int64_t min_units = L.o.cpu_wg_split ? 1 : nact;   // L18.s31 without C23
+        size = std::max<int64_t>(size, min_units);
+        size = std::min<int64_t>(size, hi_cur - lo_cpu);
+        cur_hi = hi_cur; cur_lo = hi_cur - size; cur_size = size;
+        const int parts = (L.o.cpu_wg_split && size < nact) ? (int)((nact + size - 1) / size) : 1;
+        if (L.o.host_delay_us > 0) std::this_thread::sleep_for(std::chrono::microseconds(L.o.host_delay_us));
+        if (nch < 64) info.chunk_sizes[nch] = (int32_t)size;
+        ++nch;
+        t_start = now_ms();
+        ex.submit(L.a, L.g, cur_lo, cur_hi, parts, nact);
+        in_flight = true;
+    };
+    auto stage_chunk = [&](int64_t clo, int64_t chi) -> fcl_status {
+        for (int q = 0; q < L.nout; ++q) {
+            fcl_buffer b = L.bufs[L.out_idx[q]];
+            size_t b0, b1;
+            out_span(L.a, L.g, L.out_idx[q], clo, chi, &b0, &b1);
+            if (b1 > b0) {
+                CK(ctx, cudaMemcpyAsync((char *)stage[q] + b0, (char *)b->host + b0, b1 - b0, cudaMemcpyHostToDevice, ctx->hd));
+                info.h2d_bytes += (int64_t)(b1 - b0);
+            }
+        }
+        if (!forced && !L.o.drop_publish) {
+            fcl_status st = publish(ctx, (uint32_t)clo, ctx->hd);
+            if (st != FCL_SUCCESS) return st;
+        }
+        cudaEvent_t e = ev_get(ctx, nev);
+        if (!e) return set_err(ctx, FCL_OUT_OF_RESOURCES, "event pool");
+        CK(ctx, cudaEventRecord(e, ctx->hd));
+        published.push_back({clo, nev});
+        ++nev;
+        info.published_watermark = clo;
+        return FCL_SUCCESS;
+    };
+
+    info.published_watermark = L.hi;
+    if (hi_cur > lo_cpu) start_chunk();
+    else cpu_all = !gpu_launched || forced;
+    while (in_flight) {
+        if (!forced && !gpu_done && poll_exit(ctx, &wmin, &gtasks)) {
+            gpu_done = true;
+            break;
+        }
+        if (ex.finished()) {
+            const double dt = now_ms() - t_start;
+            busy += dt;
+            in_flight = false;
+            cpu_done_wgs += cur_size;
+            const double avg = dt / (double)cur_size;
+            if (nch == 1 || avg < prev_avg) pct += std::max(0, L.o.step_pct);   // C11
+            prev_avg = avg;
+            const int64_t clo = cur_lo, chi = cur_hi;
+            hi_cur = clo;
+            const bool more = hi_cur > lo_cpu;
+            if (more) start_chunk();          // keep the workers busy while this chunk is staged
+            fcl_status st = stage_chunk(clo, chi);
+            if (st != FCL_SUCCESS) { ex.abort_flag = 1; ex.wait(); release(); return st; }
+            if (!more) { cpu_all = true; break; }
+        } else {
+            _mm_pause();
+        }
+    }
+    if (in_flight) {   // GPU finished first: abandon the running chunk (L18.s19)
+        ex.abort_flag = 1;
+        ex.wait();
+        busy += now_ms() - t_start;
+        ex.abort_flag = 0;
+    }
+    info.t_host_ms = busy;
+    info.n_chunks = nch;
+    info.cpu_wgs = cpu_done_wgs;
+    info.gpu_watermark = L.hi;
+
+    // Decide the merge domain and the device->host return (C15/C17)
+    int64_t merge_lo = L.hi, ret_hi = L.hi;
+    size_t wait_ev = (size_t)-1;
+    if (forced) {
+        merge_lo = s_forced;
+        ret_hi = s_forced;
+        if (!published.empty()) wait_ev = published.back().second;
+        info.gpu_watermark = s_forced;
+        if (s_forced == L.lo) info.cpu_did_all = 1;
+    } else if (cpu_all && !gpu_done) {
+        // the host covered the range first: host copy authoritative (L16.s21); the device copy
+        // is made coherent by merging everything once the GPU has stopped (stream order)
+        merge_lo = L.lo;
+        ret_hi = L.lo;
+        if (!published.empty()) wait_ev = published.back().second;
+        info.cpu_did_all = 1;
+        info.gpu_watermark = L.lo;   // resolved when the exit record arrives (see fcl_finish)
+    } else {
+        const int64_t wm = (wmin == 0xFFFFFFFFu) ? L.hi : (int64_t)wmin;
+        info.gpu_watermark = wm;
+        info.gpu_tasks = (int64_t)gtasks;
+        merge_lo = wm;
+        ret_hi = wm;
+        if (wm < L.hi) {
+            for (auto &pe : published)
+                if (pe.first == wm) wait_ev = pe.second;
+            if (wait_ev == (size_t)-1 && !published.empty()) wait_ev = published.back().second;
+        }
+        if (wm <= L.lo) info.cpu_did_all = 1;
+    }
+    if (merge_lo < L.hi) {
+        if (wait_ev != (size_t)-1) CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->evpool[wait_ev], 0));
+        fcl_status st = enqueue_merges(ctx, L, twin, stage, merge_lo, L.hi);
+        if (st != FCL_SUCCESS) { release(); return st; }
+    }
+    fcl_status st = FCL_SUCCESS;
+    if (L.o.defer_merge && merge_lo < L.hi) {
+        // the return copy must follow the merge: fcl_merge performs both
+        for (int q = 0; q < L.nout; ++q) {
+            fcl_buffer b = L.bufs[L.out_idx[q]];
+            out_span(L.a, L.g, L.out_idx[q], L.lo, ret_hi, &b->r_b0, &b->r_b1);
+        }
+    } else {
+        st = enqueue_d2h(ctx, L, L.lo, ret_hi, merge_lo < L.hi);
+    }
+    CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
+    release();
+    return st;
+}
+
+fcl_status check_ctx(fcl_context ctx) {
+    if (!ctx) return FCL_INVALID_CONTEXT;
+    if (ctx->sticky != FCL_SUCCESS) return ctx->sticky;
+    cudaSetDevice(ctx->device);
+    return FCL_SUCCESS;
+}
+
+}  // namespace
+
+// ==========================================================================================
+// C-ABI
+// ==========================================================================================
+extern "C" {
+
+const char *fcl_version(void) { return "fcl-b200 0.1 sm_100a"; }
+
+const char *fcl_status_string(fcl_status s) {
+    switch (s) {
+    case FCL_SUCCESS: return "FCL_SUCCESS";
+    case FCL_DEVICE_NOT_AVAILABLE: return "FCL_DEVICE_NOT_AVAILABLE";
+    case FCL_OUT_OF_RESOURCES: return "FCL_OUT_OF_RESOURCES";
+    case FCL_INVALID_VALUE: return "FCL_INVALID_VALUE";
+    case FCL_INVALID_CONTEXT: return "FCL_INVALID_CONTEXT";
+    case FCL_INVALID_MEM_OBJECT: return "FCL_INVALID_MEM_OBJECT";
+    case FCL_INVALID_KERNEL_NAME: return "FCL_INVALID_KERNEL_NAME";
+    case FCL_INVALID_KERNEL: return "FCL_INVALID_KERNEL";
+    case FCL_INVALID_KERNEL_ARGS: return "FCL_INVALID_KERNEL_ARGS";
+    case FCL_INVALID_WORK_DIMENSION: return "FCL_INVALID_WORK_DIMENSION";
+    case FCL_INVALID_WORK_GROUP_SIZE: return "FCL_INVALID_WORK_GROUP_SIZE";
+    case FCL_INVALID_GLOBAL_WORK_SIZE: return "FCL_INVALID_GLOBAL_WORK_SIZE";
+    case FCL_CONTEXT_LOST: return "FCL_CONTEXT_LOST";
+    case FCL_CUDA_ERROR: return "FCL_CUDA_ERROR";
+    case FCL_NOT_SUPPORTED: return "FCL_NOT_SUPPORTED";
+    default: return "FCL_UNKNOWN_STATUS";
+    }
+}
+
+const char *fcl_last_error(fcl_context ctx) { return ctx ? ctx->err.c_str() : "no context"; }
+
+fcl_status fcl_default_launch_opts(fcl_launch_opts *o) {
+    if (!o) return FCL_INVALID_VALUE;
+    std::memset(o, 0, sizeof *o);
+    o->mode = FCL_MODE_COOP;
+    o->forced_split = -1;
+    o->init_chunk_pct = 2;
+    o->step_pct = 2;
+    o->cpu_wg_split = 1;
+    o->abort_period = 0;
+    o->wg_lo = 0;
+    o->wg_hi = 0;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
+    if (!out) return FCL_INVALID_VALUE;
+    *out = nullptr;
+    fcl_context_desc d{};
+    if (desc) d = *desc;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) { cudaGetLastError(); return FCL_DEVICE_NOT_AVAILABLE; }
+    if (d.device < 0 || d.device >= ndev) return FCL_INVALID_VALUE;
+    if (d.status_location != FCL_STATUS_HOST_MAPPED && d.status_location != FCL_STATUS_DEVICE) return FCL_INVALID_VALUE;
+    fcl_context ctx = new fcl_context_st();
+    ctx->device = d.device;
+    ctx->status_location = d.status_location;
+    auto fail = [&](cudaError_t e, const char *what) {
+        set_err(ctx, FCL_CUDA_ERROR, "%s: %s", what, cudaGetErrorString(e));
+        fprintf(stderr, "fcl_create_context: %s\n", ctx->err.c_str());
+        delete ctx;
+        return FCL_CUDA_ERROR;
+    };
+    cudaError_t e;
+    if ((e = cudaSetDevice(d.device)) != cudaSuccess) return fail(e, "cudaSetDevice");
+    if ((e = cudaFree(nullptr)) != cudaSuccess) return fail(e, "context init");
+    cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, d.device);
+    auto mk = [&](void *given, cudaStream_t *s, bool *own) -> cudaError_t {
+        if (given) { *s = (cudaStream_t)given; *own = false; return cudaSuccess; }
+        *own = true;
+        return cudaStreamCreateWithFlags(s, cudaStreamNonBlocking);
+    };
+    if ((e = mk(d.main_stream, &ctx->main, &ctx->own_main)) != cudaSuccess) return fail(e, "main stream");
+    if ((e = mk(d.hd_stream, &ctx->hd, &ctx->own_hd)) != cudaSuccess) return fail(e, "hd stream");
+    if ((e = mk(d.dh_stream, &ctx->dh, &ctx->own_dh)) != cudaSuccess) return fail(e, "dh stream");
+    // status word and exit record
+    void *hp = nullptr;
+    if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "exit record");
+    std::memset(hp, 0, 64);
+    ctx->exit_host = (unsigned long long *)hp;
+    void *dp = nullptr;
+    if ((e = cudaHostGetDevicePointer(&dp, hp, 0)) != cudaSuccess) return fail(e, "exit record mapping");
+    ctx->exit_dptr = (unsigned long long *)dp;
+    if (d.status_location == FCL_STATUS_HOST_MAPPED) {
+        if ((e = cudaHostAlloc(&hp, 8 * fcl_context_st::kSlots, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "status word");
+        std::memset(hp, 0, 8 * fcl_context_st::kSlots);
+        ctx->status_host = (unsigned long long *)hp;
+        if ((e = cudaHostGetDevicePointer(&dp, hp, 0)) != cudaSuccess) return fail(e, "status mapping");
+        ctx->status_dptr = (unsigned long long *)dp;
+    } else {
+        if ((e = cudaMalloc(&dp, 8 * fcl_context_st::kSlots)) != cudaSuccess) return fail(e, "status word");
+        cudaMemset(dp, 0, 8 * fcl_context_st::kSlots);
+        ctx->status_dptr = (unsigned long long *)dp;
+    }
+    // device counters: claim (u64), tasks (u64), done (u32), wmin (u32)
+    if ((e = cudaMalloc(&dp, 64)) != cudaSuccess) return fail(e, "counters");
+    cudaMemset(dp, 0, 64);
+    ctx->dclaim = (unsigned long long *)dp;
+    ctx->dtasks = ctx->dclaim + 1;
+    ctx->ddone = (unsigned int *)(ctx->dclaim + 2);
+    ctx->dwmin = ctx->ddone + 1;
+    const unsigned int ff = 0xFFFFFFFFu;
+    if ((e = cudaMemcpy(ctx->dwmin, &ff, 4, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "counter init");
+    for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1, &ctx->ev_m0, &ctx->ev_m1})
+        if ((e = cudaEventCreate(pe)) != cudaSuccess) return fail(e, "events");
+    if ((e = cudaEventCreateWithFlags(&ctx->ev_hd_last, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
+    if ((e = cudaEventCreateWithFlags(&ctx->ev_mark, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
+    // stream memory operations for publication (driver entry point; fall back to a kernel store)
+    {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue64", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess && fn)
+            ctx->write64 = (PFN_writeValue64)fn;
+        else
+            cudaGetLastError();
+    }
+    if (getenv("FCL_NO_MEMOPS")) ctx->write64 = nullptr;
+    if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail(e, "init sync");
+    const char *pin = getenv("FCL_PIN_THREADS");
+    const bool do_pin = d.pin_threads ? true : (pin ? atoi(pin) != 0 : true);
+    int nthr = d.n_host_threads;
+    if (nthr <= 0 && getenv("FCL_HOST_THREADS")) nthr = atoi(getenv("FCL_HOST_THREADS"));
+    ctx->ex.start(nthr, do_pin);
+    *out = ctx;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_release_context(fcl_context ctx) {
+    if (!ctx) return FCL_INVALID_CONTEXT;
+    cudaSetDevice(ctx->device);
+    cudaDeviceSynchronize();
+    ctx->ex.shutdown();
+    for (auto &pe : ctx->pool) cudaFree(pe.p);
+    for (auto e : ctx->evpool) cudaEventDestroy(e);
+    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_k1, ctx->ev_m0, ctx->ev_m1, ctx->ev_hd_last, ctx->ev_mark})
+        if (e) cudaEventDestroy(e);
+    if (ctx->status_host) cudaFreeHost(ctx->status_host);
+    else if (ctx->status_dptr) cudaFree(ctx->status_dptr);
+    if (ctx->exit_host) cudaFreeHost(ctx->exit_host);
+    if (ctx->dclaim) cudaFree(ctx->dclaim);
+    if (ctx->own_main) cudaStreamDestroy(ctx->main);
+    if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
+    if (ctx->own_dh) cudaStreamDestroy(ctx->dh);
+    delete ctx;
+    return FCL_SUCCESS;
+}
+
+static fcl_status create_buffer_impl(fcl_context ctx, uint32_t flags, size_t bytes, uint32_t elem_size,
+                                     const void *host_init, void *host_ptr, void *device_ptr, fcl_buffer *out) {
+    fcl_status s = check_ctx(ctx);
+    if (s != FCL_SUCCESS) return s;
+    if (!out || bytes == 0) return set_err(ctx, FCL_INVALID_VALUE, "bytes must be > 0");
+    if (!(elem_size == 1 || elem_size == 2 || elem_size == 4 || elem_size == 8) || bytes % elem_size)
+        return set_err(ctx, FCL_INVALID_VALUE, "elem_size %u invalid for %zu bytes", elem_size, bytes);
+    if ((flags & FCL_MEM_USE_HOST_PTR) && !host_ptr) return set_err(ctx, FCL_INVALID_VALUE, "USE_HOST_PTR without host_ptr");
+    if ((flags & FCL_MEM_USE_DEVICE_PTR) && !device_ptr) return set_err(ctx, FCL_INVALID_VALUE, "USE_DEVICE_PTR without device_ptr");
+    fcl_buffer b = new fcl_buffer_st();
+    b->ctx = ctx; b->bytes = bytes; b->elem_size = elem_size; b->flags = flags;
+    cudaError_t e;
+    if (flags & FCL_MEM_USE_DEVICE_PTR) { b->dev = device_ptr; b->own_dev = false; }
+    else {
+        if ((e = cudaMalloc(&b->dev, bytes)) != cudaSuccess) { cudaGetLastError(); delete b; return set_err(ctx, FCL_OUT_OF_RESOURCES, "cudaMalloc(%zu)", bytes); }
+        b->own_dev = true;
+    }
+    if (flags & FCL_MEM_USE_HOST_PTR) { b->host = host_ptr; b->own_host = false; }
+    else {
+        if ((e = cudaHostAlloc(&b->host, bytes, cudaHostAllocPortable)) != cudaSuccess) {
+            cudaGetLastError();
+            if (b->own_dev) cudaFree(b->dev);
+            delete b;
+            return set_err(ctx, FCL_OUT_OF_RESOURCES, "cudaHostAlloc(%zu)", bytes);
+        }
+        b->own_host = true;
+    }
+    if ((e = cudaEventCreateWithFlags(&b->d2h_ev, cudaEventDisableTiming)) != cudaSuccess) { delete b; return cuda_fail(ctx, e, "event"); }
+    const bool ext_host = (flags & FCL_MEM_USE_HOST_PTR) != 0, ext_dev = (flags & FCL_MEM_USE_DEVICE_PTR) != 0;
+    if (host_init) {
+        std::memcpy(b->host, host_init, bytes);
+        if ((e = cudaMemcpy(b->dev, b->host, bytes, cudaMemcpyHostToDevice)) != cudaSuccess) return cuda_fail(ctx, e, "initial H2D");
+    } else if (ext_host && !ext_dev) {
+        if ((e = cudaMemcpy(b->dev, b->host, bytes, cudaMemcpyHostToDevice)) != cudaSuccess) return cuda_fail(ctx, e, "initial H2D");
+    } else if (ext_dev && !ext_host) {
+        if ((e = cudaMemcpy(b->host, b->dev, bytes, cudaMemcpyDeviceToHost)) != cudaSuccess) return cuda_fail(ctx, e, "initial D2H");
+    } else if (!ext_host && !ext_dev) {
+        std::memset(b->host, 0, bytes);
+        if ((e = cudaMemset(b->dev, 0, bytes)) != cudaSuccess) return cuda_fail(ctx, e, "memset");
+    }
+    b->host_valid = b->dev_valid = true;
+    *out = b;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_create_buffer(fcl_context ctx, uint32_t flags, size_t bytes, uint32_t elem_size,
+                             const void *host_init, fcl_buffer *out) {
+    if (flags & (FCL_MEM_USE_HOST_PTR | FCL_MEM_USE_DEVICE_PTR))
+        return set_err(ctx, FCL_INVALID_VALUE, "use fcl_create_buffer_ext for caller-owned memory");
+    return create_buffer_impl(ctx, flags, bytes, elem_size, host_init, nullptr, nullptr, out);
+}
+
+fcl_status fcl_create_buffer_ext(fcl_context ctx, uint32_t flags, size_t bytes, uint32_t elem_size,
+                                 void *host_ptr, void *device_ptr, fcl_buffer *out) {
+    if (host_ptr) flags |= FCL_MEM_USE_HOST_PTR;
+    if (device_ptr) flags |= FCL_MEM_USE_DEVICE_PTR;
+    return create_buffer_impl(ctx, flags, bytes, elem_size, nullptr, host_ptr, device_ptr, out);
+}
+
+fcl_status fcl_release_buffer(fcl_buffer b) {
+    if (!b) return FCL_INVALID_MEM_OBJECT;
+    fcl_context ctx = b->ctx;
+    cudaSetDevice(ctx->device);
+    cudaStreamSynchronize(ctx->main);
+    cudaStreamSynchronize(ctx->hd);
+    cudaStreamSynchronize(ctx->dh);
+    if (b->merge_pending) {
+        if (b->twin) pool_put(ctx, b->twin);
+        if (b->stage) pool_put(ctx, b->stage);
+        ctx->defer_list.erase(std::remove(ctx->defer_list.begin(), ctx->defer_list.end(), b), ctx->defer_list.end());
+    }
+    if (b->own_dev) cudaFree(b->dev);
+    if (b->own_host) cudaFreeHost(b->host);
+    cudaEventDestroy(b->d2h_ev);
+    delete b;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t n, const void *src, int32_t blocking) {
+    fcl_status s = check_ctx(ctx);
+    if (s != FCL_SUCCESS) return s;
+    if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
+    if (!src || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "write range");
+    if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
+    // the rest of the buffer must be current on both sides before a partial write
+    char *h = (char *)b->host + offset;
+    if (n < b->bytes) {
+        fcl_status st = make_valid(ctx, b, true, true);
+        if (st != FCL_SUCCESS) return st;
+    }
+    // overwriting the pinned mirror: no queued copy may still read its old contents
+    if (src != h) CK(ctx, cudaStreamSynchronize(ctx->main));
+    if (src != h) std::memcpy(h, src, n);
+    CK(ctx, cudaMemcpyAsync((char *)b->dev + offset, h, n, cudaMemcpyHostToDevice, ctx->main));
+    ctx->info.h2d_bytes += (int64_t)n;
+    b->host_valid = b->dev_valid = true;
+    if (blocking) CK(ctx, cudaStreamSynchronize(ctx->main));
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t n, void *dst, int32_t blocking) {
+    fcl_status s = check_ctx(ctx);
+    if (s != FCL_SUCCESS) return s;
+    if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
+    if (!dst || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "read range");
+    (void)blocking;
+    if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
+    if (b->host_valid) {   // location tracking (L20.s31-33): no transfer when the host is current
+        const char *h = (const char *)b->host + offset;
+        if (dst != h) std::memcpy(dst, h, n);
+        return FCL_SUCCESS;
+    }
+    CK(ctx, cudaStreamSynchronize(ctx->main));
+    CK(ctx, cudaMemcpy((char *)b->host + offset, (char *)b->dev + offset, n, cudaMemcpyDeviceToHost));
+    if (n == b->bytes) b->host_valid = true;
+    const char *h = (const char *)b->host + offset;
+    if (dst != h) std::memcpy(dst, h, n);
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_buffer_info(fcl_buffer b, void **host_ptr, void **device_ptr, size_t *bytes, uint32_t *elem_size) {
+    if (!b) return FCL_INVALID_MEM_OBJECT;
+    if (host_ptr) *host_ptr = b->host;
+    if (device_ptr) *device_ptr = b->dev;
+    if (bytes) *bytes = b->bytes;
+    if (elem_size) *elem_size = b->elem_size;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_get_kernel(fcl_context ctx, const char *name, fcl_kernel *out) {
+    (void)ctx;
+    if (!name || !out) return FCL_INVALID_VALUE;
+    static fcl_kernel_st handles[kNumKernels];
+    for (int k = 0; k < kNumKernels; ++k)
+        if (!std::strcmp(kKernels[k].name, name)) {
+            handles[k].def = &kKernels[k];
+            *out = &handles[k];
+            return FCL_SUCCESS;
+        }
+    return FCL_INVALID_KERNEL_NAME;
+}
+
+fcl_status fcl_kernel_signature(fcl_kernel k, char *buf, size_t len) {
+    if (!k || !buf || len == 0) return FCL_INVALID_VALUE;
+    std::string s;
+    for (int a = 0; a < k->def->nargs; ++a) {
+        const ArgSpec &sp = k->def->args[a];
+        if (a) s += ' ';
+        s += sp.name;
+        s += ':';
+        if (sp.kind == 'b') s += (sp.acc == 1 ? "in" : sp.acc == 2 ? "out" : "inout");
+        else s += (sp.kind == 'i' ? "i" : "f");
+    }
+    std::snprintf(buf, len, "%s", s.c_str());
+    return s.size() < len ? FCL_SUCCESS : FCL_INVALID_VALUE;
+}
+
+static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work_dim, const size_t gws[3],
+                               const size_t lws[3], const fcl_arg *args, uint32_t n_args, const fcl_launch_opts *opts,
+                               Launch &L) {
+    if (!kernel) return FCL_INVALID_KERNEL;
+    const KernelDef *kd = kernel->def;
+    if (work_dim < 1 || work_dim > 3) return set_err(ctx, FCL_INVALID_WORK_DIMENSION, "work_dim %u", work_dim);
+    if (!gws || !lws) return set_err(ctx, FCL_INVALID_VALUE, "gws/lws required");
+    Geom g{};
+    g.work_dim = (int)work_dim;
+    int64_t lprod = 1;
+    g.n_wg = 1;
+    for (uint32_t d = 0; d < 3; ++d) {
+        g.gws[d] = d < work_dim ? (int64_t)gws[d] : 1;
+        g.lws[d] = d < work_dim ? (int64_t)lws[d] : 1;
+        if (g.lws[d] <= 0 || g.gws[d] <= 0) return set_err(ctx, FCL_INVALID_WORK_GROUP_SIZE, "zero size in dim %u", d);
+        if (g.gws[d] % g.lws[d]) return set_err(ctx, FCL_INVALID_WORK_GROUP_SIZE, "gws %% lws != 0 in dim %u", d);
+        g.ng[d] = g.gws[d] / g.lws[d];
+        lprod *= g.lws[d];
+        g.n_wg *= g.ng[d];
+    }
+    if (lprod > 1024) return set_err(ctx, FCL_INVALID_WORK_GROUP_SIZE, "work-group of %lld > 1024 items", (long long)lprod);
+    if (g.n_wg >= 0xFFFFFFFFll) return set_err(ctx, FCL_INVALID_GLOBAL_WORK_SIZE, "too many work-groups");
+    if ((int)n_args != kd->nargs || !args) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "%s takes %d args", kd->name, kd->nargs);
+    KArgs a{};
+    a.kernel = kd->id;
+    a.integer = kd->integer;
+    a.alpha = 1.5f; a.beta = 1.2f; a.eps = 0.1f; a.ialpha = 3; a.ibeta = 2;
+    int nb = 0, ni = 0;
+    int64_t ints[2] = {0, 0};
+    L.nout = 0;
+    for (int k = 0; k < kd->nargs; ++k) {
+        const ArgSpec &sp = kd->args[k];
+        const fcl_arg &ar = args[k];
+        if (sp.kind == 'b') {
+            if (ar.kind != FCL_ARG_BUFFER || !ar.buffer || ar.buffer->ctx != ctx)
+                return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %d (%s) must be a buffer of this context", k, sp.name);
+            const int acc = ar.access ? ar.access : sp.acc;
+            if ((sp.acc & 2) && !(acc & 2))
+                return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %s is written by %s: access must be OUT/INOUT", sp.name, kd->name);
+            if (ar.buffer->elem_size != 4) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %s: elem_size must be 4", sp.name);
+            L.bufs[nb] = ar.buffer;
+            a.dev[nb] = ar.buffer->dev;
+            a.host[nb] = ar.buffer->host;
+            if (sp.acc & 2) L.out_idx[L.nout++] = nb;
+            ++nb;
+        } else if (sp.kind == 'i') {
+            if (ar.kind != FCL_ARG_INT) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %d (%s) must be an int", k, sp.name);
+            if (!std::strcmp(sp.name, "alpha")) a.ialpha = (int32_t)ar.i;
+            else if (!std::strcmp(sp.name, "beta")) a.ibeta = (int32_t)ar.i;
+            else if (ni < 2) ints[ni++] = ar.i;
+        } else {
+            if (ar.kind != FCL_ARG_FLOAT) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %d (%s) must be a float", k, sp.name);
+            if (!std::strcmp(sp.name, "alpha")) a.alpha = (float)ar.f;
+            else if (!std::strcmp(sp.name, "beta")) a.beta = (float)ar.f;
+            else if (!std::strcmp(sp.name, "eps")) a.eps = (float)ar.f;
+        }
+    }
+    a.nbuf = nb;
+    a.n0 = ints[0];
+    a.n1 = ni >= 2 ? ints[1] : ints[0];
+    if (a.n0 <= 0 || a.n1 <= 0) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "problem sizes must be > 0");
+    for (int k = 0; k < nb; ++k) {
+        const int64_t need = required_elems(a.kernel, k, a.n0, a.n1) * 4;
+        if ((int64_t)L.bufs[k]->bytes < need)
+            return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "buffer arg %d holds %zu bytes, needs %lld", k, L.bufs[k]->bytes, (long long)need);
+    }
+    int64_t ext[3];
+    required_extent(a.kernel, a.n0, a.n1, ext);
+    for (uint32_t d = 0; d < work_dim; ++d)
+        if (g.gws[d] < ext[d] || g.gws[d] >= ext[d] + g.lws[d])
+            return set_err(ctx, FCL_INVALID_GLOBAL_WORK_SIZE, "gws[%u]=%lld must be the extent %lld padded to lws", d,
+                           (long long)g.gws[d], (long long)ext[d]);
+    const char *why = nullptr;
+    if (!gpu_geometry_ok(a, g, &why)) return set_err(ctx, FCL_INVALID_WORK_GROUP_SIZE, "%s: %s", kd->name, why);
+    fcl_launch_opts o;
+    fcl_default_launch_opts(&o);
+    if (opts) o = *opts;
+    if (o.mode < FCL_MODE_COOP || o.mode > FCL_MODE_CPU_ONLY) return set_err(ctx, FCL_INVALID_VALUE, "mode");
+    int64_t lo = o.wg_lo, hi = o.wg_hi > 0 ? o.wg_hi : g.n_wg;
+    if (lo < 0 || hi > g.n_wg || lo >= hi) return set_err(ctx, FCL_INVALID_VALUE, "wg range [%lld, %lld)", (long long)lo, (long long)hi);
+    const int64_t al = gpu_slice_align(a, g);
+    if ((lo % al) || (hi % al && hi != g.n_wg))
+        return set_err(ctx, FCL_INVALID_VALUE, "wg range must be aligned to %lld work-groups (fcl_slice_range)", (long long)al);
+    L.ctx = ctx; L.kd = kd; L.a = a; L.g = g; L.lo = lo; L.hi = hi; L.o = o;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work_dim, const size_t gws[3],
+                               const size_t lws[3], const fcl_arg *args, uint32_t n_args, const fcl_launch_opts *opts,
+                               fcl_launch_info *info_out) {
+    fcl_status s = check_ctx(ctx);
+    if (s != FCL_SUCCESS) return s;
+    const double t_call = now_ms();
+    Launch L{};
+    s = build_launch(ctx, kernel, work_dim, gws, lws, args, n_args, opts, L);
+    if (s != FCL_SUCCESS) return s;
+    if (!ctx->defer_list.empty()) return set_err(ctx, FCL_INVALID_VALUE, "a deferred merge is pending (call fcl_merge)");
+    std::memset(&ctx->info, 0, sizeof ctx->info);
+    ctx->have_k = ctx->have_m = false;
+    fcl_launch_info &info = ctx->info;
+    info.n_wg = L.hi - L.lo;
+    info.wg_lo = L.lo;
+    info.wg_hi = L.hi;
+    info.gpu_watermark = info.published_watermark = L.hi;
+    // coherence of every argument for the chosen mode (minimal location tracking)
+    for (int k = 0; k < L.a.nbuf; ++k) {
+        const bool is_out = std::find(L.out_idx, L.out_idx + L.nout, k) != L.out_idx + L.nout;
+        const bool need_host = L.o.mode != FCL_MODE_GPU_ONLY || is_out;
+        const bool need_dev = L.o.mode != FCL_MODE_CPU_ONLY;
+        s = make_valid(ctx, L.bufs[k], need_host, need_dev);
+        if (s != FCL_SUCCESS) return s;
+    }
+    switch (L.o.mode) {
+    case FCL_MODE_GPU_ONLY: s = run_gpu_only(L); break;
+    case FCL_MODE_CPU_ONLY: s = run_cpu_only(L); break;
+    default: s = run_coop(L); break;
+    }
+    pool_trim(ctx);
+    info.t_call_ms = now_ms() - t_call;
+    if (info_out) *info_out = info;
+    return s;
+}
+
+fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
+    fcl_status s = check_ctx(ctx);
+    if (s != FCL_SUCCESS) return s;
+    if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
+    if (!b->merge_pending) return FCL_SUCCESS;
+    if (gpu_launch_merge((char *)b->dev + b->m_b0, (char *)b->stage + b->m_b0, (char *)b->twin + b->m_b0,
+                         b->m_b1 - b->m_b0, (int)b->elem_size, ctx->num_sms, ctx->main) < 0)
+        return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    CK(ctx, cudaEventRecord(ctx->ev_mark, ctx->main));
+    CK(ctx, cudaStreamWaitEvent(ctx->hd, ctx->ev_mark, 0));   // pool reuse is ordered after the merge
+    if (b->r_b1 > b->r_b0) {
+        CK(ctx, cudaStreamWaitEvent(ctx->dh, ctx->ev_mark, 0));
+        CK(ctx, cudaMemcpyAsync((char *)b->host + b->r_b0, (char *)b->dev + b->r_b0, b->r_b1 - b->r_b0,
+                                cudaMemcpyDeviceToHost, ctx->dh));
+        CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
+        b->d2h_pending = true;
+    }
+    b->r_b0 = b->r_b1 = 0;
+    pool_put(ctx, b->twin);
+    pool_put(ctx, b->stage);
+    b->twin = b->stage = nullptr;
+    b->merge_pending = false;
+    ctx->defer_list.erase(std::remove(ctx->defer_list.begin(), ctx->defer_list.end(), b), ctx->defer_list.end());
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_merge_raw(void *gpu, const void *cpu, const void *twin, size_t bytes, uint32_t elem_size, void *stream) {
+    if (!(elem_size == 1 || elem_size == 2 || elem_size == 4 || elem_size == 8) || bytes % elem_size) return FCL_INVALID_VALUE;
+    if (bytes && (!gpu || !cpu || !twin)) return FCL_INVALID_VALUE;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (gpu_launch_merge(gpu, cpu, twin, bytes, (int)elem_size, sms, stream) < 0) return FCL_CUDA_ERROR;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_finish(fcl_context ctx) {
+    if (!ctx) return FCL_INVALID_CONTEXT;
+    if (ctx->sticky != FCL_SUCCESS) return ctx->sticky;
+    cudaSetDevice(ctx->device);
+    CK(ctx, cudaStreamSynchronize(ctx->main));
+    CK(ctx, cudaStreamSynchronize(ctx->hd));
+    CK(ctx, cudaStreamSynchronize(ctx->dh));
+    CK(ctx, cudaGetLastError());
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info) {
+    if (!ctx) return FCL_INVALID_CONTEXT;
+    if (!info) return FCL_INVALID_VALUE;
+    cudaSetDevice(ctx->device);
+    if (ctx->have_k) {
+        float ms = 0.f;
+        if (cudaEventSynchronize(ctx->ev_k1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_k0, ctx->ev_k1) == cudaSuccess)
+            ctx->info.t_gpu_kernel_ms = ms;
+        // the exit record of a cooperative launch that finished after the host returned
+        uint32_t wm;
+        uint64_t nt;
+        if (poll_exit(ctx, &wm, &nt)) {
+            ctx->info.gpu_tasks = (int64_t)nt;
+            if (!ctx->info.cpu_did_all) ctx->info.gpu_watermark = (wm == 0xFFFFFFFFu) ? ctx->info.wg_hi : (int64_t)wm;
+        }
+    }
+    if (ctx->have_m) {
+        float ms = 0.f;
+        if (cudaEventSynchronize(ctx->ev_m1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_m0, ctx->ev_m1) == cudaSuccess)
+            ctx->info.t_merge_ms = ms;
+    }
+    cudaGetLastError();
+    *info = ctx->info;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_slice_range(fcl_kernel kernel, uint32_t work_dim, const size_t gws[3], const size_t lws[3],
+                           int32_t rank, int32_t nranks, int64_t *wg_lo, int64_t *wg_hi) {
+    if (!kernel || !gws || !lws || !wg_lo || !wg_hi || nranks < 1 || rank < 0 || rank >= nranks) return FCL_INVALID_VALUE;
+    if (work_dim < 1 || work_dim > 3) return FCL_INVALID_WORK_DIMENSION;
+    Geom g{};
+    g.work_dim = (int)work_dim;
+    g.n_wg = 1;
+    for (uint32_t d = 0; d < 3; ++d) {
+        g.gws[d] = d < work_dim ? (int64_t)gws[d] : 1;
+        g.lws[d] = d < work_dim ? (int64_t)lws[d] : 1;
+        if (g.lws[d] <= 0 || g.gws[d] % g.lws[d]) return FCL_INVALID_WORK_GROUP_SIZE;
+        g.ng[d] = g.gws[d] / g.lws[d];
+        g.n_wg *= g.ng[d];
+    }
+    KArgs a{};
+    a.kernel = kernel->def->id;
+    a.integer = kernel->def->integer;
+    int64_t ext[3] = {g.gws[0], g.gws[1], 1};
+    (void)ext;
+    a.n0 = a.n1 = 0;
+    const int64_t al = gpu_slice_align(a, g);
+    const int64_t units = (g.n_wg + al - 1) / al;
+    const int64_t u0 = units * rank / nranks, u1 = units * (rank + 1) / nranks;
+    *wg_lo = std::min<int64_t>(u0 * al, g.n_wg);
+    *wg_hi = std::min<int64_t>(u1 * al, g.n_wg);
+    return FCL_SUCCESS;
+}
+
+}  // extern "C"

@@ -1,0 +1,221 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the oracle, every kernel.
+
+Each case checks, at sizes that span several tiles and a ragged tail:
+  * GPU-only (plain grid) and CPU-only (host executor) against the oracle (bit-exact int32,
+    1e-5 relative fp32);
+  * the bit-identity of the two device bodies;
+  * FluidiCL cooperative execution at forced split points and free-running: host copy
+    and device copy both equal the single-device result bit for bit.
+"""
+import numpy as np
+import pytest
+
+import fcl_harness as H
+import workloads as W
+from _util import assert_bits, assert_parity, oracle_outputs
+
+pytestmark = pytest.mark.gpu
+
+CASES = [
+    # kernel, n0, n1, integer, lws1d, lws2d
+    ("atax_tmp", 300, 200, False, 32, None),
+    ("atax_tmp", 300, 200, True, 32, None),
+    ("atax_y", 300, 200, False, 32, None),
+    ("atax_y", 300, 200, True, 32, None),
+    ("bicg_s", 257, 384, False, 64, None),
+    ("bicg_s", 257, 384, True, 64, None),
+    ("bicg_q", 384, 257, False, 64, None),
+    ("bicg_q", 384, 257, True, 64, None),
+    ("gesummv", 300, 300, False, 32, None),
+    ("gesummv", 300, 300, True, 32, None),
+    ("gesummv", 512, 512, False, 256, None),
+    ("syrk", 200, 70, False, None, (32, 8)),
+    ("syrk", 256, 128, False, None, (32, 8)),
+    ("syrk", 200, 70, True, None, (32, 8)),
+    ("syr2k", 200, 70, False, None, (32, 8)),
+    ("syr2k", 256, 64, True, None, (32, 8)),
+    ("conv2d", 150, 300, False, None, (32, 8)),
+    ("conv2d", 150, 300, True, None, (32, 8)),
+    ("corr_mean", 200, 300, False, 64, None),
+    ("corr_std", 200, 300, False, 64, None),
+    ("corr_reduce", 200, 300, False, None, (32, 8)),
+    ("corr_corr", 200, 300, False, 64, None),
+]
+
+
+def _ids(c):
+    return f"{c[0]}-{'i32' if c[3] else 'f32'}-{c[1]}x{c[2]}"
+
+
+def _problem(c, seed=0):
+    kernel, n0, n1, integer, l1, l2 = c
+    return W.make(kernel, n0, n1, integer=integer, seed=seed, lws1d=l1 or 256, lws2d=l2 or (32, 8))
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    from paper_conf_cgo_panditg14_b200 import _build, fcl
+    _build.build()
+    c = fcl.Context(0)
+    yield c
+    c.release()
+
+
+@pytest.mark.parametrize("case", CASES, ids=_ids)
+def test_single_device_modes_vs_oracle(ctx, oracle_mod, case):
+    P = _problem(case)
+    R = oracle_outputs(oracle_mod, P)
+    g_out, g_info = H.run(ctx, P, mode="gpu")
+    c_out, c_info = H.run(ctx, P, mode="cpu")
+    assert g_info["gpu_launches"] >= 1 and c_info["cpu_did_all"] == 1
+    for k in P.out_indices:
+        assert_parity(g_out[k], R[k], P.integer, f"{_ids(case)} gpu-only buf{k}")
+        assert_parity(c_out[k], R[k], P.integer, f"{_ids(case)} cpu-only buf{k}")
+        assert_bits(g_out[k], c_out[k], f"{_ids(case)} gpu vs cpu body buf{k}")
+
+
+@pytest.mark.parametrize("case", CASES, ids=_ids)
+def test_forced_splits_bit_identical(ctx, oracle_mod, case):
+    """Every (or a spread of) split point(s): merge(G, C, T) equals the single-device result."""
+    P = _problem(case, seed=1)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    R = oracle_outputs(oracle_mod, P)
+    n = P.num_groups
+    splits = range(n + 1) if n <= 20 else sorted({0, 1, n // 3, n // 2, n - 1, n})
+    for s in splits:
+        bufs = H.create_buffers(ctx, P)
+        out, info = H.run(ctx, P, mode="coop", bufs=bufs, forced_split=s)
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], f"{_ids(case)} split {s} host copy buf{k}")
+            dev = H.device_array(bufs[k], np.int32 if P.integer else np.float32)
+            assert_bits(dev, ref[k], f"{_ids(case)} split {s} device copy buf{k}")
+        if s == n:
+            assert info["merged"] == 0
+        for b in bufs:
+            b.release()
+    for k in P.out_indices:
+        assert_parity(ref[k], R[k], P.integer, _ids(case))
+
+
+@pytest.mark.parametrize("case", CASES, ids=_ids)
+@pytest.mark.parametrize("status", ["host_mapped", "device"])
+def test_free_running_coop(oracle_mod, case, status):
+    from paper_conf_cgo_panditg14_b200 import fcl
+    ctx = fcl.Context(0, status_location=status)
+    try:
+        P = _problem(case, seed=2)
+        R = oracle_outputs(oracle_mod, P)
+        ref, _ = H.run(ctx, P, mode="gpu")
+        for trial in range(3):
+            bufs = H.create_buffers(ctx, P)
+            out, info = H.run(ctx, P, mode="coop", bufs=bufs, host_delay_us=[0, 50, 500][trial])
+            for k in P.out_indices:
+                assert_bits(out[k], ref[k], f"{_ids(case)} coop host buf{k} trial {trial}")
+                dev = H.device_array(bufs[k], np.int32 if P.integer else np.float32)
+                assert_bits(dev, ref[k], f"{_ids(case)} coop device buf{k} trial {trial}")
+                assert_parity(out[k], R[k], P.integer, _ids(case))
+            for b in bufs:
+                b.release()
+    finally:
+        ctx.release()
+
+
+@pytest.mark.parametrize("case", [CASES[0], CASES[9], CASES[12], CASES[16]], ids=_ids)
+def test_fault_injection(ctx, oracle_mod, case):
+    """Dropped publications, slow host, tiny and huge chunks: the result never changes."""
+    P = _problem(case, seed=3)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    for kw in [dict(drop_publish=1), dict(host_delay_us=2000), dict(init_chunk_pct=50, step_pct=0),
+               dict(init_chunk_pct=1, step_pct=1), dict(cpu_wg_split=0), dict(n_host_threads=1),
+               dict(abort_period=1), dict(abort_period=-1)]:
+        out, info = H.run(ctx, P, mode="coop", **kw)
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], f"{_ids(case)} {kw}")
+
+
+def test_cpu_first_returns_host_authoritative(ctx):
+    """L16.s21: when the host covers everything first the host copy is final, no D2H."""
+    P = W.make("gesummv", 512, integer=True, seed=4, lws1d=256)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    bufs = H.create_buffers(ctx, P)
+    out, info = H.run(ctx, P, mode="coop", bufs=bufs, forced_split=0)
+    assert info["cpu_did_all"] == 1 and info["d2h_bytes"] == 0
+    for k in P.out_indices:
+        assert_bits(out[k], ref[k], "host")
+        assert_bits(H.device_array(bufs[k], np.int32), ref[k], "device (merged)")
+
+
+def test_slices_cover_only_their_range(ctx):
+    """opts.wg_lo/wg_hi: a rank's slice writes exactly its work-groups (multi-GPU building block)."""
+    P = W.make("conv2d", 130, 260, integer=True, seed=5)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    k = ctx.kernel(H.kernel_name(P))
+    nwg = P.num_groups
+    for nranks in (2, 3):
+        acc = P.bufs[1].copy()
+        for r in range(nranks):
+            lo, hi = ctx.slice_range(k, P.gws, P.lws, r, nranks)
+            bufs = H.create_buffers(ctx, P)
+            out, info = H.run(ctx, P, mode="coop", bufs=bufs, wg_lo=lo, wg_hi=hi)
+            assert info["n_wg"] == hi - lo
+            # rows owned by the slice
+            ngx = P.gws[0] // P.lws[0]
+            r0, r1 = (lo // ngx) * P.lws[1], min((hi // ngx) * P.lws[1], P.n0) if hi < nwg else P.n0
+            o2, a2 = out[1].reshape(P.n0, P.n1), acc.reshape(P.n0, P.n1)
+            a2[r0:r1] = o2[r0:r1]
+            # untouched outside the slice
+            np.testing.assert_array_equal(np.delete(o2, np.s_[r0:r1], axis=0),
+                                          np.delete(P.bufs[1].reshape(P.n0, P.n1), np.s_[r0:r1], axis=0))
+            for b in bufs:
+                b.release()
+        assert_bits(acc, ref[1], f"{nranks} slices concatenated")
+
+
+def test_multi_kernel_chain_location_tracking(ctx, oracle_mod):
+    """ATAX tmp -> y with the two kernels on different devices (C22 minimal form)."""
+    n = 384
+    P1 = W.make("atax_tmp", n, n, seed=6, lws1d=64)
+    P2 = W.make("atax_y", n, n, seed=7, lws1d=64)
+    P2.bufs[0] = P1.bufs[0]
+    A, x, tmp = (ctx.buffer_from_array(b) for b in P1.bufs)
+    y = ctx.buffer_from_array(P2.bufs[2])
+    R1 = oracle_outputs(oracle_mod, P1)[2]
+    for m1, m2 in [("cpu", "gpu"), ("gpu", "cpu"), ("coop", "coop"), ("cpu", "coop")]:
+        ctx.enqueue_ndrange("atax_tmp_f32", P1.gws, P1.lws, [A, x, tmp, n, n], mode=m1)
+        ctx.enqueue_ndrange("atax_y_f32", P2.gws, P2.lws, [A, tmp, y, n, n], mode=m2)
+        ctx.finish()
+        got = y.read_array(np.float32)
+        L2 = oracle_mod.Launch("atax_y", False, n, n, list(P2.gws), list(P2.lws),
+                               [P1.bufs[0].astype(np.float64), R1.copy(), np.zeros(n)])
+        oracle_mod.run_range(L2, 0, L2.num_groups())
+        assert_parity(got, L2.bufs[2], False, f"atax chain {m1}->{m2}")
+    for b in (A, x, tmp, y):
+        b.release()
+
+
+def test_corr_chain_coop_vs_oracle(ctx, oracle_mod):
+    n, m = 300, 200
+    data = W.corr_chain_inputs(n, m, seed=8)
+    gws1, lws1 = W.geometry("corr_mean", n, m, lws1d=64)
+    gws2, lws2 = W.geometry("corr_reduce", n, m)
+    d = ctx.buffer_from_array(data)
+    mean = ctx.buffer_from_array(np.zeros(m, np.float32))
+    std = ctx.buffer_from_array(np.zeros(m, np.float32))
+    sym = ctx.buffer_from_array(np.full(m * m, -3.0, np.float32))
+    ctx.enqueue_ndrange("corr_mean_f32", gws1, lws1, [d, mean, n, m])
+    ctx.enqueue_ndrange("corr_std_f32", gws1, lws1, [d, mean, std, n, m, 0.1])
+    ctx.enqueue_ndrange("corr_reduce_f32", gws2, lws2, [d, mean, std, n, m])
+    ctx.enqueue_ndrange("corr_corr_f32", gws1, lws1, [d, sym, n, m])
+    ctx.finish()
+    got = sym.read_array(np.float32)
+    # the oracle's chain on the same inputs
+    d64, mean64, std64, sym64 = data.astype(np.float64), np.zeros(m), np.zeros(m), np.full(m * m, -3.0)
+    for kname, bl, g in [("corr_mean", [d64, mean64], (gws1, lws1)), ("corr_std", [d64, mean64, std64], (gws1, lws1)),
+                         ("corr_reduce", [d64, mean64, std64], (gws2, lws2)), ("corr_corr", [d64, sym64], (gws1, lws1))]:
+        L = oracle_mod.Launch(kname, False, n, m, list(g[0]), list(g[1]), bl)
+        oracle_mod.run_range(L, 0, L.num_groups())
+    assert_parity(got, sym64, False, "corr chain")
+    assert_parity(mean.read_array(np.float32), mean64, False, "corr mean")
+    assert_parity(d.read_array(np.float32), d64, False, "corr reduced data")
+    for b in (d, mean, std, sym):
+        b.release()
