@@ -1,0 +1,379 @@
+#!/usr/bin/env python
+"""bench.py -- FluidiCL on B200: end-to-end cooperative kernel time, roofline, oracle baseline.
+
+Default workload (BASELINE.json configs[1]): GESUMMV + BICG (both kernels), N = 4096, fp32,
+on one B200 plus the host cores.  One step = the three kernel launches through the C-ABI in
+FluidiCL cooperative mode (GPU dispatcher + host executor + staging + diff-merge + return of
+outputs), outputs coherent on the host at the end.  Inputs are resident in HBM and in the
+pinned host mirrors when the timed region starts; L2 is flushed between steps.
+
+Reported value: algorithmic GB/s of the step (bytes the kernels must move: every matrix
+read once per kernel, vectors read/written) / device-timed step duration, summed over ranks.
+Multi-GPU (torchrun): each rank runs an independent problem of the same size ("replicas",
+weak scaling, no data-path collective); the max step time over ranks is used.
+
+Also reported: GPU-only / CPU-only step times (the paper's two baselines, Fig 13), the merge
+kernel's HBM bandwidth on a 1 GiB diff-merge, the dispatcher's roofline, the oracle timed
+on the host cores (cpu_baseline) and an end-to-end number with the inputs' host->device
+copies inside the timed region (e2e).
+
+--impl reference times the oracle (the tier's reference arm) on the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np
+
+METRIC = "end-to-end kernel time vs GPU-only/CPU-only; merge HBM GB/s vs peak"
+N = 4096
+
+
+def algorithmic_bytes(n: int) -> dict:
+    f = 4
+    return {
+        "gesummv": 2 * n * n * f + 3 * n * f,   # A, B, x read; tmp, y written
+        "bicg_s": n * n * f + 2 * n * f,        # A, r read; s written
+        "bicg_q": n * n * f + 2 * n * f,        # A, p read; q written
+    }
+
+
+def problems(seed: int):
+    import workloads as W
+    P1 = W.make("gesummv", N, seed=seed, lws1d=256, out_init="zero")
+    P2 = W.make("bicg_s", N, N, seed=seed + 1, lws1d=256, out_init="zero")
+    P3 = W.make("bicg_q", N, N, seed=seed + 2, lws1d=256, out_init="zero")
+    P3.bufs[0] = P2.bufs[0]          # BICG: both kernels read the same A
+    return [P1, P2, P3]
+
+
+# ---------------------------------------------------------------------------------- clocks
+class ClockSampler:
+    def __init__(self, index: int):
+        self.index, self.proc, self.lines = index, None, []
+
+    def __enter__(self):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                          "-i", str(self.index), "-lms", "20"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self) -> dict:
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            p = [x.strip() for x in l.split(",")]
+            if len(p) < 9:
+                continue
+            try:
+                sm.append(float(p[1])); mx = float(p[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, p[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def measured_peaks() -> dict:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "source": "measured"}
+    return {"hbm_gbs": 6650.0, "source": "fallback (B200_PROFILING.md)"}
+
+
+def ncu_traffic(kernel: str):
+    """DRAM bytes per launch of `kernel` from the committed ncu capture, or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f).get(kernel)
+    return None
+
+
+# ---------------------------------------------------------------------------------- oracle legs
+def oracle_step_seconds(Ps, reps: int = 1) -> float:
+    import oracle  # test infrastructure: only the cpu_baseline / --impl reference legs use it
+    Ls = []
+    for P in Ps:
+        bufs = [b.astype(np.float64) for b in P.bufs]
+        Ls.append(oracle.Launch(P.kernel, P.integer, P.n0, P.n1, list(P.gws), list(P.lws), bufs,
+                                alpha=P.alpha, beta=P.beta))
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        for L in Ls:
+            oracle.run_range(L, 0, L.num_groups())
+    return (time.perf_counter() - t0) / reps
+
+
+def run_reference(args, rank: int, world: int):
+    if rank != 0:
+        return
+    Ps = problems(0)
+    step_bytes = sum(algorithmic_bytes(N).values())
+    for _ in range(args.warmup):
+        oracle_step_seconds(Ps)
+    times = [oracle_step_seconds(Ps) for _ in range(args.steps)]
+    t = sum(times) / len(times)
+    v = step_bytes / t / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": "gesummv_bicg4096", "n": N, "kernels": ["gesummv", "bicg_s", "bicg_q"]},
+            "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": "full step: serial C oracle (fp64) of GESUMMV + BICG s/q at N=4096"},
+            "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------------- product leg
+def run_fcl(args, rank: int, world: int, local_rank: int):
+    import torch
+    import fcl_harness as H
+    from paper_conf_cgo_panditg14_b200 import _build, fcl
+
+    if rank == 0:
+        _build.build()
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    stream = torch.cuda.Stream(device=dev)
+    cores = len(os.sched_getaffinity(0))
+    per_rank = max(2, cores // max(1, int(os.environ.get("LOCAL_WORLD_SIZE", world))))
+    host_threads = max(1, per_rank - 1)
+    ctx = fcl.Context(local_rank, n_host_threads=host_threads, streams=(stream.cuda_stream, None, None))
+
+    Ps = problems(1000 * rank)
+    step_bytes = sum(algorithmic_bytes(N).values())
+    # buffers: BICG's A shared by both kernels
+    bufs = [H.create_buffers(ctx, Ps[0])]
+    b2 = H.create_buffers(ctx, Ps[1])
+    b3 = H.create_buffers(ctx, Ps[2])
+    b3[0].release()
+    b3[0] = b2[0]
+    bufs += [b2, b3]
+    prepared = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m)
+                    for P, b in zip(Ps, bufs)] for m in ("coop", "gpu", "cpu")}
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def step(mode: str, infos: list = None):
+        for launch in prepared[mode]:
+            launch()
+            if infos is not None:
+                ctx.finish()
+                infos.append(ctx.launch_info())
+        ctx.finish()
+
+    def timed(mode: str, k: int, collect=False):
+        ts, infos = [], []
+        for _ in range(k):
+            with torch.cuda.stream(stream):
+                flush.fill_(1.0)          # L2 flush (outside the timed interval)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            step(mode, infos if collect else None)
+            e1.record(stream)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        return ts, infos
+
+    def max_over_ranks(x: float) -> float:
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # warm-up (all modes), then the timed COOP steps
+    for m in ("gpu", "cpu", "coop"):
+        for _ in range(max(1, args.warmup)):
+            step(m)
+    if dist is not None:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local_rank) as clk:
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t_wall0 = time.perf_counter()
+        coop_ts, _ = timed("coop", args.steps)
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter() - t_wall0
+        if dist is not None:
+            dist.barrier()
+        # the timed region can be shorter than nvidia-smi's sampling period: keep the same
+        # workload running (untimed) until the sampler has seen the clocks under this load
+        t_s = time.perf_counter()
+        while len(clk.lines) < 5 and time.perf_counter() - t_s < 3.0:
+            step("coop")
+    coop_ms = max_over_ranks(sum(coop_ts) / len(coop_ts))
+
+    # per-launch detail (dispatcher CUDA-event time, merges, host share) from separate steps
+    _, infos = timed("coop", max(2, min(args.steps, 5)), collect=True)
+    gpu_ts, _ = timed("gpu", max(3, min(args.steps, 10)))
+    cpu_ts, _ = timed("cpu", max(2, min(args.steps, 5)))
+    gpu_ms = max_over_ranks(statistics.mean(gpu_ts))
+    cpu_ms = max_over_ranks(statistics.mean(cpu_ts))
+    ideal_ms = 1.0 / (1.0 / gpu_ms + 1.0 / cpu_ms)
+
+    # dominant kernel: the GESUMMV dispatcher (2 N^2 floats); CUDA-event duration on main
+    ges = [i for i in infos if i["n_wg"] == Ps[0].num_groups and i["gpu_launches"] >= 1][::3] or infos[::3]
+    k_ms = statistics.mean(i["t_gpu_kernel_ms"] for i in ges if i["t_gpu_kernel_ms"] > 0)
+    peaks = measured_peaks()
+    achieved = algorithmic_bytes(N)["gesummv"] / (k_ms * 1e-3) / 1e9
+    launches_per_step = statistics.mean(
+        sum(i["gpu_launches"] for i in infos[j:j + 3]) for j in range(0, len(infos) - 2, 3))
+
+    # merge microbench: 1 GiB per stream, 10% of words changed (suffix), L2 flushed
+    merge = None
+    if rank == 0:
+        nw = (1 << 30) // 4
+        g = torch.randint(0, 2**31 - 1, (nw,), dtype=torch.int32, device=dev)
+        t = torch.randint(0, 2**31 - 1, (nw,), dtype=torch.int32, device=dev)
+        c = t.clone()
+        c[-nw // 10:] ^= 1
+        mts = []
+        for r in range(8):
+            with torch.cuda.stream(stream):
+                flush.fill_(2.0)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            fcl.merge_raw(g.data_ptr(), c.data_ptr(), t.data_ptr(), nw * 4, 4, stream.cuda_stream)
+            e1.record(stream)
+            e1.synchronize()
+            if r >= 2:
+                mts.append(e0.elapsed_time(e1))
+        mms = statistics.median(mts)
+        alg = nw * 8 + (nw // 10) * 4
+        merge = {"bytes_per_stream": nw * 4, "changed_frac": 0.1, "ms": round(mms, 4),
+                 "gbs": round(alg / (mms * 1e-3) / 1e9, 1),
+                 "frac": round(alg / (mms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4),
+                 "traffic": ncu_traffic("merge_kernel")}
+        del g, t, c
+
+    # e2e: the same step with every input copied host->device inside the timed region
+    in_bufs = [bufs[0][0], bufs[0][1], bufs[0][2], bufs[1][0], bufs[1][1], bufs[2][1]]
+    out_bufs = [bufs[0][3], bufs[0][4], bufs[1][2], bufs[2][2]]
+    h2d = sum(b.nbytes for b in in_bufs)
+    d2h = sum(b.nbytes for b in out_bufs)
+    outs = [np.empty(b.nbytes // 4, np.float32) for b in out_bufs]
+    e2e_ts = []
+    for r in range(args.warmup + args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(3.0)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for b in in_bufs:
+            b.write(b.host_ptr, blocking=False)     # pinned mirror -> device
+        step("coop")
+        for b, o in zip(out_bufs, outs):
+            b.read(o.ctypes.data)
+        e1.record(stream)
+        e1.synchronize()
+        if r >= args.warmup:
+            e2e_ts.append(e0.elapsed_time(e1))
+    e2e_ms = max_over_ranks(statistics.mean(e2e_ts))
+
+    # oracle on the host cores (rank 0, N=1 only): one bounded full step
+    cpu_baseline = None
+    if rank == 0 and world == 1:
+        t_or = oracle_step_seconds(problems(0))
+        cpu_baseline = {"value": round(step_bytes / t_or / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                        "sample": f"one full step (GESUMMV + BICG s/q, N={N}) in the serial fp64 C oracle: "
+                                  f"{t_or * 1e3:.0f} ms"}
+
+    if rank == 0:
+        value = step_bytes * world / (coop_ms * 1e-3) / 1e9
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(coop_ms, 4), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "gesummv_bicg4096", "n": N, "kernels": ["gesummv", "bicg_s", "bicg_q"],
+                       "mode": "coop", "lws": 256, "work_groups_per_kernel": 16, "host_threads": host_threads,
+                       "l2": "flushed between steps (256 MiB write)", "parallelism": f"replicas{world}"},
+            "coop_ms": round(coop_ms, 4), "gpu_only_ms": round(gpu_ms, 4), "cpu_only_ms": round(cpu_ms, 4),
+            "ideal_coop_ms": round(ideal_ms, 4), "frac_of_ideal": round(ideal_ms / coop_ms, 4),
+            "coop_vs_best_single": round(min(gpu_ms, cpu_ms) / coop_ms, 4),
+            "wall_ms_per_step": round(t_wall * 1e3 / args.steps, 4),
+            "roofline": {"kernel": "coop_kernel<RowDotBody<float,2>> (GESUMMV dispatcher)", "bound": "hbm",
+                         "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                         "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": ncu_traffic("gesummv"),
+                         "algorithmic_bytes": algorithmic_bytes(N)["gesummv"], "kernel_ms": round(k_ms, 4),
+                         "peak_source": peaks["source"]},
+            "merge": merge,
+            "cpu_baseline": cpu_baseline,
+            "e2e": {"value": round(step_bytes * world / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GB/s",
+                    "ms_per_step": round(e2e_ms, 4), "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+            "gpu_launches": int(round(launches_per_step * args.steps)),
+            "clocks": clk.summary(),
+            "host_cores": cores,
+        }
+        print(json.dumps(line), flush=True)
+    ctx.release()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="fcl", choices=["fcl", "reference"])
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    run_fcl(args, rank, world, local_rank)
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -57,14 +57,17 @@ def run(ctx: fcl.Context, P: W.Problem, mode: str = "coop", bufs: Optional[List[
     return outs, info
 
 
+class _CudaView:
+    def __init__(self, ptr: int, n: int, typestr: str):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
 def device_array(buf: fcl.Buffer, dtype) -> np.ndarray:
     """Copy a buffer's DEVICE copy to a numpy array (bypassing the host mirror), via torch."""
     import torch
-    n = buf.nbytes // np.dtype(dtype).itemsize
-    t = torch.empty(n, dtype=torch.int32 if np.dtype(dtype) == np.int32 else torch.float32, device="cuda")
+    dt = np.dtype(dtype)
+    n = buf.nbytes // dt.itemsize
     torch.cuda.synchronize()
-    import ctypes
-    cudart = torch.cuda.cudart()
-    res = cudart.cudaMemcpy(t.data_ptr(), buf.device_ptr, buf.nbytes, 3)  # device-to-device
-    torch.cuda.synchronize()
-    return t.cpu().numpy().view(dtype)
+    t = torch.as_tensor(_CudaView(buf.device_ptr, n, dt.str), device="cuda")
+    return t.clone().cpu().numpy().view(dtype)

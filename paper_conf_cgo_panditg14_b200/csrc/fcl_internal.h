@@ -57,8 +57,23 @@ struct CoopCtl {
     unsigned int *wmin;                 // lowest watermark acted on (0xFFFFFFFF on entry)
     unsigned long long *tasks;          // tasks executed (0 on entry)
     unsigned long long *exit_rec;       // device-visible address of the mapped host exit record
+    unsigned long long *wm_out;         // device word: {epoch | lowest watermark acted on}
     long long task_lo, task_hi;         // task index range of this launch
     int abort_period;                   // in-task poll period (body-specific units); 0 = none
+    int check_first;                    // 1: check the watermark before a CTA's first task too
+};
+
+// Device-side merge of a cooperative launch's output buffers (domain read from wm_word).
+struct DevMergeList {
+    unsigned char *gpu[6];
+    const unsigned char *cpu[6];
+    const unsigned char *twin[6];
+    long long unit_wgs[6], unit_bytes[6], total[6];   // span descriptor (unit_wgs 0 = whole buffer)
+    int es[6];
+    int n;
+    const unsigned long long *wm_word;
+    unsigned int epoch;
+    long long hi;
 };
 
 // ---- GPU side (kernels.cu) ----
@@ -80,6 +95,10 @@ int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t tas
 // Fig 9 diff-merge on [0, bytes) of three device buffers.
 int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes, int elem_size,
                      int num_sms, void *stream);
+int gpu_launch_merge_dev(const DevMergeList &L, size_t max_bytes, int num_sms, void *stream);
+// Copy up to 6 (dst, src, bytes) device regions in one launch (16-byte aligned pointers).
+int gpu_launch_copies(int n, void *const *dst, const void *const *src, const size_t *bytes, int num_sms,
+                      void *stream);
 // One-thread kernel that stores `value` to `addr` (status publication fallback).
 int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream);
 const char *gpu_last_error_string();
@@ -95,5 +114,9 @@ void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
 // work-groups [lo, hi) (superset of the exact footprint; the diff-merge tolerates it).
 void out_span(const KArgs &a, const Geom &g, int buf_index, int64_t lo, int64_t hi,
               size_t *b0, size_t *b1);
+// The same spans in closed form: span_lo(W) = min(floor(W / unit_wgs) * unit_bytes, total),
+// span_hi(W) = min(ceil(W / unit_wgs) * unit_bytes, total); unit_wgs == 0: the whole buffer.
+void out_span_desc(const KArgs &a, const Geom &g, int buf_index, long long *unit_wgs,
+                   long long *unit_bytes, long long *total);
 
 }  // namespace fcl

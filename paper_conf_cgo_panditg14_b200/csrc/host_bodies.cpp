@@ -369,4 +369,23 @@ void out_span(const KArgs &a, const Geom &g, int k, int64_t lo, int64_t hi, size
     (void)k;
 }
 
+void out_span_desc(const KArgs &a, const Geom &g, int k, long long *unit_wgs, long long *unit_bytes,
+                   long long *total) {
+    (void)k;
+    const long long es = 4;
+    switch (a.kernel) {
+    case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV:
+        *unit_wgs = 1; *unit_bytes = g.lws[0] * es; *total = a.n0 * es; break;
+    case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD:
+        *unit_wgs = 1; *unit_bytes = g.lws[0] * es; *total = a.n1 * es; break;
+    case K_SYRK: case K_SYR2K:
+        *unit_wgs = g.ng[0]; *unit_bytes = g.lws[1] * a.n0 * es; *total = a.n0 * a.n0 * es; break;
+    case K_CORR_REDUCE: case K_CONV2D:
+        *unit_wgs = g.ng[0]; *unit_bytes = g.lws[1] * a.n1 * es; *total = a.n0 * a.n1 * es; break;
+    case K_CORR_CORR:
+    default:
+        *unit_wgs = 0; *unit_bytes = 0; *total = a.n1 * a.n1 * es; break;
+    }
+}
+
 }  // namespace fcl

@@ -104,21 +104,30 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
     __shared__ int s_flag;
     __shared__ __align__(16) typename Body::Smem smem;
 
-    long long t_next = 0;
-    unsigned long long st_next = 0;
-    unsigned long long executed = 0;
-    if (threadIdx.x == 0) {
-        t_next = c.task_lo + (long long)atomicAdd(c.claim, 1ull);
-        st_next = ld_status(c.status);
-    }
-    for (;;) {
-        if (threadIdx.x == 0) { s_task = t_next; s_w = decode_w(st_next, c); }
+    // The first task of every CTA is blockIdx.x: no claim and no status wait before it starts.
+    // Running a work-group the host already covers is never wrong (the merge keeps the host's
+    // words), and long tasks still poll the status inside their loops; the status load issued
+    // here is consumed at that first poll.  Later tasks are claimed from the device counter
+    // and checked against the watermark (Fig 8) with the load prefetched during the previous
+    // task, so neither the claim nor the check is on the critical path.
+    long long t = c.task_lo + (long long)blockIdx.x;
+    unsigned int w = c.w_default;
+    bool checked = false;
+    if (c.check_first) {   // deterministic mode (forced split): check before the first task too
+        if (threadIdx.x == 0) s_w = decode_w(ld_status(c.status), c);
         __syncthreads();
-        const long long t = s_task;
-        const unsigned int w = s_w;
+        w = s_w;
+        checked = true;
+        __syncthreads();
+    }
+    long long t_next = 0;
+    unsigned long long st_next = 0, st_first = 0;
+    unsigned long long executed = 0;
+    if (threadIdx.x == 0) st_first = ld_status(c.status);
+    for (;;) {
         if (t >= c.task_hi) break;
         const long long key = Body::key(bp, t);
-        if ((unsigned long long)key >= (unsigned long long)w) {   // covered by the host (Fig 8)
+        if (checked && (unsigned long long)key >= (unsigned long long)w) {   // covered by the host
             if (threadIdx.x == 0) atomicMin(c.wmin, w);
             break;
         }
@@ -126,9 +135,9 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
         tc.c = &c; tc.key = key; tc.s_flag = &s_flag; tc.abort_w = 0; tc.pending = 0;
         if (threadIdx.x == 0) {
             // claim the next task and prefetch the status while this one runs
-            t_next = c.task_lo + (long long)atomicAdd(c.claim, 1ull);
+            t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
             st_next = ld_status(c.status);
-            tc.pending = st_next;
+            tc.pending = checked ? st_next : st_first;
         }
         const bool aborted = Body::run(bp, t, tc, smem);
         if (aborted) {
@@ -136,6 +145,11 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
             break;
         }
         ++executed;
+        if (threadIdx.x == 0) { s_task = t_next; s_w = decode_w(st_next, c); }
+        __syncthreads();
+        t = s_task;
+        w = s_w;
+        checked = true;
         __syncthreads();
     }
     // Exit protocol: the last CTA out publishes the exit record to mapped host memory and
@@ -150,9 +164,10 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
             const unsigned long long nt = atomicExch(c.tasks, 0ull);
             atomicExch(c.claim, 0ull);
             atomicExch(c.done, 0u);
-            __threadfence_system();
+            // device copy of the watermark the GPU acted on, read by the merge kernel queued
+            // behind this launch (the merge domain is decided on the device, no host round trip)
+            atomicExch(c.wm_out, ((unsigned long long)c.epoch << 32) | wm);
             asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(c.exit_rec + 1), "l"(nt) : "memory");
-            __threadfence_system();
             const unsigned long long rec = ((unsigned long long)c.epoch << 32) | wm;
             asm volatile("st.release.sys.global.b64 [%0], %1;" ::"l"(c.exit_rec), "l"(rec) : "memory");
         }
@@ -167,6 +182,22 @@ plain_kernel(const typename Body::Params bp, long long task_lo) {
     TaskCtx tc;
     tc.c = nullptr; tc.key = 0; tc.pending = 0; tc.s_flag = &s_flag; tc.abort_w = 0;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
+}
+
+// Twin capture (C5, L16.s2-3): copy every OUT/INOUT buffer to its twin in ONE launch.
+struct CopyList { uint8_t *dst[6]; const uint8_t *src[6]; size_t bytes[6]; int n; };
+
+__global__ void __launch_bounds__(256) copies_kernel(const CopyList L) {
+    const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const size_t nth = (size_t)gridDim.x * blockDim.x;
+    for (int b = 0; b < L.n; ++b) {
+        const size_t nv = L.bytes[b] / 16;
+        const uint4 *s = reinterpret_cast<const uint4 *>(L.src[b]);
+        uint4 *d = reinterpret_cast<uint4 *>(L.dst[b]);
+        for (size_t v = tid; v < nv; v += nth) d[v] = __ldcs(s + v);
+        const size_t tail = L.bytes[b] - 16 * nv;
+        if (tid < tail) L.dst[b][16 * nv + tid] = L.src[b][16 * nv + tid];
+    }
 }
 
 __global__ void store64_kernel(unsigned long long *addr, unsigned long long v) {
@@ -685,15 +716,20 @@ __device__ __forceinline__ uint4 ld_nc_v4(const uint8_t *p) {
     return v;
 }
 
+// Merge [0, nbytes) of one buffer with all threads of the grid (head/tail bytes scalar).
 template <int ES>
-__global__ void __launch_bounds__(256)
-merge_kernel(uint8_t *__restrict__ gpu, const uint8_t *__restrict__ cpu, const uint8_t *__restrict__ twin,
-             size_t head, size_t nvec, size_t tail) {
-    // bytes: [0, head) scalar, [head, head + 16*nvec) vector, then `tail` scalar bytes
-    const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const size_t nthreads = (size_t)gridDim.x * blockDim.x;
+__device__ __forceinline__ void merge_range(uint8_t *gpu, const uint8_t *cpu, const uint8_t *twin, size_t nbytes,
+                                            size_t tid, size_t nthreads) {
+    size_t head = 0, nvec = 0, tail = nbytes;
+    const uintptr_t ag = reinterpret_cast<uintptr_t>(gpu) & 15u;
+    if (ag == (reinterpret_cast<uintptr_t>(cpu) & 15u) && ag == (reinterpret_cast<uintptr_t>(twin) & 15u)) {
+        head = ag ? 16 - ag : 0;
+        if (head > nbytes) head = nbytes;
+        nvec = (nbytes - head) / 16;
+        tail = nbytes - head - 16 * nvec;
+    }
     if (tid == 0 && head) merge_scalar<ES>(gpu, cpu, twin, head);
-    if (tid == 1 % nthreads && tail) {
+    if (tid == (nthreads > 1 ? 1 : 0) && tail) {
         const size_t off = head + 16 * nvec;
         merge_scalar<ES>(gpu + off, cpu + off, twin + off, tail);
     }
@@ -715,6 +751,45 @@ merge_kernel(uint8_t *__restrict__ gpu, const uint8_t *__restrict__ cpu, const u
     for (; v < nvec; v += nthreads) {
         const uint4 cv = ld_nc_v4(c + 16 * v), tv = ld_nc_v4(t + 16 * v);
         if ((cv.x != tv.x) | (cv.y != tv.y) | (cv.z != tv.z) | (cv.w != tv.w)) merge_vec<ES>(g + 16 * v, cv, tv);
+    }
+}
+
+template <int ES>
+__global__ void __launch_bounds__(256)
+merge_kernel(uint8_t *__restrict__ gpu, const uint8_t *__restrict__ cpu, const uint8_t *__restrict__ twin,
+             size_t nbytes) {
+    merge_range<ES>(gpu, cpu, twin, nbytes, (size_t)blockIdx.x * blockDim.x + threadIdx.x,
+                    (size_t)gridDim.x * blockDim.x);
+}
+
+// Merge of every OUT/INOUT buffer of a cooperative launch, queued behind the dispatcher.
+// The domain [span_lo(wm), span_hi(hi)) of each buffer comes from the watermark the
+// dispatcher acted on (it skipped only work-groups >= wm, whose host results were staged
+// before the watermark was published, L16.s15); nothing is merged if it never skipped.
+__global__ void __launch_bounds__(256) merge_dev_kernel(const DevMergeList L) {
+    __shared__ unsigned long long s_wm;
+    if (threadIdx.x == 0) s_wm = ld_status(L.wm_word);
+    __syncthreads();
+    const unsigned long long r = s_wm;
+    if ((unsigned int)(r >> 32) != L.epoch) return;
+    const long long wm = (long long)(unsigned int)r;
+    if ((unsigned int)r == 0xFFFFFFFFu || wm >= L.hi) return;
+    const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
+    for (int b = 0; b < L.n; ++b) {
+        long long b0 = 0, b1 = L.total[b];
+        if (L.unit_wgs[b] > 0) {
+            b0 = (wm / L.unit_wgs[b]) * L.unit_bytes[b];
+            b1 = ((L.hi + L.unit_wgs[b] - 1) / L.unit_wgs[b]) * L.unit_bytes[b];
+            if (b0 > L.total[b]) b0 = L.total[b];
+            if (b1 > L.total[b]) b1 = L.total[b];
+        }
+        if (b1 <= b0) continue;
+        switch (L.es[b]) {
+        case 1: merge_range<1>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        case 2: merge_range<2>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        case 4: merge_range<4>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        default: merge_range<8>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        }
     }
 }
 
@@ -1008,30 +1083,51 @@ int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes,
     if (bytes == 0) return 0;
     uint8_t *g = (uint8_t *)gpu;
     const uint8_t *c = (const uint8_t *)cpu, *t = (const uint8_t *)twin;
-    size_t head = 0, nvec = 0, tail = bytes;
-    const uintptr_t ag = reinterpret_cast<uintptr_t>(g) & 15u;
-    if (ag == (reinterpret_cast<uintptr_t>(c) & 15u) && ag == (reinterpret_cast<uintptr_t>(t) & 15u)) {
-        head = ag ? 16 - ag : 0;
-        if (head > bytes) head = bytes;
-        // head must hold whole elements: alignment of the buffers is a multiple of elem_size
-        nvec = (bytes - head) / 16;
-        tail = bytes - head - 16 * nvec;
-    }
-    size_t threads_needed = (nvec + 3) / 4;
-    long long grid = (long long)((threads_needed + 255) / 256);
+    long long grid = (long long)((bytes / 64 + 255) / 256);
     const long long cap = (long long)num_sms * 8;
     if (grid > cap) grid = cap;
     if (grid < 1) grid = 1;
     cudaStream_t s = (cudaStream_t)stream;
     switch (elem_size) {
-    case 1: merge_kernel<1><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
-    case 2: merge_kernel<2><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
-    case 4: merge_kernel<4><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
-    case 8: merge_kernel<8><<<(unsigned)grid, 256, 0, s>>>(g, c, t, head, nvec, tail); break;
+    case 1: merge_kernel<1><<<(unsigned)grid, 256, 0, s>>>(g, c, t, bytes); break;
+    case 2: merge_kernel<2><<<(unsigned)grid, 256, 0, s>>>(g, c, t, bytes); break;
+    case 4: merge_kernel<4><<<(unsigned)grid, 256, 0, s>>>(g, c, t, bytes); break;
+    case 8: merge_kernel<8><<<(unsigned)grid, 256, 0, s>>>(g, c, t, bytes); break;
     default: return -1;
     }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return seterr(e, "merge_kernel launch");
+    return 1;
+}
+
+int gpu_launch_merge_dev(const DevMergeList &L, size_t max_bytes, int num_sms, void *stream) {
+    long long grid = (long long)((max_bytes / 64 + 255) / 256);
+    const long long cap = (long long)num_sms * 8;
+    if (grid > cap) grid = cap;
+    if (grid < 1) grid = 1;
+    merge_dev_kernel<<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(L);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return seterr(e, "merge_dev_kernel launch");
+    return 1;
+}
+
+int gpu_launch_copies(int n, void *const *dst, const void *const *src, const size_t *bytes, int num_sms,
+                      void *stream) {
+    CopyList L;
+    size_t total = 0;
+    L.n = n;
+    for (int b = 0; b < n && b < 6; ++b) {
+        if ((reinterpret_cast<uintptr_t>(dst[b]) | reinterpret_cast<uintptr_t>(src[b])) & 15u) return -1;
+        L.dst[b] = (uint8_t *)dst[b]; L.src[b] = (const uint8_t *)src[b]; L.bytes[b] = bytes[b];
+        total += bytes[b];
+    }
+    if (total == 0) return 0;
+    long long grid = (long long)((total / 16 + 255) / 256);
+    if (grid > (long long)num_sms * 8) grid = (long long)num_sms * 8;
+    if (grid < 1) grid = 1;
+    copies_kernel<<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(L);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return seterr(e, "copies_kernel launch");
     return 1;
 }
 

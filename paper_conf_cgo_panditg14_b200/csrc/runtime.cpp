@@ -272,7 +272,7 @@ struct fcl_context_st {
     int num_sms = 148;
     cudaStream_t main = nullptr, hd = nullptr, dh = nullptr;
     bool own_main = false, own_hd = false, own_dh = false;
-    int status_location = FCL_STATUS_HOST_MAPPED;
+    int status_location = FCL_STATUS_DEVICE;
     // One 64-bit status word per launch slot (epoch % kSlots): a dispatcher that is still
     // running after its host side returned never sees a later launch's watermark.
     static constexpr int kSlots = 16;
@@ -281,7 +281,7 @@ struct fcl_context_st {
     uint32_t slot_epoch[kSlots] = {0};           // epoch of the dispatcher that last used a slot
     unsigned long long *exit_host = nullptr;     // mapped exit record [2]
     unsigned long long *exit_dptr = nullptr;
-    unsigned long long *dclaim = nullptr, *dtasks = nullptr;
+    unsigned long long *dclaim = nullptr, *dtasks = nullptr, *dwm = nullptr;
     unsigned int *ddone = nullptr, *dwmin = nullptr;
     uint32_t epoch = 0;
     PFN_writeValue64 write64 = nullptr;
@@ -295,6 +295,7 @@ struct fcl_context_st {
     bool have_k = false, have_m = false;
     fcl_launch_info info{};
     std::vector<fcl_buffer> defer_list;
+    size_t eager_return_bytes = 8u << 20;   // outputs up to this size return right behind the merge
 };
 
 namespace {
@@ -441,6 +442,7 @@ struct Launch {
     fcl_buffer bufs[6];
     int out_idx[6];
     int nout;
+    bool any_inout;   // some output is read-modify-write (INOUT)
     int64_t lo, hi;
     fcl_launch_opts o;
 };
@@ -560,12 +562,22 @@ fcl_status run_coop(Launch &L) {
 
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
     void *twin[6] = {nullptr}, *stage[6] = {nullptr};
+    const void *srcs[6];
+    size_t nbytes[6];
     for (int q = 0; q < L.nout; ++q) {
         fcl_buffer b = L.bufs[L.out_idx[q]];
         twin[q] = pool_get(ctx, b->bytes);
         stage[q] = pool_get(ctx, b->bytes);
         if (!twin[q] || !stage[q]) return set_err(ctx, FCL_OUT_OF_RESOURCES, "twin/stage allocation of %zu bytes failed", b->bytes);
-        CK(ctx, cudaMemcpyAsync(twin[q], b->dev, b->bytes, cudaMemcpyDeviceToDevice, ctx->main));
+        srcs[q] = b->dev;
+        nbytes[q] = b->bytes;
+    }
+    if (gpu_launch_copies(L.nout, twin, srcs, nbytes, ctx->num_sms, ctx->main) < 0) {
+        // unaligned caller memory: fall back to per-buffer copies
+        for (int q = 0; q < L.nout; ++q)
+            CK(ctx, cudaMemcpyAsync(twin[q], srcs[q], nbytes[q], cudaMemcpyDeviceToDevice, ctx->main));
+    } else {
+        info.gpu_launches += 1;
     }
     auto release = [&]() {
         for (int q = 0; q < L.nout; ++q) {
@@ -589,6 +601,8 @@ fcl_status run_coop(Launch &L) {
     c.w_default = (unsigned int)L.hi;
     c.claim = ctx->dclaim; c.done = ctx->ddone; c.wmin = ctx->dwmin; c.tasks = ctx->dtasks;
     c.exit_rec = ctx->exit_dptr;
+    c.wm_out = ctx->dwm;
+    c.check_first = forced ? 1 : 0;
     c.task_lo = t0; c.task_hi = t1;
     c.abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
     bool gpu_launched = false;
@@ -603,6 +617,50 @@ fcl_status run_coop(Launch &L) {
         info.gpu_launches += 1;
         gpu_launched = true;
         ctx->slot_epoch[ctx->epoch % fcl_context_st::kSlots] = ctx->epoch;
+    }
+    // Free-running mode: the merge is queued right behind the dispatcher and decides its
+    // domain on the device from the watermark the dispatcher acted on, and small outputs are
+    // returned eagerly behind it -- no host round trip between the GPU finishing and the
+    // result being coherent.
+    const bool dev_merge = gpu_launched && !forced && !L.o.defer_merge;
+    size_t out_total = 0;
+    for (int q = 0; q < L.nout; ++q) {
+        size_t b0, b1;
+        out_span(L.a, L.g, L.out_idx[q], L.lo, L.hi, &b0, &b1);
+        out_total += b1 - b0;
+    }
+    // An INOUT buffer is read-modify-written in place by the host bodies: its return copy
+    // must wait until the host workers have stopped (an abandoned chunk may still be running
+    // when the GPU finishes), so only pure-OUT launches return eagerly.
+    const bool eager = dev_merge && !L.any_inout && out_total <= ctx->eager_return_bytes;
+    if (dev_merge) {
+        DevMergeList M{};
+        M.n = L.nout;
+        size_t maxb = 0;
+        for (int q = 0; q < L.nout; ++q) {
+            fcl_buffer b = L.bufs[L.out_idx[q]];
+            M.gpu[q] = (unsigned char *)b->dev;
+            M.cpu[q] = (const unsigned char *)stage[q];
+            M.twin[q] = (const unsigned char *)twin[q];
+            M.es[q] = (int)b->elem_size;
+            out_span_desc(L.a, L.g, L.out_idx[q], &M.unit_wgs[q], &M.unit_bytes[q], &M.total[q]);
+            maxb = std::max(maxb, (size_t)M.total[q]);
+        }
+        M.wm_word = ctx->dwm;
+        M.epoch = ctx->epoch;
+        M.hi = L.hi;
+        CK(ctx, cudaEventRecord(ctx->ev_m0, ctx->main));
+        if (gpu_launch_merge_dev(M, maxb, ctx->num_sms, ctx->main) < 0) {
+            release();
+            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        }
+        CK(ctx, cudaEventRecord(ctx->ev_m1, ctx->main));
+        ctx->have_m = true;
+        info.gpu_launches += 1;
+        if (eager) {
+            fcl_status st = enqueue_d2h(ctx, L, L.lo, L.hi, true);
+            if (st != FCL_SUCCESS) { release(); return st; }
+        }
     }
 
     // CPU: descending adaptive chunks (C9-C11), staged and published after each (C13)
@@ -696,7 +754,33 @@ fcl_status run_coop(Launch &L) {
     info.cpu_wgs = cpu_done_wgs;
     info.gpu_watermark = L.hi;
 
-    // Decide the merge domain and the device->host return (C15/C17)
+    if (dev_merge) {
+        // merge already queued; only the precise return of large outputs is left to decide
+        fcl_status st = FCL_SUCCESS;
+        if (gpu_done) {
+            const int64_t wm = (wmin == 0xFFFFFFFFu) ? L.hi : (int64_t)wmin;
+            info.gpu_watermark = wm;
+            info.gpu_tasks = (int64_t)gtasks;
+            info.merged = wm < L.hi;
+            if (wm <= L.lo) info.cpu_did_all = 1;
+            if (!eager) st = enqueue_d2h(ctx, L, L.lo, wm, true);
+        } else {
+            info.cpu_did_all = 1;       // host authoritative (L16.s21); device merged behind
+            info.gpu_watermark = L.lo;  // refined from the exit record in fcl_get_launch_info
+            info.merged = 1;
+        }
+        for (int q = 0; q < L.nout; ++q) {
+            size_t b0, b1;
+            out_span(L.a, L.g, L.out_idx[q], L.lo, L.hi, &b0, &b1);
+            if (info.merged) info.merge_bytes += (int64_t)(b1 - b0);
+        }
+        CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
+        release();
+        return st;
+    }
+
+    // Forced split / deferred merge: the host decides the merge domain and the return
+    // (C15/C17)
     int64_t merge_lo = L.hi, ret_hi = L.hi;
     size_t wait_ev = (size_t)-1;
     if (forced) {
@@ -855,6 +939,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->dtasks = ctx->dclaim + 1;
     ctx->ddone = (unsigned int *)(ctx->dclaim + 2);
     ctx->dwmin = ctx->ddone + 1;
+    ctx->dwm = ctx->dclaim + 3;
     const unsigned int ff = 0xFFFFFFFFu;
     if ((e = cudaMemcpy(ctx->dwmin, &ff, 4, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "counter init");
     for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1, &ctx->ev_m0, &ctx->ev_m1})
@@ -872,6 +957,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
             cudaGetLastError();
     }
     if (getenv("FCL_NO_MEMOPS")) ctx->write64 = nullptr;
+    if (getenv("FCL_EAGER_RETURN_BYTES")) ctx->eager_return_bytes = (size_t)atoll(getenv("FCL_EAGER_RETURN_BYTES"));
     if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail(e, "init sync");
     const char *pin = getenv("FCL_PIN_THREADS");
     const bool do_pin = d.pin_threads ? true : (pin ? atoi(pin) != 0 : true);
@@ -1089,6 +1175,7 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
     int nb = 0, ni = 0;
     int64_t ints[2] = {0, 0};
     L.nout = 0;
+    L.any_inout = false;
     for (int k = 0; k < kd->nargs; ++k) {
         const ArgSpec &sp = kd->args[k];
         const fcl_arg &ar = args[k];
@@ -1103,6 +1190,7 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
             a.dev[nb] = ar.buffer->dev;
             a.host[nb] = ar.buffer->host;
             if (sp.acc & 2) L.out_idx[L.nout++] = nb;
+            if (sp.acc == 3) L.any_inout = true;
             ++nb;
         } else if (sp.kind == 'i') {
             if (ar.kind != FCL_ARG_INT) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %d (%s) must be an int", k, sp.name);

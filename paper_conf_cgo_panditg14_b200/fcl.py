@@ -24,7 +24,7 @@ MEM_USE_HOST_PTR, MEM_USE_DEVICE_PTR = 8, 16
 ARG_BUFFER, ARG_INT, ARG_FLOAT = 0, 1, 2
 ACCESS_IN, ACCESS_OUT, ACCESS_INOUT = 1, 2, 3
 MODE_COOP, MODE_GPU_ONLY, MODE_CPU_ONLY = 0, 1, 2
-STATUS_HOST_MAPPED, STATUS_DEVICE = 0, 1
+STATUS_DEVICE, STATUS_HOST_MAPPED = 0, 1
 MODES = {"coop": MODE_COOP, "gpu": MODE_GPU_ONLY, "gpu_only": MODE_GPU_ONLY,
          "cpu": MODE_CPU_ONLY, "cpu_only": MODE_CPU_ONLY}
 
@@ -225,11 +225,11 @@ def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg
 class Context:
     """A FluidiCL context on one CUDA device plus the host executor threads."""
 
-    def __init__(self, device: int = 0, n_host_threads: int = 0, status_location: str = "host_mapped",
+    def __init__(self, device: int = 0, n_host_threads: int = 0, status_location: str = "device",
                  streams: Optional[Sequence[int]] = None, pin_threads: bool = True):
         d = ContextDesc()
         d.device, d.n_host_threads, d.pin_threads = int(device), int(n_host_threads), int(pin_threads)
-        d.status_location = STATUS_DEVICE if status_location == "device" else STATUS_HOST_MAPPED
+        d.status_location = STATUS_HOST_MAPPED if status_location == "host_mapped" else STATUS_DEVICE
         if streams:
             d.main_stream, d.hd_stream, d.dh_stream = [int(s) if s else None for s in streams]
         h = ctypes.c_void_p()
@@ -295,6 +295,10 @@ class Context:
                f"fcl_enqueue_ndrange({k.name})", self.handle)
         return info.as_dict()
 
+    def prepare(self, kernel, gws: Sequence[int], lws: Sequence[int], args: Iterable, **kw) -> "PreparedLaunch":
+        """Marshal a launch once; calling the result enqueues it with one C call."""
+        return PreparedLaunch(self, kernel, gws, lws, args, **kw)
+
     def merge(self, buf: Buffer):
         _check(load().fcl_merge(self.handle, buf.handle), "fcl_merge", self.handle)
 
@@ -320,6 +324,40 @@ class Context:
         if self.handle:
             _check(load().fcl_release_context(self.handle), "fcl_release_context")
             self.handle = None
+
+
+class PreparedLaunch:
+    """A launch whose C structs are built once (argument marshalling off the critical path)."""
+
+    def __init__(self, ctx: Context, kernel, gws, lws, args, **kw):
+        k = ctx.kernel(kernel) if isinstance(kernel, str) else kernel
+        args = list(args)
+        if len(args) != len(k.params):
+            raise ValueError(f"{k.name} takes {k.signature}")
+        self.ctx, self.k = ctx, k
+        self.arr = (Arg * len(args))()
+        for n, (v, (pname, pkind)) in enumerate(zip(args, k.params)):
+            if isinstance(v, Buffer):
+                self.arr[n].kind, self.arr[n].buffer = ARG_BUFFER, v.handle
+                self.arr[n].access = {"in": ACCESS_IN, "out": ACCESS_OUT, "inout": ACCESS_INOUT}[pkind]
+            elif pkind == "i":
+                self.arr[n].kind, self.arr[n].i = ARG_INT, int(v)
+            else:
+                self.arr[n].kind, self.arr[n].f = ARG_FLOAT, float(v)
+        self.nargs = len(args)
+        self.wd = len(gws)
+        self.gws, self.lws = _sizes3(gws), _sizes3(lws)
+        self.opts = make_opts(**kw)
+        self.info = LaunchInfo()
+        self._fn = load().fcl_enqueue_ndrange
+        self._args = (ctx.handle, k.handle, self.wd, self.gws, self.lws, self.arr, self.nargs,
+                      ctypes.byref(self.opts), ctypes.byref(self.info))
+
+    def __call__(self):
+        st = self._fn(*self._args)
+        if st != SUCCESS:
+            _check(st, f"fcl_enqueue_ndrange({self.k.name})", self.ctx.handle)
+        return self.info
 
 
 def merge_raw(gpu_ptr: int, cpu_ptr: int, twin_ptr: int, nbytes: int, elem_size: int, stream: int = 0):
