@@ -176,7 +176,14 @@ typedef struct {
     int32_t drop_publish;    /* fault injection: stage chunks but never publish the watermark */
     int64_t wg_lo, wg_hi;    /* execute only flattened ids [wg_lo, wg_hi) (multi-GPU slice);
                                 wg_hi <= 0 means the whole NDRange */
+    int32_t blocking;        /* 1 = return only when the launch's host side is done (the paper's
+                                blocking calls, L22.s14); 0 (default) = OpenCL-style enqueue */
+    int32_t flags;           /* FCL_LAUNCH_* bits */
 } fcl_launch_opts;
+
+/* opts.flags: record CUDA events around the GPU kernel (info.t_gpu_kernel_ms); off by default
+ * because each event costs host time on the launch path. */
+#define FCL_LAUNCH_TIMING 1u
 
 /* Fill *opts with the defaults above. */
 fcl_status fcl_default_launch_opts(fcl_launch_opts *opts);
@@ -203,10 +210,14 @@ typedef struct {
 
 /* Launch `kernel` over the NDRange (work_dim in 1..3, gws[k] % lws[k] == 0,
  * prod(lws) <= 1024) with args in the kernel's signature order.
- * COOP: the GPU dispatcher and the host executor race over the range; on
- * return every output buffer is current on the host (or will be once the
- * queued device->host copy completes -- see fcl_finish) and, once the queued
- * device work completes, on the device.  opts / info may be NULL.
+ * COOP: the GPU dispatcher and the host executor race over the range.  The
+ * call queues the GPU work and hands the host side to the context's
+ * coordinator thread, then returns (like clEnqueueNDRangeKernel); a launch
+ * that writes a buffer a pending launch touches (or vice versa) first waits
+ * for the pending launches.  After fcl_finish every output buffer is coherent
+ * on host and device.  GPU_ONLY / CPU_ONLY wait for pending launches first.
+ * opts / info may be NULL; info receives what is known at return (complete
+ * with opts.blocking = 1, otherwise use fcl_get_launch_info after fcl_finish).
  * Errors: FCL_INVALID_WORK_DIMENSION, FCL_INVALID_WORK_GROUP_SIZE,
  * FCL_INVALID_GLOBAL_WORK_SIZE, FCL_INVALID_KERNEL_ARGS, FCL_INVALID_VALUE,
  * FCL_OUT_OF_RESOURCES, FCL_CONTEXT_LOST. */

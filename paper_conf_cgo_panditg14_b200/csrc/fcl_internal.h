@@ -47,22 +47,6 @@ struct KArgs {
     int32_t ialpha, ibeta;
 };
 
-// Parameters of one cooperative (FluidiCL) dispatcher launch.
-struct CoopCtl {
-    const unsigned long long *status;   // {epoch:32 | W:32}; device-visible address
-    unsigned int epoch;                 // this launch's kernel id (C14)
-    unsigned int w_default;             // watermark when the status is stale: the range end
-    unsigned long long *claim;          // device claim counter (0 on entry, reset by last CTA)
-    unsigned int *done;                 // CTA exit counter (0 on entry, reset by last CTA)
-    unsigned int *wmin;                 // lowest watermark acted on (0xFFFFFFFF on entry)
-    unsigned long long *tasks;          // tasks executed (0 on entry)
-    unsigned long long *exit_rec;       // device-visible address of the mapped host exit record
-    unsigned long long *wm_out;         // device word: {epoch | lowest watermark acted on}
-    long long task_lo, task_hi;         // task index range of this launch
-    int abort_period;                   // in-task poll period (body-specific units); 0 = none
-    int check_first;                    // 1: check the watermark before a CTA's first task too
-};
-
 // Device-side merge of a cooperative launch's output buffers (domain read from wm_word).
 struct DevMergeList {
     unsigned char *gpu[6];
@@ -74,7 +58,43 @@ struct DevMergeList {
     const unsigned long long *wm_word;
     unsigned int epoch;
     long long hi;
+    unsigned long long *tstamp;         // optional %globaltimer stamps [start, end] (stats mode)
+    unsigned long long *exit_word;      // mapped host word: set to `epoch` when this kernel starts
 };
+
+// Parameters of one cooperative (FluidiCL) dispatcher launch.
+struct CoopCtl {
+    const unsigned long long *status;   // {epoch:32 | W:32}; device-visible address
+    unsigned int epoch;                 // this launch's kernel id (C14)
+    unsigned int w_default;             // watermark when the status is stale: the range end
+    unsigned long long *claim;          // this launch's claim counter (0 on entry)
+    unsigned long long *claim_next;     // the next launch's claim counter (reset here)
+    unsigned long long *tasks;          // optional: tasks executed (0 on entry), nullptr = off
+    unsigned long long *tasks_next;     // optional: next launch's task counter (reset here)
+    unsigned long long *wm_out;         // {epoch | ~lowest watermark acted on}, atomicMax
+    long long task_lo, task_hi;         // task index range of this launch
+    int abort_period;                   // in-task poll period (body-specific units); 0 = none
+    int check_first;                    // 1: check the watermark before a CTA's first task too
+    unsigned long long *tstamp;         // optional %globaltimer stamps [start, end] (stats mode)
+    unsigned long long *tstamp_next;    // the next launch's stamps (its end stamp is reset here)
+    int fused;                          // 1: grid barrier + exit signal + merge in this kernel
+    unsigned int *barrier;              // this launch's grid-barrier counter (0 on entry)
+    unsigned int *barrier_next;         // the next launch's counter (reset here)
+    unsigned long long *exit_word;      // mapped host word set to `epoch` after the barrier
+    DevMergeList mg;                    // merge list (mg.n == 0: nothing to merge in-kernel)
+};
+
+// Decode the dispatcher's wm word: the lowest watermark launch `epoch` acted on, or
+// 0xFFFFFFFF if it never skipped a task.
+#ifdef __CUDACC__
+#define FCL_HD __host__ __device__
+#else
+#define FCL_HD
+#endif
+FCL_HD inline unsigned int decode_wm_word(unsigned long long r, unsigned int epoch) {
+    return ((unsigned int)(r >> 32) == epoch) ? 0xFFFFFFFFu - (unsigned int)r : 0xFFFFFFFFu;
+}
+
 
 // ---- GPU side (kernels.cu) ----
 struct TaskSpace {

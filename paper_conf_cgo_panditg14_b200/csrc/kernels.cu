@@ -20,6 +20,7 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 
 #include "fcl_internal.h"
 
@@ -64,6 +65,12 @@ __device__ __forceinline__ unsigned long long ld_status(const unsigned long long
     asm volatile("ld.relaxed.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
 __device__ __forceinline__ unsigned int decode_w(unsigned long long st, const CoopCtl &c) {
     // A status word from another kernel (stale epoch) means "nothing covered" (C14, L20.s9).
     return ((unsigned int)(st >> 32) == c.epoch) ? (unsigned int)st : c.w_default;
@@ -94,8 +101,176 @@ struct TaskCtx {
 };
 
 // ------------------------------------------------------------------------------------------
+// Diff-merge (Fig 9): gpu[e] = (cpu[e] != twin[e]) ? cpu[e] : gpu[e], bitwise, per element.
+// cpu/twin are streamed once with 128-bit no-L1-allocate loads (4 vectors in flight per
+// thread); changed elements are stored with predicated element stores (a fully changed vector
+// with one 128-bit store), so the GPU copy is never read: traffic = 8 B/word read + 4 B per
+// changed word written.  Byte/half-word element sizes blend within the 32-bit lane.
+// ------------------------------------------------------------------------------------------
+template <int ES>
+__device__ __forceinline__ void merge_vec(uint8_t *g, const uint4 c, const uint4 t) {
+    const uint32_t cw[4] = {c.x, c.y, c.z, c.w}, tw[4] = {t.x, t.y, t.z, t.w};
+    if (ES == 4) {
+        const bool ch0 = cw[0] != tw[0], ch1 = cw[1] != tw[1], ch2 = cw[2] != tw[2], ch3 = cw[3] != tw[3];
+        if (ch0 && ch1 && ch2 && ch3) { *reinterpret_cast<uint4 *>(g) = c; return; }
+        uint32_t *gw = reinterpret_cast<uint32_t *>(g);
+        if (ch0) gw[0] = cw[0];
+        if (ch1) gw[1] = cw[1];
+        if (ch2) gw[2] = cw[2];
+        if (ch3) gw[3] = cw[3];
+    } else if (ES == 8) {
+        const bool ch0 = (cw[0] != tw[0]) || (cw[1] != tw[1]);
+        const bool ch1 = (cw[2] != tw[2]) || (cw[3] != tw[3]);
+        if (ch0 && ch1) { *reinterpret_cast<uint4 *>(g) = c; return; }
+        unsigned long long *gd = reinterpret_cast<unsigned long long *>(g);
+        if (ch0) gd[0] = ((unsigned long long)cw[1] << 32) | cw[0];
+        if (ch1) gd[1] = ((unsigned long long)cw[3] << 32) | cw[2];
+    } else {
+        uint32_t m[4];
+        bool all = true, any = false;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            if (ES == 1) m[q] = __vcmpne4(cw[q], tw[q]);
+            else m[q] = __vcmpne2(cw[q], tw[q]);
+            all &= (m[q] == 0xFFFFFFFFu);
+            any |= (m[q] != 0u);
+        }
+        if (all) { *reinterpret_cast<uint4 *>(g) = c; return; }
+        if (!any) return;
+        uint32_t *gw = reinterpret_cast<uint32_t *>(g);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            if (m[q] == 0xFFFFFFFFu) gw[q] = cw[q];
+            else if (m[q]) gw[q] = (cw[q] & m[q]) | (gw[q] & ~m[q]);
+        }
+    }
+}
+
+template <int ES>
+__device__ __forceinline__ void merge_scalar(uint8_t *g, const uint8_t *c, const uint8_t *t, size_t nbytes) {
+    for (size_t e = 0; e + ES <= nbytes; e += ES) {
+        bool ch = false;
+#pragma unroll
+        for (int b = 0; b < ES; ++b) ch |= (c[e + b] != t[e + b]);
+        if (ch) {
+#pragma unroll
+            for (int b = 0; b < ES; ++b) g[e + b] = c[e + b];
+        }
+    }
+}
+
+// The twin stream may alias the destination (twin := device copy for exact spans), so it is
+// read through the coherent path.
+__device__ __forceinline__ uint4 ld_na_v4(const uint8_t *p) {
+    uint4 v;
+    asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ uint4 ld_nc_v4(const uint8_t *p) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+
+// Merge [0, nbytes) of one buffer with all threads of the grid (head/tail bytes scalar).
+template <int ES>
+__device__ __forceinline__ void merge_range(uint8_t *gpu, const uint8_t *cpu, const uint8_t *twin, size_t nbytes,
+                                            size_t tid, size_t nthreads) {
+    size_t head = 0, nvec = 0, tail = nbytes;
+    const uintptr_t ag = reinterpret_cast<uintptr_t>(gpu) & 15u;
+    if (ag == (reinterpret_cast<uintptr_t>(cpu) & 15u) && ag == (reinterpret_cast<uintptr_t>(twin) & 15u)) {
+        head = ag ? 16 - ag : 0;
+        if (head > nbytes) head = nbytes;
+        nvec = (nbytes - head) / 16;
+        tail = nbytes - head - 16 * nvec;
+    }
+    if (tid == 0 && head) merge_scalar<ES>(gpu, cpu, twin, head);
+    if (tid == (nthreads > 1 ? 1 : 0) && tail) {
+        const size_t off = head + 16 * nvec;
+        merge_scalar<ES>(gpu + off, cpu + off, twin + off, tail);
+    }
+    uint8_t *g = gpu + head;
+    const uint8_t *c = cpu + head, *t = twin + head;
+    constexpr int U = 4;
+    size_t v = tid;
+    for (; v + (U - 1) * nthreads < nvec; v += U * nthreads) {
+        uint4 cv[U], tv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) { cv[u] = ld_nc_v4(c + 16 * (v + u * nthreads)); tv[u] = ld_na_v4(t + 16 * (v + u * nthreads)); }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const bool diff = (cv[u].x != tv[u].x) | (cv[u].y != tv[u].y) | (cv[u].z != tv[u].z) | (cv[u].w != tv[u].w);
+            // warp vote: a warp whose 512-byte segment is unchanged skips the store path
+            if (__ballot_sync(__activemask(), diff) && diff) merge_vec<ES>(g + 16 * (v + u * nthreads), cv[u], tv[u]);
+        }
+    }
+    for (; v < nvec; v += nthreads) {
+        const uint4 cv = ld_nc_v4(c + 16 * v), tv = ld_na_v4(t + 16 * v);
+        if ((cv.x != tv.x) | (cv.y != tv.y) | (cv.z != tv.z) | (cv.w != tv.w)) merge_vec<ES>(g + 16 * v, cv, tv);
+    }
+}
+
+template <int ES>
+__global__ void __launch_bounds__(256)
+merge_kernel(uint8_t *gpu, const uint8_t *cpu, const uint8_t *twin, size_t nbytes) {
+    merge_range<ES>(gpu, cpu, twin, nbytes, (size_t)blockIdx.x * blockDim.x + threadIdx.x,
+                    (size_t)gridDim.x * blockDim.x);
+}
+
+// Merge of every OUT/INOUT buffer of a cooperative launch, queued behind the dispatcher.
+// The domain [span_lo(wm), span_hi(hi)) of each buffer comes from the watermark the
+// dispatcher acted on (it skipped only work-groups >= wm, whose host results were staged
+// before the watermark was published, L16.s15); nothing is merged if it never skipped.
+__device__ __forceinline__ void merge_dev_body(const DevMergeList &L, unsigned long long r, size_t tid, size_t nth) {
+    const unsigned int w32 = decode_wm_word(r, L.epoch);
+    const long long wm = (long long)w32;
+    if (w32 == 0xFFFFFFFFu || wm >= L.hi) return;
+    for (int b = 0; b < L.n; ++b) {
+        long long b0 = 0, b1 = L.total[b];
+        if (L.unit_wgs[b] > 0) {
+            b0 = (wm / L.unit_wgs[b]) * L.unit_bytes[b];
+            b1 = ((L.hi + L.unit_wgs[b] - 1) / L.unit_wgs[b]) * L.unit_bytes[b];
+            if (b0 > L.total[b]) b0 = L.total[b];
+            if (b1 > L.total[b]) b1 = L.total[b];
+        }
+        if (b1 <= b0) continue;
+        switch (L.es[b]) {
+        case 1: merge_range<1>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        case 2: merge_range<2>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        case 4: merge_range<4>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        default: merge_range<8>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256) merge_dev_kernel(const DevMergeList L) {
+    __shared__ unsigned long long s_wm;
+    if (threadIdx.x == 0) s_wm = ld_status(L.wm_word);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        // the dispatcher has finished (stream order): tell the host executor (L18.s19)
+        if (L.exit_word)
+            asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(L.exit_word), "l"((unsigned long long)L.epoch) : "memory");
+        if (L.tstamp) L.tstamp[0] = globaltimer();
+    }
+    __syncthreads();
+    struct StampEnd {
+        unsigned long long *p;
+        __device__ ~StampEnd() { if (p && threadIdx.x == 0) atomicMax(p + 1, globaltimer()); }
+    } stamp_end{L.tstamp};
+    merge_dev_body(L, s_wm, (size_t)blockIdx.x * blockDim.x + threadIdx.x, (size_t)gridDim.x * blockDim.x);
+}
+
+// ------------------------------------------------------------------------------------------
 // Dispatcher (persistent, ascending claim) and plain grid
 // ------------------------------------------------------------------------------------------
+__device__ __forceinline__ void record_wm(const CoopCtl &c, unsigned int w) {
+    // epoch-tagged: a later launch's word always wins, within a launch the smallest watermark
+    atomicMax(c.wm_out, ((unsigned long long)c.epoch << 32) | (unsigned long long)(0xFFFFFFFFu - w));
+}
+
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
 coop_kernel(const CoopCtl c, const typename Body::Params bp) {
@@ -104,6 +279,16 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
     __shared__ int s_flag;
     __shared__ __align__(16) typename Body::Smem smem;
 
+    if (blockIdx.x == 0 && threadIdx.x == 0) {   // counters of the next launch (stream-ordered)
+        *c.claim_next = 0ull;
+        if (c.barrier_next) *c.barrier_next = 0u;
+        if (c.tasks_next) *c.tasks_next = 0ull;
+        if (c.tstamp) {   // stats mode: start stamp, reset this launch's merge end and the next end
+            c.tstamp[0] = globaltimer();
+            c.tstamp[3] = 0ull;
+            c.tstamp_next[1] = 0ull;
+        }
+    }
     // The first task of every CTA is blockIdx.x: no claim and no status wait before it starts.
     // Running a work-group the host already covers is never wrong (the merge keeps the host's
     // words), and long tasks still poll the status inside their loops; the status load issued
@@ -128,7 +313,7 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
         if (t >= c.task_hi) break;
         const long long key = Body::key(bp, t);
         if (checked && (unsigned long long)key >= (unsigned long long)w) {   // covered by the host
-            if (threadIdx.x == 0) atomicMin(c.wmin, w);
+            if (threadIdx.x == 0) record_wm(c, w);
             break;
         }
         TaskCtx tc;
@@ -141,7 +326,7 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
         }
         const bool aborted = Body::run(bp, t, tc, smem);
         if (aborted) {
-            if (threadIdx.x == 0) atomicMin(c.wmin, tc.abort_w);
+            if (threadIdx.x == 0) record_wm(c, tc.abort_w);
             break;
         }
         ++executed;
@@ -152,26 +337,34 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
         checked = true;
         __syncthreads();
     }
-    // Exit protocol: the last CTA out publishes the exit record to mapped host memory and
-    // resets the device counters for the next launch (stream order serialises launches).
+    if (c.tasks && threadIdx.x == 0 && executed) atomicAdd(c.tasks, executed);
+    if (c.tstamp && threadIdx.x == 0) atomicMax(c.tstamp + 1, globaltimer());
+    if (!c.fused) return;
+    // Fused tail (the kernel is launched cooperatively, so every CTA is resident): a grid
+    // barrier, then the GPU-exit signal for the host executor (L18.s19) and the diff-merge
+    // (Fig 9) over the domain given by the lowest watermark any CTA acted on -- no second
+    // kernel launch and no host round trip between the dispatcher and the merge.
+    __syncthreads();
     if (threadIdx.x == 0) {
-        if (executed) atomicAdd(c.tasks, executed);
         __threadfence();
-        const unsigned int prev = atomicAdd(c.done, 1u);
-        if (prev == gridDim.x - 1) {
-            __threadfence();
-            const unsigned int wm = atomicExch(c.wmin, 0xFFFFFFFFu);
-            const unsigned long long nt = atomicExch(c.tasks, 0ull);
-            atomicExch(c.claim, 0ull);
-            atomicExch(c.done, 0u);
-            // device copy of the watermark the GPU acted on, read by the merge kernel queued
-            // behind this launch (the merge domain is decided on the device, no host round trip)
-            atomicExch(c.wm_out, ((unsigned long long)c.epoch << 32) | wm);
-            asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(c.exit_rec + 1), "l"(nt) : "memory");
-            const unsigned long long rec = ((unsigned long long)c.epoch << 32) | wm;
-            asm volatile("st.release.sys.global.b64 [%0], %1;" ::"l"(c.exit_rec), "l"(rec) : "memory");
+        atomicAdd(c.barrier, 1u);
+        unsigned int v;
+        for (;;) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(c.barrier) : "memory");
+            if (v >= gridDim.x) break;
+            __nanosleep(64);
+        }
+        s_task = (long long)ld_status(c.mg.wm_word);
+        if (blockIdx.x == 0) {
+            asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(c.exit_word), "l"((unsigned long long)c.epoch) : "memory");
+            if (c.mg.tstamp) c.mg.tstamp[0] = globaltimer();
         }
     }
+    __syncthreads();
+    if (c.mg.n > 0)
+        merge_dev_body(c.mg, (unsigned long long)s_task, (size_t)blockIdx.x * blockDim.x + threadIdx.x,
+                       (size_t)gridDim.x * blockDim.x);
+    if (c.mg.tstamp && threadIdx.x == 0) atomicMax(c.mg.tstamp + 1, globaltimer());
 }
 
 template <class Body>
@@ -215,8 +408,12 @@ struct EmptySmem { int dummy; };
 
 template <typename T, int NMAT>
 struct RowDotBody {
-    static constexpr int kThreads = 256;
-    static constexpr int kMinBlocks = 2;
+    // 4 warps, one row each: 64 registers allow 8 CTAs (32 warps) per SM, so a 4096-row
+    // launch (1024 tasks) is resident in a single wave with 2 KB of loads in flight per warp.
+    static constexpr int kThreads = 128;
+    static constexpr int kMinBlocks = 8;
+    static constexpr int kWarps = kThreads / 32;
+    static constexpr int U = (NMAT == 2) ? 2 : 4;   // 128-column blocks whose loads are issued together
     struct Params {
         const T *A; const T *B; const T *x; T *out0; T *out1;
         long long nrows, ncols, lws; int R; T alpha, beta; int vec4;
@@ -234,70 +431,71 @@ struct RowDotBody {
 
     __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
         const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-        if (warp >= p.R) return false;
-        const long long i = t * p.R + warp;
-        if (i >= p.nrows) return false;
-        const T *Ar = p.A + i * p.ncols;
-        const T *Br = (NMAT == 2) ? p.B + i * p.ncols : nullptr;
-        T a0 = 0, a1 = 0, a2 = 0, a3 = 0, b0 = 0, b1 = 0, b2 = 0, b3 = 0;
-        const long long nfull = p.ncols / 128;
-        long long k = 0;
-        if (p.vec4) {
-            // main loop: loads of 4 blocks issued before their FMAs (memory-level parallelism)
-            for (; k + 4 <= nfull; k += 4) {
-                typename V4<T>::type av[4], bv[4], xv[4];
+        for (int r = warp; r < p.R; r += kWarps) {
+            const long long i = t * p.R + r;
+            if (i >= p.nrows) return false;
+            const T *Ar = p.A + i * p.ncols;
+            const T *Br = (NMAT == 2) ? p.B + i * p.ncols : nullptr;
+            T a0 = 0, a1 = 0, a2 = 0, a3 = 0, b0 = 0, b1 = 0, b2 = 0, b3 = 0;
+            const long long nfull = p.ncols / 128;
+            long long k = 0;
+            if (p.vec4) {
+                for (; k + U <= nfull; k += U) {
+                    typename V4<T>::type av[U], bv[U], xv[U];
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const long long j = (k + u) * 128 + 4 * lane;
-                    av[u] = ld_stream4(Ar + j);
-                    if (NMAT == 2) bv[u] = ld_stream4(Br + j);
-                    xv[u] = ld_cached4(p.x + j);
+                    for (int u = 0; u < U; ++u) {
+                        const long long j = (k + u) * 128 + 4 * lane;
+                        av[u] = ld_stream4(Ar + j);
+                        if (NMAT == 2) bv[u] = ld_stream4(Br + j);
+                    }
+#pragma unroll
+                    for (int u = 0; u < U; ++u) xv[u] = ld_cached4(p.x + (k + u) * 128 + 4 * lane);
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        a0 = op_fma(av[u].x, xv[u].x, a0); a1 = op_fma(av[u].y, xv[u].y, a1);
+                        a2 = op_fma(av[u].z, xv[u].z, a2); a3 = op_fma(av[u].w, xv[u].w, a3);
+                        if (NMAT == 2) {
+                            b0 = op_fma(bv[u].x, xv[u].x, b0); b1 = op_fma(bv[u].y, xv[u].y, b1);
+                            b2 = op_fma(bv[u].z, xv[u].z, b2); b3 = op_fma(bv[u].w, xv[u].w, b3);
+                        }
+                    }
                 }
-#pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    a0 = op_fma(av[u].x, xv[u].x, a0); a1 = op_fma(av[u].y, xv[u].y, a1);
-                    a2 = op_fma(av[u].z, xv[u].z, a2); a3 = op_fma(av[u].w, xv[u].w, a3);
+                for (; k < nfull; ++k) {
+                    const long long j = k * 128 + 4 * lane;
+                    typename V4<T>::type av = ld_stream4(Ar + j), xv = ld_cached4(p.x + j);
+                    a0 = op_fma(av.x, xv.x, a0); a1 = op_fma(av.y, xv.y, a1);
+                    a2 = op_fma(av.z, xv.z, a2); a3 = op_fma(av.w, xv.w, a3);
                     if (NMAT == 2) {
-                        b0 = op_fma(bv[u].x, xv[u].x, b0); b1 = op_fma(bv[u].y, xv[u].y, b1);
-                        b2 = op_fma(bv[u].z, xv[u].z, b2); b3 = op_fma(bv[u].w, xv[u].w, b3);
+                        typename V4<T>::type bv = ld_stream4(Br + j);
+                        b0 = op_fma(bv.x, xv.x, b0); b1 = op_fma(bv.y, xv.y, b1);
+                        b2 = op_fma(bv.z, xv.z, b2); b3 = op_fma(bv.w, xv.w, b3);
                     }
                 }
             }
-            for (; k < nfull; ++k) {
+            // scalar path (unaligned rows) and the ragged tail, same partition order
+            for (; k * 128 < p.ncols; ++k) {
                 const long long j = k * 128 + 4 * lane;
-                typename V4<T>::type av = ld_stream4(Ar + j), xv = ld_cached4(p.x + j);
-                a0 = op_fma(av.x, xv.x, a0); a1 = op_fma(av.y, xv.y, a1);
-                a2 = op_fma(av.z, xv.z, a2); a3 = op_fma(av.w, xv.w, a3);
-                if (NMAT == 2) {
-                    typename V4<T>::type bv = ld_stream4(Br + j);
-                    b0 = op_fma(bv.x, xv.x, b0); b1 = op_fma(bv.y, xv.y, b1);
-                    b2 = op_fma(bv.z, xv.z, b2); b3 = op_fma(bv.w, xv.w, b3);
-                }
-            }
-        }
-        // scalar path (unaligned rows) and the ragged tail, same partition order
-        for (; k * 128 < p.ncols; ++k) {
-            const long long j = k * 128 + 4 * lane;
 #define FCL_ROWDOT_TAIL(C, AC, BC)                                             \
-            if (j + C < p.ncols) {                                             \
-                const T xv = p.x[j + C];                                       \
-                AC = op_fma(Ar[j + C], xv, AC);                                \
-                if (NMAT == 2) BC = op_fma(Br[j + C], xv, BC);                 \
-            }
-            FCL_ROWDOT_TAIL(0, a0, b0)
-            FCL_ROWDOT_TAIL(1, a1, b1)
-            FCL_ROWDOT_TAIL(2, a2, b2)
-            FCL_ROWDOT_TAIL(3, a3, b3)
+                if (j + C < p.ncols) {                                         \
+                    const T xv = p.x[j + C];                                   \
+                    AC = op_fma(Ar[j + C], xv, AC);                            \
+                    if (NMAT == 2) BC = op_fma(Br[j + C], xv, BC);             \
+                }
+                FCL_ROWDOT_TAIL(0, a0, b0)
+                FCL_ROWDOT_TAIL(1, a1, b1)
+                FCL_ROWDOT_TAIL(2, a2, b2)
+                FCL_ROWDOT_TAIL(3, a3, b3)
 #undef FCL_ROWDOT_TAIL
-        }
-        const T va = warp_fold(a0, a1, a2, a3);
-        if (NMAT == 1) {
-            if (lane == 0) p.out0[i] = va;
-        } else {
-            const T vb = warp_fold(b0, b1, b2, b3);
-            if (lane == 0) {
-                p.out0[i] = va;                                           // tmp[i]
-                p.out1[i] = op_add(op_mul(p.alpha, va), op_mul(p.beta, vb)); // y[i]
+            }
+            const T va = warp_fold(a0, a1, a2, a3);
+            if (NMAT == 1) {
+                if (lane == 0) p.out0[i] = va;
+            } else {
+                const T vb = warp_fold(b0, b1, b2, b3);
+                if (lane == 0) {
+                    p.out0[i] = va;                                              // tmp[i]
+                    p.out1[i] = op_add(op_mul(p.alpha, va), op_mul(p.beta, vb)); // y[i]
+                }
             }
         }
         return false;
@@ -651,149 +849,6 @@ struct GemmBody {
 };
 
 // ------------------------------------------------------------------------------------------
-// Diff-merge (Fig 9): gpu[e] = (cpu[e] != twin[e]) ? cpu[e] : gpu[e], bitwise, per element.
-// cpu/twin are streamed once with 128-bit no-L1-allocate loads (4 vectors in flight per
-// thread); changed elements are stored with predicated element stores (a fully changed vector
-// with one 128-bit store), so the GPU copy is never read: traffic = 8 B/word read + 4 B per
-// changed word written.  Byte/half-word element sizes blend within the 32-bit lane.
-// ------------------------------------------------------------------------------------------
-template <int ES>
-__device__ __forceinline__ void merge_vec(uint8_t *g, const uint4 c, const uint4 t) {
-    const uint32_t cw[4] = {c.x, c.y, c.z, c.w}, tw[4] = {t.x, t.y, t.z, t.w};
-    if (ES == 4) {
-        const bool ch0 = cw[0] != tw[0], ch1 = cw[1] != tw[1], ch2 = cw[2] != tw[2], ch3 = cw[3] != tw[3];
-        if (ch0 && ch1 && ch2 && ch3) { *reinterpret_cast<uint4 *>(g) = c; return; }
-        uint32_t *gw = reinterpret_cast<uint32_t *>(g);
-        if (ch0) gw[0] = cw[0];
-        if (ch1) gw[1] = cw[1];
-        if (ch2) gw[2] = cw[2];
-        if (ch3) gw[3] = cw[3];
-    } else if (ES == 8) {
-        const bool ch0 = (cw[0] != tw[0]) || (cw[1] != tw[1]);
-        const bool ch1 = (cw[2] != tw[2]) || (cw[3] != tw[3]);
-        if (ch0 && ch1) { *reinterpret_cast<uint4 *>(g) = c; return; }
-        unsigned long long *gd = reinterpret_cast<unsigned long long *>(g);
-        if (ch0) gd[0] = ((unsigned long long)cw[1] << 32) | cw[0];
-        if (ch1) gd[1] = ((unsigned long long)cw[3] << 32) | cw[2];
-    } else {
-        uint32_t m[4];
-        bool all = true, any = false;
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            if (ES == 1) m[q] = __vcmpne4(cw[q], tw[q]);
-            else m[q] = __vcmpne2(cw[q], tw[q]);
-            all &= (m[q] == 0xFFFFFFFFu);
-            any |= (m[q] != 0u);
-        }
-        if (all) { *reinterpret_cast<uint4 *>(g) = c; return; }
-        if (!any) return;
-        uint32_t *gw = reinterpret_cast<uint32_t *>(g);
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            if (m[q] == 0xFFFFFFFFu) gw[q] = cw[q];
-            else if (m[q]) gw[q] = (cw[q] & m[q]) | (gw[q] & ~m[q]);
-        }
-    }
-}
-
-template <int ES>
-__device__ __forceinline__ void merge_scalar(uint8_t *g, const uint8_t *c, const uint8_t *t, size_t nbytes) {
-    for (size_t e = 0; e + ES <= nbytes; e += ES) {
-        bool ch = false;
-#pragma unroll
-        for (int b = 0; b < ES; ++b) ch |= (c[e + b] != t[e + b]);
-        if (ch) {
-#pragma unroll
-            for (int b = 0; b < ES; ++b) g[e + b] = c[e + b];
-        }
-    }
-}
-
-__device__ __forceinline__ uint4 ld_nc_v4(const uint8_t *p) {
-    uint4 v;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
-    return v;
-}
-
-// Merge [0, nbytes) of one buffer with all threads of the grid (head/tail bytes scalar).
-template <int ES>
-__device__ __forceinline__ void merge_range(uint8_t *gpu, const uint8_t *cpu, const uint8_t *twin, size_t nbytes,
-                                            size_t tid, size_t nthreads) {
-    size_t head = 0, nvec = 0, tail = nbytes;
-    const uintptr_t ag = reinterpret_cast<uintptr_t>(gpu) & 15u;
-    if (ag == (reinterpret_cast<uintptr_t>(cpu) & 15u) && ag == (reinterpret_cast<uintptr_t>(twin) & 15u)) {
-        head = ag ? 16 - ag : 0;
-        if (head > nbytes) head = nbytes;
-        nvec = (nbytes - head) / 16;
-        tail = nbytes - head - 16 * nvec;
-    }
-    if (tid == 0 && head) merge_scalar<ES>(gpu, cpu, twin, head);
-    if (tid == (nthreads > 1 ? 1 : 0) && tail) {
-        const size_t off = head + 16 * nvec;
-        merge_scalar<ES>(gpu + off, cpu + off, twin + off, tail);
-    }
-    uint8_t *g = gpu + head;
-    const uint8_t *c = cpu + head, *t = twin + head;
-    constexpr int U = 4;
-    size_t v = tid;
-    for (; v + (U - 1) * nthreads < nvec; v += U * nthreads) {
-        uint4 cv[U], tv[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) { cv[u] = ld_nc_v4(c + 16 * (v + u * nthreads)); tv[u] = ld_nc_v4(t + 16 * (v + u * nthreads)); }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const bool diff = (cv[u].x != tv[u].x) | (cv[u].y != tv[u].y) | (cv[u].z != tv[u].z) | (cv[u].w != tv[u].w);
-            // warp vote: a warp whose 512-byte segment is unchanged skips the store path
-            if (__ballot_sync(__activemask(), diff) && diff) merge_vec<ES>(g + 16 * (v + u * nthreads), cv[u], tv[u]);
-        }
-    }
-    for (; v < nvec; v += nthreads) {
-        const uint4 cv = ld_nc_v4(c + 16 * v), tv = ld_nc_v4(t + 16 * v);
-        if ((cv.x != tv.x) | (cv.y != tv.y) | (cv.z != tv.z) | (cv.w != tv.w)) merge_vec<ES>(g + 16 * v, cv, tv);
-    }
-}
-
-template <int ES>
-__global__ void __launch_bounds__(256)
-merge_kernel(uint8_t *__restrict__ gpu, const uint8_t *__restrict__ cpu, const uint8_t *__restrict__ twin,
-             size_t nbytes) {
-    merge_range<ES>(gpu, cpu, twin, nbytes, (size_t)blockIdx.x * blockDim.x + threadIdx.x,
-                    (size_t)gridDim.x * blockDim.x);
-}
-
-// Merge of every OUT/INOUT buffer of a cooperative launch, queued behind the dispatcher.
-// The domain [span_lo(wm), span_hi(hi)) of each buffer comes from the watermark the
-// dispatcher acted on (it skipped only work-groups >= wm, whose host results were staged
-// before the watermark was published, L16.s15); nothing is merged if it never skipped.
-__global__ void __launch_bounds__(256) merge_dev_kernel(const DevMergeList L) {
-    __shared__ unsigned long long s_wm;
-    if (threadIdx.x == 0) s_wm = ld_status(L.wm_word);
-    __syncthreads();
-    const unsigned long long r = s_wm;
-    if ((unsigned int)(r >> 32) != L.epoch) return;
-    const long long wm = (long long)(unsigned int)r;
-    if ((unsigned int)r == 0xFFFFFFFFu || wm >= L.hi) return;
-    const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
-    for (int b = 0; b < L.n; ++b) {
-        long long b0 = 0, b1 = L.total[b];
-        if (L.unit_wgs[b] > 0) {
-            b0 = (wm / L.unit_wgs[b]) * L.unit_bytes[b];
-            b1 = ((L.hi + L.unit_wgs[b] - 1) / L.unit_wgs[b]) * L.unit_bytes[b];
-            if (b0 > L.total[b]) b0 = L.total[b];
-            if (b1 > L.total[b]) b1 = L.total[b];
-        }
-        if (b1 <= b0) continue;
-        switch (L.es[b]) {
-        case 1: merge_range<1>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
-        case 2: merge_range<2>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
-        case 4: merge_range<4>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
-        default: merge_range<8>(L.gpu[b] + b0, L.cpu[b] + b0, L.twin[b] + b0, (size_t)(b1 - b0), tid, nth); break;
-        }
-    }
-}
-
-// ------------------------------------------------------------------------------------------
 // Host-side launch plumbing
 // ------------------------------------------------------------------------------------------
 static thread_local char g_err[256];
@@ -813,10 +868,14 @@ static int largest_pow2_divisor_le(long long v, int cap) {
 
 template <class Body>
 static int occupancy_grid(int num_sms) {
-    int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, coop_kernel<Body>, Body::kThreads, 0) != cudaSuccess ||
-        per_sm < 1)
-        per_sm = 1;
+    static int per_sm = 0;   // cached per body type
+    if (per_sm == 0) {
+        int v = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, coop_kernel<Body>, Body::kThreads, 0) != cudaSuccess || v < 1)
+            v = 1;
+        cudaGetLastError();
+        per_sm = v;
+    }
     return per_sm * num_sms;
 }
 
@@ -828,6 +887,17 @@ static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long l
     if (c) {
         long long grid = occupancy_grid<Body>(num_sms);
         if (grid > n) grid = n;
+        static const bool coop_api = !(getenv("FCL_COOP_LAUNCH") && atoi(getenv("FCL_COOP_LAUNCH")) == 0);
+        if (c->fused && coop_api) {
+            // cooperative launch: all CTAs co-resident, required by the fused tail's grid barrier
+            CoopCtl cc = *c;
+            typename Body::Params pp = bp;
+            void *args[] = {(void *)&cc, (void *)&pp};
+            cudaError_t e = cudaLaunchCooperativeKernel((const void *)coop_kernel<Body>, dim3((unsigned)grid),
+                                                        dim3(Body::kThreads), args, 0, s);
+            if (e != cudaSuccess) return seterr(e, "coop_kernel cooperative launch");
+            return (int)grid;
+        }
         coop_kernel<Body><<<(unsigned)grid, Body::kThreads, 0, s>>>(*c, bp);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return seterr(e, "coop_kernel launch");
@@ -865,7 +935,7 @@ static typename RowDotBody<T, NMAT>::Params rowdot_params(const KArgs &a, const 
         p.nrows = a.n0; p.ncols = a.n1;
     }
     p.lws = g.lws[0];
-    p.R = largest_pow2_divisor_le(g.lws[0], 8);
+    p.R = largest_pow2_divisor_le(g.lws[0], 4);
     if (a.integer) { p.alpha = (T)a.ialpha; p.beta = (T)a.ibeta; }
     else { p.alpha = (T)a.alpha; p.beta = (T)a.beta; }
     p.vec4 = (p.ncols % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.x) && (NMAT == 1 || is_aligned16(p.B));
@@ -957,7 +1027,7 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
 
 // Host mirror of each body's task enumeration (must match Body::key exactly).
 static int64_t host_rowdot_key(const Geom &g, int64_t t) {
-    const int R = largest_pow2_divisor_le(g.lws[0], 8);
+    const int R = largest_pow2_divisor_le(g.lws[0], 4);
     return (t * R) / g.lws[0];
 }
 
@@ -965,9 +1035,9 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
     TaskSpace ts{0, 256};
     switch (a.kernel) {
     case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV: {
-        const int R = largest_pow2_divisor_le(g.lws[0], 8);
+        const int R = largest_pow2_divisor_le(g.lws[0], 4);
         ts.ntasks = (g.ng[0] * g.lws[0] + R - 1) / R;   // covers every row of every work-group
-        ts.threads = 256; break;
+        ts.threads = 128; break;
     }
     case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD: {
         const int CB = largest_pow2_divisor_le(g.lws[0], 32);

@@ -1,9 +1,14 @@
 // runtime.cpp -- the FluidiCL runtime for one B200 + its host cores, behind the C-ABI fcl.h.
 //
 // Components:
-//   * context: CUDA device, streams main / hd / dh (L20.s10-13), the 64-bit watermark word
-//     {epoch, W} (D1, C14) in pinned mapped host memory (or device memory), the mapped exit
-//     record written by the dispatcher's last CTA, device claim counters, kernel-id epoch;
+//   * context: CUDA device, streams main / hd / dh (L20.s10-13), the 64-bit watermark words
+//     {epoch, W} (D1, C14; one per launch slot) in device or pinned mapped memory, the mapped
+//     GPU-exit word, per-slot device claim counters, the kernel-id epoch;
+//   * launch queue: fcl_enqueue_ndrange queues a launch's GPU work (twin capture, dispatcher,
+//     merge, return copy) from the calling thread and hands its host side to the coordinator
+//     thread -- the paper's CPU scheduler thread (C10, L18.s18-21) -- so, like OpenCL's
+//     clEnqueueNDRangeKernel, the call does not block on the GPU (the paper's blocking calls
+//     were a stated limitation, L22.s14); fcl_finish waits for everything;
 //   * dual-resident buffers (C3, L14.s49-50 / L16.s1) with element-size metadata (C16, D6) and
 //     host/device validity flags (minimal data-location tracking, C22 / L20.s31-33);
 //   * twin + stage buffer pool (C5/C6, L16.s2-3, L20.s23-29);
@@ -232,10 +237,25 @@ struct Executor {
     }
 };
 
+// Optional host-side event trace (FCL_TRACE=1): (time, tag, epoch) triples printed at
+// context release; used to attribute host latency, never on by default.
+struct TraceRec { double t; const char *tag; uint32_t epoch; };
+struct Tracer {
+    bool on = false;
+    std::mutex mu;
+    std::vector<TraceRec> recs;
+    void add(const char *tag, uint32_t e) {
+        if (!on) return;
+        std::lock_guard<std::mutex> lk(mu);
+        if (recs.size() < 200000) recs.push_back({now_ms(), tag, e});
+    }
+};
+
 struct PoolEnt {
     void *p;
     size_t bytes;
     bool used;
+    bool hd_pending;      // a staging copy on hd may still write it (wait on ev_hd_release)
     uint32_t last_epoch;
 };
 
@@ -258,7 +278,7 @@ struct fcl_buffer_st {
     bool own_dev, own_host;
     bool host_valid, dev_valid;
     bool d2h_pending;
-    cudaEvent_t d2h_ev;
+    cudaEvent_t d2h_ev;    // completion of the buffer's pending return copy (recorded on dh)
     // deferred merge state (opts.defer_merge)
     bool merge_pending;
     void *twin, *stage;
@@ -266,6 +286,44 @@ struct fcl_buffer_st {
 };
 
 typedef CUresult (*PFN_writeValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+
+namespace {
+
+struct Launch {
+    fcl_context ctx;
+    const KernelDef *kd;
+    KArgs a;
+    Geom g;
+    fcl_buffer bufs[6];
+    uint8_t acc[6];   // 1 read, 2 written, 3 both
+    int out_idx[6];
+    int nout;
+    bool any_inout;   // some output is read-modify-written in place (INOUT)
+    int64_t lo, hi;
+    fcl_launch_opts o;
+};
+
+// One cooperative launch in flight: phase A (GPU side, calling thread) then phase B (host
+// side, coordinator thread).
+struct Job {
+    Launch L;
+    uint32_t epoch = 0;
+    int slot = 0;
+    int64_t t0 = 0, t1 = 0, s_forced = -1;
+    bool forced = false, dev_merge = false, eager = false, gpu_launched = false;
+    bool twin_alias = false;   // exact spans: the merge compares against the device copy itself
+    int64_t unit = 1;          // host chunk boundaries are multiples of this many work-groups
+    void *twin[6] = {nullptr}, *stage[6] = {nullptr};
+    cudaEvent_t ev_start = nullptr, ev_k0 = nullptr, ev_k1 = nullptr, ev_m0 = nullptr, ev_m1 = nullptr,
+                ev_staged = nullptr, ev_ret = nullptr, ev_wm = nullptr, ev_d2h = nullptr;
+    cudaEvent_t main_before = nullptr;   // an event on main at or after every earlier launch's merge
+    bool have_k = false, have_m = false, wm_pending = false;
+    fcl_launch_info info{};
+    fcl_status status = FCL_SUCCESS;
+    std::atomic<int> done{0};
+};
+
+}  // namespace
 
 struct fcl_context_st {
     int device = 0;
@@ -278,24 +336,46 @@ struct fcl_context_st {
     static constexpr int kSlots = 16;
     unsigned long long *status_host = nullptr;   // mapped host words (HOST_MAPPED)
     unsigned long long *status_dptr = nullptr;   // device-visible address of slot 0
-    uint32_t slot_epoch[kSlots] = {0};           // epoch of the dispatcher that last used a slot
-    unsigned long long *exit_host = nullptr;     // mapped exit record [2]
-    unsigned long long *exit_dptr = nullptr;
+    bool slot_used[kSlots] = {};
+    unsigned long long *wm_host = nullptr;       // pinned copy of the dispatcher's wm word
+    unsigned long long *exit_host = nullptr;     // mapped word: epoch of the last finished dispatcher
+    unsigned long long *exit_dptr = nullptr;     // its device-visible address
     unsigned long long *dclaim = nullptr, *dtasks = nullptr, *dwm = nullptr;
-    unsigned int *ddone = nullptr, *dwmin = nullptr;
+    unsigned long long *dstamp = nullptr;        // stats mode: %globaltimer stamps, 4 per slot
+    unsigned int *dbar = nullptr;                // grid-barrier counters, one per slot
+    bool unfused = false;                        // FCL_UNFUSED_MERGE=1: merge as a separate kernel
+    bool ktiming = false;                        // CUDA events around every kernel (FCL_KTIMING=1)
+    cudaEvent_t main_tail = nullptr;             // ev_k1 of the last cooperative dispatcher
     uint32_t epoch = 0;
     PFN_writeValue64 write64 = nullptr;
+    bool stats = false;                          // count executed GPU tasks, time merges (FCL_STATS=1)
+    size_t eager_return_bytes = 8u << 20;        // outputs up to this size return right behind the merge
+    bool force_twin = false;                     // FCL_FORCE_TWIN=1: always capture a twin (Fig 9 as printed)
+    // twin/stage pool (C6, L20.s23-29)
+    std::mutex pool_mu;
     std::vector<PoolEnt> pool;
+    cudaEvent_t ev_hd_release = nullptr;         // hd position after the last released stage copies
+    // host executor + coordinator (the CPU scheduler thread, C10)
     Executor ex;
+    std::mutex q_mu;
+    std::condition_variable q_cv;
+    std::vector<Job *> queue;                    // pending jobs, FIFO
+    std::vector<Job *> free_jobs;
+    Job *running = nullptr;
+    Job *last = nullptr;                         // most recent launch (for fcl_get_launch_info)
+    bool q_stop = false;
+    std::thread coord;
+    // errors
+    std::mutex err_mu;
     std::string err;
-    fcl_status sticky = FCL_SUCCESS;
-    std::vector<cudaEvent_t> evpool;   // timing-disabled events for chunk publication
-    cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr, ev_m0 = nullptr, ev_m1 = nullptr, ev_hd_last = nullptr;
-    cudaEvent_t ev_mark = nullptr;   // main-stream progress marker for the dh stream
-    bool have_k = false, have_m = false;
-    fcl_launch_info info{};
+    std::atomic<fcl_status> sticky{FCL_SUCCESS};
+    // single-device modes
+    cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr, ev_mark = nullptr;
+    cudaEvent_t ev_gd2h = nullptr;               // completion of single-device / deferred returns (on dh)
+    fcl_launch_info sync_info{};
+    bool sync_have_k = false;
     std::vector<fcl_buffer> defer_list;
-    size_t eager_return_bytes = 8u << 20;   // outputs up to this size return right behind the merge
+    Tracer tr;
 };
 
 namespace {
@@ -307,6 +387,7 @@ fcl_status set_err(fcl_context ctx, fcl_status s, const char *fmt, ...) {
         va_start(ap, fmt);
         vsnprintf(b, sizeof b, fmt, ap);
         va_end(ap);
+        std::lock_guard<std::mutex> lk(ctx->err_mu);
         ctx->err = b;
     }
     return s;
@@ -324,16 +405,21 @@ fcl_status cuda_fail(fcl_context ctx, cudaError_t e, const char *what) {
         if (_e != cudaSuccess) return cuda_fail((ctx), _e, #call);      \
     } while (0)
 
-void *pool_get(fcl_context ctx, size_t bytes) {
+// ---- pool ----
+// Returns the buffer and whether main must wait for ctx->ev_hd_release before writing it.
+void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait) {
+    std::lock_guard<std::mutex> lk(ctx->pool_mu);
     int best = -1;
     for (size_t k = 0; k < ctx->pool.size(); ++k) {
         const PoolEnt &e = ctx->pool[k];
         if (!e.used && e.bytes >= bytes && (best < 0 || e.bytes < ctx->pool[(size_t)best].bytes)) best = (int)k;
     }
     if (best >= 0) {
-        ctx->pool[(size_t)best].used = true;
-        ctx->pool[(size_t)best].last_epoch = ctx->epoch;
-        return ctx->pool[(size_t)best].p;
+        PoolEnt &e = ctx->pool[(size_t)best];
+        e.used = true;
+        e.last_epoch = ctx->epoch;
+        if (e.hd_pending) { *hd_wait = true; e.hd_pending = false; }
+        return e.p;
     }
     void *p = nullptr;
     if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) {
@@ -345,19 +431,21 @@ void *pool_get(fcl_context ctx, size_t bytes) {
         }
         if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) { cudaGetLastError(); return nullptr; }
     }
-    ctx->pool.push_back({p, bytes, true, ctx->epoch});
+    ctx->pool.push_back({p, bytes, true, false, ctx->epoch});
     return p;
 }
 
-void pool_put(fcl_context ctx, void *p) {
+void pool_put(fcl_context ctx, void *p, bool hd_pending) {
+    std::lock_guard<std::mutex> lk(ctx->pool_mu);
     for (auto &e : ctx->pool)
-        if (e.p == p) { e.used = false; e.last_epoch = ctx->epoch; }
+        if (e.p == p) { e.used = false; e.hd_pending = e.hd_pending || hd_pending; e.last_epoch = ctx->epoch; }
 }
 
 // "At the end of each kernel execution, older unused buffers are freed" (L20.s29).
 void pool_trim(fcl_context ctx) {
+    std::lock_guard<std::mutex> lk(ctx->pool_mu);
     for (auto it = ctx->pool.begin(); it != ctx->pool.end();) {
-        if (!it->used && it->last_epoch + 16 < ctx->epoch) {
+        if (!it->used && !it->hd_pending && it->last_epoch + 16 < ctx->epoch) {
             cudaFree(it->p);
             it = ctx->pool.erase(it);
         } else {
@@ -366,43 +454,28 @@ void pool_trim(fcl_context ctx) {
     }
 }
 
-cudaEvent_t ev_get(fcl_context ctx, size_t k) {
-    while (ctx->evpool.size() <= k) {
-        cudaEvent_t e;
-        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
-        ctx->evpool.push_back(e);
-    }
-    return ctx->evpool[k];
-}
-
-// Store {epoch, W} after everything already queued on `s` (status follows data, L16.s15).
-unsigned long long *status_slot(fcl_context ctx) {
-    return ctx->status_dptr + (ctx->epoch % fcl_context_st::kSlots);
-}
-
-fcl_status publish(fcl_context ctx, uint32_t w, cudaStream_t s) {
-    const unsigned long long v = ((unsigned long long)ctx->epoch << 32) | w;
-    unsigned long long *dst = status_slot(ctx);
+// Store `v` to `dst` after everything already queued on `s` (stream memory operation; a
+// one-thread kernel store if the driver lacks 64-bit memops).
+fcl_status stream_store(fcl_context ctx, unsigned long long *dst, unsigned long long v, cudaStream_t s,
+                        bool barrier = true) {
     if (ctx->write64) {
-        CUresult r = ctx->write64((CUstream)s, (CUdeviceptr)dst, v, 0);
+        // with a barrier the store is ordered after the data of earlier operations on `s`
+        // (needed for publication, C13); a bare completion signal skips it (it costs ~12 us)
+        CUresult r = ctx->write64((CUstream)s, (CUdeviceptr)dst, v, barrier ? 0u : (unsigned)CU_STREAM_WRITE_VALUE_NO_MEMORY_BARRIER);
         if (r == CUDA_SUCCESS) return FCL_SUCCESS;
         ctx->write64 = nullptr;   // fall back to the kernel store from now on
     }
-    if (gpu_launch_store64(dst, v, s) < 0)
-        return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    if (gpu_launch_store64(dst, v, s) < 0) return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
     return FCL_SUCCESS;
 }
 
-bool poll_exit(fcl_context ctx, uint32_t *wmin, uint64_t *tasks) {
-    const unsigned long long r = __atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE);
-    if ((uint32_t)(r >> 32) != ctx->epoch) return false;
-    *wmin = (uint32_t)r;
-    *tasks = __atomic_load_n(ctx->exit_host + 1, __ATOMIC_ACQUIRE);
-    return true;
+// Publish {epoch, W} behind everything queued on hd: status follows data (C13, L16.s15).
+fcl_status publish(fcl_context ctx, const Job &j, uint32_t w) {
+    const unsigned long long v = ((unsigned long long)j.epoch << 32) | w;
+    return stream_store(ctx, ctx->status_dptr + j.slot, v, ctx->hd);
 }
 
-// Bring a buffer's copies to the validity a launch needs.
-fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_dev) {
+fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_dev, fcl_launch_info *info) {
     if (b->d2h_pending) {
         CK(ctx, cudaEventSynchronize(b->d2h_ev));
         b->d2h_pending = false;
@@ -410,13 +483,13 @@ fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_d
     if (need_dev && !b->dev_valid) {
         CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
         b->dev_valid = true;
-        ctx->info.h2d_bytes += (int64_t)b->bytes;
+        if (info) info->h2d_bytes += (int64_t)b->bytes;
     }
     if (need_host && !b->host_valid) {
         CK(ctx, cudaMemcpyAsync(b->host, b->dev, b->bytes, cudaMemcpyDeviceToHost, ctx->main));
         CK(ctx, cudaStreamSynchronize(ctx->main));
         b->host_valid = true;
-        ctx->info.d2h_bytes += (int64_t)b->bytes;
+        if (info) info->d2h_bytes += (int64_t)b->bytes;
     }
     return FCL_SUCCESS;
 }
@@ -434,40 +507,30 @@ int64_t first_task_at(const KArgs &a, const Geom &g, int64_t ntasks, int64_t f) 
     return lo;
 }
 
-struct Launch {
-    fcl_context ctx;
-    const KernelDef *kd;
-    KArgs a;
-    Geom g;
-    fcl_buffer bufs[6];
-    int out_idx[6];
-    int nout;
-    bool any_inout;   // some output is read-modify-write (INOUT)
-    int64_t lo, hi;
-    fcl_launch_opts o;
-};
-
-fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, bool after_merge) {
+// Device->host return of the outputs' spans of work-groups [wlo, whi), on dh behind
+// `main_mark` (an event already recorded on main after the kernel / merge).
+fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, fcl_launch_info &info,
+                       cudaEvent_t main_mark) {
     if (whi <= wlo) return FCL_SUCCESS;
-    (void)after_merge;
-    CK(ctx, cudaEventRecord(ctx->ev_mark, ctx->main));   // after the kernel (and merge) on main
-    CK(ctx, cudaStreamWaitEvent(ctx->dh, ctx->ev_mark, 0));
+    CK(ctx, cudaStreamWaitEvent(ctx->dh, main_mark, 0));
     for (int q = 0; q < L.nout; ++q) {
         fcl_buffer b = L.bufs[L.out_idx[q]];
         size_t b0, b1;
         out_span(L.a, L.g, L.out_idx[q], wlo, whi, &b0, &b1);
         if (b1 <= b0) continue;
         CK(ctx, cudaMemcpyAsync((char *)b->host + b0, (char *)b->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
-        ctx->info.d2h_bytes += (int64_t)(b1 - b0);
+        info.d2h_bytes += (int64_t)(b1 - b0);
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
         b->d2h_pending = true;
     }
     return FCL_SUCCESS;
 }
 
-fcl_status enqueue_merges(fcl_context ctx, Launch &L, void **twin, void **stage, int64_t mlo, int64_t mhi) {
+// Host-decided merges (forced split, deferred merge) on main.
+fcl_status enqueue_merges(fcl_context ctx, Job &j, int64_t mlo, int64_t mhi) {
+    Launch &L = j.L;
     if (mhi <= mlo) return FCL_SUCCESS;
-    if (!ctx->have_m) CK(ctx, cudaEventRecord(ctx->ev_m0, ctx->main));
+    if (ctx->stats && !L.o.defer_merge) CK(ctx, cudaEventRecord(j.ev_m0, ctx->main));
     for (int q = 0; q < L.nout; ++q) {
         fcl_buffer b = L.bufs[L.out_idx[q]];
         size_t b0, b1;
@@ -475,154 +538,189 @@ fcl_status enqueue_merges(fcl_context ctx, Launch &L, void **twin, void **stage,
         if (b1 <= b0) continue;
         if (L.o.defer_merge) {
             b->merge_pending = true;
-            b->twin = twin[q]; b->stage = stage[q];
+            b->twin = j.twin[q];   // nullptr: twin aliases the device copy
+            b->stage = j.stage[q];
             b->m_b0 = b0; b->m_b1 = b1;
-            twin[q] = stage[q] = nullptr;   // ownership moves to the buffer until fcl_merge
+            j.twin[q] = j.stage[q] = nullptr;   // ownership moves to the buffer until fcl_merge
             ctx->defer_list.push_back(b);
             continue;
         }
-        if (gpu_launch_merge((char *)b->dev + b0, (char *)stage[q] + b0, (char *)twin[q] + b0, b1 - b0,
+        const char *tw = j.twin_alias ? (const char *)b->dev : (const char *)j.twin[q];
+        ctx->main_tail = nullptr;
+        if (gpu_launch_merge((char *)b->dev + b0, (char *)j.stage[q] + b0, tw + b0, b1 - b0,
                              (int)b->elem_size, ctx->num_sms, ctx->main) < 0)
             return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
-        ctx->info.gpu_launches += 1;
-        ctx->info.merge_bytes += (int64_t)(b1 - b0);
-        ctx->info.merged = 1;
+        j.info.gpu_launches += 1;
+        j.info.merge_bytes += (int64_t)(b1 - b0);
     }
-    if (!L.o.defer_merge) {
-        CK(ctx, cudaEventRecord(ctx->ev_m1, ctx->main));
-        ctx->have_m = true;
+    if (ctx->stats && !L.o.defer_merge) {
+        CK(ctx, cudaEventRecord(j.ev_m1, ctx->main));
+        j.have_m = true;
     }
     return FCL_SUCCESS;
 }
 
-// ---- the three modes ----
-fcl_status run_gpu_only(Launch &L) {
-    fcl_context ctx = L.ctx;
-    const TaskSpace ts = gpu_task_space(L.a, L.g);
-    const int64_t t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo), t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
-    CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
-    if (gpu_launch_plain(L.a, L.g, t0, t1, ctx->main) < 0)
-        return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
-    CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
-    ctx->have_k = true;
-    ctx->info.gpu_launches += 1;
-    ctx->info.gpu_tasks = ctx->info.gpu_tasks_total = t1 - t0;
-    return enqueue_d2h(ctx, L, L.lo, L.hi, false);
-}
-
-fcl_status run_cpu_only(Launch &L) {
-    fcl_context ctx = L.ctx;
-    Executor &ex = ctx->ex;
-    const int nact = L.o.n_host_threads > 0 ? L.o.n_host_threads : ex.T;
-    const int64_t nwg = L.hi - L.lo;
-    const int parts = (L.o.cpu_wg_split && nwg < nact) ? (int)((nact + nwg - 1) / nwg) : 1;
-    const double t0 = now_ms();
-    ex.abort_flag = 0;
-    ex.executed.store(0);
-    ex.submit(L.a, L.g, L.lo, L.hi, parts, nact);
-    ex.wait();
-    ctx->info.t_host_ms = now_ms() - t0;
-    ctx->info.cpu_wgs = nwg;
-    ctx->info.n_chunks = 1;
-    ctx->info.chunk_sizes[0] = (int32_t)nwg;
-    ctx->info.cpu_did_all = 1;
-    ctx->info.published_watermark = L.lo;
-    for (int q = 0; q < L.nout; ++q) L.bufs[L.out_idx[q]]->dev_valid = false;   // lazy H2D on next GPU use
+// Lowest watermark the dispatcher of job j acted on (hi if it never skipped); a synchronous
+// 8-byte read used off the fast path.  Only valid until a later dispatcher touches the word.
+fcl_status read_gpu_watermark(fcl_context ctx, Job &j, int64_t *wm) {
+    CK(ctx, cudaStreamWaitEvent(ctx->dh, j.ev_k1, 0));
+    CK(ctx, cudaMemcpyAsync(ctx->wm_host, ctx->dwm, 8, cudaMemcpyDeviceToHost, ctx->dh));
+    CK(ctx, cudaEventRecord(j.ev_wm, ctx->dh));
+    CK(ctx, cudaEventSynchronize(j.ev_wm));
+    const unsigned int w = decode_wm_word(*ctx->wm_host, j.epoch);
+    *wm = (w == 0xFFFFFFFFu) ? j.L.hi : std::min<int64_t>(j.L.hi, (int64_t)w);
     return FCL_SUCCESS;
 }
 
-fcl_status run_coop(Launch &L) {
-    fcl_context ctx = L.ctx;
-    Executor &ex = ctx->ex;
-    fcl_launch_info &info = ctx->info;
+Job *job_alloc(fcl_context ctx) {
+    Job *j = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(ctx->q_mu);
+        if (!ctx->free_jobs.empty()) { j = ctx->free_jobs.back(); ctx->free_jobs.pop_back(); }
+    }
+    if (!j) {
+        j = new Job();
+        for (cudaEvent_t *pe : {&j->ev_k0, &j->ev_k1, &j->ev_m0, &j->ev_m1})
+            if (cudaEventCreate(pe) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+        for (cudaEvent_t *pe : {&j->ev_start, &j->ev_staged, &j->ev_ret, &j->ev_wm, &j->ev_d2h})
+            if (cudaEventCreateWithFlags(pe, cudaEventDisableTiming) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+    }
+    j->status = FCL_SUCCESS;
+    j->done.store(0);
+    j->have_k = j->have_m = j->wm_pending = false;
+    j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = false;
+    j->unit = 1;
+    std::memset(&j->info, 0, sizeof j->info);
+    for (int q = 0; q < 6; ++q) j->twin[q] = j->stage[q] = nullptr;
+    return j;
+}
+
+void job_release_buffers(fcl_context ctx, Job &j, bool staged) {
+    if (staged) cudaEventRecord(ctx->ev_hd_release, ctx->hd);
+    for (int q = 0; q < j.L.nout; ++q) {
+        if (j.twin[q]) pool_put(ctx, j.twin[q], staged);
+        if (j.stage[q]) pool_put(ctx, j.stage[q], staged);
+        j.twin[q] = j.stage[q] = nullptr;
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// Phase A (calling thread): everything the GPU does for a cooperative launch is queued here.
+// ------------------------------------------------------------------------------------------
+fcl_status coop_phase_a(fcl_context ctx, Job &j) {
+    Launch &L = j.L;
+    fcl_launch_info &info = j.info;
     const TaskSpace ts = gpu_task_space(L.a, L.g);
-    const int64_t t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo), t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
-    info.gpu_tasks_total = t1 - t0;
-    const int64_t nwg = L.hi - L.lo;
-    const bool forced = L.o.forced_split >= 0;
-    const int64_t s_forced = forced ? std::min<int64_t>(std::max<int64_t>(L.o.forced_split, L.lo), L.hi) : -1;
+    j.t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo);
+    j.t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
+    info.gpu_tasks_total = j.t1 - j.t0;
+    info.gpu_tasks = -1;
+    j.forced = L.o.forced_split >= 0;
+    j.s_forced = j.forced ? std::min<int64_t>(std::max<int64_t>(L.o.forced_split, L.lo), L.hi) : -1;
+    constexpr int kSlots = fcl_context_st::kSlots;
 
     // a new kernel id (C14); stale status words are ignored by the dispatcher
     ctx->epoch += 1;
-    {
-        // the dispatcher that last used this launch's status slot must have exited
-        const uint32_t prev = ctx->slot_epoch[ctx->epoch % fcl_context_st::kSlots];
-        if (prev) {
-            const double tw = now_ms();
-            while ((uint32_t)(__atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE) >> 32) < prev) {
-                if (cudaStreamQuery(ctx->main) == cudaSuccess) break;
-                if (now_ms() - tw > 60000.0) return set_err(ctx, FCL_CONTEXT_LOST, "dispatcher %u never exited", prev);
-                _mm_pause();
-            }
+    j.epoch = ctx->epoch;
+    j.slot = (int)(j.epoch % kSlots);
+    if (ctx->slot_used[j.slot]) {
+        // the dispatcher that used this status slot 16 launches ago must have finished
+        const uint32_t prev = j.epoch - kSlots;
+        while (__atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE) < prev) {
+            const cudaError_t q = cudaStreamQuery(ctx->main);
+            if (q == cudaSuccess) break;
+            if (q != cudaErrorNotReady) return cuda_fail(ctx, q, "slot reuse");
+            _mm_pause();
         }
     }
-    // previous staging copies on hd must be done before the pool hands their stages out again
-    CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
-    CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_last, 0));
+    // main-stream position before this launch: this job's first staging copy waits for it,
+    // so no pool buffer is overwritten while an earlier merge still reads it.  The previous
+    // launch's end-of-dispatcher event (its merge is fused into the dispatcher) serves.
+    if (ctx->main_tail && !ctx->unfused) {
+        j.main_before = ctx->main_tail;
+    } else {
+        CK(ctx, cudaEventRecord(j.ev_start, ctx->main));
+        j.main_before = j.ev_start;
+    }
 
+    // Host chunk boundaries are aligned to the output span unit (1 work-group for 1-D kernels,
+    // one work-group row for 2-D row-major ones).  The staged spans are then exactly the host's
+    // footprint, and the only words the GPU can have written inside a merge domain are its own
+    // redundant (bit-identical) copies of host work-groups, so the device copy itself is a
+    // valid twin.  A twin is captured only when the footprint is not one span
+    // (CORR symmat: a row plus a column) or a forced split point is not span-aligned.
+    {
+        long long uw = 0, ub = 0, tot = 0;
+        bool contiguous = true;
+        for (int q = 0; q < L.nout; ++q) {
+            out_span_desc(L.a, L.g, L.out_idx[q], &uw, &ub, &tot);
+            if (uw <= 0) contiguous = false;
+            else j.unit = std::max<int64_t>(j.unit, uw);
+        }
+        const bool aligned_split = !j.forced || j.s_forced % j.unit == 0 || j.s_forced == L.hi;
+        j.twin_alias = contiguous && aligned_split && !ctx->force_twin;
+    }
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
-    void *twin[6] = {nullptr}, *stage[6] = {nullptr};
     const void *srcs[6];
     size_t nbytes[6];
+    bool hd_wait = false;
     for (int q = 0; q < L.nout; ++q) {
         fcl_buffer b = L.bufs[L.out_idx[q]];
-        twin[q] = pool_get(ctx, b->bytes);
-        stage[q] = pool_get(ctx, b->bytes);
-        if (!twin[q] || !stage[q]) return set_err(ctx, FCL_OUT_OF_RESOURCES, "twin/stage allocation of %zu bytes failed", b->bytes);
+        if (!j.twin_alias) j.twin[q] = pool_get(ctx, b->bytes, &hd_wait);
+        j.stage[q] = pool_get(ctx, b->bytes, &hd_wait);
+        if ((!j.twin_alias && !j.twin[q]) || !j.stage[q]) {
+            job_release_buffers(ctx, j, false);
+            return set_err(ctx, FCL_OUT_OF_RESOURCES, "twin/stage allocation of %zu bytes failed", b->bytes);
+        }
         srcs[q] = b->dev;
         nbytes[q] = b->bytes;
     }
-    if (gpu_launch_copies(L.nout, twin, srcs, nbytes, ctx->num_sms, ctx->main) < 0) {
-        // unaligned caller memory: fall back to per-buffer copies
-        for (int q = 0; q < L.nout; ++q)
-            CK(ctx, cudaMemcpyAsync(twin[q], srcs[q], nbytes[q], cudaMemcpyDeviceToDevice, ctx->main));
-    } else {
-        info.gpu_launches += 1;
-    }
-    auto release = [&]() {
-        for (int q = 0; q < L.nout; ++q) {
-            if (twin[q]) pool_put(ctx, twin[q]);
-            if (stage[q]) pool_put(ctx, stage[q]);
+    ctx->tr.add("A_pool", j.epoch);
+    if (hd_wait) CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_release, 0));
+    if (!j.twin_alias) {
+        if (gpu_launch_copies(L.nout, j.twin, srcs, nbytes, ctx->num_sms, ctx->main) < 0) {
+            for (int q = 0; q < L.nout; ++q)   // unaligned caller memory: per-buffer copies
+                CK(ctx, cudaMemcpyAsync(j.twin[q], srcs[q], nbytes[q], cudaMemcpyDeviceToDevice, ctx->main));
+        } else {
+            info.gpu_launches += 1;
         }
-    };
+    }
 
-    if (forced) {
+    if (j.forced) {
         // test hook: the GPU is told the split before it starts
-        fcl_status st = publish(ctx, (uint32_t)s_forced, ctx->hd);
-        if (st != FCL_SUCCESS) { release(); return st; }
-        CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
-        CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_last, 0));
+        CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
+        fcl_status st = publish(ctx, j, (uint32_t)j.s_forced);
+        if (st != FCL_SUCCESS) return st;
+        CK(ctx, cudaEventRecord(j.ev_staged, ctx->hd));
+        CK(ctx, cudaStreamWaitEvent(ctx->main, j.ev_staged, 0));
     }
 
     // GPU: the whole range, persistent dispatcher (C8)
     CoopCtl c;
-    c.status = status_slot(ctx);
-    c.epoch = ctx->epoch;
+    c.status = ctx->status_dptr + j.slot;
+    c.epoch = j.epoch;
     c.w_default = (unsigned int)L.hi;
-    c.claim = ctx->dclaim; c.done = ctx->ddone; c.wmin = ctx->dwmin; c.tasks = ctx->dtasks;
-    c.exit_rec = ctx->exit_dptr;
+    c.claim = ctx->dclaim + j.slot;
+    c.claim_next = ctx->dclaim + (j.slot + 1) % kSlots;
+    c.tasks = ctx->stats ? ctx->dtasks + j.slot : nullptr;
+    c.tasks_next = ctx->stats ? ctx->dtasks + (j.slot + 1) % kSlots : nullptr;
     c.wm_out = ctx->dwm;
-    c.check_first = forced ? 1 : 0;
-    c.task_lo = t0; c.task_hi = t1;
+    c.check_first = j.forced ? 1 : 0;
+    c.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot : nullptr;
+    c.tstamp_next = ctx->stats ? ctx->dstamp + 4 * ((j.slot + 1) % kSlots) : nullptr;
+    c.task_lo = j.t0; c.task_hi = j.t1;
     c.abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
-    bool gpu_launched = false;
-    if (t1 > t0) {
-        CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
-        if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0) {
-            release();
-            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
-        }
-        CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
-        ctx->have_k = true;
-        info.gpu_launches += 1;
-        gpu_launched = true;
-        ctx->slot_epoch[ctx->epoch % fcl_context_st::kSlots] = ctx->epoch;
-    }
-    // Free-running mode: the merge is queued right behind the dispatcher and decides its
-    // domain on the device from the watermark the dispatcher acted on, and small outputs are
-    // returned eagerly behind it -- no host round trip between the GPU finishing and the
-    // result being coherent.
-    const bool dev_merge = gpu_launched && !forced && !L.o.defer_merge;
+    c.barrier = ctx->dbar + j.slot;
+    c.barrier_next = ctx->dbar + (j.slot + 1) % kSlots;
+    c.exit_word = ctx->exit_dptr;
+    c.mg = DevMergeList{};
+    c.mg.n = 0;
+
+    // Free-running mode: the merge decides its domain on the device from the watermark the
+    // dispatcher acted on and runs in the dispatcher's fused tail (or right behind it), and
+    // small outputs are returned eagerly behind it -- no host round trip between the GPU
+    // finishing and the result being coherent.
+    j.dev_merge = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge;
     size_t out_total = 0;
     for (int q = 0; q < L.nout; ++q) {
         size_t b0, b1;
@@ -632,57 +730,105 @@ fcl_status run_coop(Launch &L) {
     // An INOUT buffer is read-modify-written in place by the host bodies: its return copy
     // must wait until the host workers have stopped (an abandoned chunk may still be running
     // when the GPU finishes), so only pure-OUT launches return eagerly.
-    const bool eager = dev_merge && !L.any_inout && out_total <= ctx->eager_return_bytes;
-    if (dev_merge) {
-        DevMergeList M{};
+    j.eager = j.dev_merge && !L.any_inout && out_total <= ctx->eager_return_bytes;
+    DevMergeList M{};
+    size_t maxb = 0;
+    if (j.dev_merge) {
         M.n = L.nout;
-        size_t maxb = 0;
         for (int q = 0; q < L.nout; ++q) {
             fcl_buffer b = L.bufs[L.out_idx[q]];
             M.gpu[q] = (unsigned char *)b->dev;
-            M.cpu[q] = (const unsigned char *)stage[q];
-            M.twin[q] = (const unsigned char *)twin[q];
+            M.cpu[q] = (const unsigned char *)j.stage[q];
+            M.twin[q] = (const unsigned char *)(j.twin_alias ? b->dev : j.twin[q]);
             M.es[q] = (int)b->elem_size;
             out_span_desc(L.a, L.g, L.out_idx[q], &M.unit_wgs[q], &M.unit_bytes[q], &M.total[q]);
             maxb = std::max(maxb, (size_t)M.total[q]);
         }
         M.wm_word = ctx->dwm;
-        M.epoch = ctx->epoch;
+        M.epoch = j.epoch;
         M.hi = L.hi;
-        CK(ctx, cudaEventRecord(ctx->ev_m0, ctx->main));
-        if (gpu_launch_merge_dev(M, maxb, ctx->num_sms, ctx->main) < 0) {
-            release();
+        M.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot + 2 : nullptr;
+        M.exit_word = ctx->exit_dptr;
+    }
+    M.wm_word = ctx->dwm;
+    M.epoch = j.epoch;
+    M.hi = L.hi;
+    c.fused = ctx->unfused ? 0 : 1;
+    if (c.fused) c.mg = M;   // mg.n == 0 (forced / deferred): barrier + exit signal only
+    c.mg.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot + 2 : nullptr;
+
+    if (j.t1 > j.t0) {
+        const bool timing = ctx->ktiming || (L.o.flags & FCL_LAUNCH_TIMING);
+        if (timing) CK(ctx, cudaEventRecord(j.ev_k0, ctx->main));
+        ctx->tr.add("A_prelaunch", j.epoch);
+        if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0)
             return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        ctx->tr.add("A_launched", j.epoch);
+        CK(ctx, cudaEventRecord(j.ev_k1, ctx->main));
+        ctx->tr.add("A_k1", j.epoch);
+        // GPU exit signal for the host executor (L18.s19): the fused tail stores the epoch to
+        // mapped host memory after its grid barrier; unfused, a bare memop does it.
+        if (!c.fused) {
+            fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->main, false);
+            if (xs != FCL_SUCCESS) return xs;
         }
-        CK(ctx, cudaEventRecord(ctx->ev_m1, ctx->main));
-        ctx->have_m = true;
+        ctx->slot_used[j.slot] = true;
+        ctx->main_tail = j.ev_k1;
+        j.have_k = timing;
         info.gpu_launches += 1;
-        if (eager) {
-            fcl_status st = enqueue_d2h(ctx, L, L.lo, L.hi, true);
-            if (st != FCL_SUCCESS) { release(); return st; }
+        j.gpu_launched = true;
+    } else {
+        // no dispatcher: reset the next launch's counters here
+        CK(ctx, cudaMemsetAsync(ctx->dclaim + (j.slot + 1) % kSlots, 0, 8, ctx->main));
+        CK(ctx, cudaMemsetAsync(ctx->dtasks + (j.slot + 1) % kSlots, 0, 8, ctx->main));
+        CK(ctx, cudaMemsetAsync(ctx->dbar + (j.slot + 1) % kSlots, 0, 4, ctx->main));
+        ctx->main_tail = nullptr;
+    }
+    if (j.dev_merge && !c.fused) {
+        if (gpu_launch_merge_dev(M, maxb, ctx->num_sms, ctx->main) < 0)
+            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        info.gpu_launches += 1;
+    }
+    if (j.dev_merge && j.eager) {
+        cudaEvent_t mark = j.ev_k1;
+        if (!c.fused) { CK(ctx, cudaEventRecord(j.ev_ret, ctx->main)); mark = j.ev_ret; }
+        fcl_status st = enqueue_d2h(ctx, L, L.lo, L.hi, info, mark);
+        if (st != FCL_SUCCESS) return st;
+    }
+    return FCL_SUCCESS;
+}
+
+// ------------------------------------------------------------------------------------------
+// Phase B (coordinator thread): descending adaptive chunks on the host (C9-C11), staged and
+// published after each (C13), until the GPU exits or the host covers the range.
+// ------------------------------------------------------------------------------------------
+fcl_status coop_phase_b(fcl_context ctx, Job &j) {
+    Launch &L = j.L;
+    Executor &ex = ctx->ex;
+    fcl_launch_info &info = j.info;
+    // host copies of every argument must be current (pending returns of earlier launches)
+    for (int k = 0; k < L.a.nbuf; ++k) {
+        fcl_buffer b = L.bufs[k];
+        if (b->d2h_pending && !(j.eager && (L.acc[k] & 2))) {
+            CK(ctx, cudaEventSynchronize(b->d2h_ev));
         }
     }
-
-    // CPU: descending adaptive chunks (C9-C11), staged and published after each (C13)
+    const int64_t nwg = L.hi - L.lo;
     const int nact = L.o.n_host_threads > 0 ? std::min(L.o.n_host_threads, ex.T) : ex.T;
-    const int64_t hi_cpu = L.hi, lo_cpu = forced ? s_forced : L.lo;
-    int64_t hi_cur = hi_cpu;
+    const int64_t lo_cpu = j.forced ? j.s_forced : L.lo;
+    int64_t hi_cur = L.hi;
     int pct = std::max(1, L.o.init_chunk_pct);
     double prev_avg = -1.0, t_start = 0.0, busy = 0.0;
     int nch = 0;
-    bool in_flight = false, gpu_done = !gpu_launched, cpu_all = false;
-    uint32_t wmin = 0xFFFFFFFFu;
-    uint64_t gtasks = 0;
+    bool in_flight = false, gpu_done = !j.gpu_launched, cpu_all = false, staged_any = false, hd_joined = false;
     int64_t cur_lo = 0, cur_hi = 0, cur_size = 0, cpu_done_wgs = 0;
-    std::vector<std::pair<int64_t, size_t>> published;   // (watermark, event index)
-    size_t nev = 0;
     ex.abort_flag = 0;
-    ex.executed.store(0);
 
     auto start_chunk = [&]() {
         int64_t size = ceil_pct(pct, nwg);
         const int64_t min_units = L.o.cpu_wg_split ? 1 : nact;   // L18.s31 without C23
         size = std::max<int64_t>(size, min_units);
+        if (j.twin_alias) size = (size + j.unit - 1) / j.unit * j.unit;   // span-aligned chunks
         size = std::min<int64_t>(size, hi_cur - lo_cpu);
         cur_hi = hi_cur; cur_lo = hi_cur - size; cur_size = size;
         const int parts = (L.o.cpu_wg_split && size < nact) ? (int)((nact + size - 1) / size) : 1;
@@ -694,35 +840,42 @@ fcl_status run_coop(Launch &L) {
         in_flight = true;
     };
     auto stage_chunk = [&](int64_t clo, int64_t chi) -> fcl_status {
+        if (!hd_joined) {
+            CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
+            hd_joined = true;
+        }
         for (int q = 0; q < L.nout; ++q) {
             fcl_buffer b = L.bufs[L.out_idx[q]];
             size_t b0, b1;
             out_span(L.a, L.g, L.out_idx[q], clo, chi, &b0, &b1);
             if (b1 > b0) {
-                CK(ctx, cudaMemcpyAsync((char *)stage[q] + b0, (char *)b->host + b0, b1 - b0, cudaMemcpyHostToDevice, ctx->hd));
+                CK(ctx, cudaMemcpyAsync((char *)j.stage[q] + b0, (char *)b->host + b0, b1 - b0, cudaMemcpyHostToDevice, ctx->hd));
                 info.h2d_bytes += (int64_t)(b1 - b0);
             }
         }
-        if (!forced && !L.o.drop_publish) {
-            fcl_status st = publish(ctx, (uint32_t)clo, ctx->hd);
+        if (!j.forced && !L.o.drop_publish) {
+            fcl_status st = publish(ctx, j, (uint32_t)clo);
             if (st != FCL_SUCCESS) return st;
         }
-        cudaEvent_t e = ev_get(ctx, nev);
-        if (!e) return set_err(ctx, FCL_OUT_OF_RESOURCES, "event pool");
-        CK(ctx, cudaEventRecord(e, ctx->hd));
-        published.push_back({clo, nev});
-        ++nev;
+        CK(ctx, cudaEventRecord(j.ev_staged, ctx->hd));
+        staged_any = true;
         info.published_watermark = clo;
         return FCL_SUCCESS;
     };
 
     info.published_watermark = L.hi;
     if (hi_cur > lo_cpu) start_chunk();
-    else cpu_all = !gpu_launched || forced;
+    else cpu_all = true;
+    unsigned spin = 0;
     while (in_flight) {
-        if (!forced && !gpu_done && poll_exit(ctx, &wmin, &gtasks)) {
-            gpu_done = true;
+        if (!j.forced && !gpu_done && __atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch) {
+            gpu_done = true;   // GPU exit (L18.s19)
+            ctx->tr.add("gpu_exit_seen", j.epoch);
             break;
+        }
+        if ((++spin & 0xFFFF) == 0 && j.gpu_launched) {   // a failed dispatcher never signals
+            const cudaError_t q = cudaEventQuery(j.ev_k1);
+            if (q != cudaSuccess && q != cudaErrorNotReady) { ex.abort_flag = 1; ex.wait(); return cuda_fail(ctx, q, "dispatcher"); }
         }
         if (ex.finished()) {
             const double dt = now_ms() - t_start;
@@ -737,7 +890,7 @@ fcl_status run_coop(Launch &L) {
             const bool more = hi_cur > lo_cpu;
             if (more) start_chunk();          // keep the workers busy while this chunk is staged
             fcl_status st = stage_chunk(clo, chi);
-            if (st != FCL_SUCCESS) { ex.abort_flag = 1; ex.wait(); release(); return st; }
+            if (st != FCL_SUCCESS) { ex.abort_flag = 1; ex.wait(); return st; }
             if (!more) { cpu_all = true; break; }
         } else {
             _mm_pause();
@@ -753,87 +906,154 @@ fcl_status run_coop(Launch &L) {
     info.n_chunks = nch;
     info.cpu_wgs = cpu_done_wgs;
     info.gpu_watermark = L.hi;
+    fcl_status st = FCL_SUCCESS;
 
-    if (dev_merge) {
-        // merge already queued; only the precise return of large outputs is left to decide
-        fcl_status st = FCL_SUCCESS;
+    if (j.dev_merge) {
+        // the merge is already queued; only the precise return of large outputs is left
         if (gpu_done) {
-            const int64_t wm = (wmin == 0xFFFFFFFFu) ? L.hi : (int64_t)wmin;
-            info.gpu_watermark = wm;
-            info.gpu_tasks = (int64_t)gtasks;
-            info.merged = wm < L.hi;
-            if (wm <= L.lo) info.cpu_did_all = 1;
-            if (!eager) st = enqueue_d2h(ctx, L, L.lo, wm, true);
+            if (!j.eager) {
+                int64_t wm = L.hi;
+                st = read_gpu_watermark(ctx, j, &wm);
+                if (st == FCL_SUCCESS) {
+                    info.gpu_watermark = wm;
+                    if (wm < L.hi) info.merged = 1;
+                    cudaEvent_t mark = j.ev_k1;
+                    st = enqueue_d2h(ctx, L, L.lo, wm, info, mark);
+                }
+            } else {
+                j.wm_pending = true;   // resolved lazily by fcl_get_launch_info
+            }
         } else {
-            info.cpu_did_all = 1;       // host authoritative (L16.s21); device merged behind
-            info.gpu_watermark = L.lo;  // refined from the exit record in fcl_get_launch_info
+            info.cpu_did_all = 1;      // host authoritative (L16.s21); device merged behind
+            info.gpu_watermark = L.lo;
             info.merged = 1;
         }
-        for (int q = 0; q < L.nout; ++q) {
-            size_t b0, b1;
-            out_span(L.a, L.g, L.out_idx[q], L.lo, L.hi, &b0, &b1);
-            if (info.merged) info.merge_bytes += (int64_t)(b1 - b0);
-        }
-        CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
-        release();
-        return st;
-    }
-
-    // Forced split / deferred merge: the host decides the merge domain and the return
-    // (C15/C17)
-    int64_t merge_lo = L.hi, ret_hi = L.hi;
-    size_t wait_ev = (size_t)-1;
-    if (forced) {
-        merge_lo = s_forced;
-        ret_hi = s_forced;
-        if (!published.empty()) wait_ev = published.back().second;
-        info.gpu_watermark = s_forced;
-        if (s_forced == L.lo) info.cpu_did_all = 1;
-    } else if (cpu_all && !gpu_done) {
-        // the host covered the range first: host copy authoritative (L16.s21); the device copy
-        // is made coherent by merging everything once the GPU has stopped (stream order)
-        merge_lo = L.lo;
-        ret_hi = L.lo;
-        if (!published.empty()) wait_ev = published.back().second;
-        info.cpu_did_all = 1;
-        info.gpu_watermark = L.lo;   // resolved when the exit record arrives (see fcl_finish)
     } else {
-        const int64_t wm = (wmin == 0xFFFFFFFFu) ? L.hi : (int64_t)wmin;
-        info.gpu_watermark = wm;
-        info.gpu_tasks = (int64_t)gtasks;
-        merge_lo = wm;
-        ret_hi = wm;
-        if (wm < L.hi) {
-            for (auto &pe : published)
-                if (pe.first == wm) wait_ev = pe.second;
-            if (wait_ev == (size_t)-1 && !published.empty()) wait_ev = published.back().second;
+        // Forced split / deferred merge: the host decides merge domain and return (C15/C17)
+        int64_t merge_lo = L.hi;
+        bool wait_staged = false;
+        if (j.forced) {
+            merge_lo = j.s_forced;
+            wait_staged = staged_any;
+        } else if (cpu_all && !gpu_done) {
+            merge_lo = L.lo;
+            wait_staged = staged_any;
+        } else if (j.gpu_launched) {
+            int64_t wm = L.hi;
+            st = read_gpu_watermark(ctx, j, &wm);
+            if (st != FCL_SUCCESS) return st;
+            merge_lo = wm;
+            wait_staged = staged_any && wm < L.hi;
         }
-        if (wm <= L.lo) info.cpu_did_all = 1;
-    }
-    if (merge_lo < L.hi) {
-        if (wait_ev != (size_t)-1) CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->evpool[wait_ev], 0));
-        fcl_status st = enqueue_merges(ctx, L, twin, stage, merge_lo, L.hi);
-        if (st != FCL_SUCCESS) { release(); return st; }
-    }
-    fcl_status st = FCL_SUCCESS;
-    if (L.o.defer_merge && merge_lo < L.hi) {
-        // the return copy must follow the merge: fcl_merge performs both
-        for (int q = 0; q < L.nout; ++q) {
-            fcl_buffer b = L.bufs[L.out_idx[q]];
-            out_span(L.a, L.g, L.out_idx[q], L.lo, ret_hi, &b->r_b0, &b->r_b1);
+        if (merge_lo <= L.lo) info.cpu_did_all = 1;
+        info.gpu_watermark = merge_lo;
+        if (merge_lo < L.hi) {
+            info.merged = 1;
+            if (wait_staged) CK(ctx, cudaStreamWaitEvent(ctx->main, j.ev_staged, 0));
+            st = enqueue_merges(ctx, j, merge_lo, L.hi);
+            if (st != FCL_SUCCESS) return st;
         }
-    } else {
-        st = enqueue_d2h(ctx, L, L.lo, ret_hi, merge_lo < L.hi);
+        if (L.o.defer_merge && merge_lo < L.hi) {
+            for (int q = 0; q < L.nout; ++q) {   // the return copy must follow the deferred merge
+                fcl_buffer b = L.bufs[L.out_idx[q]];
+                out_span(L.a, L.g, L.out_idx[q], L.lo, merge_lo, &b->r_b0, &b->r_b1);
+            }
+        } else {
+            CK(ctx, cudaEventRecord(j.ev_ret, ctx->main));   // after the host-side merges
+            st = enqueue_d2h(ctx, L, L.lo, merge_lo, info, j.ev_ret);
+        }
     }
-    CK(ctx, cudaEventRecord(ctx->ev_hd_last, ctx->hd));
-    release();
+    job_release_buffers(ctx, j, staged_any);
     return st;
+}
+
+// ------------------------------------------------------------------------------------------
+// Coordinator thread and the launch queue
+// ------------------------------------------------------------------------------------------
+void coordinator(fcl_context ctx) {
+    cudaSetDevice(ctx->device);
+    for (;;) {
+        Job *j = nullptr;
+        {
+            std::unique_lock<std::mutex> lk(ctx->q_mu);
+            ctx->q_cv.wait(lk, [&] { return ctx->q_stop || !ctx->queue.empty(); });
+            if (ctx->queue.empty()) return;   // stop requested and nothing pending
+            j = ctx->queue.front();
+            ctx->running = j;
+        }
+        fcl_status st = FCL_SUCCESS;
+        ctx->tr.add("phaseB_begin", j->epoch);
+        if (ctx->sticky.load() == FCL_SUCCESS) st = coop_phase_b(ctx, *j);
+        else st = ctx->sticky.load();
+        ctx->tr.add("phaseB_end", j->epoch);
+        {
+            std::lock_guard<std::mutex> lk(ctx->q_mu);
+            j->status = st;
+            if (st != FCL_SUCCESS && ctx->sticky.load() == FCL_SUCCESS) ctx->sticky = st;
+            ctx->queue.erase(ctx->queue.begin());
+            ctx->running = nullptr;
+            j->done.store(1, std::memory_order_release);
+            if (j != ctx->last) ctx->free_jobs.push_back(j);
+        }
+        ctx->q_cv.notify_all();
+    }
+}
+
+// Wait until every queued launch's host side is done.
+void drain(fcl_context ctx) {
+    std::unique_lock<std::mutex> lk(ctx->q_mu);
+    ctx->q_cv.wait(lk, [&] { return ctx->queue.empty(); });
+}
+
+// A new launch conflicts with a pending one if either writes a buffer the other touches.
+bool conflicts_with_pending(fcl_context ctx, const Launch &L) {
+    std::lock_guard<std::mutex> lk(ctx->q_mu);
+    for (Job *p : ctx->queue) {
+        for (int a = 0; a < L.a.nbuf; ++a)
+            for (int b = 0; b < p->L.a.nbuf; ++b)
+                if (L.bufs[a] == p->L.bufs[b] && ((L.acc[a] & 2) || (p->L.acc[b] & 2))) return true;
+    }
+    return false;
 }
 
 fcl_status check_ctx(fcl_context ctx) {
     if (!ctx) return FCL_INVALID_CONTEXT;
-    if (ctx->sticky != FCL_SUCCESS) return ctx->sticky;
+    if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
     cudaSetDevice(ctx->device);
+    return FCL_SUCCESS;
+}
+
+// ---- single-device modes (run with the queue drained) ----
+fcl_status run_gpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
+    const TaskSpace ts = gpu_task_space(L.a, L.g);
+    const int64_t t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo), t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
+    const bool timing = ctx->ktiming || (L.o.flags & FCL_LAUNCH_TIMING);
+    if (timing) CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
+    if (gpu_launch_plain(L.a, L.g, t0, t1, ctx->main) < 0)
+        return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
+    ctx->sync_have_k = timing;
+    info.gpu_launches += 1;
+    info.gpu_tasks = info.gpu_tasks_total = t1 - t0;
+    return enqueue_d2h(ctx, L, L.lo, L.hi, info, ctx->ev_k1);
+}
+
+fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
+    Executor &ex = ctx->ex;
+    const int nact = L.o.n_host_threads > 0 ? L.o.n_host_threads : ex.T;
+    const int64_t nwg = L.hi - L.lo;
+    const int parts = (L.o.cpu_wg_split && nwg < nact) ? (int)((nact + nwg - 1) / nwg) : 1;
+    const double t0 = now_ms();
+    ex.abort_flag = 0;
+    ex.submit(L.a, L.g, L.lo, L.hi, parts, nact);
+    ex.wait();
+    info.t_host_ms = now_ms() - t0;
+    info.cpu_wgs = nwg;
+    info.n_chunks = 1;
+    info.chunk_sizes[0] = (int32_t)nwg;
+    info.cpu_did_all = 1;
+    info.published_watermark = L.lo;
+    for (int q = 0; q < L.nout; ++q) L.bufs[L.out_idx[q]]->dev_valid = false;   // lazy H2D on next GPU use
     return FCL_SUCCESS;
 }
 
@@ -844,7 +1064,7 @@ fcl_status check_ctx(fcl_context ctx) {
 // ==========================================================================================
 extern "C" {
 
-const char *fcl_version(void) { return "fcl-b200 0.1 sm_100a"; }
+const char *fcl_version(void) { return "fcl-b200 0.2 sm_100a"; }
 
 const char *fcl_status_string(fcl_status s) {
     switch (s) {
@@ -867,7 +1087,13 @@ const char *fcl_status_string(fcl_status s) {
     }
 }
 
-const char *fcl_last_error(fcl_context ctx) { return ctx ? ctx->err.c_str() : "no context"; }
+const char *fcl_last_error(fcl_context ctx) {
+    if (!ctx) return "no context";
+    std::lock_guard<std::mutex> lk(ctx->err_mu);
+    static thread_local std::string copy;
+    copy = ctx->err;
+    return copy.c_str();
+}
 
 fcl_status fcl_default_launch_opts(fcl_launch_opts *o) {
     if (!o) return FCL_INVALID_VALUE;
@@ -880,6 +1106,7 @@ fcl_status fcl_default_launch_opts(fcl_launch_opts *o) {
     o->abort_period = 0;
     o->wg_lo = 0;
     o->wg_hi = 0;
+    o->blocking = 0;
     return FCL_SUCCESS;
 }
 
@@ -896,8 +1123,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->device = d.device;
     ctx->status_location = d.status_location;
     auto fail = [&](cudaError_t e, const char *what) {
-        set_err(ctx, FCL_CUDA_ERROR, "%s: %s", what, cudaGetErrorString(e));
-        fprintf(stderr, "fcl_create_context: %s\n", ctx->err.c_str());
+        fprintf(stderr, "fcl_create_context: %s: %s\n", what, cudaGetErrorString(e));
         delete ctx;
         return FCL_CUDA_ERROR;
     };
@@ -913,13 +1139,15 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if ((e = mk(d.main_stream, &ctx->main, &ctx->own_main)) != cudaSuccess) return fail(e, "main stream");
     if ((e = mk(d.hd_stream, &ctx->hd, &ctx->own_hd)) != cudaSuccess) return fail(e, "hd stream");
     if ((e = mk(d.dh_stream, &ctx->dh, &ctx->own_dh)) != cudaSuccess) return fail(e, "dh stream");
-    // status word and exit record
-    void *hp = nullptr;
-    if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "exit record");
+    // status words (one per launch slot), GPU-exit word, pinned copy of the wm word
+    void *hp = nullptr, *dp = nullptr;
+    if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocPortable)) != cudaSuccess) return fail(e, "pinned scratch");
+    std::memset(hp, 0, 64);
+    ctx->wm_host = (unsigned long long *)hp;
+    if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "exit word");
     std::memset(hp, 0, 64);
     ctx->exit_host = (unsigned long long *)hp;
-    void *dp = nullptr;
-    if ((e = cudaHostGetDevicePointer(&dp, hp, 0)) != cudaSuccess) return fail(e, "exit record mapping");
+    if ((e = cudaHostGetDevicePointer(&dp, hp, 0)) != cudaSuccess) return fail(e, "exit word mapping");
     ctx->exit_dptr = (unsigned long long *)dp;
     if (d.status_location == FCL_STATUS_HOST_MAPPED) {
         if ((e = cudaHostAlloc(&hp, 8 * fcl_context_st::kSlots, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "status word");
@@ -932,20 +1160,18 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
         cudaMemset(dp, 0, 8 * fcl_context_st::kSlots);
         ctx->status_dptr = (unsigned long long *)dp;
     }
-    // device counters: claim (u64), tasks (u64), done (u32), wmin (u32)
-    if ((e = cudaMalloc(&dp, 64)) != cudaSuccess) return fail(e, "counters");
-    cudaMemset(dp, 0, 64);
+    // device counters: claim[kSlots], tasks[kSlots], wm word, stamps[4 * kSlots], barrier[kSlots]
+    if ((e = cudaMalloc(&dp, 8 * (7 * fcl_context_st::kSlots + 2))) != cudaSuccess) return fail(e, "counters");
+    cudaMemset(dp, 0, 8 * (7 * fcl_context_st::kSlots + 2));
     ctx->dclaim = (unsigned long long *)dp;
-    ctx->dtasks = ctx->dclaim + 1;
-    ctx->ddone = (unsigned int *)(ctx->dclaim + 2);
-    ctx->dwmin = ctx->ddone + 1;
-    ctx->dwm = ctx->dclaim + 3;
-    const unsigned int ff = 0xFFFFFFFFu;
-    if ((e = cudaMemcpy(ctx->dwmin, &ff, 4, cudaMemcpyHostToDevice)) != cudaSuccess) return fail(e, "counter init");
-    for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1, &ctx->ev_m0, &ctx->ev_m1})
+    ctx->dtasks = ctx->dclaim + fcl_context_st::kSlots;
+    ctx->dwm = ctx->dtasks + fcl_context_st::kSlots;
+    ctx->dstamp = ctx->dwm + 2;
+    ctx->dbar = (unsigned int *)(ctx->dstamp + 4 * fcl_context_st::kSlots);
+    for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1})
         if ((e = cudaEventCreate(pe)) != cudaSuccess) return fail(e, "events");
-    if ((e = cudaEventCreateWithFlags(&ctx->ev_hd_last, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
-    if ((e = cudaEventCreateWithFlags(&ctx->ev_mark, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
+    for (cudaEvent_t *pe : {&ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h})
+        if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
     // stream memory operations for publication (driver entry point; fall back to a kernel store)
     {
         void *fn = nullptr;
@@ -958,12 +1184,18 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     }
     if (getenv("FCL_NO_MEMOPS")) ctx->write64 = nullptr;
     if (getenv("FCL_EAGER_RETURN_BYTES")) ctx->eager_return_bytes = (size_t)atoll(getenv("FCL_EAGER_RETURN_BYTES"));
+    ctx->stats = getenv("FCL_STATS") && atoi(getenv("FCL_STATS")) != 0;
+    ctx->tr.on = getenv("FCL_TRACE") && atoi(getenv("FCL_TRACE")) != 0;
+    ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
+    ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
+    if (getenv("FCL_KTIMING")) ctx->ktiming = atoi(getenv("FCL_KTIMING")) != 0;
     if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail(e, "init sync");
     const char *pin = getenv("FCL_PIN_THREADS");
     const bool do_pin = d.pin_threads ? true : (pin ? atoi(pin) != 0 : true);
     int nthr = d.n_host_threads;
     if (nthr <= 0 && getenv("FCL_HOST_THREADS")) nthr = atoi(getenv("FCL_HOST_THREADS"));
     ctx->ex.start(nthr, do_pin);
+    ctx->coord = std::thread(coordinator, ctx);
     *out = ctx;
     return FCL_SUCCESS;
 }
@@ -971,14 +1203,40 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
 fcl_status fcl_release_context(fcl_context ctx) {
     if (!ctx) return FCL_INVALID_CONTEXT;
     cudaSetDevice(ctx->device);
+    drain(ctx);
+    if (ctx->tr.on) {
+        const char *path = getenv("FCL_TRACE_FILE");
+        FILE *f = path ? fopen(path, "w") : stderr;
+        if (f) {
+            for (auto &r : ctx->tr.recs) fprintf(f, "%.4f %s %u\n", r.t, r.tag, r.epoch);
+            if (f != stderr) fclose(f);
+        }
+    }
+    {
+        std::lock_guard<std::mutex> lk(ctx->q_mu);
+        ctx->q_stop = true;
+    }
+    ctx->q_cv.notify_all();
+    if (ctx->coord.joinable()) ctx->coord.join();
     cudaDeviceSynchronize();
     ctx->ex.shutdown();
     for (auto &pe : ctx->pool) cudaFree(pe.p);
-    for (auto e : ctx->evpool) cudaEventDestroy(e);
-    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_k1, ctx->ev_m0, ctx->ev_m1, ctx->ev_hd_last, ctx->ev_mark})
+    for (Job *j : ctx->free_jobs) {
+        for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
+            if (e) cudaEventDestroy(e);
+        delete j;
+    }
+    if (ctx->last && ctx->last->done.load()) {
+        Job *j = ctx->last;
+        for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
+            if (e) cudaEventDestroy(e);
+        delete j;
+    }
+    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_k1, ctx->ev_mark, ctx->ev_hd_release, ctx->ev_gd2h})
         if (e) cudaEventDestroy(e);
     if (ctx->status_host) cudaFreeHost(ctx->status_host);
     else if (ctx->status_dptr) cudaFree(ctx->status_dptr);
+    if (ctx->wm_host) cudaFreeHost(ctx->wm_host);
     if (ctx->exit_host) cudaFreeHost(ctx->exit_host);
     if (ctx->dclaim) cudaFree(ctx->dclaim);
     if (ctx->own_main) cudaStreamDestroy(ctx->main);
@@ -1051,12 +1309,13 @@ fcl_status fcl_release_buffer(fcl_buffer b) {
     if (!b) return FCL_INVALID_MEM_OBJECT;
     fcl_context ctx = b->ctx;
     cudaSetDevice(ctx->device);
+    drain(ctx);
     cudaStreamSynchronize(ctx->main);
     cudaStreamSynchronize(ctx->hd);
     cudaStreamSynchronize(ctx->dh);
     if (b->merge_pending) {
-        if (b->twin) pool_put(ctx, b->twin);
-        if (b->stage) pool_put(ctx, b->stage);
+        if (b->twin) pool_put(ctx, b->twin, false);
+        if (b->stage) pool_put(ctx, b->stage, false);
         ctx->defer_list.erase(std::remove(ctx->defer_list.begin(), ctx->defer_list.end(), b), ctx->defer_list.end());
     }
     if (b->own_dev) cudaFree(b->dev);
@@ -1071,18 +1330,17 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
     if (s != FCL_SUCCESS) return s;
     if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
     if (!src || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "write range");
+    drain(ctx);
     if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
-    // the rest of the buffer must be current on both sides before a partial write
     char *h = (char *)b->host + offset;
     if (n < b->bytes) {
-        fcl_status st = make_valid(ctx, b, true, true);
-        if (st != FCL_SUCCESS) return st;
+        s = make_valid(ctx, b, true, true, nullptr);
+        if (s != FCL_SUCCESS) return s;
     }
     // overwriting the pinned mirror: no queued copy may still read its old contents
     if (src != h) CK(ctx, cudaStreamSynchronize(ctx->main));
     if (src != h) std::memcpy(h, src, n);
     CK(ctx, cudaMemcpyAsync((char *)b->dev + offset, h, n, cudaMemcpyHostToDevice, ctx->main));
-    ctx->info.h2d_bytes += (int64_t)n;
     b->host_valid = b->dev_valid = true;
     if (blocking) CK(ctx, cudaStreamSynchronize(ctx->main));
     return FCL_SUCCESS;
@@ -1094,6 +1352,7 @@ fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t 
     if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
     if (!dst || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "read range");
     (void)blocking;
+    drain(ctx);
     if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
     if (b->host_valid) {   // location tracking (L20.s31-33): no transfer when the host is current
         const char *h = (const char *)b->host + offset;
@@ -1187,6 +1446,7 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
                 return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %s is written by %s: access must be OUT/INOUT", sp.name, kd->name);
             if (ar.buffer->elem_size != 4) return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "arg %s: elem_size must be 4", sp.name);
             L.bufs[nb] = ar.buffer;
+            L.acc[nb] = sp.acc;
             a.dev[nb] = ar.buffer->dev;
             a.host[nb] = ar.buffer->host;
             if (sp.acc & 2) L.out_idx[L.nout++] = nb;
@@ -1213,6 +1473,10 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
         if ((int64_t)L.bufs[k]->bytes < need)
             return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "buffer arg %d holds %zu bytes, needs %lld", k, L.bufs[k]->bytes, (long long)need);
     }
+    for (int x = 0; x < nb; ++x)
+        for (int y = x + 1; y < nb; ++y)
+            if (L.bufs[x] == L.bufs[y] && ((L.acc[x] & 2) || (L.acc[y] & 2)))
+                return set_err(ctx, FCL_INVALID_KERNEL_ARGS, "a written buffer is passed twice (args alias)");
     int64_t ext[3];
     required_extent(a.kernel, a.n0, a.n1, ext);
     for (uint32_t d = 0; d < work_dim; ++d)
@@ -1243,28 +1507,83 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     Launch L{};
     s = build_launch(ctx, kernel, work_dim, gws, lws, args, n_args, opts, L);
     if (s != FCL_SUCCESS) return s;
-    if (!ctx->defer_list.empty()) return set_err(ctx, FCL_INVALID_VALUE, "a deferred merge is pending (call fcl_merge)");
-    std::memset(&ctx->info, 0, sizeof ctx->info);
-    ctx->have_k = ctx->have_m = false;
-    fcl_launch_info &info = ctx->info;
-    info.n_wg = L.hi - L.lo;
-    info.wg_lo = L.lo;
-    info.wg_hi = L.hi;
+    if (!ctx->defer_list.empty()) {
+        drain(ctx);
+        if (!ctx->defer_list.empty()) return set_err(ctx, FCL_INVALID_VALUE, "a deferred merge is pending (call fcl_merge)");
+    }
+    const bool coop = L.o.mode == FCL_MODE_COOP;
+    ctx->tr.add("enq_begin", ctx->epoch + 1);
+    // The single-device modes and any launch that conflicts with a pending one wait for the
+    // pending launches' host sides first (the cross-launch hazards the paper's version
+    // tracking resolves, L20.s1-9; here conservatively by draining).
+    bool host_needed = false;
+    for (int k = 0; k < L.a.nbuf; ++k) host_needed |= !L.bufs[k]->host_valid || !L.bufs[k]->dev_valid;
+    if (!coop || host_needed || L.o.blocking || conflicts_with_pending(ctx, L)) drain(ctx);
+    if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
+
+    if (!coop) {
+        ctx->main_tail = nullptr;   // later launches record their own main position
+        fcl_launch_info &info = ctx->sync_info;
+        std::memset(&info, 0, sizeof info);
+        info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
+        info.gpu_watermark = info.published_watermark = L.hi;
+        ctx->sync_have_k = false;
+        for (int k = 0; k < L.a.nbuf; ++k) {
+            const bool is_out = (L.acc[k] & 2) != 0;
+            const bool need_host = L.o.mode != FCL_MODE_GPU_ONLY || is_out;
+            const bool need_dev = L.o.mode != FCL_MODE_CPU_ONLY;
+            s = make_valid(ctx, L.bufs[k], need_host, need_dev, &info);
+            if (s != FCL_SUCCESS) return s;
+        }
+        s = (L.o.mode == FCL_MODE_GPU_ONLY) ? run_gpu_only(ctx, L, info) : run_cpu_only(ctx, L, info);
+        info.t_call_ms = now_ms() - t_call;
+        {
+            std::lock_guard<std::mutex> lk(ctx->q_mu);
+            if (ctx->last && ctx->last->done.load()) ctx->free_jobs.push_back(ctx->last);
+            ctx->last = nullptr;
+        }
+        if (info_out) *info_out = info;
+        return s;
+    }
+
+    // cooperative launch: both copies of every argument must be current
+    Job *j = job_alloc(ctx);
+    if (!j) return set_err(ctx, FCL_OUT_OF_RESOURCES, "job allocation");
+    j->L = L;
+    fcl_launch_info &info = j->info;
+    info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
     info.gpu_watermark = info.published_watermark = L.hi;
-    // coherence of every argument for the chosen mode (minimal location tracking)
     for (int k = 0; k < L.a.nbuf; ++k) {
-        const bool is_out = std::find(L.out_idx, L.out_idx + L.nout, k) != L.out_idx + L.nout;
-        const bool need_host = L.o.mode != FCL_MODE_GPU_ONLY || is_out;
-        const bool need_dev = L.o.mode != FCL_MODE_CPU_ONLY;
-        s = make_valid(ctx, L.bufs[k], need_host, need_dev);
-        if (s != FCL_SUCCESS) return s;
+        fcl_buffer b = L.bufs[k];
+        // (both copies are valid here: anything else drained above.)  A pending return copy
+        // of a buffer this launch writes still reads its device copy: order the overwrite
+        // behind it on the device; the host side of the hazard is resolved in phase B.
+        if (b->d2h_pending && (L.acc[k] & 2)) {
+            const cudaError_t e = cudaStreamWaitEvent(ctx->main, b->d2h_ev, 0);
+            if (e != cudaSuccess) { s = cuda_fail(ctx, e, "stream wait"); break; }
+        }
     }
-    switch (L.o.mode) {
-    case FCL_MODE_GPU_ONLY: s = run_gpu_only(L); break;
-    case FCL_MODE_CPU_ONLY: s = run_cpu_only(L); break;
-    default: s = run_coop(L); break;
+    ctx->tr.add("phaseA_begin", ctx->epoch + 1);
+    if (s == FCL_SUCCESS) s = coop_phase_a(ctx, *j);
+    ctx->tr.add("phaseA_end", j->epoch);
+    if (s != FCL_SUCCESS) {
+        job_release_buffers(ctx, *j, false);
+        std::lock_guard<std::mutex> lk(ctx->q_mu);
+        ctx->free_jobs.push_back(j);
+        return s;
     }
+    {
+        std::lock_guard<std::mutex> lk(ctx->q_mu);
+        if (ctx->last && ctx->last != j && ctx->last->done.load()) ctx->free_jobs.push_back(ctx->last);
+        ctx->last = j;
+        ctx->queue.push_back(j);
+    }
+    ctx->q_cv.notify_all();
     pool_trim(ctx);
+    if (L.o.blocking) {
+        drain(ctx);
+        s = j->status;
+    }
     info.t_call_ms = now_ms() - t_call;
     if (info_out) *info_out = info;
     return s;
@@ -1274,10 +1593,13 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
     fcl_status s = check_ctx(ctx);
     if (s != FCL_SUCCESS) return s;
     if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
+    drain(ctx);
     if (!b->merge_pending) return FCL_SUCCESS;
-    if (gpu_launch_merge((char *)b->dev + b->m_b0, (char *)b->stage + b->m_b0, (char *)b->twin + b->m_b0,
+    const char *tw = b->twin ? (const char *)b->twin : (const char *)b->dev;
+    if (gpu_launch_merge((char *)b->dev + b->m_b0, (char *)b->stage + b->m_b0, tw + b->m_b0,
                          b->m_b1 - b->m_b0, (int)b->elem_size, ctx->num_sms, ctx->main) < 0)
         return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    ctx->main_tail = nullptr;
     CK(ctx, cudaEventRecord(ctx->ev_mark, ctx->main));
     CK(ctx, cudaStreamWaitEvent(ctx->hd, ctx->ev_mark, 0));   // pool reuse is ordered after the merge
     if (b->r_b1 > b->r_b0) {
@@ -1288,8 +1610,8 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
         b->d2h_pending = true;
     }
     b->r_b0 = b->r_b1 = 0;
-    pool_put(ctx, b->twin);
-    pool_put(ctx, b->stage);
+    if (b->twin) pool_put(ctx, b->twin, false);
+    pool_put(ctx, b->stage, false);
     b->twin = b->stage = nullptr;
     b->merge_pending = false;
     ctx->defer_list.erase(std::remove(ctx->defer_list.begin(), ctx->defer_list.end(), b), ctx->defer_list.end());
@@ -1308,12 +1630,28 @@ fcl_status fcl_merge_raw(void *gpu, const void *cpu, const void *twin, size_t by
 
 fcl_status fcl_finish(fcl_context ctx) {
     if (!ctx) return FCL_INVALID_CONTEXT;
-    if (ctx->sticky != FCL_SUCCESS) return ctx->sticky;
     cudaSetDevice(ctx->device);
+    ctx->tr.add("finish_begin", ctx->epoch);
+    drain(ctx);
+    ctx->tr.add("finish_drained", ctx->epoch);
+    if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
     CK(ctx, cudaStreamSynchronize(ctx->main));
     CK(ctx, cudaStreamSynchronize(ctx->hd));
     CK(ctx, cudaStreamSynchronize(ctx->dh));
     CK(ctx, cudaGetLastError());
+    ctx->tr.add("finish_end", ctx->epoch);
+    if (ctx->tr.on && ctx->stats) {
+        unsigned long long st[4 * fcl_context_st::kSlots];
+        if (cudaMemcpy(st, ctx->dstamp, sizeof st, cudaMemcpyDeviceToHost) == cudaSuccess) {
+            std::lock_guard<std::mutex> lk(ctx->tr.mu);
+            for (int k = 0; k < fcl_context_st::kSlots; ++k) {
+                static const char *names[4] = {"gpu_disp_start_ns", "gpu_disp_end_ns", "gpu_merge_start_ns", "gpu_merge_end_ns"};
+                for (int q = 0; q < 4; ++q)
+                    if (st[4 * k + q] && st[4 * k + q] != ~0ull)
+                        ctx->tr.recs.push_back({(double)(st[4 * k + q] % 1000000000000ull) * 1e-6, names[q], (uint32_t)k});
+            }
+        }
+    }
     return FCL_SUCCESS;
 }
 
@@ -1321,25 +1659,46 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info) {
     if (!ctx) return FCL_INVALID_CONTEXT;
     if (!info) return FCL_INVALID_VALUE;
     cudaSetDevice(ctx->device);
-    if (ctx->have_k) {
+    drain(ctx);
+    Job *j = ctx->last;
+    if (!j) {   // the last launch was a single-device one
+        if (ctx->sync_have_k) {
+            float ms = 0.f;
+            if (cudaEventSynchronize(ctx->ev_k1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_k0, ctx->ev_k1) == cudaSuccess)
+                ctx->sync_info.t_gpu_kernel_ms = ms;
+        }
+        cudaGetLastError();
+        *info = ctx->sync_info;
+        return FCL_SUCCESS;
+    }
+    if (j->have_k) {
         float ms = 0.f;
-        if (cudaEventSynchronize(ctx->ev_k1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_k0, ctx->ev_k1) == cudaSuccess)
-            ctx->info.t_gpu_kernel_ms = ms;
-        // the exit record of a cooperative launch that finished after the host returned
-        uint32_t wm;
-        uint64_t nt;
-        if (poll_exit(ctx, &wm, &nt)) {
-            ctx->info.gpu_tasks = (int64_t)nt;
-            if (!ctx->info.cpu_did_all) ctx->info.gpu_watermark = (wm == 0xFFFFFFFFu) ? ctx->info.wg_hi : (int64_t)wm;
+        if (cudaEventSynchronize(j->ev_k1) == cudaSuccess && cudaEventElapsedTime(&ms, j->ev_k0, j->ev_k1) == cudaSuccess)
+            j->info.t_gpu_kernel_ms = ms;
+        // the watermark of a cooperative launch whose host side did not need it (valid while
+        // no later dispatcher has run: this is the most recent launch and the queue is drained)
+        if (j->wm_pending) {
+            int64_t wm = j->L.hi;
+            if (read_gpu_watermark(ctx, *j, &wm) == FCL_SUCCESS) {
+                j->info.gpu_watermark = wm;
+                j->info.merged = wm < j->L.hi;
+                if (wm <= j->L.lo) j->info.cpu_did_all = 1;
+            }
+            j->wm_pending = false;
+        }
+        if (ctx->stats && j->info.gpu_tasks < 0) {
+            unsigned long long nt = 0;
+            if (cudaMemcpy(&nt, ctx->dtasks + j->slot, 8, cudaMemcpyDeviceToHost) == cudaSuccess)
+                j->info.gpu_tasks = (int64_t)nt;
         }
     }
-    if (ctx->have_m) {
+    if (j->have_m) {
         float ms = 0.f;
-        if (cudaEventSynchronize(ctx->ev_m1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_m0, ctx->ev_m1) == cudaSuccess)
-            ctx->info.t_merge_ms = ms;
+        if (cudaEventSynchronize(j->ev_m1) == cudaSuccess && cudaEventElapsedTime(&ms, j->ev_m0, j->ev_m1) == cudaSuccess)
+            j->info.t_merge_ms = ms;
     }
     cudaGetLastError();
-    *info = ctx->info;
+    *info = j->info;
     return FCL_SUCCESS;
 }
 
@@ -1360,9 +1719,6 @@ fcl_status fcl_slice_range(fcl_kernel kernel, uint32_t work_dim, const size_t gw
     KArgs a{};
     a.kernel = kernel->def->id;
     a.integer = kernel->def->integer;
-    int64_t ext[3] = {g.gws[0], g.gws[1], 1};
-    (void)ext;
-    a.n0 = a.n1 = 0;
     const int64_t al = gpu_slice_align(a, g);
     const int64_t units = (g.n_wg + al - 1) / al;
     const int64_t u0 = units * rank / nranks, u1 = units * (rank + 1) / nranks;

@@ -25,6 +25,7 @@ ARG_BUFFER, ARG_INT, ARG_FLOAT = 0, 1, 2
 ACCESS_IN, ACCESS_OUT, ACCESS_INOUT = 1, 2, 3
 MODE_COOP, MODE_GPU_ONLY, MODE_CPU_ONLY = 0, 1, 2
 STATUS_DEVICE, STATUS_HOST_MAPPED = 0, 1
+LAUNCH_TIMING = 1
 MODES = {"coop": MODE_COOP, "gpu": MODE_GPU_ONLY, "gpu_only": MODE_GPU_ONLY,
          "cpu": MODE_CPU_ONLY, "cpu_only": MODE_CPU_ONLY}
 
@@ -56,7 +57,8 @@ class LaunchOpts(ctypes.Structure):
                 ("cpu_wg_split", ctypes.c_int32), ("abort_period", ctypes.c_int32),
                 ("defer_merge", ctypes.c_int32), ("n_host_threads", ctypes.c_int32),
                 ("host_delay_us", ctypes.c_int32), ("drop_publish", ctypes.c_int32),
-                ("wg_lo", ctypes.c_int64), ("wg_hi", ctypes.c_int64)]
+                ("wg_lo", ctypes.c_int64), ("wg_hi", ctypes.c_int64),
+                ("blocking", ctypes.c_int32), ("flags", ctypes.c_int32)]
 
 
 class LaunchInfo(ctypes.Structure):
@@ -210,7 +212,7 @@ class Kernel:
 
 def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg_split=1,
               abort_period=0, defer_merge=0, n_host_threads=0, host_delay_us=0, drop_publish=0,
-              wg_lo=0, wg_hi=0) -> LaunchOpts:
+              wg_lo=0, wg_hi=0, blocking=0, timing=0) -> LaunchOpts:
     o = LaunchOpts()
     load().fcl_default_launch_opts(ctypes.byref(o))
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
@@ -219,6 +221,8 @@ def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg
     o.abort_period, o.defer_merge, o.n_host_threads = int(abort_period), int(defer_merge), int(n_host_threads)
     o.host_delay_us, o.drop_publish = int(host_delay_us), int(drop_publish)
     o.wg_lo, o.wg_hi = int(wg_lo), int(wg_hi)
+    o.blocking = int(blocking)
+    o.flags = LAUNCH_TIMING if timing else 0
     return o
 
 

@@ -52,7 +52,7 @@ def test_struct_layouts_match_header():
     # offsets the C compiler uses for the public structs (x86-64 SysV)
     assert ctypes.sizeof(fcl.ContextDesc) == 40
     assert ctypes.sizeof(fcl.Arg) == 32
-    assert fcl.LaunchOpts.forced_split.offset == 8 and ctypes.sizeof(fcl.LaunchOpts) == 64
+    assert fcl.LaunchOpts.forced_split.offset == 8 and ctypes.sizeof(fcl.LaunchOpts) == 72
     assert fcl.LaunchInfo.t_call_ms.offset == 104 and ctypes.sizeof(fcl.LaunchInfo) == 392
 
 

@@ -98,9 +98,12 @@ def test_forced_splits_bit_identical(ctx, oracle_mod, case):
 
 
 @pytest.mark.parametrize("case", CASES, ids=_ids)
-@pytest.mark.parametrize("status", ["host_mapped", "device"])
-def test_free_running_coop(oracle_mod, case, status):
+@pytest.mark.parametrize("status,twin", [("device", "alias"), ("device", "twin"), ("host_mapped", "alias")])
+def test_free_running_coop(oracle_mod, case, status, twin, monkeypatch):
+    """Free-running race; with the twin aliased to the device copy (exact spans, default) and
+    with a captured twin (Fig 9 as printed, FCL_FORCE_TWIN=1)."""
     from paper_conf_cgo_panditg14_b200 import fcl
+    monkeypatch.setenv("FCL_FORCE_TWIN", "1" if twin == "twin" else "0")
     ctx = fcl.Context(0, status_location=status)
     try:
         P = _problem(case, seed=2)
@@ -218,4 +221,38 @@ def test_corr_chain_coop_vs_oracle(ctx, oracle_mod):
     assert_parity(mean.read_array(np.float32), mean64, False, "corr mean")
     assert_parity(d.read_array(np.float32), d64, False, "corr reduced data")
     for b in (d, mean, std, sym):
+        b.release()
+
+
+def test_async_independent_launches(ctx):
+    """Non-blocking enqueue: independent launches queue their GPU work back to back while the
+    coordinator runs their host sides in order; results match the single-device ones."""
+    cases = [CASES[8], CASES[9], CASES[4], CASES[6], CASES[11], CASES[16], CASES[19], CASES[1]]
+    probs = [_problem(c, seed=9 + k) for k, c in enumerate(cases)]
+    refs = [H.run(ctx, P, mode="gpu")[0] for P in probs]
+    bufs = [H.create_buffers(ctx, P) for P in probs]
+    for rep in range(3):
+        for P, b in zip(probs, bufs):
+            ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode="coop",
+                                host_delay_us=[0, 30, 300][rep])
+        ctx.finish()
+        for P, b, ref in zip(probs, bufs, refs):
+            if P.inout_indices:      # INOUT kernels accumulate across repetitions: reset input
+                continue
+            dt = np.int32 if P.integer else np.float32
+            for k in P.out_indices:
+                assert_bits(b[k].read_array(dt), ref[k], f"{P.kernel} rep {rep} host")
+                assert_bits(H.device_array(b[k], dt), ref[k], f"{P.kernel} rep {rep} device")
+    for bl in bufs:
+        for b in bl:
+            b.release()
+
+
+def test_blocking_launch_reports_complete_info(ctx):
+    P = W.make("gesummv", 1024, seed=5, lws1d=256)
+    bufs = H.create_buffers(ctx, P)
+    info = ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, bufs), mode="coop", blocking=1)
+    assert info["n_wg"] == 4 and info["gpu_launches"] >= 1
+    ctx.finish()
+    for b in bufs:
         b.release()
