@@ -234,12 +234,16 @@ void wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, 
     // transposed column operands: Xt[k * wc + jj] = X[j0 + jj][k]
     thread_local std::vector<T> At, Bt, acc;
     At.resize((size_t)m * (size_t)wc);
-    for (int64_t jj = 0; jj < wc; ++jj)
+    for (int64_t jj = 0; jj < wc; ++jj) {
+        if (aborted(ab)) return;
         for (int64_t k = 0; k < m; ++k) At[(size_t)(k * wc + jj)] = A[(j0 + jj) * m + k];
+    }
     if (TWO) {
         Bt.resize((size_t)m * (size_t)wc);
-        for (int64_t jj = 0; jj < wc; ++jj)
+        for (int64_t jj = 0; jj < wc; ++jj) {
+            if (aborted(ab)) return;
             for (int64_t k = 0; k < m; ++k) Bt[(size_t)(k * wc + jj)] = B[(j0 + jj) * m + k];
+        }
     }
     acc.resize((size_t)wc);
     for (int64_t i = w.r0 + rlo; i < w.r0 + rhi; ++i) {
@@ -249,6 +253,7 @@ void wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, 
         const T *ai = A + i * m;
         const T *bi = TWO ? B + i * m : nullptr;
         for (int64_t k = 0; k < m; ++k) {
+            if ((k & 511) == 511 && aborted(ab)) return;   // write-once: nothing stored yet
             const T aik = ai[k];
             if (TWO) {
                 const T bik = bi[k];

@@ -475,10 +475,18 @@ fcl_status publish(fcl_context ctx, const Job &j, uint32_t w) {
     return stream_store(ctx, ctx->status_dptr + j.slot, v, ctx->hd);
 }
 
-fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_dev, fcl_launch_info *info) {
+// Bring a buffer's copies to what a launch needs.  A pending return copy is waited for on the
+// host only when the host copy is needed; a device-only use of a buffer the launch writes is
+// ordered behind it on the device (write-after-read), and device-only reads need nothing.
+fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_dev, fcl_launch_info *info,
+                      bool dev_write = true) {
     if (b->d2h_pending) {
-        CK(ctx, cudaEventSynchronize(b->d2h_ev));
-        b->d2h_pending = false;
+        if (need_host || !b->dev_valid) {
+            CK(ctx, cudaEventSynchronize(b->d2h_ev));
+            b->d2h_pending = false;
+        } else if (dev_write) {
+            CK(ctx, cudaStreamWaitEvent(ctx->main, b->d2h_ev, 0));
+        }
     }
     if (need_dev && !b->dev_valid) {
         CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
@@ -912,17 +920,13 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         // the merge is already queued; only the precise return of large outputs is left
         if (gpu_done) {
             if (!j.eager) {
-                int64_t wm = L.hi;
-                st = read_gpu_watermark(ctx, j, &wm);
-                if (st == FCL_SUCCESS) {
-                    info.gpu_watermark = wm;
-                    if (wm < L.hi) info.merged = 1;
-                    cudaEvent_t mark = j.ev_k1;
-                    st = enqueue_d2h(ctx, L, L.lo, wm, info, mark);
-                }
-            } else {
-                j.wm_pending = true;   // resolved lazily by fcl_get_launch_info
+                // The host copy already holds every published chunk, and the GPU acted on some
+                // watermark >= the lowest one published, so returning the device copy (merged
+                // by the fused tail) below the host's own published watermark is complete --
+                // no device read of the GPU's watermark on this path.
+                st = enqueue_d2h(ctx, L, L.lo, info.published_watermark, info, j.ev_k1);
             }
+            j.wm_pending = true;   // info.gpu_watermark resolved lazily by fcl_get_launch_info
         } else {
             info.cpu_did_all = 1;      // host authoritative (L16.s21); device merged behind
             info.gpu_watermark = L.lo;
@@ -1530,10 +1534,18 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         ctx->sync_have_k = false;
         for (int k = 0; k < L.a.nbuf; ++k) {
             const bool is_out = (L.acc[k] & 2) != 0;
-            const bool need_host = L.o.mode != FCL_MODE_GPU_ONLY || is_out;
+            // GPU-only: the host copy of an output is only rewritten by the return copy (which
+            // is ordered behind earlier ones on dh), so it need not be current; CPU-only reads
+            // and writes host copies
+            const bool need_host = L.o.mode == FCL_MODE_CPU_ONLY;
             const bool need_dev = L.o.mode != FCL_MODE_CPU_ONLY;
-            s = make_valid(ctx, L.bufs[k], need_host, need_dev, &info);
+            s = make_valid(ctx, L.bufs[k], need_host, need_dev, &info, is_out);
             if (s != FCL_SUCCESS) return s;
+            if (L.o.mode == FCL_MODE_GPU_ONLY && is_out && !L.bufs[k]->host_valid) {
+                // partially returned outputs: the rest of the host copy must be current first
+                s = make_valid(ctx, L.bufs[k], true, true, &info);
+                if (s != FCL_SUCCESS) return s;
+            }
         }
         s = (L.o.mode == FCL_MODE_GPU_ONLY) ? run_gpu_only(ctx, L, info) : run_cpu_only(ctx, L, info);
         info.t_call_ms = now_ms() - t_call;
