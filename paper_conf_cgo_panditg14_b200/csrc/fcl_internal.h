@@ -80,6 +80,8 @@ struct CoopCtl {
     int fused;                          // 1: grid barrier + exit signal + merge in this kernel
     unsigned int *barrier;              // this launch's grid-barrier counter (0 on entry)
     unsigned int *barrier_next;         // the next launch's counter (reset here)
+    unsigned long long *merge_ctr;      // fused merge: chunk counter (0 on entry)
+    unsigned long long *merge_ctr_next; // the next launch's chunk counter (reset here)
     unsigned long long *exit_word;      // mapped host word set to `epoch` after the barrier
     DevMergeList mg;                    // merge list (mg.n == 0: nothing to merge in-kernel)
 };

@@ -246,6 +246,43 @@ __device__ __forceinline__ void merge_dev_body(const DevMergeList &L, unsigned l
     }
 }
 
+// The same merge shared out dynamically: 64 KB chunks of the concatenated domains are claimed
+// from `ctr` by whole CTAs (any number of CTAs may take part).
+__device__ void merge_dev_chunks(const DevMergeList &L, long long wm, unsigned long long *ctr) {
+    constexpr long long CH = 64 * 1024;
+    long long b0[6], b1[6], nch[6];
+    long long total = 0;
+    for (int b = 0; b < L.n; ++b) {
+        b0[b] = 0; b1[b] = L.total[b];
+        if (L.unit_wgs[b] > 0) {
+            b0[b] = (wm / L.unit_wgs[b]) * L.unit_bytes[b];
+            b1[b] = ((L.hi + L.unit_wgs[b] - 1) / L.unit_wgs[b]) * L.unit_bytes[b];
+            if (b0[b] > L.total[b]) b0[b] = L.total[b];
+            if (b1[b] > L.total[b]) b1[b] = L.total[b];
+        }
+        nch[b] = b1[b] > b0[b] ? (b1[b] - b0[b] + CH - 1) / CH : 0;
+        total += nch[b];
+    }
+    __shared__ long long s_chunk;
+    for (;;) {
+        if (threadIdx.x == 0) s_chunk = (long long)atomicAdd(ctr, 1ull);
+        __syncthreads();
+        long long k = s_chunk;
+        __syncthreads();
+        if (k >= total) return;
+        int b = 0;
+        while (k >= nch[b]) { k -= nch[b]; ++b; }
+        const long long off = b0[b] + k * CH;
+        const size_t len = (size_t)((off + CH < b1[b]) ? CH : b1[b] - off);
+        switch (L.es[b]) {
+        case 1: merge_range<1>(L.gpu[b] + off, L.cpu[b] + off, L.twin[b] + off, len, threadIdx.x, blockDim.x); break;
+        case 2: merge_range<2>(L.gpu[b] + off, L.cpu[b] + off, L.twin[b] + off, len, threadIdx.x, blockDim.x); break;
+        case 4: merge_range<4>(L.gpu[b] + off, L.cpu[b] + off, L.twin[b] + off, len, threadIdx.x, blockDim.x); break;
+        default: merge_range<8>(L.gpu[b] + off, L.cpu[b] + off, L.twin[b] + off, len, threadIdx.x, blockDim.x); break;
+        }
+    }
+}
+
 __global__ void __launch_bounds__(256) merge_dev_kernel(const DevMergeList L) {
     __shared__ unsigned long long s_wm;
     if (threadIdx.x == 0) s_wm = ld_status(L.wm_word);
@@ -281,7 +318,9 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
 
     if (blockIdx.x == 0 && threadIdx.x == 0) {   // counters of the next launch (stream-ordered)
         *c.claim_next = 0ull;
-        if (c.barrier_next) *c.barrier_next = 0u;
+        if (c.barrier_next)
+            for (int q = 0; q < 17; ++q) c.barrier_next[q] = 0u;
+        if (c.merge_ctr_next) *c.merge_ctr_next = 0ull;
         if (c.tasks_next) *c.tasks_next = 0ull;
         if (c.tstamp) {   // stats mode: start stamp, reset this launch's merge end and the next end
             c.tstamp[0] = globaltimer();
@@ -319,9 +358,15 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
         TaskCtx tc;
         tc.c = &c; tc.key = key; tc.s_flag = &s_flag; tc.abort_w = 0; tc.pending = 0;
         if (threadIdx.x == 0) {
-            // claim the next task and prefetch the status while this one runs
-            t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
-            st_next = ld_status(c.status);
+            // claim the next task and prefetch the status while this one runs (no claim at all
+            // when the grid already covers every task: no contention on the counter)
+            if (c.task_lo + (long long)gridDim.x < c.task_hi) {
+                t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
+                st_next = ld_status(c.status);
+            } else {
+                t_next = c.task_hi;
+                st_next = st_first;
+            }
             tc.pending = checked ? st_next : st_first;
         }
         const bool aborted = Body::run(bp, t, tc, smem);
@@ -340,30 +385,50 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
     if (c.tasks && threadIdx.x == 0 && executed) atomicAdd(c.tasks, executed);
     if (c.tstamp && threadIdx.x == 0) atomicMax(c.tstamp + 1, globaltimer());
     if (!c.fused) return;
-    // Fused tail (the kernel is launched cooperatively, so every CTA is resident): a grid
-    // barrier, then the GPU-exit signal for the host executor (L18.s19) and the diff-merge
-    // (Fig 9) over the domain given by the lowest watermark any CTA acted on -- no second
-    // kernel launch and no host round trip between the dispatcher and the merge.
+    // Fused tail.  Every CTA registers its arrival; the LAST one to arrive publishes the
+    // GPU-exit signal (L18.s19).  The diff-merge (Fig 9) then runs over the domain given by the
+    // lowest watermark any CTA acted on, shared out in 64 KB chunks from a counter, by the CTAs
+    // still present: the last one, plus those that had already seen a skip when they arrived
+    // (they wait for the last arrival, since a merge is certain).  With nothing to merge -- the
+    // GPU-favoured case -- no CTA waits at all.
     __syncthreads();
     if (threadIdx.x == 0) {
         __threadfence();
-        atomicAdd(c.barrier, 1u);
-        unsigned int v;
-        for (;;) {
-            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(c.barrier) : "memory");
-            if (v >= gridDim.x) break;
-            __nanosleep(64);
+        // hierarchical arrival count: 16 leaf counters, the CTA completing a leaf bumps the
+        // root, the CTA completing the root is the last one (no 1000-way contention on a word)
+        const unsigned int leaf = blockIdx.x & 15u;
+        const unsigned int nleaf = (gridDim.x > 16u) ? 16u : gridDim.x;
+        const unsigned int leaf_size = (gridDim.x - leaf + 15u) / 16u;
+        bool last = false;
+        if (atomicAdd(c.barrier + 1 + leaf, 1u) == leaf_size - 1) {
+            __threadfence();
+            last = atomicAdd(c.barrier, 1u) == nleaf - 1;
         }
-        s_task = (long long)ld_status(c.mg.wm_word);
-        if (blockIdx.x == 0) {
+        const bool skip_seen = decode_wm_word(ld_status(c.mg.wm_word), c.epoch) != 0xFFFFFFFFu;
+        int role = last ? 2 : (skip_seen && c.mg.n > 0 ? 1 : 0);
+        if (role == 1) {   // wait for the last arrival (the kernel is cooperative: all resident)
+            unsigned int v;
+            unsigned int ns = 256;
+            for (;;) {
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(c.barrier) : "memory");
+                if (v >= nleaf) break;
+                __nanosleep(ns);
+                if (ns < 4096) ns *= 2;
+            }
+        }
+        if (last) {
+            __threadfence();
             asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(c.exit_word), "l"((unsigned long long)c.epoch) : "memory");
             if (c.mg.tstamp) c.mg.tstamp[0] = globaltimer();
         }
+        s_task = role ? (long long)ld_status(c.mg.wm_word) : 0;
+        s_w = (unsigned int)role;
     }
     __syncthreads();
-    if (c.mg.n > 0)
-        merge_dev_body(c.mg, (unsigned long long)s_task, (size_t)blockIdx.x * blockDim.x + threadIdx.x,
-                       (size_t)gridDim.x * blockDim.x);
+    if (s_w == 0u || c.mg.n == 0) return;
+    const unsigned int w32 = decode_wm_word((unsigned long long)s_task, c.epoch);
+    if (w32 == 0xFFFFFFFFu || (long long)w32 >= c.mg.hi) return;
+    merge_dev_chunks(c.mg, (long long)w32, c.merge_ctr);
     if (c.mg.tstamp && threadIdx.x == 0) atomicMax(c.mg.tstamp + 1, globaltimer());
 }
 
@@ -609,19 +674,85 @@ struct CorrReduceBody {
 // 2DCONV (PolyBench/GPU): interior B[i][j] = sum of 9 taps, canonical PolyBench term order
 // (column j-1 rows i-1..i+1, then column j, then column j+1): first tap a product, the other
 // eight fused multiply-adds.  Border untouched.
+// Thread mapping (vector path): a tile is 256 columns x 32 rows; a thread owns 4 consecutive
+// columns (float4) of 8 rows; its 10 input rows are loaded up front (memory-level parallelism),
+// the left/right halo columns come from the neighbouring lanes by shuffle (edge lanes load
+// them), and each output row is one 16-byte store (masked at the image border).
 template <typename T>
 struct Conv2DBody {
     static constexpr int kThreads = 256;
-    static constexpr int kMinBlocks = 4;
-    struct Params { const T *A; T *B; Tile2D tl; T c[9]; };   // c[a*3+b]: row offset a-1, col offset b-1
+    static constexpr int kMinBlocks = 2;   // 10 x 16 B of loads in flight per thread needs the registers
+    struct Params { const T *A; T *B; Tile2D tl; T c[9]; int vec4; };   // c[a*3+b]: row offset a-1, col offset b-1
     typedef EmptySmem Smem;
     __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
+
+    __device__ static T tap9(const Params &p, T l0, T l1, T l2, T m0, T m1, T m2, T r0, T r1, T r2) {
+        T s = op_mul(p.c[0], l0);
+        s = op_fma(p.c[3], l1, s);
+        s = op_fma(p.c[6], l2, s);
+        s = op_fma(p.c[1], m0, s);
+        s = op_fma(p.c[4], m1, s);
+        s = op_fma(p.c[7], m2, s);
+        s = op_fma(p.c[2], r0, s);
+        s = op_fma(p.c[5], r1, s);
+        s = op_fma(p.c[8], r2, s);
+        return s;
+    }
+
     __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
         const Tile2D &tl = p.tl;
         const long long tx = t % tl.ntx, ty = t / tl.ntx;
         const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
         const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
         const long long ni = tl.nrows, nj = tl.ncols;
+        if (p.vec4 && tcols == 256 && trows == 32) {
+            const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+            const int cg = warp & 1;                 // which 128-column half of the tile
+            const int rg = warp >> 1;                // which 8-row group
+            const long long j = c0 + cg * 128 + lane * 4;   // first of this thread's 4 columns
+            const long long ib = r0 + rg * 8;        // first output row of the group
+            if (ib >= ni) return false;
+            const bool colok = j < nj;               // nj % 4 == 0 on this path
+            typename V4<T>::type v[10];
+            T lh[10], rh[10];
+#pragma unroll
+            for (int q = 0; q < 10; ++q) {
+                const long long r = ib - 1 + q;
+                if (colok && r >= 0 && r < ni) v[q] = ld_cached4(p.A + r * nj + j);
+                else { v[q].x = v[q].y = v[q].z = v[q].w = T(0); }
+            }
+#pragma unroll
+            for (int q = 0; q < 10; ++q) {
+                T left = __shfl_up_sync(0xffffffffu, v[q].w, 1);
+                T right = __shfl_down_sync(0xffffffffu, v[q].x, 1);
+                const long long r = ib - 1 + q;
+                if (lane == 0) left = (colok && j >= 1 && r >= 0 && r < ni) ? __ldg(p.A + r * nj + j - 1) : T(0);
+                if (lane == 31) right = (j + 4 < nj && r >= 0 && r < ni) ? __ldg(p.A + r * nj + j + 4) : T(0);
+                lh[q] = left; rh[q] = right;
+            }
+            if (!colok) return false;
+#pragma unroll
+            for (int q = 1; q <= 8; ++q) {
+                const long long i = ib + q - 1;
+                if (i < 1 || i >= ni - 1) continue;
+                typename V4<T>::type o;
+                o.x = tap9(p, lh[q - 1], lh[q], lh[q + 1], v[q - 1].x, v[q].x, v[q + 1].x, v[q - 1].y, v[q].y, v[q + 1].y);
+                o.y = tap9(p, v[q - 1].x, v[q].x, v[q + 1].x, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z);
+                o.z = tap9(p, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w);
+                o.w = tap9(p, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w, rh[q - 1], rh[q], rh[q + 1]);
+                T *dst = p.B + i * nj + j;
+                if (j >= 1 && j + 4 <= nj - 1) {
+                    __stcs(reinterpret_cast<typename V4<T>::type *>(dst), o);
+                } else {   // a border column inside this vector stays untouched
+                    if (j >= 1 && j < nj - 1) __stcs(dst, o.x);
+                    if (j + 1 >= 1 && j + 1 < nj - 1) __stcs(dst + 1, o.y);
+                    if (j + 2 >= 1 && j + 2 < nj - 1) __stcs(dst + 2, o.z);
+                    if (j + 3 >= 1 && j + 3 < nj - 1) __stcs(dst + 3, o.w);
+                }
+            }
+            return false;
+        }
+        // generic path (any tile shape / alignment): one column per thread, sliding window
         for (int cc = threadIdx.x; cc < tcols; cc += kThreads) {
             const long long j = c0 + cc;
             if (j < 1 || j >= nj - 1) continue;
@@ -629,23 +760,13 @@ struct Conv2DBody {
             const long long iend = (r0 + trows < ni - 1) ? r0 + trows : ni - 1;
             if (i >= iend) continue;
             const T *a = p.A + j;
-            // sliding window: w[a][b] = A[i + a - 1][j + b - 1]
             T w0[3], w1[3], w2[3];
 #pragma unroll
             for (int b = 0; b < 3; ++b) { w0[b] = __ldg(a + (i - 1) * nj + b - 1); w1[b] = __ldg(a + i * nj + b - 1); }
             for (; i < iend; ++i) {
 #pragma unroll
                 for (int b = 0; b < 3; ++b) w2[b] = __ldg(a + (i + 1) * nj + b - 1);
-                T s = op_mul(p.c[0], w0[0]);
-                s = op_fma(p.c[3], w1[0], s);
-                s = op_fma(p.c[6], w2[0], s);
-                s = op_fma(p.c[1], w0[1], s);
-                s = op_fma(p.c[4], w1[1], s);
-                s = op_fma(p.c[7], w2[1], s);
-                s = op_fma(p.c[2], w0[2], s);
-                s = op_fma(p.c[5], w1[2], s);
-                s = op_fma(p.c[8], w2[2], s);
-                __stcs(p.B + i * nj + j, s);
+                __stcs(p.B + i * nj + j, tap9(p, w0[0], w1[0], w2[0], w0[1], w1[1], w2[1], w0[2], w1[2], w2[2]));
 #pragma unroll
                 for (int b = 0; b < 3; ++b) { w0[b] = w1[b]; w1[b] = w2[b]; }
             }
@@ -1003,6 +1124,7 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
             Conv2DBody<int32_t>::Params p;
             p.A = (const int32_t *)a.dev[0]; p.B = (int32_t *)a.dev[1];
             p.tl = make_tile(g, a.n0, a.n1, tw, th);
+            p.vec4 = (a.n1 % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.B);
             const int32_t c[9] = {2, 5, -8, -3, 6, -9, 4, 7, 1};
             for (int q = 0; q < 9; ++q) p.c[q] = c[q];
             return f.template go<Conv2DBody<int32_t>>(p);
@@ -1010,6 +1132,7 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
         Conv2DBody<float>::Params p;
         p.A = (const float *)a.dev[0]; p.B = (float *)a.dev[1];
         p.tl = make_tile(g, a.n0, a.n1, tw, th);
+        p.vec4 = (a.n1 % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.B);
         const float c[9] = {0.2f, 0.5f, -0.8f, -0.3f, 0.6f, -0.9f, 0.4f, 0.7f, 0.10f};
         for (int q = 0; q < 9; ++q) p.c[q] = c[q];
         return f.template go<Conv2DBody<float>>(p);

@@ -343,6 +343,7 @@ struct fcl_context_st {
     unsigned long long *dclaim = nullptr, *dtasks = nullptr, *dwm = nullptr;
     unsigned long long *dstamp = nullptr;        // stats mode: %globaltimer stamps, 4 per slot
     unsigned int *dbar = nullptr;                // grid-barrier counters, one per slot
+    unsigned long long *dmctr = nullptr;         // fused-merge chunk counters, one per slot
     bool unfused = false;                        // FCL_UNFUSED_MERGE=1: merge as a separate kernel
     bool ktiming = false;                        // CUDA events around every kernel (FCL_KTIMING=1)
     cudaEvent_t main_tail = nullptr;             // ev_k1 of the last cooperative dispatcher
@@ -718,8 +719,10 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     c.tstamp_next = ctx->stats ? ctx->dstamp + 4 * ((j.slot + 1) % kSlots) : nullptr;
     c.task_lo = j.t0; c.task_hi = j.t1;
     c.abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
-    c.barrier = ctx->dbar + j.slot;
-    c.barrier_next = ctx->dbar + (j.slot + 1) % kSlots;
+    c.barrier = ctx->dbar + 32 * j.slot;
+    c.barrier_next = ctx->dbar + 32 * ((j.slot + 1) % kSlots);
+    c.merge_ctr = ctx->dmctr + j.slot;
+    c.merge_ctr_next = ctx->dmctr + (j.slot + 1) % kSlots;
     c.exit_word = ctx->exit_dptr;
     c.mg = DevMergeList{};
     c.mg.n = 0;
@@ -789,7 +792,8 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         // no dispatcher: reset the next launch's counters here
         CK(ctx, cudaMemsetAsync(ctx->dclaim + (j.slot + 1) % kSlots, 0, 8, ctx->main));
         CK(ctx, cudaMemsetAsync(ctx->dtasks + (j.slot + 1) % kSlots, 0, 8, ctx->main));
-        CK(ctx, cudaMemsetAsync(ctx->dbar + (j.slot + 1) % kSlots, 0, 4, ctx->main));
+        CK(ctx, cudaMemsetAsync(ctx->dbar + 32 * ((j.slot + 1) % kSlots), 0, 128, ctx->main));
+        CK(ctx, cudaMemsetAsync(ctx->dmctr + (j.slot + 1) % kSlots, 0, 8, ctx->main));
         ctx->main_tail = nullptr;
     }
     if (j.dev_merge && !c.fused) {
@@ -1164,14 +1168,16 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
         cudaMemset(dp, 0, 8 * fcl_context_st::kSlots);
         ctx->status_dptr = (unsigned long long *)dp;
     }
-    // device counters: claim[kSlots], tasks[kSlots], wm word, stamps[4 * kSlots], barrier[kSlots]
-    if ((e = cudaMalloc(&dp, 8 * (7 * fcl_context_st::kSlots + 2))) != cudaSuccess) return fail(e, "counters");
-    cudaMemset(dp, 0, 8 * (7 * fcl_context_st::kSlots + 2));
+    // device counters: claim[kSlots], tasks[kSlots], wm word, stamps[4 * kSlots], merge chunk
+    // counters[kSlots], then barrier counters (32 u32 per slot: root + 16 leaves)
+    if ((e = cudaMalloc(&dp, 8 * (7 * fcl_context_st::kSlots + 2) + 128 * fcl_context_st::kSlots)) != cudaSuccess) return fail(e, "counters");
+    cudaMemset(dp, 0, 8 * (7 * fcl_context_st::kSlots + 2) + 128 * fcl_context_st::kSlots);
     ctx->dclaim = (unsigned long long *)dp;
     ctx->dtasks = ctx->dclaim + fcl_context_st::kSlots;
     ctx->dwm = ctx->dtasks + fcl_context_st::kSlots;
     ctx->dstamp = ctx->dwm + 2;
-    ctx->dbar = (unsigned int *)(ctx->dstamp + 4 * fcl_context_st::kSlots);
+    ctx->dmctr = ctx->dstamp + 4 * fcl_context_st::kSlots;
+    ctx->dbar = (unsigned int *)(ctx->dmctr + fcl_context_st::kSlots);
     for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1})
         if ((e = cudaEventCreate(pe)) != cudaSuccess) return fail(e, "events");
     for (cudaEvent_t *pe : {&ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h})
