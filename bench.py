@@ -209,6 +209,9 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         for _ in range(k):
             with torch.cuda.stream(stream):
                 flush.fill_(1.0)          # L2 flush (outside the timed interval)
+            # idle GPU at e0: host-side work (the CPU-only leg, the host share of a cooperative
+            # launch, launch submission) cannot hide under the flush
+            stream.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             step(mode, infos if collect else None)
@@ -303,6 +306,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     for r in range(args.warmup + args.steps):
         with torch.cuda.stream(stream):
             flush.fill_(3.0)
+        stream.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         for b in in_bufs:

@@ -35,7 +35,7 @@ def _cmd(obj: str, src: str, kind: str):
     srcp = os.path.join(CSRC, src)
     if kind == "nvcc":
         return [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
-                "-I", INCLUDE, "-c", srcp, "-o", out]
+                "-I", INCLUDE, *os.environ.get("FCL_NVCC_EXTRA", "").split(), "-c", srcp, "-o", out]
     common = ["g++", "-std=c++17", "-fPIC", "-Wall", "-Wno-unused-function", "-I", INCLUDE,
               "-I", os.path.join(CUDA_HOME, "include"), "-c", srcp, "-o", out]
     if kind == "host_fp":

@@ -76,28 +76,29 @@ __device__ __forceinline__ unsigned int decode_w(unsigned long long st, const Co
     return ((unsigned int)(st >> 32) == c.epoch) ? (unsigned int)st : c.w_default;
 }
 
-// Per-task view of the status for in-task polling (abort checks in loops, Fig 12).
+// Per-task view of the status for in-task polling (abort checks in loops, Fig 12).  Only the
+// prefetched status word lives in a register; the task key and the abort verdict are in
+// shared memory, so a polling body keeps its registers.
 struct TaskCtx {
-    const CoopCtl *c;          // nullptr for plain launches
-    long long key;
+    const CoopCtl *c;            // nullptr for plain launches (parameter space, no register copy)
     unsigned long long pending;  // thread 0: status word loaded at the previous poll
-    int *s_flag;                 // shared memory broadcast slot (D2: the local 'completedatcpu')
-    unsigned int abort_w;
+    long long *s_key;            // shared: key of the running task
+    int *s_flag;                 // shared broadcast slot (D2: the local 'completedatcpu'); w + 1 after an abort
 
     // Called by ALL threads at a CTA-uniform point with a CTA-uniform iteration count.
     __device__ __forceinline__ bool poll(int it) {
         if (c == nullptr || c->abort_period <= 0 || it == 0 || (it % c->abort_period) != 0) return false;
         if (threadIdx.x == 0) {
-            unsigned int w = decode_w(pending, *c);
+            const unsigned int w = decode_w(pending, *c);
             pending = ld_status(c->status);   // prefetch: consumed at the next poll
-            *s_flag = ((unsigned long long)key >= (unsigned long long)w) ? (int)(w + 1u) : 0;
+            *s_flag = ((unsigned long long)*s_key >= (unsigned long long)w) ? (int)(w + 1u) : 0;
         }
         __syncthreads();
-        int f = *s_flag;
+        const int f = *s_flag;
         __syncthreads();
-        if (f) { abort_w = (unsigned int)(f - 1); return true; }
-        return false;
+        return f != 0;
     }
+    __device__ __forceinline__ unsigned int abort_w() const { return (unsigned int)(*s_flag - 1); }
 };
 
 // ------------------------------------------------------------------------------------------
@@ -310,8 +311,8 @@ __device__ __forceinline__ void record_wm(const CoopCtl &c, unsigned int w) {
 
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
-coop_kernel(const CoopCtl c, const typename Body::Params bp) {
-    __shared__ long long s_task;
+coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename Body::Params bp) {
+    __shared__ long long s_task, s_key;
     __shared__ unsigned int s_w;
     __shared__ int s_flag;
     __shared__ __align__(16) typename Body::Smem smem;
@@ -333,7 +334,9 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
     // words), and long tasks still poll the status inside their loops; the status load issued
     // here is consumed at that first poll.  Later tasks are claimed from the device counter
     // and checked against the watermark (Fig 8) with the load prefetched during the previous
-    // task, so neither the claim nor the check is on the critical path.
+    // task, so neither the claim nor the check is on the critical path.  Only the claimed index
+    // and one status word stay live across a task (thread 0's); everything else is in shared
+    // memory or the parameter bank, so the dispatcher does not take registers from the body.
     long long t = c.task_lo + (long long)blockIdx.x;
     unsigned int w = c.w_default;
     bool checked = false;
@@ -344,45 +347,40 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
         checked = true;
         __syncthreads();
     }
-    long long t_next = 0;
-    unsigned long long st_next = 0, st_first = 0;
-    unsigned long long executed = 0;
-    if (threadIdx.x == 0) st_first = ld_status(c.status);
+    const bool claims = c.task_lo + (long long)gridDim.x < c.task_hi;
+    TaskCtx tc;
+    tc.c = &c; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.pending = 0;
+    if (threadIdx.x == 0) tc.pending = ld_status(c.status);
+    bool marked = false;   // thread 0: this CTA recorded a watermark (skip or abort)
     for (;;) {
         if (t >= c.task_hi) break;
         const long long key = Body::key(bp, t);
         if (checked && (unsigned long long)key >= (unsigned long long)w) {   // covered by the host
-            if (threadIdx.x == 0) record_wm(c, w);
+            if (threadIdx.x == 0) { record_wm(c, w); marked = true; }
             break;
         }
-        TaskCtx tc;
-        tc.c = &c; tc.key = key; tc.s_flag = &s_flag; tc.abort_w = 0; tc.pending = 0;
-        if (threadIdx.x == 0) {
-            // claim the next task and prefetch the status while this one runs (no claim at all
-            // when the grid already covers every task: no contention on the counter)
-            if (c.task_lo + (long long)gridDim.x < c.task_hi) {
-                t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
-                st_next = ld_status(c.status);
-            } else {
-                t_next = c.task_hi;
-                st_next = st_first;
-            }
-            tc.pending = checked ? st_next : st_first;
-        }
+        if (threadIdx.x == 0) s_key = key;   // read back by thread 0 only
+        // claim the next task while this one runs (no claim at all when the grid already
+        // covers every task: no contention on the counter)
+        long long t_next = c.task_hi;
+        if (threadIdx.x == 0 && claims) t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
         const bool aborted = Body::run(bp, t, tc, smem);
         if (aborted) {
-            if (threadIdx.x == 0) record_wm(c, tc.abort_w);
+            if (threadIdx.x == 0) { record_wm(c, tc.abort_w()); marked = true; }
             break;
         }
-        ++executed;
-        if (threadIdx.x == 0) { s_task = t_next; s_w = decode_w(st_next, c); }
+        if (threadIdx.x == 0) {
+            if (c.tasks) atomicAdd(c.tasks, 1ull);
+            s_task = t_next;
+            s_w = decode_w(tc.pending, c);
+            tc.pending = ld_status(c.status);   // prefetch for the next task's polls
+        }
         __syncthreads();
         t = s_task;
         w = s_w;
         checked = true;
         __syncthreads();
     }
-    if (c.tasks && threadIdx.x == 0 && executed) atomicAdd(c.tasks, executed);
     if (c.tstamp && threadIdx.x == 0) atomicMax(c.tstamp + 1, globaltimer());
     if (!c.fused) return;
     // Fused tail.  Every CTA registers its arrival; the LAST one to arrive publishes the
@@ -393,7 +391,12 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
     // GPU-favoured case -- no CTA waits at all.
     __syncthreads();
     if (threadIdx.x == 0) {
-        __threadfence();
+        // Only a CTA that recorded a watermark must make that record (and the partial writes
+        // of an aborted task) visible before it arrives; complete work-groups are bit-identical
+        // to the host's, so when their writes land does not matter.  The merge-role probe is
+        // issued before the arrival atomics so the two round trips overlap.
+        const unsigned long long wm_probe = ld_status(c.mg.wm_word);
+        if (marked) __threadfence();
         // hierarchical arrival count: 16 leaf counters, the CTA completing a leaf bumps the
         // root, the CTA completing the root is the last one (no 1000-way contention on a word)
         const unsigned int leaf = blockIdx.x & 15u;
@@ -404,7 +407,7 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
             __threadfence();
             last = atomicAdd(c.barrier, 1u) == nleaf - 1;
         }
-        const bool skip_seen = decode_wm_word(ld_status(c.mg.wm_word), c.epoch) != 0xFFFFFFFFu;
+        const bool skip_seen = decode_wm_word(wm_probe, c.epoch) != 0xFFFFFFFFu;
         int role = last ? 2 : (skip_seen && c.mg.n > 0 ? 1 : 0);
         if (role == 1) {   // wait for the last arrival (the kernel is cooperative: all resident)
             unsigned int v;
@@ -434,11 +437,12 @@ coop_kernel(const CoopCtl c, const typename Body::Params bp) {
 
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
-plain_kernel(const typename Body::Params bp, long long task_lo) {
+plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo) {
     __shared__ int s_flag;
     __shared__ __align__(16) typename Body::Smem smem;
+    __shared__ long long s_key;
     TaskCtx tc;
-    tc.c = nullptr; tc.key = 0; tc.pending = 0; tc.s_flag = &s_flag; tc.abort_w = 0;
+    tc.c = nullptr; tc.pending = 0; tc.s_flag = &s_flag; tc.s_key = &s_key;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
 }
 
@@ -778,17 +782,22 @@ struct Conv2DBody {
 // ------------------------------------------------------------------------------------------
 // GEMM-like bodies on CUDA cores (fp32 FFMA / int32 IMAD; no tensor cores: fp32 parity, see
 // DESIGN.md §6): SYRK, SYR2K and CORR's symmat.  Output tile 128 x 128, 256 threads, 8 x 8
-// outputs per thread, k-tile 8, double-buffered shared memory.  Every output accumulates its
-// k-chain in ascending k with one fma per term (SYR2K: A_i*B_j then B_i*A_j per k).
+// outputs per thread, k-tile 16, double-buffered shared memory plus register double-buffered
+// fragments.  Every output accumulates its k-chain in ascending k with one fma per term.
+// SYR2K is one GEMM over the interleaved K' = 2M: k' = 2k holds (A_i[k], B_j[k]) and
+// k' = 2k+1 holds (B_i[k], A_j[k]) -- exactly the canonical "A_i*B_j then B_i*A_j" per-k order.
 // ------------------------------------------------------------------------------------------
 enum { G_SYRK = 0, G_SYR2K = 1, G_CORR = 2 };
-constexpr int GBM = 128, GBK = 8, GPAD = 4;
+constexpr int GBM = 128, GBK = 16, GPAD = 4;
 
 template <typename T, int OP>
 struct GemmBody {
     static constexpr int kThreads = 256;
-    static constexpr int kMinBlocks = 2;
-    static constexpr int kOps = (OP == G_SYR2K) ? 4 : 2;   // operand tiles per stage
+#ifndef FCL_GEMM_MINB
+#define FCL_GEMM_MINB 2
+#endif
+    static constexpr int kMinBlocks = FCL_GEMM_MINB;
+    typedef typename V4<T>::type T4;
     struct Params {
         const T *A; const T *B; T *C;
         long long n;      // output is n x n (CORR: M x M)
@@ -799,7 +808,7 @@ struct GemmBody {
         long long ngx, lws0, lws1, lws;  // work-group geometry for keys
         int vec4;
     };
-    struct Smem { T s[2][kOps][GBK][GBM + GPAD]; };
+    struct Smem { T s[2][2][GBK][GBM + GPAD]; };   // [stage][A|B][k'][m]
 
     __device__ static void tile_of(const Params &p, long long t, long long &bi, long long &bj) {
         if (OP == G_CORR) {  // upper triangle, row-major over (b1 <= b2)
@@ -817,44 +826,74 @@ struct GemmBody {
         return (bj * GBM) / p.lws0 + p.ngx * ((bi * GBM) / p.lws1);
     }
 
-    // Load one k-tile of operand `which` into registers (4 elements per thread).
-    // K-contiguous operands (SYRK/SYR2K): element (row r, k) at X[(row0 + r) * ld + k].
-    // MN-contiguous operands (CORR): element (k, col c) at X[k * ld + col0 + c].
-    __device__ static void gload(const Params &p, const T *X, long long base, long long k0, T r[4]) {
-        const int tid = threadIdx.x;
-        if (OP == G_CORR) {
-            const int kk = tid >> 5, c = (tid & 31) * 4;
-            const long long k = k0 + kk, col = base + c;
-            if (k < p.m && p.vec4 && col + 3 < p.n) {
-                typename V4<T>::type v = ld_cached4(X + k * p.ld + col);
-                r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
-            } else {
-#pragma unroll
-                for (int q = 0; q < 4; ++q) r[q] = (k < p.m && col + q < p.n) ? X[k * p.ld + col + q] : T(0);
-            }
+    // 4 consecutive k of row `row` of X (K-contiguous operands), zero outside the matrix
+    __device__ static void load4_k(const Params &p, const T *X, long long row, long long k, T *r) {
+        if (row < p.n && p.vec4 && k + 3 < p.m) {
+            const T4 v = ld_cached4(X + row * p.ld + k);
+            r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
         } else {
-            const int row = tid >> 1, kq = (tid & 1) * 4;
-            const long long gr = base + row, k = k0 + kq;
-            if (gr < p.n && p.vec4 && k + 3 < p.m) {
-                typename V4<T>::type v = ld_cached4(X + gr * p.ld + k);
-                r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
-            } else {
 #pragma unroll
-                for (int q = 0; q < 4; ++q) r[q] = (gr < p.n && k + q < p.m) ? X[gr * p.ld + k + q] : T(0);
-            }
+            for (int q = 0; q < 4; ++q) r[q] = (row < p.n && k + q < p.m) ? X[row * p.ld + k + q] : T(0);
         }
     }
-    __device__ static void sstore(T (*S)[GBM + GPAD], const T r[4]) {
+    // 4 consecutive columns of data row k (CORR: MN-contiguous operand)
+    __device__ static void load4_row(const Params &p, const T *X, long long k, long long col, T *r) {
+        if (k < p.m && p.vec4 && col + 3 < p.n) {
+            const T4 v = ld_cached4(X + k * p.ld + col);
+            r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
+        } else {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) r[q] = (k < p.m && col + q < p.n) ? X[k * p.ld + col + q] : T(0);
+        }
+    }
+
+    // One k'-tile into registers: 8 elements of each operand tile per thread.
+    __device__ static void gload(const Params &p, long long i0, long long j0, long long kt, T ra[8], T rb[8]) {
         const int tid = threadIdx.x;
         if (OP == G_CORR) {
-            const int kk = tid >> 5, c = (tid & 31) * 4;
+            const int kk = tid >> 4, c = (tid & 15) * 8;
+            const long long k = kt * GBK + kk;
+            load4_row(p, p.A, k, i0 + c, ra); load4_row(p, p.A, k, i0 + c + 4, ra + 4);
+            load4_row(p, p.A, k, j0 + c, rb); load4_row(p, p.A, k, j0 + c + 4, rb + 4);
+        } else if (OP == G_SYRK) {
+            const int row = tid >> 1;
+            const long long k = kt * GBK + (tid & 1) * 8;
+            load4_k(p, p.A, i0 + row, k, ra); load4_k(p, p.A, i0 + row, k + 4, ra + 4);
+            load4_k(p, p.A, j0 + row, k, rb); load4_k(p, p.A, j0 + row, k + 4, rb + 4);
+        } else {   // SYR2K: this k'-tile covers k in [kt*GBK/2, (kt+1)*GBK/2)
+            const int row = tid >> 1;
+            const long long k = kt * (GBK / 2) + (tid & 1) * 4;
+            T x[4], y[4];
+            load4_k(p, p.A, i0 + row, k, x); load4_k(p, p.B, i0 + row, k, y);
 #pragma unroll
-            for (int q = 0; q < 4; ++q) S[kk][c + q] = r[q];
-        } else {
-            const int row = tid >> 1, kq = (tid & 1) * 4;
+            for (int q = 0; q < 4; ++q) { ra[2 * q] = x[q]; ra[2 * q + 1] = y[q]; }   // A_i[k], B_i[k]
+            load4_k(p, p.B, j0 + row, k, x); load4_k(p, p.A, j0 + row, k, y);
 #pragma unroll
-            for (int q = 0; q < 4; ++q) S[kq + q][row] = r[q];
+            for (int q = 0; q < 4; ++q) { rb[2 * q] = x[q]; rb[2 * q + 1] = y[q]; }   // B_j[k], A_j[k]
         }
+    }
+    __device__ static T4 mk4(T a, T b, T c, T d) { T4 v; v.x = a; v.y = b; v.z = c; v.w = d; return v; }
+    __device__ static void sstore(Smem &sm, int st, const T ra[8], const T rb[8]) {
+        const int tid = threadIdx.x;
+        if (OP == G_CORR) {
+            const int kk = tid >> 4, c = (tid & 15) * 8;
+            *reinterpret_cast<T4 *>(&sm.s[st][0][kk][c]) = mk4(ra[0], ra[1], ra[2], ra[3]);
+            *reinterpret_cast<T4 *>(&sm.s[st][0][kk][c + 4]) = mk4(ra[4], ra[5], ra[6], ra[7]);
+            *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c]) = mk4(rb[0], rb[1], rb[2], rb[3]);
+            *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c + 4]) = mk4(rb[4], rb[5], rb[6], rb[7]);
+        } else {
+            const int row = tid >> 1, kq = (tid & 1) * 8;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) { sm.s[st][0][kq + q][row] = ra[q]; sm.s[st][1][kq + q][row] = rb[q]; }
+        }
+    }
+    __device__ static void frag(const Smem &sm, int st, int kk, int tx, int ty, T a[8], T b[8]) {
+        const T4 a0 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][ty * 4]);
+        const T4 a1 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][64 + ty * 4]);
+        const T4 b0 = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][tx * 4]);
+        const T4 b1 = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][64 + tx * 4]);
+        a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w; a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
+        b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w; b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
     }
 
     __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &sm) {
@@ -862,72 +901,34 @@ struct GemmBody {
         tile_of(p, t, bi, bj);
         const long long i0 = bi * GBM, j0 = bj * GBM;
         const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
-        // operand sources: SYRK: (A rows i, A rows j); SYR2K: (A_i, B_j, B_i, A_j); CORR: (D cols i, D cols j)
-        const T *src[4];
-        long long base[4];
-        if (OP == G_SYR2K) {
-            src[0] = p.A; base[0] = i0; src[1] = p.B; base[1] = j0;
-            src[2] = p.B; base[2] = i0; src[3] = p.A; base[3] = j0;
-        } else {
-            src[0] = p.A; base[0] = i0; src[1] = p.A; base[1] = j0;
-            src[2] = src[3] = nullptr; base[2] = base[3] = 0;
-        }
         T acc[8][8];
 #pragma unroll
         for (int r = 0; r < 8; ++r)
 #pragma unroll
             for (int c = 0; c < 8; ++c) acc[r][c] = 0;
 
-        const long long nkt = (p.m + GBK - 1) / GBK;
-        T reg[kOps][4];
-#pragma unroll
-        for (int o = 0; o < kOps; ++o) gload(p, src[o], base[o], 0, reg[o]);
-#pragma unroll
-        for (int o = 0; o < kOps; ++o) sstore(sm.s[0][o], reg[o]);
+        const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;   // K'
+        const long long nkt = (kdim + GBK - 1) / GBK;
+        T ra[8], rb[8];
+        gload(p, i0, j0, 0, ra, rb);
+        sstore(sm, 0, ra, rb);
         __syncthreads();
         for (long long kt = 0; kt < nkt; ++kt) {
             const int st = (int)(kt & 1);
-            if (kt + 1 < nkt) {
-#pragma unroll
-                for (int o = 0; o < kOps; ++o) gload(p, src[o], base[o], (kt + 1) * GBK, reg[o]);
-            }
+            if (kt + 1 < nkt) gload(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
+            T a[2][8], b[2][8];
+            frag(sm, st, 0, tx, ty, a[0], b[0]);
 #pragma unroll
             for (int kk = 0; kk < GBK; ++kk) {
-                T a[8], b[8];
-                const typename V4<T>::type a0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][0][kk][ty * 4]);
-                const typename V4<T>::type a1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][0][kk][64 + ty * 4]);
-                const typename V4<T>::type b0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][1][kk][tx * 4]);
-                const typename V4<T>::type b1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][1][kk][64 + tx * 4]);
-                a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w; a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
-                b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w; b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
-                if (OP == G_SYR2K) {
-                    T a2[8], b2[8];
-                    const typename V4<T>::type c0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][2][kk][ty * 4]);
-                    const typename V4<T>::type c1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][2][kk][64 + ty * 4]);
-                    const typename V4<T>::type d0 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][3][kk][tx * 4]);
-                    const typename V4<T>::type d1 = *reinterpret_cast<const typename V4<T>::type *>(&sm.s[st][3][kk][64 + tx * 4]);
-                    a2[0] = c0.x; a2[1] = c0.y; a2[2] = c0.z; a2[3] = c0.w; a2[4] = c1.x; a2[5] = c1.y; a2[6] = c1.z; a2[7] = c1.w;
-                    b2[0] = d0.x; b2[1] = d0.y; b2[2] = d0.z; b2[3] = d0.w; b2[4] = d1.x; b2[5] = d1.y; b2[6] = d1.z; b2[7] = d1.w;
+                if (kk + 1 < GBK) frag(sm, st, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
 #pragma unroll
-                    for (int r = 0; r < 8; ++r)
+                for (int r = 0; r < 8; ++r)
 #pragma unroll
-                        for (int c = 0; c < 8; ++c) {
-                            acc[r][c] = op_fma(a[r], b[c], acc[r][c]);     // alpha*A[i][k]*B[j][k]
-                            acc[r][c] = op_fma(a2[r], b2[c], acc[r][c]);   // alpha*B[i][k]*A[j][k]
-                        }
-                } else {
-#pragma unroll
-                    for (int r = 0; r < 8; ++r)
-#pragma unroll
-                        for (int c = 0; c < 8; ++c) acc[r][c] = op_fma(a[r], b[c], acc[r][c]);
-                }
+                    for (int c = 0; c < 8; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
             }
-            if (kt + 1 < nkt) {
-#pragma unroll
-                for (int o = 0; o < kOps; ++o) sstore(sm.s[st ^ 1][o], reg[o]);
-            }
+            if (kt + 1 < nkt) sstore(sm, st ^ 1, ra, rb);
             __syncthreads();
-            if (tc.poll((int)(kt + 1))) return true;   // abort check every abort_period k-tiles (Fig 12)
+            if (tc.poll((int)(kt + 1))) return true;   // abort check every abort_period k'-tiles (Fig 12)
         }
         // epilogue: write-once stores
 #pragma unroll
@@ -949,12 +950,12 @@ struct GemmBody {
                     if (i >= p.n) continue;
                     T *crow = p.C + i * p.n;
                     if (p.vec4 && jb + 3 < p.n) {
-                        typename V4<T>::type cv = *reinterpret_cast<typename V4<T>::type *>(crow + jb);
+                        T4 cv = *reinterpret_cast<T4 *>(crow + jb);
                         cv.x = op_fma(p.alpha, acc[r][half * 4 + 0], op_mul(p.beta, cv.x));
                         cv.y = op_fma(p.alpha, acc[r][half * 4 + 1], op_mul(p.beta, cv.y));
                         cv.z = op_fma(p.alpha, acc[r][half * 4 + 2], op_mul(p.beta, cv.z));
                         cv.w = op_fma(p.alpha, acc[r][half * 4 + 3], op_mul(p.beta, cv.w));
-                        *reinterpret_cast<typename V4<T>::type *>(crow + jb) = cv;
+                        *reinterpret_cast<T4 *>(crow + jb) = cv;
                     } else {
 #pragma unroll
                         for (int c = 0; c < 4; ++c) {
@@ -1243,7 +1244,7 @@ int64_t gpu_slice_align(const KArgs &a, const Geom &g) {
 
 int gpu_default_abort_period(const KArgs &a) {
     switch (a.kernel) {
-    case K_SYRK: case K_SYR2K: case K_CORR_CORR: return 16;   // every 16 k-tiles (128 k)
+    case K_SYRK: case K_SYR2K: case K_CORR_CORR: return 8;    // every 8 k'-tiles (128 k')
     default: return 0;
     }
 }

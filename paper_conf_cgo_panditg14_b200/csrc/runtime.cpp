@@ -1573,9 +1573,15 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     info.gpu_watermark = info.published_watermark = L.hi;
     for (int k = 0; k < L.a.nbuf; ++k) {
         fcl_buffer b = L.bufs[k];
-        // (both copies are valid here: anything else drained above.)  A pending return copy
-        // of a buffer this launch writes still reads its device copy: order the overwrite
-        // behind it on the device; the host side of the hazard is resolved in phase B.
+        // A device copy left stale by a CPU-only launch is refreshed first (lazy H2D; the
+        // queue is drained above whenever a copy is stale).
+        if (!b->dev_valid) {
+            s = make_valid(ctx, b, false, true, &info);
+            if (s != FCL_SUCCESS) break;
+        }
+        // A pending return copy of a buffer this launch writes still reads its device copy:
+        // order the overwrite behind it on the device; the host side of the hazard is
+        // resolved in phase B.
         if (b->d2h_pending && (L.acc[k] & 2)) {
             const cudaError_t e = cudaStreamWaitEvent(ctx->main, b->d2h_ev, 0);
             if (e != cudaSuccess) { s = cuda_fail(ctx, e, "stream wait"); break; }

@@ -109,6 +109,7 @@ def run_config(name, steps, cpu_steps, modes):
             ctx.finish()
             with torch.cuda.stream(stream):
                 flush.fill_(1.0)
+            stream.synchronize()   # idle GPU at e0: host work cannot hide under the flush
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             for k, L in enumerate(prepared):

@@ -13,14 +13,15 @@ import workloads as W
 from paper_conf_cgo_panditg14_b200 import fcl
 
 mode = sys.argv[1] if len(sys.argv) > 1 else "coop"
+which = sys.argv[2] if len(sys.argv) > 2 else "gesummv_bicg4096"
+sys.path.insert(0, os.path.join(ROOT, "scripts"))
+from bench_configs import cfg_problems
 ctx = fcl.Context(0)
-Ps = [W.make("gesummv", 4096, seed=0, lws1d=256, out_init="zero"),
-      W.make("bicg_s", 4096, 4096, seed=1, lws1d=256, out_init="zero"),
-      W.make("bicg_q", 4096, 4096, seed=2, lws1d=256, out_init="zero")]
-launches = []
-for P in Ps:
-    b = H.create_buffers(ctx, P)
-    launches.append(ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode))
+Ps, meta = cfg_problems(which)
+bufs = [H.create_buffers(ctx, P) for P in Ps]
+for dl, db, sl, sb in meta.get("shared", []):
+    bufs[dl][db] = bufs[sl][sb]
+launches = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode) for P, b in zip(Ps, bufs)]
 for rep in range(30):
     for L in launches:
         L()

@@ -196,6 +196,35 @@ def test_multi_kernel_chain_location_tracking(ctx, oracle_mod):
         b.release()
 
 
+def test_cpu_only_then_coop_refreshes_device_copy(ctx, oracle_mod):
+    """A CPU-only launch leaves the device copy of its output stale; a following cooperative
+    launch reading that buffer must see the host's values (lazy H2D), not the old device ones."""
+    n = 384
+    P1 = W.make("atax_tmp", n, n, seed=16, lws1d=64)
+    P2 = W.make("atax_y", n, n, seed=17, lws1d=64)
+    A, x, tmp = (ctx.buffer_from_array(b) for b in P1.bufs)
+    y = ctx.buffer_from_array(P2.bufs[2])
+    # device copy of tmp <- A x (GPU); then x changes and tmp is recomputed on the host only
+    ctx.enqueue_ndrange("atax_tmp_f32", P1.gws, P1.lws, [A, x, tmp, n, n], mode="gpu")
+    ctx.finish()
+    x2 = (P1.bufs[1] * 2.0 + 1.0).astype(np.float32)
+    x.write_array(x2)
+    ctx.enqueue_ndrange("atax_tmp_f32", P1.gws, P1.lws, [A, x, tmp, n, n], mode="cpu")
+    ctx.enqueue_ndrange("atax_y_f32", P2.gws, P2.lws, [A, tmp, y, n, n], mode="coop", forced_split=0)
+    ctx.enqueue_ndrange("atax_y_f32", P2.gws, P2.lws, [A, tmp, y, n, n], mode="coop")
+    ctx.finish()
+    L1 = oracle_mod.Launch("atax_tmp", False, n, n, list(P1.gws), list(P1.lws),
+                           [P1.bufs[0].astype(np.float64), x2.astype(np.float64), np.zeros(n)])
+    oracle_mod.run_range(L1, 0, L1.num_groups())
+    L2 = oracle_mod.Launch("atax_y", False, n, n, list(P2.gws), list(P2.lws),
+                           [P1.bufs[0].astype(np.float64), L1.bufs[2].copy(), np.zeros(n)])
+    oracle_mod.run_range(L2, 0, L2.num_groups())
+    assert_parity(y.read_array(np.float32), L2.bufs[2], False, "cpu -> coop chain with a stale device copy")
+    assert_parity(H.device_array(y, np.float32), L2.bufs[2], False, "device copy of y")
+    for b in (A, x, tmp, y):
+        b.release()
+
+
 def test_corr_chain_coop_vs_oracle(ctx, oracle_mod):
     n, m = 300, 200
     data = W.corr_chain_inputs(n, m, seed=8)
