@@ -177,9 +177,15 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     stream = torch.cuda.Stream(device=dev)
+    # each local rank gets its own slice of the host cores (its host executor is pinned inside
+    # it); within a slice one core is the coordinator's and one the caller's (runtime default)
+    all_cores = sorted(os.sched_getaffinity(0))
+    lws_ranks = max(1, int(os.environ.get("LOCAL_WORLD_SIZE", world)))
+    per_rank = max(1, len(all_cores) // lws_ranks)
+    if lws_ranks > 1:
+        os.sched_setaffinity(0, all_cores[local_rank * per_rank:(local_rank + 1) * per_rank] or all_cores)
     cores = len(os.sched_getaffinity(0))
-    per_rank = max(2, cores // max(1, int(os.environ.get("LOCAL_WORLD_SIZE", world))))
-    host_threads = max(1, per_rank - 1)
+    host_threads = max(1, cores - 2)
     ctx = fcl.Context(local_rank, n_host_threads=host_threads, streams=(stream.cuda_stream, None, None))
 
     Ps = problems(1000 * rank)

@@ -70,7 +70,8 @@ typedef struct fcl_kernel_st  *fcl_kernel;
 
 typedef struct {
     int32_t device;          /* CUDA device ordinal */
-    int32_t n_host_threads;  /* host executor threads; 0 = (cores in affinity mask) - 1 */
+    int32_t n_host_threads;  /* host executor threads; 0 = (cores in affinity mask) - 2: one core
+                                is the coordinator's, one is left to the calling thread */
     int32_t pin_threads;     /* 1 = pin executor threads to cores of the affinity mask */
     int32_t status_location; /* FCL_STATUS_DEVICE (default) | FCL_STATUS_HOST_MAPPED */
     void   *main_stream;     /* optional cudaStream_t for kernels/merge; NULL = own stream */

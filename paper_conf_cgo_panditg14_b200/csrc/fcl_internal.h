@@ -112,8 +112,18 @@ int gpu_default_abort_period(const KArgs &a);
 int64_t gpu_slice_align(const KArgs &a, const Geom &g);
 // Launch the persistent cooperative dispatcher; returns the grid size used (<= 0 on error).
 int gpu_launch_coop(const KArgs &a, const Geom &g, const CoopCtl &c, int num_sms, void *stream);
-// Plain grid over tasks [task_lo, task_hi) with no status reads (GPU-only baseline).
-int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream);
+// Plain grid over tasks [task_lo, task_hi) with no status reads (GPU-only baseline, and the
+// cooperative single-wave case, see gpu_coop_capacity).  `reset` (nullable): the dispatcher
+// counters of the next launch slot, zeroed by block 0 as a dispatcher would.
+struct SlotReset {
+    unsigned long long *claim, *tasks, *merge_ctr;
+    unsigned int *barrier;   // 17 words
+};
+int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream,
+                     const SlotReset *reset = nullptr);
+// CTAs of the persistent dispatcher resident at once (occupancy x SMs): a launch with no more
+// tasks than this runs in a single wave, every CTA's only task unchecked.
+int64_t gpu_coop_capacity(const KArgs &a, const Geom &g, int num_sms);
 // Fig 9 diff-merge on [0, bytes) of three device buffers.
 int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes, int elem_size,
                      int num_sms, void *stream);

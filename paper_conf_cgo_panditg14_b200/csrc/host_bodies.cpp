@@ -39,11 +39,14 @@ inline void part_range(int64_t n, int part, int nparts, int64_t &lo, int64_t &hi
 // ---------------------------------------------------------------- row-dot (ATAX k1, BICG k2, GESUMMV)
 // Canonical order: 128 column partitions (q = j % 128, ascending j), per-lane fold of 4
 // partials, xor-butterfly over 32 lanes.  Mirrors RowDotBody in kernels.cu.
+// Returns false (and no value) when the abort flag is seen: it is polled every 1024 columns,
+// so an abandoned chunk stops within a fraction of a microsecond.
 template <typename T>
-T rowdot(const T *Ar, const T *x, int64_t ncols) {
+bool rowdot(const T *Ar, const T *x, int64_t ncols, const volatile int *ab, T *res) {
     T p[kRowPartitions];
     for (int q = 0; q < kRowPartitions; ++q) p[q] = 0;
     for (int64_t j0 = 0; j0 < ncols; j0 += kRowPartitions) {
+        if ((j0 & 1023) == 0 && aborted(ab)) return false;
         const int w = (int)std::min<int64_t>(kRowPartitions, ncols - j0);
         const T *a = Ar + j0;
         const T *xv = x + j0;
@@ -53,7 +56,8 @@ T rowdot(const T *Ar, const T *x, int64_t ncols) {
     for (int l = 0; l < 32; ++l) v[l] = op_add(op_add(op_add(p[4 * l], p[4 * l + 1]), p[4 * l + 2]), p[4 * l + 3]);
     for (int off = 16; off > 0; off >>= 1)
         for (int l = 0; l < off; ++l) v[l] = op_add(v[l], v[l + off]);
-    return v[0];
+    *res = v[0];
+    return true;
 }
 
 template <typename T>
@@ -70,8 +74,9 @@ void wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
         const T *x = (const T *)a.host[1];
         T *out = (T *)a.host[2];
         for (int64_t i = r0 + lo; i < r0 + hi; ++i) {
-            if (aborted(ab)) return;
-            out[i] = rowdot<T>(A + i * ncols, x, ncols);
+            T v;
+            if (!rowdot<T>(A + i * ncols, x, ncols, ab, &v)) return;
+            out[i] = v;
         }
     } else {
         const T *B = (const T *)a.host[1];
@@ -80,9 +85,8 @@ void wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
         const T alpha = a.integer ? (T)(uint32_t)a.ialpha : (T)a.alpha;
         const T beta = a.integer ? (T)(uint32_t)a.ibeta : (T)a.beta;
         for (int64_t i = r0 + lo; i < r0 + hi; ++i) {
-            if (aborted(ab)) return;
-            const T va = rowdot<T>(A + i * ncols, x, ncols);
-            const T vb = rowdot<T>(B + i * ncols, x, ncols);
+            T va, vb;
+            if (!rowdot<T>(A + i * ncols, x, ncols, ab, &va) || !rowdot<T>(B + i * ncols, x, ncols, ab, &vb)) return;
             tmp[i] = va;
             y[i] = op_add(op_mul(alpha, va), op_mul(beta, vb));
         }
@@ -111,7 +115,7 @@ void wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
     thread_local std::vector<T> P;
     P.assign((size_t)kColPartitions * (size_t)w, T(0));
     for (int64_t i = 0; i < nrows; ++i) {
-        if ((i & 255) == 0 && aborted(ab)) return;
+        if ((i & 31) == 0 && aborted(ab)) return;
         T *pq = P.data() + (size_t)(i & (kColPartitions - 1)) * (size_t)w;
         const T *ar = A + i * ncols + pc0;
         if (MODE == COL_DOT) {

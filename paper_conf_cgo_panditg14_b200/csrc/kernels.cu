@@ -437,8 +437,14 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
 
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
-plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo) {
+plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo, const SlotReset r) {
     __shared__ int s_flag;
+    if (r.claim && blockIdx.x == 0 && threadIdx.x == 0) {   // next slot's dispatcher counters
+        *r.claim = 0ull;
+        for (int q = 0; q < 17; ++q) r.barrier[q] = 0u;
+        *r.merge_ctr = 0ull;
+        if (r.tasks) *r.tasks = 0ull;
+    }
     __shared__ __align__(16) typename Body::Smem smem;
     __shared__ long long s_key;
     TaskCtx tc;
@@ -509,16 +515,19 @@ struct RowDotBody {
             const long long nfull = p.ncols / 128;
             long long k = 0;
             if (p.vec4) {
-                for (; k + U <= nfull; k += U) {
+                // explicit pointer walk (no per-load index arithmetic, whatever the register
+                // budget of the kernel the body is compiled into)
+                const T *pa = Ar + 4 * lane, *pb = (NMAT == 2) ? Br + 4 * lane : nullptr, *px = p.x + 4 * lane;
+                for (; k + U <= nfull; k += U, pa += U * 128, px += U * 128) {
                     typename V4<T>::type av[U], bv[U], xv[U];
 #pragma unroll
                     for (int u = 0; u < U; ++u) {
-                        const long long j = (k + u) * 128 + 4 * lane;
-                        av[u] = ld_stream4(Ar + j);
-                        if (NMAT == 2) bv[u] = ld_stream4(Br + j);
+                        av[u] = ld_stream4(pa + u * 128);
+                        if (NMAT == 2) bv[u] = ld_stream4(pb + u * 128);
                     }
+                    if (NMAT == 2) pb += U * 128;
 #pragma unroll
-                    for (int u = 0; u < U; ++u) xv[u] = ld_cached4(p.x + (k + u) * 128 + 4 * lane);
+                    for (int u = 0; u < U; ++u) xv[u] = ld_cached4(px + u * 128);
 #pragma unroll
                     for (int u = 0; u < U; ++u) {
                         a0 = op_fma(av[u].x, xv[u].x, a0); a1 = op_fma(av[u].y, xv[u].y, a1);
@@ -605,16 +614,18 @@ struct ColDotBody {
         T acc = 0;
         if (active) {
             const T mj = (MODE == COL_SQDEV) ? p.mean[j] : T(0);
-            const T *col = p.A + j;
+            // explicit pointer walk down the column (rows w, w + 32, ...)
+            const long long stride = 32 * p.ncols;
+            const T *pc = p.A + j + (long long)w * p.ncols;
             long long i = w;
             for (; i + 7 * 32 < p.nrows; i += 8 * 32) {
                 T a[8];
 #pragma unroll
-                for (int u = 0; u < 8; ++u) a[u] = __ldcs(col + (i + 32 * u) * p.ncols);
+                for (int u = 0; u < 8; ++u) { a[u] = __ldcs(pc); pc += stride; }
 #pragma unroll
                 for (int u = 0; u < 8; ++u) acc = term(p, a[u], i + 32 * u, mj, acc);
             }
-            for (; i < p.nrows; i += 32) acc = term(p, __ldcs(col + i * p.ncols), i, mj, acc);
+            for (; i < p.nrows; i += 32, pc += stride) acc = term(p, __ldcs(pc), i, mj, acc);
         }
         sm.red[w][lane] = acc;
         __syncthreads();
@@ -1003,7 +1014,7 @@ static int occupancy_grid(int num_sms) {
 
 template <class Body>
 static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long long task_lo, long long task_hi,
-                       int num_sms, cudaStream_t s) {
+                       int num_sms, cudaStream_t s, const SlotReset *reset = nullptr) {
     const long long n = task_hi - task_lo;
     if (n <= 0) return 0;
     if (c) {
@@ -1025,7 +1036,9 @@ static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long l
         if (e != cudaSuccess) return seterr(e, "coop_kernel launch");
         return (int)grid;
     }
-    plain_kernel<Body><<<(unsigned)n, Body::kThreads, 0, s>>>(bp, task_lo);
+    SlotReset r{};
+    if (reset) r = *reset;
+    plain_kernel<Body><<<(unsigned)n, Body::kThreads, 0, s>>>(bp, task_lo, r);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return seterr(e, "plain_kernel launch");
     return (int)n;
@@ -1256,19 +1269,29 @@ struct CoopLauncher {
     }
 };
 struct PlainLauncher {
-    long long lo, hi; cudaStream_t s;
+    long long lo, hi; cudaStream_t s; const SlotReset *reset;
     template <class Body> int go(const typename Body::Params &bp) {
-        return launch_body<Body>(bp, nullptr, lo, hi, 0, s);
+        return launch_body<Body>(bp, nullptr, lo, hi, 0, s, reset);
     }
 };
+struct CapacityQuery {
+    int num_sms;
+    template <class Body> int go(const typename Body::Params &) { return occupancy_grid<Body>(num_sms); }
+};
+
+int64_t gpu_coop_capacity(const KArgs &a, const Geom &g, int num_sms) {
+    CapacityQuery q{num_sms};
+    return with_body(a, g, q);
+}
 
 int gpu_launch_coop(const KArgs &a, const Geom &g, const CoopCtl &c, int num_sms, void *stream) {
     CoopLauncher L{&c, num_sms, (cudaStream_t)stream};
     return with_body(a, g, L);
 }
 
-int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream) {
-    PlainLauncher L{task_lo, task_hi, (cudaStream_t)stream};
+int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream,
+                     const SlotReset *reset) {
+    PlainLauncher L{task_lo, task_hi, (cudaStream_t)stream, reset};
     return with_body(a, g, L);
 }
 

@@ -166,7 +166,9 @@ struct Executor {
                 if (CPU_ISSET(c, &set)) cores.push_back(c);
         }
         if (cores.empty()) cores.push_back(0);
-        T = nthreads > 0 ? nthreads : std::max<int>(1, (int)cores.size() - 1);
+        // default: every core but two -- one for the coordinator (cores[0]), one left free for
+        // the calling thread -- so no spinning party ever time-slices with another
+        T = nthreads > 0 ? nthreads : std::max<int>(1, (int)cores.size() - 2);
         active = T;
         for (int k = 0; k < T; ++k) threads.emplace_back([this, k, pin] { worker(k, pin); });
     }
@@ -183,7 +185,9 @@ struct Executor {
         if (pin && cores.size() > 1) {
             cpu_set_t s;
             CPU_ZERO(&s);
-            CPU_SET(cores[(size_t)(idx + 1) % cores.size()], &s);   // leave cores[0] to the coordinator
+            // cores[0]: the coordinator; cores[1]: the caller (unless there are too few cores)
+            const size_t skip = cores.size() > 2 ? 2 : 1;
+            CPU_SET(cores[(size_t)(idx + skip) % cores.size()], &s);
             sched_setaffinity(0, sizeof s, &s);
         }
         uint64_t seen = 0;
@@ -311,6 +315,7 @@ struct Job {
     int slot = 0;
     int64_t t0 = 0, t1 = 0, s_forced = -1;
     bool forced = false, dev_merge = false, eager = false, gpu_launched = false;
+    bool lite = false;         // single wave, no in-task polls: plain grid + exit memop, never a merge
     bool twin_alias = false;   // exact spans: the merge compares against the device copy itself
     int64_t unit = 1;          // host chunk boundaries are multiples of this many work-groups
     void *twin[6] = {nullptr}, *stage[6] = {nullptr};
@@ -330,6 +335,7 @@ struct fcl_context_st {
     int num_sms = 148;
     cudaStream_t main = nullptr, hd = nullptr, dh = nullptr;
     bool own_main = false, own_hd = false, own_dh = false;
+    cudaStream_t xs = nullptr;   // exit-signal memops of lite launches (never carries data)
     int status_location = FCL_STATUS_DEVICE;
     // One 64-bit status word per launch slot (epoch % kSlots): a dispatcher that is still
     // running after its host side returned never sees a later launch's watermark.
@@ -345,6 +351,7 @@ struct fcl_context_st {
     unsigned int *dbar = nullptr;                // grid-barrier counters, one per slot
     unsigned long long *dmctr = nullptr;         // fused-merge chunk counters, one per slot
     bool unfused = false;                        // FCL_UNFUSED_MERGE=1: merge as a separate kernel
+    bool no_lite = false;                        // FCL_NO_LITE=1: always the full dispatcher
     bool ktiming = false;                        // CUDA events around every kernel (FCL_KTIMING=1)
     cudaEvent_t main_tail = nullptr;             // ev_k1 of the last cooperative dispatcher
     uint32_t epoch = 0;
@@ -361,10 +368,16 @@ struct fcl_context_st {
     std::mutex q_mu;
     std::condition_variable q_cv;
     std::vector<Job *> queue;                    // pending jobs, FIFO
+    // Lock-free mirrors for the spin waits (coordinator wake-up, drain): a futex wake costs
+    // several microseconds on the launch path, so both sides spin for a while before sleeping.
+    std::atomic<int> q_len{0};                   // queue.size()
+    std::atomic<int> coord_sleeping{0}, drain_sleeping{0};
+    std::atomic<int> q_stop_flag{0};
     std::vector<Job *> free_jobs;
     Job *running = nullptr;
     Job *last = nullptr;                         // most recent launch (for fcl_get_launch_info)
     bool q_stop = false;
+    int coord_core = -1;                         // core the coordinator is pinned to (-1: none)
     std::thread coord;
     // errors
     std::mutex err_mu;
@@ -521,7 +534,7 @@ int64_t first_task_at(const KArgs &a, const Geom &g, int64_t ntasks, int64_t f) 
 fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, fcl_launch_info &info,
                        cudaEvent_t main_mark) {
     if (whi <= wlo) return FCL_SUCCESS;
-    CK(ctx, cudaStreamWaitEvent(ctx->dh, main_mark, 0));
+    if (main_mark) CK(ctx, cudaStreamWaitEvent(ctx->dh, main_mark, 0));   // nullptr: dh already waits
     for (int q = 0; q < L.nout; ++q) {
         fcl_buffer b = L.bufs[L.out_idx[q]];
         size_t b0, b1;
@@ -597,7 +610,7 @@ Job *job_alloc(fcl_context ctx) {
     j->status = FCL_SUCCESS;
     j->done.store(0);
     j->have_k = j->have_m = j->wm_pending = false;
-    j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = false;
+    j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = j->lite = false;
     j->unit = 1;
     std::memset(&j->info, 0, sizeof j->info);
     for (int q = 0; q < 6; ++q) j->twin[q] = j->stage[q] = nullptr;
@@ -669,11 +682,20 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         const bool aligned_split = !j.forced || j.s_forced % j.unit == 0 || j.s_forced == L.hi;
         j.twin_alias = contiguous && aligned_split && !ctx->force_twin;
     }
+    // Single wave without in-task polls: every CTA runs exactly one task, unchecked (the first
+    // task of a CTA never waits for the status), so no work-group can be skipped or aborted,
+    // the GPU computes the whole range and no merge can be needed.  The dispatcher reduces to
+    // the plain grid plus the exit signal, without status loads or arrival tail, and the host
+    // neither stages nor publishes: its finished chunks only bound the return copy.
+    const int abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
+    j.lite = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && abort_period == 0 && !ctx->no_lite &&
+             (j.t1 - j.t0) <= gpu_coop_capacity(L.a, L.g, ctx->num_sms);
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
     const void *srcs[6];
     size_t nbytes[6];
     bool hd_wait = false;
-    for (int q = 0; q < L.nout; ++q) {
+    if (j.lite) j.twin_alias = true;   // no twin and no stage
+    for (int q = 0; q < L.nout && !j.lite; ++q) {
         fcl_buffer b = L.bufs[L.out_idx[q]];
         if (!j.twin_alias) j.twin[q] = pool_get(ctx, b->bytes, &hd_wait);
         j.stage[q] = pool_get(ctx, b->bytes, &hd_wait);
@@ -718,7 +740,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     c.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot : nullptr;
     c.tstamp_next = ctx->stats ? ctx->dstamp + 4 * ((j.slot + 1) % kSlots) : nullptr;
     c.task_lo = j.t0; c.task_hi = j.t1;
-    c.abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
+    c.abort_period = abort_period;
     c.barrier = ctx->dbar + 32 * j.slot;
     c.barrier_next = ctx->dbar + 32 * ((j.slot + 1) % kSlots);
     c.merge_ctr = ctx->dmctr + j.slot;
@@ -731,7 +753,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     // dispatcher acted on and runs in the dispatcher's fused tail (or right behind it), and
     // small outputs are returned eagerly behind it -- no host round trip between the GPU
     // finishing and the result being coherent.
-    j.dev_merge = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge;
+    j.dev_merge = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && !j.lite;
     size_t out_total = 0;
     for (int q = 0; q < L.nout; ++q) {
         size_t b0, b1;
@@ -741,7 +763,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     // An INOUT buffer is read-modify-written in place by the host bodies: its return copy
     // must wait until the host workers have stopped (an abandoned chunk may still be running
     // when the GPU finishes), so only pure-OUT launches return eagerly.
-    j.eager = j.dev_merge && !L.any_inout && out_total <= ctx->eager_return_bytes;
+    j.eager = (j.dev_merge || j.lite) && !L.any_inout && out_total <= ctx->eager_return_bytes;
     DevMergeList M{};
     size_t maxb = 0;
     if (j.dev_merge) {
@@ -772,14 +794,27 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         const bool timing = ctx->ktiming || (L.o.flags & FCL_LAUNCH_TIMING);
         if (timing) CK(ctx, cudaEventRecord(j.ev_k0, ctx->main));
         ctx->tr.add("A_prelaunch", j.epoch);
-        if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0)
+        if (j.lite) {
+            const int nx = (j.slot + 1) % kSlots;
+            SlotReset r{ctx->dclaim + nx, ctx->stats ? ctx->dtasks + nx : nullptr, ctx->dmctr + nx, ctx->dbar + 32 * nx};
+            if (gpu_launch_plain(L.a, L.g, j.t0, j.t1, ctx->main, &r) < 0)
+                return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        } else if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0) {
             return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        }
         ctx->tr.add("A_launched", j.epoch);
         CK(ctx, cudaEventRecord(j.ev_k1, ctx->main));
         ctx->tr.add("A_k1", j.epoch);
         // GPU exit signal for the host executor (L18.s19): the fused tail stores the epoch to
-        // mapped host memory after its grid barrier; unfused, a bare memop does it.
-        if (!c.fused) {
+        // mapped host memory after its grid barrier; unfused, a bare memop does it.  Lite: the
+        // memop goes on its own stream behind the kernel's event, so that the main stream
+        // carries kernels only (a memop between two kernels stalls the second) and the signal
+        // does not queue behind return copies.
+        if (j.lite) {
+            CK(ctx, cudaStreamWaitEvent(ctx->xs, j.ev_k1, 0));
+            fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->xs, false);
+            if (xs != FCL_SUCCESS) return xs;
+        } else if (!c.fused) {
             fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->main, false);
             if (xs != FCL_SUCCESS) return xs;
         }
@@ -801,9 +836,9 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
             return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
         info.gpu_launches += 1;
     }
-    if (j.dev_merge && j.eager) {
+    if (j.eager) {
         cudaEvent_t mark = j.ev_k1;
-        if (!c.fused) { CK(ctx, cudaEventRecord(j.ev_ret, ctx->main)); mark = j.ev_ret; }
+        if (!c.fused && !j.lite) { CK(ctx, cudaEventRecord(j.ev_ret, ctx->main)); mark = j.ev_ret; }
         fcl_status st = enqueue_d2h(ctx, L, L.lo, L.hi, info, mark);
         if (st != FCL_SUCCESS) return st;
     }
@@ -852,6 +887,10 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         in_flight = true;
     };
     auto stage_chunk = [&](int64_t clo, int64_t chi) -> fcl_status {
+        if (j.lite) {   // the GPU computes everything: the finished chunk only bounds the return
+            info.published_watermark = clo;
+            return FCL_SUCCESS;
+        }
         if (!hd_joined) {
             CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
             hd_joined = true;
@@ -920,8 +959,9 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     info.gpu_watermark = L.hi;
     fcl_status st = FCL_SUCCESS;
 
-    if (j.dev_merge) {
-        // the merge is already queued; only the precise return of large outputs is left
+    if (j.dev_merge || j.lite) {
+        // the merge is already queued (or, lite, cannot be needed); only the precise return
+        // of large outputs is left
         if (gpu_done) {
             if (!j.eager) {
                 // The host copy already holds every published chunk, and the GPU acted on some
@@ -930,11 +970,11 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
                 // no device read of the GPU's watermark on this path.
                 st = enqueue_d2h(ctx, L, L.lo, info.published_watermark, info, j.ev_k1);
             }
-            j.wm_pending = true;   // info.gpu_watermark resolved lazily by fcl_get_launch_info
+            j.wm_pending = !j.lite;   // info.gpu_watermark resolved lazily by fcl_get_launch_info
         } else {
             info.cpu_did_all = 1;      // host authoritative (L16.s21); device merged behind
-            info.gpu_watermark = L.lo;
-            info.merged = 1;
+            info.gpu_watermark = j.lite ? L.hi : L.lo;   // lite: the GPU computes every work-group
+            info.merged = j.lite ? 0 : 1;
         }
     } else {
         // Forced split / deferred merge: the host decides merge domain and return (C15/C17)
@@ -980,12 +1020,32 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
 // ------------------------------------------------------------------------------------------
 void coordinator(fcl_context ctx) {
     cudaSetDevice(ctx->device);
+    if (ctx->coord_core >= 0) {   // its own core: it spins on the GPU exit word and the workers
+        cpu_set_t cs;
+        CPU_ZERO(&cs);
+        CPU_SET(ctx->coord_core, &cs);
+        sched_setaffinity(0, sizeof cs, &cs);
+    }
     for (;;) {
         Job *j = nullptr;
+        // spin for work for a while (launches come in bursts), then sleep on the condvar
+        auto t0 = Clock::now();
+        while (ctx->q_len.load(std::memory_order_acquire) == 0 && !ctx->q_stop_flag.load(std::memory_order_relaxed)) {
+            _mm_pause();
+            if (std::chrono::duration_cast<std::chrono::nanoseconds>(Clock::now() - t0).count() > ctx->ex.spin_ns) {
+                std::unique_lock<std::mutex> lk(ctx->q_mu);
+                ctx->coord_sleeping.store(1);
+                ctx->q_cv.wait(lk, [&] { return ctx->q_stop || !ctx->queue.empty(); });
+                ctx->coord_sleeping.store(0);
+                t0 = Clock::now();
+            }
+        }
         {
-            std::unique_lock<std::mutex> lk(ctx->q_mu);
-            ctx->q_cv.wait(lk, [&] { return ctx->q_stop || !ctx->queue.empty(); });
-            if (ctx->queue.empty()) return;   // stop requested and nothing pending
+            std::lock_guard<std::mutex> lk(ctx->q_mu);
+            if (ctx->queue.empty()) {
+                if (ctx->q_stop) return;   // stop requested and nothing pending
+                continue;
+            }
             j = ctx->queue.front();
             ctx->running = j;
         }
@@ -999,18 +1059,29 @@ void coordinator(fcl_context ctx) {
             j->status = st;
             if (st != FCL_SUCCESS && ctx->sticky.load() == FCL_SUCCESS) ctx->sticky = st;
             ctx->queue.erase(ctx->queue.begin());
+            ctx->q_len.fetch_sub(1, std::memory_order_release);
             ctx->running = nullptr;
             j->done.store(1, std::memory_order_release);
             if (j != ctx->last) ctx->free_jobs.push_back(j);
         }
-        ctx->q_cv.notify_all();
+        if (ctx->drain_sleeping.load()) ctx->q_cv.notify_all();
     }
 }
 
-// Wait until every queued launch's host side is done.
+// Wait until every queued launch's host side is done (spin first, then sleep).
 void drain(fcl_context ctx) {
-    std::unique_lock<std::mutex> lk(ctx->q_mu);
-    ctx->q_cv.wait(lk, [&] { return ctx->queue.empty(); });
+    auto t0 = Clock::now();
+    while (ctx->q_len.load(std::memory_order_acquire) > 0) {
+        _mm_pause();
+        if (std::chrono::duration_cast<std::chrono::nanoseconds>(Clock::now() - t0).count() > ctx->ex.spin_ns) {
+            std::unique_lock<std::mutex> lk(ctx->q_mu);
+            ctx->drain_sleeping.fetch_add(1);
+            ctx->q_cv.wait(lk, [&] { return ctx->queue.empty(); });
+            ctx->drain_sleeping.fetch_sub(1);
+            return;
+        }
+    }
+    std::lock_guard<std::mutex> lk(ctx->q_mu);   // acquire the coordinator's last critical section
 }
 
 // A new launch conflicts with a pending one if either writes a buffer the other touches.
@@ -1147,6 +1218,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if ((e = mk(d.main_stream, &ctx->main, &ctx->own_main)) != cudaSuccess) return fail(e, "main stream");
     if ((e = mk(d.hd_stream, &ctx->hd, &ctx->own_hd)) != cudaSuccess) return fail(e, "hd stream");
     if ((e = mk(d.dh_stream, &ctx->dh, &ctx->own_dh)) != cudaSuccess) return fail(e, "dh stream");
+    if ((e = cudaStreamCreateWithFlags(&ctx->xs, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "exit-signal stream");
     // status words (one per launch slot), GPU-exit word, pinned copy of the wm word
     void *hp = nullptr, *dp = nullptr;
     if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocPortable)) != cudaSuccess) return fail(e, "pinned scratch");
@@ -1198,6 +1270,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->tr.on = getenv("FCL_TRACE") && atoi(getenv("FCL_TRACE")) != 0;
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
     ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
+    ctx->no_lite = getenv("FCL_NO_LITE") && atoi(getenv("FCL_NO_LITE")) != 0;
     if (getenv("FCL_KTIMING")) ctx->ktiming = atoi(getenv("FCL_KTIMING")) != 0;
     if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail(e, "init sync");
     const char *pin = getenv("FCL_PIN_THREADS");
@@ -1205,6 +1278,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     int nthr = d.n_host_threads;
     if (nthr <= 0 && getenv("FCL_HOST_THREADS")) nthr = atoi(getenv("FCL_HOST_THREADS"));
     ctx->ex.start(nthr, do_pin);
+    ctx->coord_core = (do_pin && !ctx->ex.cores.empty()) ? ctx->ex.cores[0] : -1;
     ctx->coord = std::thread(coordinator, ctx);
     *out = ctx;
     return FCL_SUCCESS;
@@ -1225,6 +1299,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     {
         std::lock_guard<std::mutex> lk(ctx->q_mu);
         ctx->q_stop = true;
+        ctx->q_stop_flag.store(1);
     }
     ctx->q_cv.notify_all();
     if (ctx->coord.joinable()) ctx->coord.join();
@@ -1252,6 +1327,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->own_main) cudaStreamDestroy(ctx->main);
     if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
     if (ctx->own_dh) cudaStreamDestroy(ctx->dh);
+    if (ctx->xs) cudaStreamDestroy(ctx->xs);
     delete ctx;
     return FCL_SUCCESS;
 }
@@ -1601,8 +1677,9 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         if (ctx->last && ctx->last != j && ctx->last->done.load()) ctx->free_jobs.push_back(ctx->last);
         ctx->last = j;
         ctx->queue.push_back(j);
+        ctx->q_len.fetch_add(1, std::memory_order_release);
     }
-    ctx->q_cv.notify_all();
+    if (ctx->coord_sleeping.load()) ctx->q_cv.notify_all();
     pool_trim(ctx);
     if (L.o.blocking) {
         drain(ctx);
@@ -1660,8 +1737,11 @@ fcl_status fcl_finish(fcl_context ctx) {
     ctx->tr.add("finish_drained", ctx->epoch);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
     CK(ctx, cudaStreamSynchronize(ctx->main));
+    ctx->tr.add("finish_main", ctx->epoch);
     CK(ctx, cudaStreamSynchronize(ctx->hd));
+    ctx->tr.add("finish_hd", ctx->epoch);
     CK(ctx, cudaStreamSynchronize(ctx->dh));
+    ctx->tr.add("finish_dh", ctx->epoch);
     CK(ctx, cudaGetLastError());
     ctx->tr.add("finish_end", ctx->epoch);
     if (ctx->tr.on && ctx->stats) {

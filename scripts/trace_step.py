@@ -27,19 +27,24 @@ for rep in range(30):
         L()
     ctx.finish()
 ctx.release()
-# summarize the last 10 steps
+# summarize the last steps: host events per step, device stamps separately
 recs = [l.split() for l in open(os.environ["FCL_TRACE_FILE"])]
+host = [(float(t), tag, int(e)) for t, tag, e in recs if not tag.startswith("gpu_")]
 steps, cur = [], []
-for t, tag, e in recs:
-    cur.append((float(t), tag, int(e)))
+for t, tag, e in host:
+    cur.append((t, tag, e))
     if tag == "finish_end":
         steps.append(cur); cur = []
 for st in steps[-3:]:
     t0 = st[0][0]
-    print(" | ".join(f"{tag}:{e}@{(t - t0) * 1000:.1f}us" for t, tag, e in st))
-gpu = [(float(t), tag, int(e)) for t, tag, e in recs if tag.startswith("gpu_")]
-# last 6 slots' device stamps, relative to the earliest shown
-gpu = sorted(gpu)[-12:]
+    print(" | ".join(f"{tag}:{e}@{(t - t0) * 1000:.1f}" for t, tag, e in st))
+gpu = sorted((float(t), tag, int(e)) for t, tag, e in recs if tag.startswith("gpu_"))
 if gpu:
-    g0 = gpu[0][0]
-    print("GPU:", " | ".join(f"{tag}[slot{e}]@{(t - g0) * 1000:.1f}us" for t, tag, e in gpu))
+    # device stamps of the last few slots, relative to the earliest of them (us)
+    by_slot = {}
+    for t, tag, e in gpu:
+        by_slot.setdefault(e, {})[tag] = t
+    last = sorted(by_slot.items(), key=lambda kv: min(kv[1].values()))[-6:]
+    g0 = min(last[0][1].values())
+    for slot, d in last:
+        print("GPU slot", slot, " ".join(f"{k[4:-3]}@{(v - g0) * 1000:.1f}" for k, v in sorted(d.items(), key=lambda kv: kv[1])))
