@@ -358,6 +358,13 @@ struct fcl_context_st {
     PFN_writeValue64 write64 = nullptr;
     bool stats = false;                          // count executed GPU tasks, time merges (FCL_STATS=1)
     size_t eager_return_bytes = 8u << 20;        // outputs up to this size return right behind the merge
+    // Return race: when the GPU finishes first and a large output is still to come
+    // back, it is returned in ascending pieces while the host keeps computing from the top.
+    bool no_race = false;                        // FCL_NO_RACE=1
+    size_t race_min_bytes = 32u << 20;           // only for returns at least this large
+    size_t race_piece_bytes = 8u << 20;          // return-copy piece
+    double race_chunk_ms = 1.0;                  // host chunk length during the race
+    cudaEvent_t race_ev[4] = {};                 // completion of the outstanding pieces (on dh)
     bool force_twin = false;                     // FCL_FORCE_TWIN=1: always capture a twin (Fig 9 as printed)
     // twin/stage pool (C6, L20.s23-29)
     std::mutex pool_mu;
@@ -947,7 +954,92 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             _mm_pause();
         }
     }
-    if (in_flight) {   // GPU finished first: abandon the running chunk (L18.s19)
+    // Return race: the GPU finished first (its copy is complete: it ran every work-group it did
+    // not skip, and the skipped ones were merged in its tail), but the host still needs the
+    // device's results below its own frontier hi_cur.  Instead of abandoning the running chunk
+    // and copying everything, the result comes back in ascending pieces on dh while the host
+    // goes on computing chunks from the top; the two meet in the middle.  A piece never
+    // overlaps a running chunk (INOUT outputs are updated in place on the host); when the copy
+    // front reaches the running chunk, that chunk is abandoned and its range copied too.
+    auto out_bytes = [&](int64_t a, int64_t b) -> size_t {
+        size_t t = 0;
+        for (int q = 0; q < L.nout; ++q) {
+            size_t b0, b1;
+            out_span(L.a, L.g, L.out_idx[q], a, b, &b0, &b1);
+            t += b1 - b0;
+        }
+        return t;
+    };
+    const bool race = gpu_done && !j.forced && (j.dev_merge || j.lite) && !j.eager && !ctx->no_race &&
+                      hi_cur > L.lo && out_bytes(L.lo, hi_cur) >= ctx->race_min_bytes;
+    if (race) {
+        ctx->tr.add("race_begin", j.epoch);
+        CK(ctx, cudaStreamWaitEvent(ctx->dh, j.ev_k1, 0));
+        const size_t unit_b = std::max<size_t>(1, out_bytes(L.lo, std::min<int64_t>(L.lo + j.unit, L.hi)));
+        const int64_t piece = j.unit * std::max<int64_t>(1, (int64_t)(ctx->race_piece_bytes / unit_b));
+        int64_t F = L.lo;   // end of the prefix whose return is queued
+        int qh = 0, qn = 0;
+        auto race_chunk = [&]() {
+            const double per_wg = cpu_done_wgs > 0 ? busy / (double)cpu_done_wgs : -1.0;
+            int64_t size = per_wg > 0 ? (int64_t)(ctx->race_chunk_ms / per_wg) : ceil_pct(pct, nwg);
+            size = std::max<int64_t>(size, nact);
+            size = (size + j.unit - 1) / j.unit * j.unit;
+            const int64_t room = (hi_cur - (F + piece)) / j.unit * j.unit;   // leave the next piece alone
+            if (room < j.unit) return;
+            size = std::min(size, room);
+            cur_hi = hi_cur; cur_lo = hi_cur - size; cur_size = size;
+            if (nch < 64) info.chunk_sizes[nch] = (int32_t)size;
+            ++nch;
+            t_start = now_ms();
+            ex.submit(L.a, L.g, cur_lo, cur_hi, 1, nact);
+            in_flight = true;
+        };
+        for (;;) {
+            if (in_flight && ex.finished()) {
+                busy += now_ms() - t_start;
+                in_flight = false;
+                cpu_done_wgs += cur_size;
+                hi_cur = cur_lo;
+                info.published_watermark = hi_cur;   // the host's frontier
+                race_chunk();
+            }
+            const int64_t limit = in_flight ? cur_lo : hi_cur;
+            if (F >= limit) {
+                if (!in_flight) break;   // everything below the host's frontier is on its way
+                ex.abort_flag = 1;       // the copy front reached the running chunk
+                ex.wait();
+                busy += now_ms() - t_start;
+                ex.abort_flag = 0;
+                in_flight = false;
+                continue;
+            }
+            if (qn < 2) {
+                const int64_t b = std::min<int64_t>(F + piece, limit);
+                for (int q = 0; q < L.nout; ++q) {
+                    fcl_buffer ob = L.bufs[L.out_idx[q]];
+                    size_t b0, b1;
+                    out_span(L.a, L.g, L.out_idx[q], F, b, &b0, &b1);
+                    if (b1 <= b0) continue;
+                    CK(ctx, cudaMemcpyAsync((char *)ob->host + b0, (char *)ob->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
+                    info.d2h_bytes += (int64_t)(b1 - b0);
+                }
+                CK(ctx, cudaEventRecord(ctx->race_ev[(qh + qn) & 3], ctx->dh));
+                ++qn;
+                F = b;
+            } else {
+                const cudaError_t q = cudaEventQuery(ctx->race_ev[qh & 3]);
+                if (q == cudaSuccess) { ++qh; --qn; }
+                else if (q != cudaErrorNotReady) return cuda_fail(ctx, q, "return race");
+                else for (int k = 0; k < 64; ++k) _mm_pause();
+            }
+        }
+        for (int q = 0; q < L.nout; ++q) {   // the buffers' return events follow the last piece
+            fcl_buffer ob = L.bufs[L.out_idx[q]];
+            CK(ctx, cudaEventRecord(ob->d2h_ev, ctx->dh));
+            ob->d2h_pending = true;
+        }
+        ctx->tr.add("race_end", j.epoch);
+    } else if (in_flight) {   // GPU finished first: abandon the running chunk (L18.s19)
         ex.abort_flag = 1;
         ex.wait();
         busy += now_ms() - t_start;
@@ -963,7 +1055,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         // the merge is already queued (or, lite, cannot be needed); only the precise return
         // of large outputs is left
         if (gpu_done) {
-            if (!j.eager) {
+            if (!j.eager && !race) {
                 // The host copy already holds every published chunk, and the GPU acted on some
                 // watermark >= the lowest one published, so returning the device copy (merged
                 // by the fused tail) below the host's own published watermark is complete --
@@ -1252,7 +1344,8 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->dbar = (unsigned int *)(ctx->dmctr + fcl_context_st::kSlots);
     for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1})
         if ((e = cudaEventCreate(pe)) != cudaSuccess) return fail(e, "events");
-    for (cudaEvent_t *pe : {&ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h})
+    for (cudaEvent_t *pe : {&ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h, &ctx->race_ev[0], &ctx->race_ev[1],
+                            &ctx->race_ev[2], &ctx->race_ev[3]})
         if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
     // stream memory operations for publication (driver entry point; fall back to a kernel store)
     {
@@ -1271,6 +1364,10 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
     ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
     ctx->no_lite = getenv("FCL_NO_LITE") && atoi(getenv("FCL_NO_LITE")) != 0;
+    ctx->no_race = getenv("FCL_NO_RACE") && atoi(getenv("FCL_NO_RACE")) != 0;
+    if (getenv("FCL_RACE_MIN_BYTES")) ctx->race_min_bytes = (size_t)atoll(getenv("FCL_RACE_MIN_BYTES"));
+    if (getenv("FCL_RACE_PIECE_BYTES")) ctx->race_piece_bytes = std::max<size_t>(4096, (size_t)atoll(getenv("FCL_RACE_PIECE_BYTES")));
+    if (getenv("FCL_RACE_CHUNK_MS")) ctx->race_chunk_ms = atof(getenv("FCL_RACE_CHUNK_MS"));
     if (getenv("FCL_KTIMING")) ctx->ktiming = atoi(getenv("FCL_KTIMING")) != 0;
     if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail(e, "init sync");
     const char *pin = getenv("FCL_PIN_THREADS");
@@ -1317,7 +1414,8 @@ fcl_status fcl_release_context(fcl_context ctx) {
             if (e) cudaEventDestroy(e);
         delete j;
     }
-    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_k1, ctx->ev_mark, ctx->ev_hd_release, ctx->ev_gd2h})
+    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_k1, ctx->ev_mark, ctx->ev_hd_release, ctx->ev_gd2h, ctx->race_ev[0],
+                          ctx->race_ev[1], ctx->race_ev[2], ctx->race_ev[3]})
         if (e) cudaEventDestroy(e);
     if (ctx->status_host) cudaFreeHost(ctx->status_host);
     else if (ctx->status_dptr) cudaFree(ctx->status_dptr);

@@ -123,6 +123,39 @@ def test_free_running_coop(oracle_mod, case, status, twin, monkeypatch):
         ctx.release()
 
 
+RACE_CASES = [("conv2d", 600, 1000, False, None, (32, 8)), ("conv2d", 333, 515, True, None, (32, 8)),
+              ("syrk", 512, 96, False, None, (32, 8)), ("corr_reduce", 700, 600, False, None, (32, 8)),
+              ("gesummv", 2048, 2048, False, 64, None), ("atax_y", 1500, 3000, True, 32, None)]
+
+
+@pytest.mark.parametrize("case", RACE_CASES, ids=_ids)
+def test_return_race(oracle_mod, case, monkeypatch):
+    """Return race: the output comes back in small ascending pieces while the
+    host keeps computing chunks from the top; INOUT outputs (SYRK, CORR reduce), two outputs
+    (GESUMMV) and 2-D spans.  Host and device copies equal the single-device result."""
+    from paper_conf_cgo_panditg14_b200 import fcl
+    for k, v in dict(FCL_RACE_MIN_BYTES="1", FCL_RACE_PIECE_BYTES="4096", FCL_RACE_CHUNK_MS="0.02",
+                     FCL_EAGER_RETURN_BYTES="0").items():
+        monkeypatch.setenv(k, v)
+    ctx = fcl.Context(0)
+    try:
+        P = _problem(case, seed=12)
+        R = oracle_outputs(oracle_mod, P)
+        ref, _ = H.run(ctx, P, mode="gpu")
+        for trial, kw in enumerate([{}, dict(host_delay_us=30), dict(init_chunk_pct=1, step_pct=0)]):
+            bufs = H.create_buffers(ctx, P)
+            out, info = H.run(ctx, P, mode="coop", bufs=bufs, **kw)
+            for k in P.out_indices:
+                assert_bits(out[k], ref[k], f"{_ids(case)} race host buf{k} {kw}")
+                dev = H.device_array(bufs[k], np.int32 if P.integer else np.float32)
+                assert_bits(dev, ref[k], f"{_ids(case)} race device buf{k} {kw}")
+                assert_parity(out[k], R[k], P.integer, _ids(case))
+            for b in bufs:
+                b.release()
+    finally:
+        ctx.release()
+
+
 @pytest.mark.parametrize("case", [CASES[0], CASES[9], CASES[12], CASES[16]], ids=_ids)
 def test_fault_injection(ctx, oracle_mod, case):
     """Dropped publications, slow host, tiny and huge chunks: the result never changes."""
