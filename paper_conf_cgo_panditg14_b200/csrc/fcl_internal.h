@@ -141,6 +141,9 @@ const char *gpu_last_error_string();
 // storing an incomplete value (write-once).
 void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts,
                   const volatile int *abort_flag);
+// Work-groups per executor claim (host_exec_range) and the range executor itself.
+int64_t host_batch(const KArgs &a, const Geom &g);
+void host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *abort_flag);
 
 // Conservative contiguous byte span [*b0, *b1) of output buffer `buf_index` written by
 // work-groups [lo, hi) (superset of the exact footprint; the diff-merge tolerates it).

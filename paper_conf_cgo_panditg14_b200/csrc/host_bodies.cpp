@@ -156,34 +156,35 @@ inline Wg2D wg2d(const Geom &g, int64_t fgid, int64_t nrows, int64_t ncols) {
 }
 
 // ---------------------------------------------------------------- CORR reduce (in place)
-void wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+// Rectangle [r0, r1) x [c0, c1) of the output (a work-group, or a batch of work-groups of one
+// work-group row: wide rows stream and vectorize).
+void corr_reduce_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
-    Wg2D w = wg2d(g, fgid, n, m);
-    if (w.r0 >= w.r1 || w.c0 >= w.c1) return;
-    int64_t lo, hi;
-    part_range(w.r1 - w.r0, part, nparts, lo, hi);
     float *d = (float *)a.host[0];
     const float *mean = (const float *)a.host[1], *sd = (const float *)a.host[2];
     const float sqrtn = std::sqrt((float)n);
-    for (int64_t i = w.r0 + lo; i < w.r0 + hi; ++i) {
+    for (int64_t i = r0; i < r1; ++i) {
         if (aborted(ab)) return;
-        for (int64_t j = w.c0; j < w.c1; ++j) {
+        for (int64_t j = c0; j < c1; ++j) {
             const float den = sqrtn * sd[j];
             d[i * m + j] = (d[i * m + j] + (-mean[j])) / den;
         }
     }
 }
 
-// ---------------------------------------------------------------- 2DCONV
-template <typename T>
-void wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
-    const int64_t ni = a.n0, nj = a.n1;
-    Wg2D w = wg2d(g, fgid, ni, nj);
-    const int64_t r0 = std::max<int64_t>(w.r0, 1), r1 = std::min<int64_t>(w.r1, ni - 1);
-    const int64_t c0 = std::max<int64_t>(w.c0, 1), c1 = std::min<int64_t>(w.c1, nj - 1);
-    if (r0 >= r1 || c0 >= c1) return;
+void wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+    Wg2D w = wg2d(g, fgid, a.n0, a.n1);
+    if (w.r0 >= w.r1 || w.c0 >= w.c1) return;
     int64_t lo, hi;
-    part_range(r1 - r0, part, nparts, lo, hi);
+    part_range(w.r1 - w.r0, part, nparts, lo, hi);
+    corr_reduce_rect(a, w.r0 + lo, w.r0 + hi, w.c0, w.c1, ab);
+}
+
+// ---------------------------------------------------------------- 2DCONV
+// Rectangle [r0, r1) x [c0, c1) of the output, border excluded by the caller.
+template <typename T>
+void conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
+    const int64_t nj = a.n1;
     const T *A = (const T *)a.host[0];
     T *B = (T *)a.host[1];
     T c[9];
@@ -194,7 +195,7 @@ void wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
         const float cf[9] = {0.2f, 0.5f, -0.8f, -0.3f, 0.6f, -0.9f, 0.4f, 0.7f, 0.10f};
         for (int q = 0; q < 9; ++q) c[q] = (T)cf[q];
     }
-    for (int64_t i = r0 + lo; i < r0 + hi; ++i) {
+    for (int64_t i = r0; i < r1; ++i) {
         if (aborted(ab)) return;
         const T *um = A + (i - 1) * nj, *u0 = A + i * nj, *up = A + (i + 1) * nj;
         for (int64_t j = c0; j < c1; ++j) {
@@ -210,6 +211,18 @@ void wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
             B[i * nj + j] = s;
         }
     }
+}
+
+template <typename T>
+void wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+    const int64_t ni = a.n0, nj = a.n1;
+    Wg2D w = wg2d(g, fgid, ni, nj);
+    const int64_t r0 = std::max<int64_t>(w.r0, 1), r1 = std::min<int64_t>(w.r1, ni - 1);
+    const int64_t c0 = std::max<int64_t>(w.c0, 1), c1 = std::min<int64_t>(w.c1, nj - 1);
+    if (r0 >= r1 || c0 >= c1) return;
+    int64_t lo, hi;
+    part_range(r1 - r0, part, nparts, lo, hi);
+    conv2d_rect<T>(a, r0 + lo, r0 + hi, c0, c1, ab);
 }
 
 // ---------------------------------------------------------------- SYRK / SYR2K
@@ -348,6 +361,44 @@ void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
         else wg_syrk<float, true>(a, g, fgid, part, nparts, abort_flag);
         break;
     default: break;
+    }
+}
+
+// Work-groups per executor claim: 2-D row-major bodies take runs of work-groups of one
+// work-group row as one wide rectangle (2048 columns); the others one work-group at a time.
+int64_t host_batch(const KArgs &a, const Geom &g) {
+    if ((a.kernel == K_CONV2D || a.kernel == K_CORR_REDUCE) && g.work_dim == 2)
+        return std::max<int64_t>(1, 2048 / g.lws[0]);
+    return 1;
+}
+
+// Work-groups [f_lo, f_hi) (any order is valid: every work-group writes only its own outputs).
+void host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *ab) {
+    if ((a.kernel == K_CONV2D || a.kernel == K_CORR_REDUCE) && g.work_dim == 2) {
+        const int64_t ngx = g.ng[0];
+        for (int64_t f = f_lo; f < f_hi;) {   // one segment per work-group row
+            const int64_t gy = f / ngx, gx0 = f % ngx;
+            const int64_t gx1 = std::min<int64_t>(ngx, gx0 + (f_hi - f));
+            Wg2D w0 = wg2d(g, f, a.n0, a.n1);
+            const int64_t c1 = std::min<int64_t>(gx1 * g.lws[0], a.n1);
+            if (a.kernel == K_CORR_REDUCE) {
+                corr_reduce_rect(a, w0.r0, w0.r1, w0.c0, c1, ab);
+            } else {
+                const int64_t r0 = std::max<int64_t>(w0.r0, 1), r1 = std::min<int64_t>(w0.r1, a.n0 - 1);
+                const int64_t c0 = std::max<int64_t>(w0.c0, 1), cc1 = std::min<int64_t>(c1, a.n1 - 1);
+                if (r0 < r1 && c0 < cc1) {
+                    if (a.integer) conv2d_rect<uint32_t>(a, r0, r1, c0, cc1, ab);
+                    else conv2d_rect<float>(a, r0, r1, c0, cc1, ab);
+                }
+            }
+            if (aborted(ab)) return;
+            f = gy * ngx + gx1;
+        }
+        return;
+    }
+    for (int64_t f = f_hi - 1; f >= f_lo; --f) {
+        if (aborted(ab)) return;
+        host_exec_wg(a, g, f, 0, 1, ab);
     }
 }
 

@@ -154,7 +154,7 @@ struct Executor {
     // worker still looping on a finished job can never consume an item of the next one.
     std::atomic<uint64_t> next{0};
     std::atomic<int64_t> done{0};
-    std::atomic<int64_t> executed{0};
+    int64_t batch = 1;   // work-groups per claim (host_batch), 1 when work-groups are split
     volatile int abort_flag = 0;
     int64_t spin_ns = 20 * 1000 * 1000;   // spin 20 ms after a job before sleeping
 
@@ -213,9 +213,13 @@ struct Executor {
                 if (it >= total) break;
                 if (!next.compare_exchange_weak(v, v + 1, std::memory_order_acq_rel)) continue;
                 if (!abort_flag) {
-                    const int64_t fgid = hi - 1 - it / nparts;   // descending (L14.s36)
-                    host_exec_wg(a, g, fgid, (int)(it % nparts), nparts, &abort_flag);
-                    if (!abort_flag) executed.fetch_add(1, std::memory_order_relaxed);
+                    if (batch == 1) {
+                        const int64_t fgid = hi - 1 - it / nparts;   // descending (L14.s36)
+                        host_exec_wg(a, g, fgid, (int)(it % nparts), nparts, &abort_flag);
+                    } else {   // a run of work-groups, runs claimed in descending order
+                        const int64_t fh = hi - it * batch, fl = std::max<int64_t>(lo, fh - batch);
+                        host_exec_range(a, g, fl, fh, &abort_flag);
+                    }
                 }
                 done.fetch_add(1, std::memory_order_acq_rel);
             }
@@ -224,7 +228,8 @@ struct Executor {
     // Submit work-groups [lo_, hi_) split `parts` ways; returns immediately.
     void submit(const KArgs &a_, const Geom &g_, int64_t lo_, int64_t hi_, int parts, int nact) {
         a = a_; g = g_; lo = lo_; hi = hi_; nparts = parts;
-        total = (hi_ - lo_) * parts;
+        batch = parts > 1 ? 1 : std::max<int64_t>(1, host_batch(a_, g_));
+        total = parts > 1 ? (hi_ - lo_) * parts : (hi_ - lo_ + batch - 1) / batch;
         active = std::max(1, std::min(nact, T));
         done.store(0, std::memory_order_relaxed);
         const uint64_t g1 = gen.load(std::memory_order_relaxed) + 1;
