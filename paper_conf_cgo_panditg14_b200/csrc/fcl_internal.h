@@ -75,6 +75,7 @@ struct CoopCtl {
     long long task_lo, task_hi;         // task index range of this launch
     int abort_period;                   // in-task poll period (body-specific units); 0 = none
     int check_first;                    // 1: check the watermark before a CTA's first task too
+    int status_mapped;                  // 1: status in mapped host memory (synchronous loads only)
     unsigned long long *tstamp;         // optional %globaltimer stamps [start, end] (stats mode)
     unsigned long long *tstamp_next;    // the next launch's stamps (its end stamp is reset here)
     int fused;                          // 1: grid barrier + exit signal + merge in this kernel

@@ -76,21 +76,43 @@ __device__ __forceinline__ unsigned int decode_w(unsigned long long st, const Co
     return ((unsigned int)(st >> 32) == c.epoch) ? (unsigned int)st : c.w_default;
 }
 
-// Per-task view of the status for in-task polling (abort checks in loops, Fig 12).  Only the
-// prefetched status word lives in a register; the task key and the abort verdict are in
-// shared memory, so a polling body keeps its registers.
+// Status prefetch without a register: thread 0 copies the 16-byte aligned pair holding the
+// status word into shared memory with cp.async.cg (L2, never a stale L1 line; the publication
+// memop lands in L2) and collects it at the next check.  Status in mapped host memory is read
+// synchronously instead (system-scope load, no caching assumptions).
+__device__ __forceinline__ void status_prefetch(const CoopCtl &c, unsigned long long *s_st) {
+    if (c.status_mapped) return;
+    const unsigned long long *src = (const unsigned long long *)((uintptr_t)c.status & ~(uintptr_t)15);
+    const unsigned int dst = (unsigned int)__cvta_generic_to_shared(s_st);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n\tcp.async.commit_group;\n" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ unsigned long long status_take(const CoopCtl &c, const unsigned long long *s_st) {
+    if (c.status_mapped) return ld_status(c.status);
+    asm volatile("cp.async.wait_all;\n" ::: "memory");
+    return *(volatile const unsigned long long *)(s_st + (((uintptr_t)c.status >> 3) & 1));
+}
+
+// Per-task view of the status for in-task polling (abort checks in loops, Fig 12).  Nothing
+// of it lives in registers across the body: the prefetched status, the task key and the abort
+// verdict are all in shared memory, so a polling body keeps its whole register budget.
 struct TaskCtx {
     const CoopCtl *c;            // nullptr for plain launches (parameter space, no register copy)
-    unsigned long long pending;  // thread 0: status word loaded at the previous poll
+    unsigned long long *s_st;    // shared, 16-byte aligned: status pair prefetched by thread 0
     long long *s_key;            // shared: key of the running task
     int *s_flag;                 // shared broadcast slot (D2: the local 'completedatcpu'); w + 1 after an abort
 
-    // Called by ALL threads at a CTA-uniform point with a CTA-uniform iteration count.
-    __device__ __forceinline__ bool poll(int it) {
-        if (c == nullptr || c->abort_period <= 0 || it == 0 || (it % c->abort_period) != 0) return false;
+    // In-task poll period in body iterations (a huge value when there is none): bodies run
+    // their inner loop in blocks of this many iterations and call check() between blocks, so
+    // the inner loop itself carries no polling code.
+    __device__ __forceinline__ long long period() const {
+        return (c != nullptr && c->abort_period > 0) ? (long long)c->abort_period : (1ll << 62);
+    }
+    // Called by ALL threads at a CTA-uniform point.
+    __device__ __forceinline__ bool check() {
+        if (c == nullptr || c->abort_period <= 0) return false;
         if (threadIdx.x == 0) {
-            const unsigned int w = decode_w(pending, *c);
-            pending = ld_status(c->status);   // prefetch: consumed at the next poll
+            const unsigned int w = decode_w(status_take(*c, s_st), *c);
+            status_prefetch(*c, s_st);   // consumed at the next poll
             *s_flag = ((unsigned long long)*s_key >= (unsigned long long)w) ? (int)(w + 1u) : 0;
         }
         __syncthreads();
@@ -313,6 +335,7 @@ template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
 coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename Body::Params bp) {
     __shared__ long long s_task, s_key;
+    __shared__ __align__(16) unsigned long long s_st[2];
     __shared__ unsigned int s_w;
     __shared__ int s_flag;
     __shared__ __align__(16) typename Body::Smem smem;
@@ -349,8 +372,10 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     }
     const bool claims = c.task_lo + (long long)gridDim.x < c.task_hi;
     TaskCtx tc;
-    tc.c = &c; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.pending = 0;
-    if (threadIdx.x == 0) tc.pending = ld_status(c.status);
+    tc.c = &c; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.s_st = s_st;
+    // the status is needed only by in-task polls and by the check before a claimed task
+    const bool need_status = claims || c.abort_period > 0;
+    if (threadIdx.x == 0 && need_status) status_prefetch(c, s_st);
     bool marked = false;   // thread 0: this CTA recorded a watermark (skip or abort)
     for (;;) {
         if (t >= c.task_hi) break;
@@ -363,7 +388,8 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
         // claim the next task while this one runs (no claim at all when the grid already
         // covers every task: no contention on the counter)
         long long t_next = c.task_hi;
-        if (threadIdx.x == 0 && claims) t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
+        if (!Body::kLateClaim && threadIdx.x == 0 && claims)
+            t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
         const bool aborted = Body::run(bp, t, tc, smem);
         if (aborted) {
             if (threadIdx.x == 0) { record_wm(c, tc.abort_w()); marked = true; }
@@ -371,9 +397,15 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
         }
         if (threadIdx.x == 0) {
             if (c.tasks) atomicAdd(c.tasks, 1ull);
+            // long tasks claim after they finish: nothing of the dispatcher stays in a register
+            if (Body::kLateClaim && claims) t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
             s_task = t_next;
-            s_w = decode_w(tc.pending, c);
-            tc.pending = ld_status(c.status);   // prefetch for the next task's polls
+            if (need_status) {
+                s_w = decode_w(status_take(c, s_st), c);
+                status_prefetch(c, s_st);   // for the next task's polls / check
+            } else {
+                s_w = c.w_default;
+            }
         }
         __syncthreads();
         t = s_task;
@@ -381,6 +413,7 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
         checked = true;
         __syncthreads();
     }
+    if (threadIdx.x == 0 && need_status && !c.status_mapped) asm volatile("cp.async.wait_all;\n" ::: "memory");
     if (c.tstamp && threadIdx.x == 0) atomicMax(c.tstamp + 1, globaltimer());
     if (!c.fused) return;
     // Fused tail.  Every CTA registers its arrival; the LAST one to arrive publishes the
@@ -448,7 +481,7 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
     __shared__ __align__(16) typename Body::Smem smem;
     __shared__ long long s_key;
     TaskCtx tc;
-    tc.c = nullptr; tc.pending = 0; tc.s_flag = &s_flag; tc.s_key = &s_key;
+    tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = &s_flag; tc.s_key = &s_key;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
 }
 
@@ -487,6 +520,7 @@ struct RowDotBody {
     // launch (1024 tasks) is resident in a single wave with 2 KB of loads in flight per warp.
     static constexpr int kThreads = 128;
     static constexpr int kMinBlocks = 8;
+    static constexpr bool kLateClaim = false;
     static constexpr int kWarps = kThreads / 32;
     static constexpr int U = (NMAT == 2) ? 2 : 4;   // 128-column blocks whose loads are issued together
     struct Params {
@@ -592,6 +626,7 @@ template <typename T, int MODE>
 struct ColDotBody {
     static constexpr int kThreads = 1024;
     static constexpr int kMinBlocks = 1;
+    static constexpr bool kLateClaim = false;
     struct Params {
         const T *A; const T *v; const T *mean; T *out;
         long long nrows, ncols, lws; int CB; float nf, eps;
@@ -666,6 +701,7 @@ struct Tile2D {
 struct CorrReduceBody {
     static constexpr int kThreads = 256;
     static constexpr int kMinBlocks = 4;
+    static constexpr bool kLateClaim = false;
     struct Params { float *data; const float *mean; const float *std_; Tile2D tl; float sqrtn; };
     typedef EmptySmem Smem;
     __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
@@ -697,6 +733,7 @@ template <typename T>
 struct Conv2DBody {
     static constexpr int kThreads = 256;
     static constexpr int kMinBlocks = 2;   // 10 x 16 B of loads in flight per thread needs the registers
+    static constexpr bool kLateClaim = false;
     struct Params { const T *A; T *B; Tile2D tl; T c[9]; int vec4; };   // c[a*3+b]: row offset a-1, col offset b-1
     typedef EmptySmem Smem;
     __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
@@ -808,6 +845,7 @@ struct GemmBody {
 #define FCL_GEMM_MINB 2
 #endif
     static constexpr int kMinBlocks = FCL_GEMM_MINB;
+    static constexpr bool kLateClaim = true;   // tasks of ~0.1-1 ms: an exposed claim costs nothing
     typedef typename V4<T>::type T4;
     struct Params {
         const T *A; const T *B; T *C;
@@ -924,22 +962,26 @@ struct GemmBody {
         gload(p, i0, j0, 0, ra, rb);
         sstore(sm, 0, ra, rb);
         __syncthreads();
-        for (long long kt = 0; kt < nkt; ++kt) {
-            const int st = (int)(kt & 1);
-            if (kt + 1 < nkt) gload(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
-            T a[2][8], b[2][8];
-            frag(sm, st, 0, tx, ty, a[0], b[0]);
+        const long long per = tc.period();
+        for (long long kb = 0; kb < nkt; kb += per) {   // blocks of `per` k'-tiles, polls between them
+            const long long kend = (nkt - kb < per) ? nkt : kb + per;
+            for (long long kt = kb; kt < kend; ++kt) {
+                const int st = (int)(kt & 1);
+                if (kt + 1 < nkt) gload(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
+                T a[2][8], b[2][8];
+                frag(sm, st, 0, tx, ty, a[0], b[0]);
 #pragma unroll
-            for (int kk = 0; kk < GBK; ++kk) {
-                if (kk + 1 < GBK) frag(sm, st, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
+                for (int kk = 0; kk < GBK; ++kk) {
+                    if (kk + 1 < GBK) frag(sm, st, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
 #pragma unroll
-                for (int r = 0; r < 8; ++r)
+                    for (int r = 0; r < 8; ++r)
 #pragma unroll
-                    for (int c = 0; c < 8; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+                        for (int c = 0; c < 8; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+                }
+                if (kt + 1 < nkt) sstore(sm, st ^ 1, ra, rb);
+                __syncthreads();
             }
-            if (kt + 1 < nkt) sstore(sm, st ^ 1, ra, rb);
-            __syncthreads();
-            if (tc.poll((int)(kt + 1))) return true;   // abort check every abort_period k'-tiles (Fig 12)
+            if (kend < nkt && tc.check()) return true;   // abort check every abort_period k'-tiles (Fig 12)
         }
         // epilogue: write-once stores
 #pragma unroll

@@ -321,6 +321,7 @@ struct Job {
     int64_t t0 = 0, t1 = 0, s_forced = -1;
     bool forced = false, dev_merge = false, eager = false, gpu_launched = false;
     bool lite = false;         // single wave, no in-task polls: plain grid + exit memop, never a merge
+    bool exact_spans = false;  // every output's footprint of a work-group range is one exact span
     bool twin_alias = false;   // exact spans: the merge compares against the device copy itself
     int64_t unit = 1;          // host chunk boundaries are multiples of this many work-groups
     void *twin[6] = {nullptr}, *stage[6] = {nullptr};
@@ -366,6 +367,7 @@ struct fcl_context_st {
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
+    int env_abort_period = 0;                    // FCL_ABORT_PERIOD: default for opts.abort_period == 0
     size_t race_min_bytes = 32u << 20;           // only for returns at least this large
     size_t race_piece_bytes = 8u << 20;          // return-copy piece
     double race_chunk_ms = 1.0;                  // host chunk length during the race
@@ -622,7 +624,7 @@ Job *job_alloc(fcl_context ctx) {
     j->status = FCL_SUCCESS;
     j->done.store(0);
     j->have_k = j->have_m = j->wm_pending = false;
-    j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = j->lite = false;
+    j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = j->lite = j->exact_spans = false;
     j->unit = 1;
     std::memset(&j->info, 0, sizeof j->info);
     for (int q = 0; q < 6; ++q) j->twin[q] = j->stage[q] = nullptr;
@@ -693,13 +695,16 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         }
         const bool aligned_split = !j.forced || j.s_forced % j.unit == 0 || j.s_forced == L.hi;
         j.twin_alias = contiguous && aligned_split && !ctx->force_twin;
+        j.exact_spans = contiguous;
     }
     // Single wave without in-task polls: every CTA runs exactly one task, unchecked (the first
     // task of a CTA never waits for the status), so no work-group can be skipped or aborted,
     // the GPU computes the whole range and no merge can be needed.  The dispatcher reduces to
     // the plain grid plus the exit signal, without status loads or arrival tail, and the host
     // neither stages nor publishes: its finished chunks only bound the return copy.
-    const int abort_period = L.o.abort_period > 0 ? L.o.abort_period : (L.o.abort_period < 0 ? 0 : gpu_default_abort_period(L.a));
+    int opt_period = L.o.abort_period;
+    if (opt_period == 0 && ctx->env_abort_period != 0) opt_period = ctx->env_abort_period;   // FCL_ABORT_PERIOD
+    const int abort_period = opt_period > 0 ? opt_period : (opt_period < 0 ? 0 : gpu_default_abort_period(L.a));
     j.lite = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && abort_period == 0 && !ctx->no_lite &&
              (j.t1 - j.t0) <= gpu_coop_capacity(L.a, L.g, ctx->num_sms);
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
@@ -749,6 +754,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     c.tasks_next = ctx->stats ? ctx->dtasks + (j.slot + 1) % kSlots : nullptr;
     c.wm_out = ctx->dwm;
     c.check_first = j.forced ? 1 : 0;
+    c.status_mapped = ctx->status_location == FCL_STATUS_HOST_MAPPED ? 1 : 0;
     c.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot : nullptr;
     c.tstamp_next = ctx->stats ? ctx->dstamp + 4 * ((j.slot + 1) % kSlots) : nullptr;
     c.task_lo = j.t0; c.task_hi = j.t1;
@@ -975,7 +981,9 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         }
         return t;
     };
-    const bool race = gpu_done && !j.forced && (j.dev_merge || j.lite) && !j.eager && !ctx->no_race &&
+    // (only for exact spans: a piece of work-groups must map to its own bytes, not to a
+    // conservative cover such as CORR's row-plus-column symmat footprint)
+    const bool race = gpu_done && !j.forced && (j.dev_merge || j.lite) && !j.eager && !ctx->no_race && j.exact_spans &&
                       hi_cur > L.lo && out_bytes(L.lo, hi_cur) >= ctx->race_min_bytes;
     if (race) {
         ctx->tr.add("race_begin", j.epoch);
@@ -1181,13 +1189,23 @@ void drain(fcl_context ctx) {
     std::lock_guard<std::mutex> lk(ctx->q_mu);   // acquire the coordinator's last critical section
 }
 
-// A new launch conflicts with a pending one if either writes a buffer the other touches.
+// A new launch conflicts with a pending one if either writes a buffer the other touches --
+// except a pure read-after-write on a free-running pending launch (device merge in its
+// dispatcher, or lite): its device copy is complete in stream order before the new kernel
+// on main, and the new launch's host side runs after the pending one's (FIFO) and waits for
+// the buffer's return copy before reading the host copy.  So a dependent kernel is not held
+// back by the host side of the one before it (e.g. a return race still in progress).
 bool conflicts_with_pending(fcl_context ctx, const Launch &L) {
     std::lock_guard<std::mutex> lk(ctx->q_mu);
     for (Job *p : ctx->queue) {
+        const bool free_running = p->dev_merge || p->lite;
         for (int a = 0; a < L.a.nbuf; ++a)
-            for (int b = 0; b < p->L.a.nbuf; ++b)
-                if (L.bufs[a] == p->L.bufs[b] && ((L.acc[a] & 2) || (p->L.acc[b] & 2))) return true;
+            for (int b = 0; b < p->L.a.nbuf; ++b) {
+                if (L.bufs[a] != p->L.bufs[b]) continue;
+                const bool we_write = (L.acc[a] & 2) != 0, they_write = (p->L.acc[b] & 2) != 0;
+                if (we_write) return true;                        // WAR / WAW
+                if (they_write && !free_running) return true;     // RAW on a host-decided merge
+            }
     }
     return false;
 }
@@ -1370,6 +1388,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
     ctx->no_lite = getenv("FCL_NO_LITE") && atoi(getenv("FCL_NO_LITE")) != 0;
     ctx->no_race = getenv("FCL_NO_RACE") && atoi(getenv("FCL_NO_RACE")) != 0;
+    if (getenv("FCL_ABORT_PERIOD")) ctx->env_abort_period = atoi(getenv("FCL_ABORT_PERIOD"));
     if (getenv("FCL_RACE_MIN_BYTES")) ctx->race_min_bytes = (size_t)atoll(getenv("FCL_RACE_MIN_BYTES"));
     if (getenv("FCL_RACE_PIECE_BYTES")) ctx->race_piece_bytes = std::max<size_t>(4096, (size_t)atoll(getenv("FCL_RACE_PIECE_BYTES")));
     if (getenv("FCL_RACE_CHUNK_MS")) ctx->race_chunk_ms = atof(getenv("FCL_RACE_CHUNK_MS"));
