@@ -210,14 +210,17 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
                 infos.append(ctx.launch_info())
         ctx.finish()
 
-    def timed(mode: str, k: int, collect=False):
+    def timed(mode: str, k: int, collect=False, idle=True):
         ts, infos = [], []
         for _ in range(k):
             with torch.cuda.stream(stream):
                 flush.fill_(1.0)          # L2 flush (outside the timed interval)
             # idle GPU at e0: host-side work (the CPU-only leg, the host share of a cooperative
-            # launch, launch submission) cannot hide under the flush
-            stream.synchronize()
+            # launch, launch submission) cannot hide under the flush.  The per-launch detail
+            # steps (idle=False) instead queue behind the flush, so that the kernel-only events
+            # see device time and not the host's submission latency.
+            if idle:
+                stream.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             step(mode, infos if collect else None)
@@ -260,7 +263,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         print("coop step ms:", [round(t, 3) for t in coop_ts], file=sys.stderr)
 
     # per-launch detail (dispatcher CUDA-event time, merges, host share) from separate steps
-    _, infos = timed("coop", max(2, min(args.steps, 5)), collect=True)
+    _, infos = timed("coop", max(2, min(args.steps, 5)), collect=True, idle=False)
     gpu_ts, _ = timed("gpu", max(3, min(args.steps, 10)))
     cpu_ts, _ = timed("cpu", max(2, min(args.steps, 5)))
     gpu_ms = max_over_ranks(statistics.mean(gpu_ts))
@@ -270,6 +273,11 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     # dominant kernel: the GESUMMV dispatcher (2 N^2 floats); CUDA-event duration on main
     ges = infos[0::3]   # launch order per step: gesummv, bicg_s, bicg_q
     k_ms = statistics.mean(i["t_gpu_kernel_ms"] for i in ges if i["t_gpu_kernel_ms"] > 0)
+    # which GPU path the cooperative GESUMMV launches took (FCL_GPU_PATH_*): a single wave
+    # without in-task polls runs as the lite plain grid, else the persistent dispatcher
+    paths = {i.get("gpu_path", 1) for i in ges}
+    gesummv_kernel = ("plain_kernel<RowDotBody<float,2>> (GESUMMV, lite cooperative launch)" if paths == {2}
+                      else "coop_kernel<RowDotBody<float,2>> (GESUMMV dispatcher)")
     peaks = measured_peaks()
     achieved = algorithmic_bytes(N)["gesummv"] / (k_ms * 1e-3) / 1e9
     launches_per_step = statistics.mean(
@@ -347,7 +355,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
             "ideal_coop_ms": round(ideal_ms, 4), "frac_of_ideal": round(ideal_ms / coop_ms, 4),
             "coop_vs_best_single": round(min(gpu_ms, cpu_ms) / coop_ms, 4),
             "wall_ms_per_step": round(t_wall * 1e3 / args.steps, 4),
-            "roofline": {"kernel": "coop_kernel<RowDotBody<float,2>> (GESUMMV dispatcher)", "bound": "hbm",
+            "roofline": {"kernel": gesummv_kernel, "bound": "hbm",
                          "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": ncu_traffic("gesummv"),
                          "algorithmic_bytes": algorithmic_bytes(N)["gesummv"], "kernel_ms": round(k_ms, 4),

@@ -189,6 +189,13 @@ typedef struct {
 /* Fill *opts with the defaults above. */
 fcl_status fcl_default_launch_opts(fcl_launch_opts *opts);
 
+/* info.gpu_path */
+#define FCL_GPU_PATH_NONE       0  /* no GPU kernel (CPU-only mode, empty range) */
+#define FCL_GPU_PATH_DISPATCHER 1  /* persistent dispatcher: ascending claims, watermark checks, fused merge */
+#define FCL_GPU_PATH_LITE       2  /* cooperative single wave without in-task polls: every CTA's one task is
+                                      unchecked, so the dispatcher reduces to a plain grid + exit signal */
+#define FCL_GPU_PATH_PLAIN      3  /* GPU-only mode: plain grid */
+
 typedef struct {
     int64_t n_wg;                /* work-groups in the executed range */
     int64_t wg_lo, wg_hi;
@@ -207,6 +214,8 @@ typedef struct {
     double  t_merge_ms;          /* CUDA-event time of the merge kernel(s) */
     double  t_host_ms;           /* host executor busy time */
     int32_t chunk_sizes[64];     /* first chunk sizes (C11 trace) */
+    int32_t gpu_path;            /* FCL_GPU_PATH_*: how the GPU side of the launch ran */
+    int32_t race;                /* 1 = large output returned by the return race */
 } fcl_launch_info;
 
 /* Launch `kernel` over the NDRange (work_dim in 1..3, gws[k] % lws[k] == 0,

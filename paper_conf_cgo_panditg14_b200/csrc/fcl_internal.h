@@ -119,6 +119,11 @@ int gpu_launch_coop(const KArgs &a, const Geom &g, const CoopCtl &c, int num_sms
 struct SlotReset {
     unsigned long long *claim, *tasks, *merge_ctr;
     unsigned int *barrier;   // 17 words
+    // exit signal of a lite cooperative launch (nullable): the last CTA to arrive on `arrive`
+    // (this slot's 17 counters, zero on entry) stores `epoch` to the mapped host word
+    unsigned int *arrive;
+    unsigned long long *exit_word;
+    unsigned int epoch;
 };
 int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream,
                      const SlotReset *reset = nullptr);

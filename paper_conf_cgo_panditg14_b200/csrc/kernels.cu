@@ -483,6 +483,18 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
     TaskCtx tc;
     tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = &s_flag; tc.s_key = &s_key;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
+    if (r.exit_word) {   // lite cooperative launch: GPU-exit signal for the host (L18.s19)
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            // hierarchical arrival (16 leaves + root); no fence: the word publishes no data,
+            // the return copies are ordered behind the kernel on the streams
+            const unsigned int leaf = blockIdx.x & 15u;
+            const unsigned int nleaf = (gridDim.x > 16u) ? 16u : gridDim.x;
+            const unsigned int leaf_size = (gridDim.x - leaf + 15u) / 16u;
+            if (atomicAdd(r.arrive + 1 + leaf, 1u) == leaf_size - 1 && atomicAdd(r.arrive, 1u) == nleaf - 1)
+                asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(r.exit_word), "l"((unsigned long long)r.epoch) : "memory");
+        }
+    }
 }
 
 // Twin capture (C5, L16.s2-3): copy every OUT/INOUT buffer to its twin in ONE launch.

@@ -156,7 +156,7 @@ struct Executor {
     std::atomic<int64_t> done{0};
     int64_t batch = 1;   // work-groups per claim (host_batch), 1 when work-groups are split
     volatile int abort_flag = 0;
-    int64_t spin_ns = 20 * 1000 * 1000;   // spin 20 ms after a job before sleeping
+    int64_t spin_ns = 2 * 1000 * 1000;    // spin 2 ms after a job before sleeping
 
     void start(int nthreads, bool pin) {
         cpu_set_t set;
@@ -367,6 +367,7 @@ struct fcl_context_st {
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
+    bool memop_nobarrier_ok = true;              // cleared when the driver rejects NO_MEMORY_BARRIER
     int env_abort_period = 0;                    // FCL_ABORT_PERIOD: default for opts.abort_period == 0
     size_t race_min_bytes = 32u << 20;           // only for returns at least this large
     size_t race_piece_bytes = 8u << 20;          // return-copy piece
@@ -485,22 +486,32 @@ void pool_trim(fcl_context ctx) {
 // Store `v` to `dst` after everything already queued on `s` (stream memory operation; a
 // one-thread kernel store if the driver lacks 64-bit memops).
 fcl_status stream_store(fcl_context ctx, unsigned long long *dst, unsigned long long v, cudaStream_t s,
-                        bool barrier = true) {
+                        bool barrier = true, fcl_launch_info *info = nullptr) {
     if (ctx->write64) {
-        // with a barrier the store is ordered after the data of earlier operations on `s`
-        // (needed for publication, C13); a bare completion signal skips it (it costs ~12 us)
-        CUresult r = ctx->write64((CUstream)s, (CUdeviceptr)dst, v, barrier ? 0u : (unsigned)CU_STREAM_WRITE_VALUE_NO_MEMORY_BARRIER);
+        // With a barrier the store is ordered after the data of earlier operations on `s`
+        // (needed for publication, C13); a bare completion signal may skip it where the driver
+        // allows (it rejects NO_MEMORY_BARRIER for mapped host memory on some systems).
+        const bool nb = !barrier && ctx->memop_nobarrier_ok;
+        CUresult r = ctx->write64((CUstream)s, (CUdeviceptr)dst, v, nb ? (unsigned)CU_STREAM_WRITE_VALUE_NO_MEMORY_BARRIER : 0u);
         if (r == CUDA_SUCCESS) return FCL_SUCCESS;
+        if (nb) {
+            ctx->memop_nobarrier_ok = false;
+            r = ctx->write64((CUstream)s, (CUdeviceptr)dst, v, 0u);
+            if (r == CUDA_SUCCESS) return FCL_SUCCESS;
+        }
+        fprintf(stderr, "fcl: cuStreamWriteValue64 failed (CUresult %d, dst %p): stream memops disabled, "
+                        "falling back to a store kernel\n", (int)r, (void *)dst);
         ctx->write64 = nullptr;   // fall back to the kernel store from now on
     }
     if (gpu_launch_store64(dst, v, s) < 0) return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    if (info) info->gpu_launches += 1;   // the fallback is a kernel of ours
     return FCL_SUCCESS;
 }
 
 // Publish {epoch, W} behind everything queued on hd: status follows data (C13, L16.s15).
 fcl_status publish(fcl_context ctx, const Job &j, uint32_t w) {
     const unsigned long long v = ((unsigned long long)j.epoch << 32) | w;
-    return stream_store(ctx, ctx->status_dptr + j.slot, v, ctx->hd);
+    return stream_store(ctx, ctx->status_dptr + j.slot, v, ctx->hd, true, const_cast<fcl_launch_info *>(&j.info));
 }
 
 // Bring a buffer's copies to what a launch needs.  A pending return copy is waited for on the
@@ -814,7 +825,8 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         ctx->tr.add("A_prelaunch", j.epoch);
         if (j.lite) {
             const int nx = (j.slot + 1) % kSlots;
-            SlotReset r{ctx->dclaim + nx, ctx->stats ? ctx->dtasks + nx : nullptr, ctx->dmctr + nx, ctx->dbar + 32 * nx};
+            SlotReset r{ctx->dclaim + nx, ctx->stats ? ctx->dtasks + nx : nullptr, ctx->dmctr + nx, ctx->dbar + 32 * nx,
+                        ctx->dbar + 32 * j.slot, ctx->exit_dptr, j.epoch};
             if (gpu_launch_plain(L.a, L.g, j.t0, j.t1, ctx->main, &r) < 0)
                 return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
         } else if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0) {
@@ -823,21 +835,15 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         ctx->tr.add("A_launched", j.epoch);
         CK(ctx, cudaEventRecord(j.ev_k1, ctx->main));
         ctx->tr.add("A_k1", j.epoch);
-        // GPU exit signal for the host executor (L18.s19): the fused tail stores the epoch to
-        // mapped host memory after its grid barrier; unfused, a bare memop does it.  Lite: the
-        // memop goes on its own stream behind the kernel's event, so that the main stream
-        // carries kernels only (a memop between two kernels stalls the second) and the signal
-        // does not queue behind return copies.
-        if (j.lite) {
-            CK(ctx, cudaStreamWaitEvent(ctx->xs, j.ev_k1, 0));
-            fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->xs, false);
-            if (xs != FCL_SUCCESS) return xs;
-        } else if (!c.fused) {
-            fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->main, false);
+        // GPU exit signal for the host executor (L18.s19): the fused tail (or, lite, the plain
+        // grid's last CTA) stores the epoch to mapped host memory; unfused, a bare memop does it.
+        if (!c.fused && !j.lite) {
+            fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->main, false, &info);
             if (xs != FCL_SUCCESS) return xs;
         }
         ctx->slot_used[j.slot] = true;
         ctx->main_tail = j.ev_k1;
+        info.gpu_path = j.lite ? FCL_GPU_PATH_LITE : FCL_GPU_PATH_DISPATCHER;
         j.have_k = timing;
         info.gpu_launches += 1;
         j.gpu_launched = true;
@@ -987,6 +993,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
                       hi_cur > L.lo && out_bytes(L.lo, hi_cur) >= ctx->race_min_bytes;
     if (race) {
         ctx->tr.add("race_begin", j.epoch);
+        info.race = 1;
         CK(ctx, cudaStreamWaitEvent(ctx->dh, j.ev_k1, 0));
         const size_t unit_b = std::max<size_t>(1, out_bytes(L.lo, std::min<int64_t>(L.lo + j.unit, L.hi)));
         const int64_t piece = j.unit * std::max<int64_t>(1, (int64_t)(ctx->race_piece_bytes / unit_b));
@@ -1228,6 +1235,7 @@ fcl_status run_gpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
     ctx->sync_have_k = timing;
     info.gpu_launches += 1;
+    info.gpu_path = FCL_GPU_PATH_PLAIN;
     info.gpu_tasks = info.gpu_tasks_total = t1 - t0;
     return enqueue_d2h(ctx, L, L.lo, L.hi, info, ctx->ev_k1);
 }

@@ -71,7 +71,7 @@ class LaunchInfo(ctypes.Structure):
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64),
                 ("t_call_ms", ctypes.c_double), ("t_gpu_kernel_ms", ctypes.c_double),
                 ("t_merge_ms", ctypes.c_double), ("t_host_ms", ctypes.c_double),
-                ("chunk_sizes", ctypes.c_int32 * 64)]
+                ("chunk_sizes", ctypes.c_int32 * 64), ("gpu_path", ctypes.c_int32), ("race", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k, _ in self._fields_ if k != "chunk_sizes"}

@@ -9,8 +9,9 @@ if [ "$SKIP_BENCH" = "0" ]; then
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv \
     python bench.py --steps 2 --warmup 3 > gpurun_out/${TAG}_bench_under_ncu.log 2>&1
 fi
-# the dominant kernel of the bench (GESUMMV dispatcher) and its plain-grid twin, full sets
-ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:coop_kernel.*RowDotBody<float, .*2>' -s 2 -c 1 \
+# the dominant kernel of the bench (GESUMMV, cooperative launch: the lite plain grid when it
+# runs in one wave, else the dispatcher) and its GPU-only plain grid, full sets
+ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:.*_kernel.*RowDotBody<float, .*2>' -s 2 -c 1 \
     -o gpurun_out/${TAG}_gesummv_coop python scripts/profile_step.py coop 3 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*RowDotBody<float, .*2>' -s 2 -c 1 \
     -o gpurun_out/${TAG}_gesummv_plain python scripts/profile_step.py gpu 3 > /dev/null 2>&1

@@ -55,7 +55,7 @@ lines = [f"# ncu summary, round {TAG[1:]}", "",
          "Absolute ncu durations are serialised/cold-cache; compare with the CUDA-event numbers in",
          "`profiles/" + TAG + "_configs.jsonl` and the bench line for live timing.", ""]
 traffic = {}
-for name, rep in [("gesummv dispatcher (COOP)", "gesummv_coop"), ("gesummv plain grid (GPU-only)", "gesummv_plain"),
+for name, rep in [("gesummv, cooperative launch (lite plain grid when single-wave)", "gesummv_coop"), ("gesummv plain grid (GPU-only)", "gesummv_plain"),
                   ("merge_kernel 1 GiB, scatter 10 %", "merge"), ("SYRK 2048 dispatcher", "syrk"),
                   ("2DCONV 16384^2 dispatcher", "conv2d")]:
     p = os.path.join(SRC, f"{TAG}_{rep}.ncu-rep")

@@ -53,7 +53,7 @@ def test_struct_layouts_match_header():
     assert ctypes.sizeof(fcl.ContextDesc) == 40
     assert ctypes.sizeof(fcl.Arg) == 32
     assert fcl.LaunchOpts.forced_split.offset == 8 and ctypes.sizeof(fcl.LaunchOpts) == 72
-    assert fcl.LaunchInfo.t_call_ms.offset == 104 and ctypes.sizeof(fcl.LaunchInfo) == 392
+    assert fcl.LaunchInfo.t_call_ms.offset == 104 and ctypes.sizeof(fcl.LaunchInfo) == 400
 
 
 def test_kernel_table_and_signatures(lib):
