@@ -185,7 +185,10 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     if lws_ranks > 1:
         os.sched_setaffinity(0, all_cores[local_rank * per_rank:(local_rank + 1) * per_rank] or all_cores)
     cores = len(os.sched_getaffinity(0))
-    host_threads = max(1, cores - 2)
+    # host executor threads: all cores but three -- the coordinator's, the caller's, and one
+    # left free for the OS and the nvidia-smi clock sampler (a sampler that has to preempt a
+    # spinning thread stalls the launch path by milliseconds)
+    host_threads = max(1, cores - 3)
     ctx = fcl.Context(local_rank, n_host_threads=host_threads, streams=(stream.cuda_stream, None, None))
 
     Ps = problems(1000 * rank)

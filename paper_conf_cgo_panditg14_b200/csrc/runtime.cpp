@@ -368,6 +368,7 @@ struct fcl_context_st {
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
     bool memop_nobarrier_ok = true;              // cleared when the driver rejects NO_MEMORY_BARRIER
+    int exit_poll_pauses = 8;                    // pause instructions between exit-word polls (FCL_EXIT_POLL_PAUSES)
     int env_abort_period = 0;                    // FCL_ABORT_PERIOD: default for opts.abort_period == 0
     size_t race_min_bytes = 32u << 20;           // only for returns at least this large
     size_t race_piece_bytes = 8u << 20;          // return-copy piece
@@ -968,7 +969,10 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             if (st != FCL_SUCCESS) { ex.abort_flag = 1; ex.wait(); return st; }
             if (!more) { cpu_all = true; break; }
         } else {
-            _mm_pause();
+            // back off between polls: the exit word is written by the GPU over PCIe, and a core
+            // hammering that line slows the device's posted writes (and the return copies queued
+            // behind them)
+            for (int k = 0; k < ctx->exit_poll_pauses; ++k) _mm_pause();
         }
     }
     // Return race: the GPU finished first (its copy is complete: it ran every work-group it did
@@ -1397,6 +1401,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->no_lite = getenv("FCL_NO_LITE") && atoi(getenv("FCL_NO_LITE")) != 0;
     ctx->no_race = getenv("FCL_NO_RACE") && atoi(getenv("FCL_NO_RACE")) != 0;
     if (getenv("FCL_ABORT_PERIOD")) ctx->env_abort_period = atoi(getenv("FCL_ABORT_PERIOD"));
+    if (getenv("FCL_EXIT_POLL_PAUSES")) ctx->exit_poll_pauses = std::max(1, atoi(getenv("FCL_EXIT_POLL_PAUSES")));
     if (getenv("FCL_RACE_MIN_BYTES")) ctx->race_min_bytes = (size_t)atoll(getenv("FCL_RACE_MIN_BYTES"));
     if (getenv("FCL_RACE_PIECE_BYTES")) ctx->race_piece_bytes = std::max<size_t>(4096, (size_t)atoll(getenv("FCL_RACE_PIECE_BYTES")));
     if (getenv("FCL_RACE_CHUNK_MS")) ctx->race_chunk_ms = atof(getenv("FCL_RACE_CHUNK_MS"));
@@ -1866,12 +1871,14 @@ fcl_status fcl_finish(fcl_context ctx) {
     drain(ctx);
     ctx->tr.add("finish_drained", ctx->epoch);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
+    // dh first: its return copies are ordered behind the kernels, so by the time it is done
+    // main and hd usually are too and their syncs are cheap checks
+    CK(ctx, cudaStreamSynchronize(ctx->dh));
+    ctx->tr.add("finish_dh", ctx->epoch);
     CK(ctx, cudaStreamSynchronize(ctx->main));
     ctx->tr.add("finish_main", ctx->epoch);
     CK(ctx, cudaStreamSynchronize(ctx->hd));
     ctx->tr.add("finish_hd", ctx->epoch);
-    CK(ctx, cudaStreamSynchronize(ctx->dh));
-    ctx->tr.add("finish_dh", ctx->epoch);
     CK(ctx, cudaGetLastError());
     ctx->tr.add("finish_end", ctx->epoch);
     if (ctx->tr.on && ctx->stats) {
