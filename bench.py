@@ -204,6 +204,9 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     prepared = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m, timing=(k == 0))
                     for k, (P, b) in enumerate(zip(Ps, bufs))] for m in ("coop", "gpu", "cpu")}
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    # read sweep after the write flush: L2 ends full of clean, unrelated lines (no dirty
+    # write-backs charged to the next kernel)
+    sweep = torch.ones(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
 
     def step(mode: str, infos: list = None):
         for launch in prepared[mode]:
@@ -217,7 +220,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         ts, infos = [], []
         for _ in range(k):
             with torch.cuda.stream(stream):
-                flush.fill_(1.0)          # L2 flush (outside the timed interval)
+                flush.fill_(1.0); sweep.sum()          # L2 flush (outside the timed interval)
             # idle GPU at e0: host-side work (the CPU-only leg, the host share of a cooperative
             # launch, launch submission) cannot hide under the flush.  The per-launch detail
             # steps (idle=False) instead queue behind the flush, so that the kernel-only events
@@ -246,14 +249,18 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     if dist is not None:
         dist.barrier()
     torch.cuda.synchronize()
+    import gc
     with ClockSampler(local_rank) as clk:
         if dist is not None:
             dist.barrier()
         torch.cuda.synchronize()
+        gc.collect()
+        gc.disable()   # as timeit does: no cyclic collection inside the timed region
         t_wall0 = time.perf_counter()
         coop_ts, _ = timed("coop", args.steps)
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall0
+        gc.enable()
         if dist is not None:
             dist.barrier()
         # the timed region can be shorter than nvidia-smi's sampling period: keep the same
@@ -267,8 +274,10 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
 
     # per-launch detail (dispatcher CUDA-event time, merges, host share) from separate steps
     _, infos = timed("coop", max(2, min(args.steps, 5)), collect=True, idle=False)
-    gpu_ts, _ = timed("gpu", max(3, min(args.steps, 10)))
+    gc.disable()
+    gpu_ts, _ = timed("gpu", max(10, min(args.steps, 100)))
     cpu_ts, _ = timed("cpu", max(2, min(args.steps, 5)))
+    gc.enable()
     gpu_ms = max_over_ranks(statistics.mean(gpu_ts))
     cpu_ms = max_over_ranks(statistics.mean(cpu_ts))
     ideal_ms = 1.0 / (1.0 / gpu_ms + 1.0 / cpu_ms)
@@ -297,7 +306,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         mts = []
         for r in range(8):
             with torch.cuda.stream(stream):
-                flush.fill_(2.0)
+                flush.fill_(2.0); sweep.sum()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             fcl.merge_raw(g.data_ptr(), c.data_ptr(), t.data_ptr(), nw * 4, 4, stream.cuda_stream)
@@ -322,7 +331,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     e2e_ts = []
     for r in range(args.warmup + args.steps):
         with torch.cuda.stream(stream):
-            flush.fill_(3.0)
+            flush.fill_(3.0); sweep.sum()
         stream.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
@@ -353,7 +362,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": "gesummv_bicg4096", "n": N, "kernels": ["gesummv", "bicg_s", "bicg_q"],
                        "mode": "coop", "lws": 256, "work_groups_per_kernel": 16, "host_threads": host_threads,
-                       "l2": "flushed between steps (256 MiB write)", "parallelism": f"replicas{world}"},
+                       "l2": "flushed between steps (256 MiB write + 256 MiB read sweep)", "parallelism": f"replicas{world}"},
             "coop_ms": round(coop_ms, 4), "gpu_only_ms": round(gpu_ms, 4), "cpu_only_ms": round(cpu_ms, 4),
             "ideal_coop_ms": round(ideal_ms, 4), "frac_of_ideal": round(ideal_ms / coop_ms, 4),
             "coop_vs_best_single": round(min(gpu_ms, cpu_ms) / coop_ms, 4),

@@ -369,6 +369,12 @@ struct fcl_context_st {
     bool no_race = false;                        // FCL_NO_RACE=1
     bool memop_nobarrier_ok = true;              // cleared when the driver rejects NO_MEMORY_BARRIER
     int exit_poll_pauses = 8;                    // pause instructions between exit-word polls (FCL_EXIT_POLL_PAUSES)
+    // Deferred quiescence: an abandoned chunk of an eagerly returned launch may
+    // still be running; its launch's buffers are kept here until quiesce() has waited for it.
+    std::mutex qz_mu;
+    std::atomic<int> quiescing{0};
+    fcl_buffer qz_bufs[6] = {};
+    int qz_n = 0;
     int env_abort_period = 0;                    // FCL_ABORT_PERIOD: default for opts.abort_period == 0
     size_t race_min_bytes = 32u << 20;           // only for returns at least this large
     size_t race_piece_bytes = 8u << 20;          // return-copy piece
@@ -618,6 +624,29 @@ fcl_status read_gpu_watermark(fcl_context ctx, Job &j, int64_t *wm) {
     const unsigned int w = decode_wm_word(*ctx->wm_host, j.epoch);
     *wm = (w == 0xFFFFFFFFu) ? j.L.hi : std::min<int64_t>(j.L.hi, (int64_t)w);
     return FCL_SUCCESS;
+}
+
+// Wait until an abandoned chunk (deferred by an eager launch's phase B) has stopped, and clear
+// the abort flag.  Serialised with the deferral itself, so a new abandonment is never lost.
+void quiesce(fcl_context ctx) {
+    if (!ctx->quiescing.load(std::memory_order_acquire)) return;
+    std::lock_guard<std::mutex> lk(ctx->qz_mu);
+    if (!ctx->quiescing.load(std::memory_order_relaxed)) return;
+    ctx->ex.wait();
+    ctx->ex.abort_flag = 0;
+    ctx->qz_n = 0;
+    ctx->quiescing.store(0, std::memory_order_release);
+}
+
+// Does launch L write a buffer the still-quiescing chunk reads or writes?
+bool conflicts_with_quiescing(fcl_context ctx, const Launch &L) {
+    if (!ctx->quiescing.load(std::memory_order_acquire)) return false;
+    std::lock_guard<std::mutex> lk(ctx->qz_mu);
+    for (int a = 0; a < L.a.nbuf; ++a)
+        if (L.acc[a] & 2)
+            for (int b = 0; b < ctx->qz_n; ++b)
+                if (L.bufs[a] == ctx->qz_bufs[b]) return true;
+    return false;
 }
 
 Job *job_alloc(fcl_context ctx) {
@@ -894,7 +923,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     int nch = 0;
     bool in_flight = false, gpu_done = !j.gpu_launched, cpu_all = false, staged_any = false, hd_joined = false;
     int64_t cur_lo = 0, cur_hi = 0, cur_size = 0, cpu_done_wgs = 0;
-    ex.abort_flag = 0;
+    quiesce(ctx);   // an earlier launch's abandoned chunk must have stopped before ours starts
 
     auto start_chunk = [&]() {
         int64_t size = ceil_pct(pct, nwg);
@@ -1063,6 +1092,16 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             ob->d2h_pending = true;
         }
         ctx->tr.add("race_end", j.epoch);
+    } else if (in_flight && j.eager && gpu_done) {
+        // GPU finished first and the (pure-OUT) result is already on its way back: abandon the
+        // chunk without waiting for it (L18.s19).  Its workers only write words bit-identical to
+        // the returned ones; whatever could change what they read or write waits in quiesce().
+        std::lock_guard<std::mutex> lk(ctx->qz_mu);
+        ex.abort_flag = 1;
+        ctx->qz_n = 0;
+        for (int k = 0; k < L.a.nbuf; ++k) ctx->qz_bufs[ctx->qz_n++] = L.bufs[k];
+        ctx->quiescing.store(1, std::memory_order_release);
+        busy += now_ms() - t_start;
     } else if (in_flight) {   // GPU finished first: abandon the running chunk (L18.s19)
         ex.abort_flag = 1;
         ex.wait();
@@ -1250,7 +1289,7 @@ fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     const int64_t nwg = L.hi - L.lo;
     const int parts = (L.o.cpu_wg_split && nwg < nact) ? (int)((nact + nwg - 1) / nwg) : 1;
     const double t0 = now_ms();
-    ex.abort_flag = 0;
+    quiesce(ctx);
     ex.submit(L.a, L.g, L.lo, L.hi, parts, nact);
     ex.wait();
     info.t_host_ms = now_ms() - t0;
@@ -1422,6 +1461,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (!ctx) return FCL_INVALID_CONTEXT;
     cudaSetDevice(ctx->device);
     drain(ctx);
+    quiesce(ctx);
     if (ctx->tr.on) {
         const char *path = getenv("FCL_TRACE_FILE");
         FILE *f = path ? fopen(path, "w") : stderr;
@@ -1531,6 +1571,7 @@ fcl_status fcl_release_buffer(fcl_buffer b) {
     fcl_context ctx = b->ctx;
     cudaSetDevice(ctx->device);
     drain(ctx);
+    quiesce(ctx);   // no abandoned chunk may still touch the mirror being freed
     cudaStreamSynchronize(ctx->main);
     cudaStreamSynchronize(ctx->hd);
     cudaStreamSynchronize(ctx->dh);
@@ -1552,6 +1593,7 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
     if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
     if (!src || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "write range");
     drain(ctx);
+    quiesce(ctx);   // an abandoned chunk may still read or write this mirror
     if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
     char *h = (char *)b->host + offset;
     if (n < b->bytes) {
@@ -1574,6 +1616,7 @@ fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t 
     if (!dst || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "read range");
     (void)blocking;
     drain(ctx);
+    quiesce(ctx);
     if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
     if (b->host_valid) {   // location tracking (L20.s31-33): no transfer when the host is current
         const char *h = (const char *)b->host + offset;
@@ -1740,6 +1783,7 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     bool host_needed = false;
     for (int k = 0; k < L.a.nbuf; ++k) host_needed |= !L.bufs[k]->host_valid || !L.bufs[k]->dev_valid;
     if (!coop || host_needed || L.o.blocking || conflicts_with_pending(ctx, L)) drain(ctx);
+    if (!coop || conflicts_with_quiescing(ctx, L)) quiesce(ctx);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
 
     if (!coop) {
@@ -1830,6 +1874,7 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
     if (s != FCL_SUCCESS) return s;
     if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
     drain(ctx);
+    quiesce(ctx);
     if (!b->merge_pending) return FCL_SUCCESS;
     const char *tw = b->twin ? (const char *)b->twin : (const char *)b->dev;
     if (gpu_launch_merge((char *)b->dev + b->m_b0, (char *)b->stage + b->m_b0, tw + b->m_b0,
@@ -1879,6 +1924,7 @@ fcl_status fcl_finish(fcl_context ctx) {
     ctx->tr.add("finish_main", ctx->epoch);
     CK(ctx, cudaStreamSynchronize(ctx->hd));
     ctx->tr.add("finish_hd", ctx->epoch);
+    quiesce(ctx);   // abandoned host chunks have stopped (usually long ago)
     CK(ctx, cudaGetLastError());
     ctx->tr.add("finish_end", ctx->epoch);
     if (ctx->tr.on && ctx->stats) {

@@ -95,6 +95,9 @@ def run_config(name, steps, cpu_steps, modes):
     reset = meta.get("reset", [])
     originals = {li: Ps[li].bufs[0].copy() for li in reset}
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    # read sweep after the write flush: L2 ends full of clean, unrelated lines (no dirty
+    # write-backs charged to the next kernel)
+    sweep = torch.ones(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
     # dominant kernel: the one with the most algorithmic work
     dom = max(range(len(Ps)), key=lambda k: algorithmic(Ps[k])[1] / (HBM * 1e9 if algorithmic(Ps[k])[0] == "hbm" else FP32_TFLOPS * 1e12))
     out = {"config": name, "launches": [H.kernel_name(P) for P in Ps], "dominant": H.kernel_name(Ps[dom])}
@@ -108,7 +111,7 @@ def run_config(name, steps, cpu_steps, modes):
                 bufsets[li][0].write_array(originals[li])
             ctx.finish()
             with torch.cuda.stream(stream):
-                flush.fill_(1.0)
+                flush.fill_(1.0); sweep.sum()
             stream.synchronize()   # idle GPU at e0: host work cannot hide under the flush
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)

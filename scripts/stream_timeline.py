@@ -29,6 +29,9 @@ def main():
     for dl, db, sl, sb in meta.get("shared", []):
         bufs[dl][db] = bufs[sl][sb]
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    # read sweep after the write flush: L2 ends full of clean, unrelated lines (no dirty
+    # write-backs charged to the next kernel)
+    sweep = torch.ones(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
     modes = ("gpu", "coop")
     Ls = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m, timing=True)
               for P, b in zip(Ps, bufs)] for m in modes}
@@ -41,7 +44,7 @@ def main():
         for mode in modes:   # interleaved: slow drifts of the box hit both modes alike
             ctx.finish()
             with torch.cuda.stream(stream):
-                flush.fill_(1.0)
+                flush.fill_(1.0); sweep.sum()
             stream.synchronize()
             ev = [torch.cuda.Event(enable_timing=True) for _ in range(len(Ps) + 2)]
             t0 = time.perf_counter()
