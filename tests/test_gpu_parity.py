@@ -181,6 +181,30 @@ def test_cpu_first_returns_host_authoritative(ctx):
         assert_bits(H.device_array(bufs[k], np.int32), ref[k], "device (merged)")
 
 
+def test_abandoned_chunk_hazards(ctx):
+    """Deferred quiescence: the GPU wins a lite, eagerly returned GESUMMV, whose
+    host chunk is abandoned but not waited for.  Overwriting its input right away -- by a launch
+    that writes it (WAR) or by fcl_write_buffer -- must not let the abandoned workers write
+    anything derived from the new input into the first launch's outputs."""
+    n = 2048
+    P = W.make("gesummv", n, n, seed=31, lws1d=64, out_init="zero")
+    ref, _ = H.run(ctx, P, mode="gpu")
+    Q = W.make("atax_tmp", n, n, seed=32, lws1d=64, out_init="zero")   # writes a length-n vector
+    for trial in range(6):
+        bufs = H.create_buffers(ctx, P)          # A, B, x, tmp, y
+        A2, x2 = ctx.buffer_from_array(Q.bufs[0]), ctx.buffer_from_array(Q.bufs[1])
+        ctx.enqueue_ndrange("gesummv_f32", P.gws, P.lws, H.make_args(ctx, P, bufs))
+        if trial % 2 == 0:   # WAR: x of the first launch is the output of the second
+            ctx.enqueue_ndrange("atax_tmp_f32", Q.gws, Q.lws, [A2, x2, bufs[2], n, n])
+        else:
+            bufs[2].write_array(np.full(n, 7.0, np.float32))
+        ctx.finish()
+        for k in (3, 4):
+            assert_bits(bufs[k].read_array(np.float32), ref[k], f"gesummv buf{k} trial {trial}")
+        for b in bufs + [A2, x2]:
+            b.release()
+
+
 def test_slices_cover_only_their_range(ctx):
     """opts.wg_lo/wg_hi: a rank's slice writes exactly its work-groups (multi-GPU building block)."""
     P = W.make("conv2d", 130, 260, integer=True, seed=5)
