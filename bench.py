@@ -27,7 +27,6 @@ import os
 import statistics
 import subprocess
 import sys
-import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
@@ -59,28 +58,47 @@ def problems(seed: int):
 
 # ---------------------------------------------------------------------------------- clocks
 class ClockSampler:
+    """nvidia-smi sampling clocks every 100 ms into a temporary file.  No Python thread reads
+    its pipe: a reader thread competing for the GIL with the launching thread stalled
+    cooperative steps by milliseconds."""
+
     def __init__(self, index: int):
-        self.index, self.proc, self.lines = index, None, []
+        self.index, self.proc, self.path = index, None, None
 
     def __enter__(self):
         if os.environ.get("FCL_NO_CLOCKS"):
             return self
+        import tempfile
         q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
         try:
+            fd, self.path = tempfile.mkstemp(prefix="fcl_clocks_", suffix=".csv")
+            self.out = os.fdopen(fd, "w")
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}", "--format=csv,noheader,nounits",
                                           "-i", str(self.index), "-lms", "100"],
-                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
-            self.t.start()
+                                         stdout=self.out, stderr=subprocess.DEVNULL, text=True)
         except Exception:
             self.proc = None
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.lines.append(line.strip())
+    @property
+    def lines(self) -> list:
+        if not self.path:
+            return []
+        try:
+            with open(self.path) as f:
+                return [l.strip() for l in f if l.strip()]
+        except OSError:
+            return []
+
+    def wait_started(self, timeout: float = 10.0):
+        """Block until the sampler has printed its first sample: nvidia-smi's start-up (process
+        spawn, NVML init) competes with the launch path for host cores and driver locks, so it
+        must not fall inside the timed region."""
+        t0 = time.perf_counter()
+        while self.proc and not self.lines and time.perf_counter() - t0 < timeout:
+            time.sleep(0.01)
 
     def __exit__(self, *a):
         if self.proc:
@@ -89,11 +107,12 @@ class ClockSampler:
                 self.proc.wait(timeout=2)
             except Exception:
                 self.proc.kill()
+            self.out.close()
 
     def summary(self) -> dict:
         sm, mx, reasons = [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for l in self.lines:
+        for l in list(self.lines):
             p = [x.strip() for x in l.split(",")]
             if len(p) < 9:
                 continue
@@ -104,6 +123,11 @@ class ClockSampler:
             for nm, v in zip(names, p[5:9]):
                 if v.lower() == "active":
                     reasons.add(nm)
+        if self.path:
+            try:
+                os.unlink(self.path)
+            except OSError:
+                pass
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
                 "reasons": sorted(reasons), "samples": len(sm)}
 
@@ -200,9 +224,13 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     b3[0].release()
     b3[0] = b2[0]
     bufs += [b2, b3]
-    # CUDA events around the dominant kernel (GESUMMV's dispatcher / plain grid) only
-    prepared = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m, timing=(k == 0))
-                    for k, (P, b) in enumerate(zip(Ps, bufs))] for m in ("coop", "gpu", "cpu")}
+    prepared = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m)
+                    for P, b in zip(Ps, bufs)] for m in ("coop", "gpu", "cpu")}
+    # per-launch detail steps only: CUDA timing events around the dominant kernel (GESUMMV).
+    # Not in the timed steps -- a timing event between two grids keeps the second from
+    # starting under the first's tail (programmatic dependent launch) and costs ~3 us itself.
+    prepared["coop_t"] = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode="coop",
+                                      timing=(k == 0)) for k, (P, b) in enumerate(zip(Ps, bufs))]
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     # read sweep after the write flush: L2 ends full of clean, unrelated lines (no dirty
     # write-backs charged to the next kernel)
@@ -251,6 +279,9 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     torch.cuda.synchronize()
     import gc
     with ClockSampler(local_rank) as clk:
+        clk.wait_started()
+        for _ in range(max(1, args.warmup)):   # re-warm after the sampler's start-up
+            step("coop")
         if dist is not None:
             dist.barrier()
         torch.cuda.synchronize()
@@ -260,6 +291,8 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         coop_ts, _ = timed("coop", args.steps)
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall0
+        # the GPU-only baseline under the same conditions (sampler running, gc off), right after
+        gpu_ts, _ = timed("gpu", args.steps)
         gc.enable()
         if dist is not None:
             dist.barrier()
@@ -273,9 +306,8 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         print("coop step ms:", [round(t, 3) for t in coop_ts], file=sys.stderr)
 
     # per-launch detail (dispatcher CUDA-event time, merges, host share) from separate steps
-    _, infos = timed("coop", max(2, min(args.steps, 5)), collect=True, idle=False)
+    _, infos = timed("coop_t", max(2, min(args.steps, 5)), collect=True, idle=False)
     gc.disable()
-    gpu_ts, _ = timed("gpu", max(10, min(args.steps, 100)))
     cpu_ts, _ = timed("cpu", max(2, min(args.steps, 5)))
     gc.enable()
     gpu_ms = max_over_ranks(statistics.mean(gpu_ts))

@@ -124,9 +124,15 @@ struct SlotReset {
     unsigned int *arrive;
     unsigned long long *exit_word;
     unsigned int epoch;
+    unsigned long long *tstamp;   // optional (stats): [block-0 start, last CTA end] %globaltimer
 };
+// pdl: PDL_OFF = ordinary launch; PDL_NOWAIT = programmatic stream serialization, the grid may
+// start while the previous plain grid drains and does not wait for it (the runtime found no
+// buffer shared with any grid possibly still in flight); PDL_WAIT = same, but every CTA first
+// waits for the grids before it (griddepcontrol.wait).
+enum { PDL_OFF = 0, PDL_NOWAIT = 1, PDL_WAIT = 2 };
 int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream,
-                     const SlotReset *reset = nullptr);
+                     const SlotReset *reset = nullptr, int pdl = PDL_OFF);
 // CTAs of the persistent dispatcher resident at once (occupancy x SMs): a launch with no more
 // tasks than this runs in a single wave, every CTA's only task unchecked.
 int64_t gpu_coop_capacity(const KArgs &a, const Geom &g, int num_sms);

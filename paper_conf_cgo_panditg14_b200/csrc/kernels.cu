@@ -468,26 +468,46 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     if (c.mg.tstamp && threadIdx.x == 0) atomicMax(c.mg.tstamp + 1, globaltimer());
 }
 
+// Programmatic dependent launch (PDL).  Plain grids are launched with programmatic stream
+// serialization, so the next plain grid on the stream may start while this one drains (its
+// launch latency and ramp hide under our tail).  Every CTA signals launch_dependents at its
+// start -- after griddepcontrol.wait when the runtime found a dependency on a grid still in
+// flight (pdl_wait), and after block 0 has reset the next slot's counters (fenced), which the
+// next grid may use at once.
+__device__ __forceinline__ void pdl_wait_prior() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
-plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo, const SlotReset r) {
+plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo, const SlotReset r, int pdl_wait) {
     __shared__ int s_flag;
-    if (r.claim && blockIdx.x == 0 && threadIdx.x == 0) {   // next slot's dispatcher counters
-        *r.claim = 0ull;
-        for (int q = 0; q < 17; ++q) r.barrier[q] = 0u;
-        *r.merge_ctr = 0ull;
-        if (r.tasks) *r.tasks = 0ull;
+    if (pdl_wait) pdl_wait_prior();
+    if (r.tstamp && blockIdx.x == 0 && threadIdx.x == 0) r.tstamp[0] = globaltimer();
+    if (blockIdx.x == 0) {
+        if (r.claim && threadIdx.x == 0) {   // next slot's dispatcher counters
+            *r.claim = 0ull;
+            for (int q = 0; q < 17; ++q) r.barrier[q] = 0u;
+            *r.merge_ctr = 0ull;
+            if (r.tasks) *r.tasks = 0ull;
+            __threadfence();
+        }
+        __syncthreads();
     }
+    pdl_trigger();
     __shared__ __align__(16) typename Body::Smem smem;
     __shared__ long long s_key;
     TaskCtx tc;
     tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = &s_flag; tc.s_key = &s_key;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
+    if (r.tstamp) {
+        __syncthreads();
+        if (threadIdx.x == 0) atomicMax(r.tstamp + 1, globaltimer());
+    }
     if (r.exit_word) {   // lite cooperative launch: GPU-exit signal for the host (L18.s19)
         __syncthreads();
         if (threadIdx.x == 0) {
             // hierarchical arrival (16 leaves + root); no fence: the word publishes no data,
-            // the return copies are ordered behind the kernel on the streams
+            // the outputs' return copies are ordered behind the grid on the streams
             const unsigned int leaf = blockIdx.x & 15u;
             const unsigned int nleaf = (gridDim.x > 16u) ? 16u : gridDim.x;
             const unsigned int leaf_size = (gridDim.x - leaf + 15u) / 16u;
@@ -530,11 +550,13 @@ template <typename T, int NMAT>
 struct RowDotBody {
     // 4 warps, one row each: 64 registers allow 8 CTAs (32 warps) per SM, so a 4096-row
     // launch (1024 tasks) is resident in a single wave with 2 KB of loads in flight per warp.
+    // GESUMMV: 4 blocks of loads in flight at 72 registers = 7 CTAs per SM (1036 >= 1024 tasks,
+    // still one wave at N = 4096; 0.74 vs 0.71 of HBM with 2 blocks, scripts/ubench_dots.cu).
     static constexpr int kThreads = 128;
-    static constexpr int kMinBlocks = 8;
+    static constexpr int kMinBlocks = (NMAT == 2) ? 7 : 8;
     static constexpr bool kLateClaim = false;
     static constexpr int kWarps = kThreads / 32;
-    static constexpr int U = (NMAT == 2) ? 2 : 4;   // 128-column blocks whose loads are issued together
+    static constexpr int U = 4;   // 128-column blocks whose loads are issued together
     struct Params {
         const T *A; const T *B; const T *x; T *out0; T *out1;
         long long nrows, ncols, lws; int R; T alpha, beta; int vec4;
@@ -630,64 +652,97 @@ struct RowDotBody {
 // Column-dot bodies: ATAX kernel 2 (y = A^T tmp), BICG kernel 1 (s = A^T r), CORR mean / std.
 // A work-group is lws consecutive columns; a task is CB <= 32 of them, all rows.
 // Canonical order: partial q (q = i % 32) accumulates rows i = q, q+32, ... ascending; the 32
-// partials are then added sequentially q = 0..31.  Warp w of the CTA owns partial w.
+// partials are then added sequentially q = 0..31.
+// Thread t owns partial q = t / 8 of the 4 columns 4*(t % 8) .. +3 of the task, so a warp
+// reads 4 rows x 128 contiguous bytes per load and each thread keeps U = 16 row loads (16 B
+// each) in flight: 256 threads, 16 KB in flight per CTA (the 1024-thread scalar layout kept
+// only 4 B per thread in flight and reached 0.50 of HBM at N = 4096; this one 0.60,
+// scripts/ubench_dots.cu).
 // ------------------------------------------------------------------------------------------
 enum { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
 
 template <typename T, int MODE>
 struct ColDotBody {
-    static constexpr int kThreads = 1024;
-    static constexpr int kMinBlocks = 1;
+    static constexpr int kThreads = 256;
+    static constexpr int kMinBlocks = 2;
     static constexpr bool kLateClaim = false;
+    static constexpr int U = 16;
     struct Params {
         const T *A; const T *v; const T *mean; T *out;
-        long long nrows, ncols, lws; int CB; float nf, eps;
+        long long nrows, ncols, lws; int CB; float nf, eps; int vec4;
     };
     struct Smem { T red[32][33]; };
 
     __device__ static long long key(const Params &p, long long t) { return (t * p.CB) / p.lws; }
 
-    __device__ static T term(const Params &p, T a, long long i, T mj, T acc) {
-        if (MODE == COL_DOT) return op_fma(a, p.v[i], acc);
+    __device__ static T term(const Params &p, T a, T vi, T mj, T acc) {
+        if (MODE == COL_DOT) return op_fma(a, vi, acc);
         if (MODE == COL_SUM) return op_add(acc, a);
         const T c = op_add(a, -mj);   // a - mean (exact negation, then one rounding)
         return op_fma(c, c, acc);
     }
 
     __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &sm) {
-        const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-        const long long j = t * p.CB + lane;
-        const bool active = (lane < p.CB) && (j < p.ncols);
-        T acc = 0;
-        if (active) {
-            const T mj = (MODE == COL_SQDEV) ? p.mean[j] : T(0);
-            // explicit pointer walk down the column (rows w, w + 32, ...)
+        const int quad = threadIdx.x & 7, q = threadIdx.x >> 3;
+        const long long j0 = t * p.CB + 4 * quad;          // first of this thread's 4 columns
+        // columns of this thread inside the task and the matrix (CB < 4 only for tiny lws)
+        const int ncol = (int)max(0ll, min(min(4ll, (long long)p.CB - 4 * quad), p.ncols - j0));
+        T c0 = 0, c1 = 0, c2 = 0, c3 = 0;
+        if (ncol > 0) {
+            T m[4] = {0, 0, 0, 0};
+            if (MODE == COL_SQDEV)
+                for (int c = 0; c < ncol; ++c) m[c] = p.mean[j0 + c];
             const long long stride = 32 * p.ncols;
-            const T *pc = p.A + j + (long long)w * p.ncols;
-            long long i = w;
-            for (; i + 7 * 32 < p.nrows; i += 8 * 32) {
-                T a[8];
+            const T *pc = p.A + j0 + (long long)q * p.ncols;   // explicit pointer walk down the rows
+            long long i = q;
+            if (p.vec4 && ncol == 4) {
+                for (; i + (U - 1) * 32 < p.nrows; i += U * 32) {
+                    typename V4<T>::type a[U];
+                    T vi[U];
 #pragma unroll
-                for (int u = 0; u < 8; ++u) { a[u] = __ldcs(pc); pc += stride; }
+                    for (int u = 0; u < U; ++u) { a[u] = ld_stream4(pc); pc += stride; }
 #pragma unroll
-                for (int u = 0; u < 8; ++u) acc = term(p, a[u], i + 32 * u, mj, acc);
+                    for (int u = 0; u < U; ++u) vi[u] = (MODE == COL_DOT) ? __ldg(p.v + i + 32 * u) : T(0);
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        c0 = term(p, a[u].x, vi[u], m[0], c0); c1 = term(p, a[u].y, vi[u], m[1], c1);
+                        c2 = term(p, a[u].z, vi[u], m[2], c2); c3 = term(p, a[u].w, vi[u], m[3], c3);
+                    }
+                }
+                for (; i < p.nrows; i += 32, pc += stride) {
+                    const typename V4<T>::type a = ld_stream4(pc);
+                    const T vi = (MODE == COL_DOT) ? __ldg(p.v + i) : T(0);
+                    c0 = term(p, a.x, vi, m[0], c0); c1 = term(p, a.y, vi, m[1], c1);
+                    c2 = term(p, a.z, vi, m[2], c2); c3 = term(p, a.w, vi, m[3], c3);
+                }
+            } else {   // unaligned rows or the ragged last columns: scalar loads, same order
+                for (; i < p.nrows; i += 32, pc += stride) {
+                    const T vi = (MODE == COL_DOT) ? p.v[i] : T(0);
+                    c0 = term(p, __ldcs(pc), vi, m[0], c0);
+                    if (ncol > 1) c1 = term(p, __ldcs(pc + 1), vi, m[1], c1);
+                    if (ncol > 2) c2 = term(p, __ldcs(pc + 2), vi, m[2], c2);
+                    if (ncol > 3) c3 = term(p, __ldcs(pc + 3), vi, m[3], c3);
+                }
             }
-            for (; i < p.nrows; i += 32, pc += stride) acc = term(p, __ldcs(pc), i, mj, acc);
         }
-        sm.red[w][lane] = acc;
+        sm.red[q][4 * quad + 0] = c0; sm.red[q][4 * quad + 1] = c1;
+        sm.red[q][4 * quad + 2] = c2; sm.red[q][4 * quad + 3] = c3;
         __syncthreads();
-        if (w == 0 && active) {
-            T tot = sm.red[0][lane];
+        const long long j = t * p.CB + threadIdx.x;
+        if (threadIdx.x < p.CB && j < p.ncols) {
+            T tot = sm.red[0][threadIdx.x];
 #pragma unroll 8
-            for (int q = 1; q < 32; ++q) tot = op_add(tot, sm.red[q][lane]);
+            for (int qq = 1; qq < 32; ++qq) tot = op_add(tot, sm.red[qq][threadIdx.x]);
+            T o;
             if (MODE == COL_DOT) {
-                p.out[j] = tot;
+                o = tot;
             } else if (MODE == COL_SUM) {
-                p.out[j] = (T)__fdiv_rn((float)tot, p.nf);
+                o = (T)__fdiv_rn((float)tot, p.nf);
             } else {
                 float s = __fsqrt_rn(__fdiv_rn((float)tot, p.nf));
-                p.out[j] = (T)((s <= p.eps) ? 1.0f : s);
+                o = (T)((s <= p.eps) ? 1.0f : s);
             }
+            p.out[j] = o;
         }
         __syncthreads();
         return false;
@@ -1068,7 +1123,7 @@ static int occupancy_grid(int num_sms) {
 
 template <class Body>
 static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long long task_lo, long long task_hi,
-                       int num_sms, cudaStream_t s, const SlotReset *reset = nullptr) {
+                       int num_sms, cudaStream_t s, const SlotReset *reset = nullptr, int pdl = PDL_OFF) {
     const long long n = task_hi - task_lo;
     if (n <= 0) return 0;
     if (c) {
@@ -1092,8 +1147,16 @@ static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long l
     }
     SlotReset r{};
     if (reset) r = *reset;
-    plain_kernel<Body><<<(unsigned)n, Body::kThreads, 0, s>>>(bp, task_lo, r);
-    cudaError_t e = cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)n);
+    cfg.blockDim = dim3(Body::kThreads);
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl != PDL_OFF ? 1 : 0;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, plain_kernel<Body>, bp, (long long)task_lo, r, pdl == PDL_WAIT ? 1 : 0);
     if (e != cudaSuccess) return seterr(e, "plain_kernel launch");
     return (int)n;
 }
@@ -1137,10 +1200,12 @@ static typename ColDotBody<T, MODE>::Params coldot_params(const KArgs &a, const 
     p.A = (const T *)a.dev[0];
     p.v = (MODE == COL_DOT) ? (const T *)a.dev[1] : nullptr;
     p.mean = (MODE == COL_SQDEV) ? (const T *)a.dev[1] : nullptr;
-    p.out = (T *)a.dev[(MODE == COL_SQDEV) ? 2 : (MODE == COL_SUM ? 1 : 2)];
+    const int oi = (MODE == COL_SQDEV) ? 2 : (MODE == COL_SUM ? 1 : 2);
+    p.out = (T *)a.dev[oi];
     p.nrows = a.n0; p.ncols = a.n1; p.lws = g.lws[0];
     p.CB = largest_pow2_divisor_le(g.lws[0], 32);
     p.nf = (float)a.n0; p.eps = a.eps;
+    p.vec4 = (p.ncols % 4 == 0) && is_aligned16(p.A);
     return p;
 }
 
@@ -1233,7 +1298,7 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
     case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD: {
         const int CB = largest_pow2_divisor_le(g.lws[0], 32);
         ts.ntasks = (g.ng[0] * g.lws[0] + CB - 1) / CB;
-        ts.threads = 1024; break;
+        ts.threads = 256; break;
     }
     case K_CORR_REDUCE: case K_CONV2D: {
         int tw, th; tile_shape(g, 256, 32, tw, th);
@@ -1323,9 +1388,9 @@ struct CoopLauncher {
     }
 };
 struct PlainLauncher {
-    long long lo, hi; cudaStream_t s; const SlotReset *reset;
+    long long lo, hi; cudaStream_t s; const SlotReset *reset; int pdl;
     template <class Body> int go(const typename Body::Params &bp) {
-        return launch_body<Body>(bp, nullptr, lo, hi, 0, s, reset);
+        return launch_body<Body>(bp, nullptr, lo, hi, 0, s, reset, pdl);
     }
 };
 struct CapacityQuery {
@@ -1344,8 +1409,8 @@ int gpu_launch_coop(const KArgs &a, const Geom &g, const CoopCtl &c, int num_sms
 }
 
 int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t task_hi, void *stream,
-                     const SlotReset *reset) {
-    PlainLauncher L{task_lo, task_hi, (cudaStream_t)stream, reset};
+                     const SlotReset *reset, int pdl) {
+    PlainLauncher L{task_lo, task_hi, (cudaStream_t)stream, reset, pdl};
     return with_body(a, g, L);
 }
 

@@ -287,6 +287,12 @@ struct fcl_buffer_st {
     bool own_dev, own_host;
     bool host_valid, dev_valid;
     bool d2h_pending;
+    bool d2h_on_main;      // the pending return copy is queued on main (a lazy return): later
+                           // grids on main are ordered behind it without a cross-stream wait
+    bool ret_lazy;         // a lazy return of [ret_b0, ret_b1) is registered, not yet queued
+    size_t ret_b0, ret_b1;
+    uint64_t d2h_gen;      // ctx->finish_gen when the pending return was queued
+    void *host_dptr;       // device-visible address of the (mapped) host mirror, nullptr = none
     cudaEvent_t d2h_ev;    // completion of the buffer's pending return copy (recorded on dh)
     // deferred merge state (opts.defer_merge)
     bool merge_pending;
@@ -320,11 +326,16 @@ struct Job {
     int slot = 0;
     int64_t t0 = 0, t1 = 0, s_forced = -1;
     bool forced = false, dev_merge = false, eager = false, gpu_launched = false;
+    bool lazy = false;         // outputs return lazily (batched on main at the next flush point)
     bool lite = false;         // single wave, no in-task polls: plain grid + exit memop, never a merge
     bool exact_spans = false;  // every output's footprint of a work-group range is one exact span
     bool twin_alias = false;   // exact spans: the merge compares against the device copy itself
     int64_t unit = 1;          // host chunk boundaries are multiples of this many work-groups
     void *twin[6] = {nullptr}, *stage[6] = {nullptr};
+    // ev_k0/ev_t1/ev_m0/ev_m1 carry timestamps and are recorded only when timing is asked for:
+    // a timing event between two grids on main stops the second from overlapping the first
+    // (PDL) and costs ~3 us per boundary even without it (scripts/ubench_dots.cu)
+    cudaEvent_t ev_t1 = nullptr;
     cudaEvent_t ev_start = nullptr, ev_k0 = nullptr, ev_k1 = nullptr, ev_m0 = nullptr, ev_m1 = nullptr,
                 ev_staged = nullptr, ev_ret = nullptr, ev_wm = nullptr, ev_d2h = nullptr;
     cudaEvent_t main_before = nullptr;   // an event on main at or after every earlier launch's merge
@@ -350,10 +361,28 @@ struct fcl_context_st {
     unsigned long long *status_dptr = nullptr;   // device-visible address of slot 0
     bool slot_used[kSlots] = {};
     unsigned long long *wm_host = nullptr;       // pinned copy of the dispatcher's wm word
-    unsigned long long *exit_host = nullptr;     // mapped word: epoch of the last finished dispatcher
-    unsigned long long *exit_dptr = nullptr;     // its device-visible address
+    // mapped words, one per launch slot: epoch of the last finished GPU grid of that slot (per
+    // slot, because grids of consecutive launches may overlap and finish out of order, PDL)
+    unsigned long long *exit_host = nullptr;
+    unsigned long long *exit_dptr = nullptr;     // their device-visible address
+    // Programmatic dependent launch of plain grids (FCL_NO_PDL=1 disables): buffers touched by
+    // plain grids that may still be in flight -- a new grid sharing one with them (and at least
+    // one side writing) waits for them in-kernel; an op queued on main that a grid must not
+    // overtake (a stream wait, a copy on main) makes the next grid an ordinary launch.
+    struct ChainEnt { fcl_buffer b; int acc; };
+    bool pdl = true;
+    std::vector<ChainEnt> pdl_chain;
+    int pdl_chain_grids = 0;
+    std::atomic<int> main_fenced{1};
+    // fcl_finish generation: a return copy queued before the last fcl_finish has completed
+    std::atomic<uint64_t> finish_gen{1};
+    // something was queued on dh / hd since the last fcl_finish (else it skips their syncs)
+    std::atomic<int> dh_used{1}, hd_used{1};
     unsigned long long *dclaim = nullptr, *dtasks = nullptr, *dwm = nullptr;
     unsigned long long *dstamp = nullptr;        // stats mode: %globaltimer stamps, 4 per slot
+    unsigned long long *dpstamp = nullptr;       // stats mode: plain-grid stamps, 2 per grid since fcl_finish
+    int pst_n = 0;
+    static constexpr int kPlainStamps = 64;
     unsigned int *dbar = nullptr;                // grid-barrier counters, one per slot
     unsigned long long *dmctr = nullptr;         // fused-merge chunk counters, one per slot
     bool unfused = false;                        // FCL_UNFUSED_MERGE=1: merge as a separate kernel
@@ -364,11 +393,22 @@ struct fcl_context_st {
     PFN_writeValue64 write64 = nullptr;
     bool stats = false;                          // count executed GPU tasks, time merges (FCL_STATS=1)
     size_t eager_return_bytes = 8u << 20;        // outputs up to this size return right behind the merge
+    // Lazy return: small outputs of free-running and GPU-only launches are not
+    // copied back behind each grid (a copy on dh waits on an event of main, which keeps the next
+    // grid from starting under this one's tail and costs ~5 us per kernel boundary).  Their spans
+    // are registered and copied in ONE batched copy on main at the next point that needs a host
+    // copy: fcl_finish, fcl_read_buffer, a launch whose host side reads them (FCL_LAZY_BYTES,
+    // 0 = off).  At that point the device copy is authoritative for every registered span.
+    size_t lazy_max_bytes = 1u << 20;
+    std::vector<fcl_buffer> lazy;
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
     bool memop_nobarrier_ok = true;              // cleared when the driver rejects NO_MEMORY_BARRIER
     int exit_poll_pauses = 8;                    // pause instructions between exit-word polls (FCL_EXIT_POLL_PAUSES)
+    bool lite_exit_word = true;                  // FCL_LITE_EXIT=0: lite grids store no exit word, the
+                                                 // coordinator polls their completion event instead
+    unsigned exit_query_mask = 0xFFFF;           // event polls every mask+1 exit-word polls
     // Deferred quiescence: an abandoned chunk of an eagerly returned launch may
     // still be running; its launch's buffers are kept here until quiesce() has waited for it.
     std::mutex qz_mu;
@@ -406,7 +446,7 @@ struct fcl_context_st {
     std::string err;
     std::atomic<fcl_status> sticky{FCL_SUCCESS};
     // single-device modes
-    cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr, ev_mark = nullptr;
+    cudaEvent_t ev_k0 = nullptr, ev_t1 = nullptr, ev_k1 = nullptr, ev_mark = nullptr;   // k0/t1: timing only
     cudaEvent_t ev_gd2h = nullptr;               // completion of single-device / deferred returns (on dh)
     fcl_launch_info sync_info{};
     bool sync_have_k = false;
@@ -440,6 +480,13 @@ fcl_status cuda_fail(fcl_context ctx, cudaError_t e, const char *what) {
         cudaError_t _e = (call);                                        \
         if (_e != cudaSuccess) return cuda_fail((ctx), _e, #call);      \
     } while (0)
+
+// A buffer's return copy may still be reading its device copy (not if an fcl_finish has
+// synchronised dh since it was queued).
+bool d2h_busy(fcl_context ctx, fcl_buffer b) {
+    if (b->d2h_pending && b->d2h_gen < ctx->finish_gen.load(std::memory_order_acquire)) b->d2h_pending = false;
+    return b->d2h_pending;
+}
 
 // ---- pool ----
 // Returns the buffer and whether main must wait for ctx->ev_hd_release before writing it.
@@ -518,23 +565,32 @@ fcl_status stream_store(fcl_context ctx, unsigned long long *dst, unsigned long 
 // Publish {epoch, W} behind everything queued on hd: status follows data (C13, L16.s15).
 fcl_status publish(fcl_context ctx, const Job &j, uint32_t w) {
     const unsigned long long v = ((unsigned long long)j.epoch << 32) | w;
+    ctx->hd_used.store(1, std::memory_order_relaxed);
     return stream_store(ctx, ctx->status_dptr + j.slot, v, ctx->hd, true, const_cast<fcl_launch_info *>(&j.info));
 }
 
 // Bring a buffer's copies to what a launch needs.  A pending return copy is waited for on the
 // host only when the host copy is needed; a device-only use of a buffer the launch writes is
 // ordered behind it on the device (write-after-read), and device-only reads need nothing.
+fcl_status flush_returns(fcl_context ctx, bool at_finish);
+
 fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_dev, fcl_launch_info *info,
                       bool dev_write = true) {
-    if (b->d2h_pending) {
+    if (need_host && b->ret_lazy) {
+        fcl_status f = flush_returns(ctx, false);
+        if (f != FCL_SUCCESS) return f;
+    }
+    if (d2h_busy(ctx, b)) {
         if (need_host || !b->dev_valid) {
             CK(ctx, cudaEventSynchronize(b->d2h_ev));
             b->d2h_pending = false;
-        } else if (dev_write) {
+        } else if (dev_write && !b->d2h_on_main) {   // (a write-through "return" reads nothing)
             CK(ctx, cudaStreamWaitEvent(ctx->main, b->d2h_ev, 0));
+            ctx->main_fenced.store(1);
         }
     }
     if (need_dev && !b->dev_valid) {
+        ctx->main_fenced.store(1);
         CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
         b->dev_valid = true;
         if (info) info->h2d_bytes += (int64_t)b->bytes;
@@ -572,10 +628,11 @@ fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, fcl
         size_t b0, b1;
         out_span(L.a, L.g, L.out_idx[q], wlo, whi, &b0, &b1);
         if (b1 <= b0) continue;
+        ctx->dh_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaMemcpyAsync((char *)b->host + b0, (char *)b->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
         info.d2h_bytes += (int64_t)(b1 - b0);
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
-        b->d2h_pending = true;
+        b->d2h_pending = true; b->d2h_on_main = false; b->d2h_gen = ctx->finish_gen.load();
     }
     return FCL_SUCCESS;
 }
@@ -617,6 +674,7 @@ fcl_status enqueue_merges(fcl_context ctx, Job &j, int64_t mlo, int64_t mhi) {
 // Lowest watermark the dispatcher of job j acted on (hi if it never skipped); a synchronous
 // 8-byte read used off the fast path.  Only valid until a later dispatcher touches the word.
 fcl_status read_gpu_watermark(fcl_context ctx, Job &j, int64_t *wm) {
+    ctx->dh_used.store(1, std::memory_order_relaxed);
     CK(ctx, cudaStreamWaitEvent(ctx->dh, j.ev_k1, 0));
     CK(ctx, cudaMemcpyAsync(ctx->wm_host, ctx->dwm, 8, cudaMemcpyDeviceToHost, ctx->dh));
     CK(ctx, cudaEventRecord(j.ev_wm, ctx->dh));
@@ -638,6 +696,14 @@ void quiesce(fcl_context ctx) {
     ctx->quiescing.store(0, std::memory_order_release);
 }
 
+// Non-blocking quiesce: true once no abandoned chunk is running (clearing the state then).
+bool quiesce_try(fcl_context ctx) {
+    if (!ctx->quiescing.load(std::memory_order_acquire)) return true;
+    if (!ctx->ex.finished()) return false;
+    quiesce(ctx);   // (finished: returns at once)
+    return true;
+}
+
 // Does launch L write a buffer the still-quiescing chunk reads or writes?
 bool conflicts_with_quiescing(fcl_context ctx, const Launch &L) {
     if (!ctx->quiescing.load(std::memory_order_acquire)) return false;
@@ -649,6 +715,102 @@ bool conflicts_with_quiescing(fcl_context ctx, const Launch &L) {
     return false;
 }
 
+// Lazy return: register the launch's output spans [lo, hi) if they are small (returns false
+// otherwise; the caller then queues an ordinary return copy).
+bool lazy_return(fcl_context ctx, const Launch &L, fcl_launch_info &info) {
+    if (ctx->lazy_max_bytes == 0) return false;
+    size_t tot = 0, b0[6], b1[6];
+    for (int q = 0; q < L.nout; ++q) {
+        out_span(L.a, L.g, L.out_idx[q], L.lo, L.hi, &b0[q], &b1[q]);
+        tot += b1[q] - b0[q];
+    }
+    if (tot > ctx->lazy_max_bytes) return false;
+    for (int q = 0; q < L.nout; ++q) {
+        fcl_buffer b = L.bufs[L.out_idx[q]];
+        if (b1[q] <= b0[q]) continue;
+        if (!b->ret_lazy) {
+            b->ret_lazy = true;
+            b->ret_b0 = b0[q]; b->ret_b1 = b1[q];
+            ctx->lazy.push_back(b);
+        } else {
+            b->ret_b0 = std::min(b->ret_b0, b0[q]);
+            b->ret_b1 = std::max(b->ret_b1, b1[q]);
+        }
+        info.d2h_bytes += (int64_t)(b1[q] - b0[q]);
+    }
+    return true;
+}
+
+// Queue every registered lazy return as one batched copy on main.  `at_finish`: the caller
+// synchronises main next and clears the buffers itself (no per-buffer completion events).
+fcl_status flush_returns(fcl_context ctx, bool at_finish) {
+    if (ctx->lazy.empty()) return FCL_SUCCESS;
+    const size_t n = ctx->lazy.size();
+    std::vector<void *> dst(n), src(n);
+    std::vector<size_t> sz(n);
+    for (size_t k = 0; k < n; ++k) {
+        fcl_buffer b = ctx->lazy[k];
+        dst[k] = (char *)b->host + b->ret_b0;
+        src[k] = (char *)b->dev + b->ret_b0;
+        sz[k] = b->ret_b1 - b->ret_b0;
+    }
+    ctx->main_fenced.store(1);   // a copy between grids on main: the next grid is ordinary
+    cudaMemcpyAttributes at = {};
+    at.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+    at.srcLocHint.type = cudaMemLocationTypeDevice; at.srcLocHint.id = ctx->device;
+    at.dstLocHint.type = cudaMemLocationTypeHost; at.dstLocHint.id = 0;
+    size_t aidx = 0, fail = 0;
+    if (n == 1 || cudaMemcpyBatchAsync(dst.data(), src.data(), sz.data(), n, &at, &aidx, 1, &fail, ctx->main) != cudaSuccess) {
+        cudaGetLastError();   // (a driver without batched copies: one copy per buffer)
+        for (size_t k = 0; k < n; ++k)
+            CK(ctx, cudaMemcpyAsync(dst[k], src[k], sz[k], cudaMemcpyDeviceToHost, ctx->main));
+    }
+    for (size_t k = 0; k < n; ++k) {
+        fcl_buffer b = ctx->lazy[k];
+        b->ret_lazy = false;
+        if (!at_finish) {
+            CK(ctx, cudaEventRecord(b->d2h_ev, ctx->main));
+            b->d2h_pending = true; b->d2h_on_main = true; b->d2h_gen = ctx->finish_gen.load();
+        }
+    }
+    ctx->lazy.clear();
+    return FCL_SUCCESS;
+}
+
+// Stats mode: stamp pair for the next plain grid (read and cleared by fcl_finish).
+unsigned long long *plain_stamp(fcl_context ctx) {
+    if (!ctx->dpstamp || ctx->pst_n >= fcl_context_st::kPlainStamps) return nullptr;
+    return ctx->dpstamp + 2 * ctx->pst_n++;
+}
+
+// PDL mode of the next plain grid on main (see fcl_context_st::pdl_chain).
+int pdl_mode_impl(fcl_context ctx, const Launch &L);
+int pdl_mode(fcl_context ctx, const Launch &L) {
+    const int m = pdl_mode_impl(ctx, L);
+    ctx->tr.add(m == PDL_OFF ? "pdl_off" : (m == PDL_WAIT ? "pdl_wait" : "pdl_nowait"), ctx->epoch);
+    return m;
+}
+int pdl_mode_impl(fcl_context ctx, const Launch &L) {
+    if (!ctx->pdl) return PDL_OFF;
+    auto &ch = ctx->pdl_chain;
+    if (ctx->main_fenced.exchange(0)) {   // an ordinary launch: it waits for everything before it
+        ch.clear();
+        ctx->pdl_chain_grids = 1;
+        for (int a = 0; a < L.a.nbuf; ++a) ch.push_back({L.bufs[a], L.acc[a]});
+        return PDL_OFF;
+    }
+    // at most 8 grids per chain: a grid can only be in flight together with the grids since the
+    // last waiting one, which keeps the 16-entry write-through counter ring safe
+    bool dep = ctx->pdl_chain_grids >= 8;
+    for (int a = 0; a < L.a.nbuf && !dep; ++a)
+        for (const auto &e : ch)
+            if (e.b == L.bufs[a] && ((e.acc | L.acc[a]) & 2)) { dep = true; break; }
+    if (dep) { ch.clear(); ctx->pdl_chain_grids = 0; }
+    for (int a = 0; a < L.a.nbuf; ++a) ch.push_back({L.bufs[a], L.acc[a]});
+    ctx->pdl_chain_grids += 1;
+    return dep ? PDL_WAIT : PDL_NOWAIT;
+}
+
 Job *job_alloc(fcl_context ctx) {
     Job *j = nullptr;
     {
@@ -657,15 +819,16 @@ Job *job_alloc(fcl_context ctx) {
     }
     if (!j) {
         j = new Job();
-        for (cudaEvent_t *pe : {&j->ev_k0, &j->ev_k1, &j->ev_m0, &j->ev_m1})
+        for (cudaEvent_t *pe : {&j->ev_k0, &j->ev_t1, &j->ev_m0, &j->ev_m1})
             if (cudaEventCreate(pe) != cudaSuccess) { cudaGetLastError(); return nullptr; }
-        for (cudaEvent_t *pe : {&j->ev_start, &j->ev_staged, &j->ev_ret, &j->ev_wm, &j->ev_d2h})
+        for (cudaEvent_t *pe : {&j->ev_start, &j->ev_k1, &j->ev_staged, &j->ev_ret, &j->ev_wm, &j->ev_d2h})
             if (cudaEventCreateWithFlags(pe, cudaEventDisableTiming) != cudaSuccess) { cudaGetLastError(); return nullptr; }
     }
     j->status = FCL_SUCCESS;
     j->done.store(0);
     j->have_k = j->have_m = j->wm_pending = false;
     j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = j->lite = j->exact_spans = false;
+    j->lazy = false;
     j->unit = 1;
     std::memset(&j->info, 0, sizeof j->info);
     for (int q = 0; q < 6; ++q) j->twin[q] = j->stage[q] = nullptr;
@@ -673,7 +836,7 @@ Job *job_alloc(fcl_context ctx) {
 }
 
 void job_release_buffers(fcl_context ctx, Job &j, bool staged) {
-    if (staged) cudaEventRecord(ctx->ev_hd_release, ctx->hd);
+    if (staged) { ctx->hd_used.store(1, std::memory_order_relaxed); cudaEventRecord(ctx->ev_hd_release, ctx->hd); }
     for (int q = 0; q < j.L.nout; ++q) {
         if (j.twin[q]) pool_put(ctx, j.twin[q], staged);
         if (j.stage[q]) pool_put(ctx, j.stage[q], staged);
@@ -703,7 +866,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     if (ctx->slot_used[j.slot]) {
         // the dispatcher that used this status slot 16 launches ago must have finished
         const uint32_t prev = j.epoch - kSlots;
-        while (__atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE) < prev) {
+        while (__atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) < prev) {
             const cudaError_t q = cudaStreamQuery(ctx->main);
             if (q == cudaSuccess) break;
             if (q != cudaErrorNotReady) return cuda_fail(ctx, q, "slot reuse");
@@ -765,7 +928,10 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         nbytes[q] = b->bytes;
     }
     ctx->tr.add("A_pool", j.epoch);
-    if (hd_wait) CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_release, 0));
+    if (hd_wait) {
+        CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_hd_release, 0));
+        ctx->main_fenced.store(1);
+    }
     if (!j.twin_alias) {
         if (gpu_launch_copies(L.nout, j.twin, srcs, nbytes, ctx->num_sms, ctx->main) < 0) {
             for (int q = 0; q < L.nout; ++q)   // unaligned caller memory: per-buffer copies
@@ -777,11 +943,13 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
 
     if (j.forced) {
         // test hook: the GPU is told the split before it starts
+        ctx->hd_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
         fcl_status st = publish(ctx, j, (uint32_t)j.s_forced);
         if (st != FCL_SUCCESS) return st;
         CK(ctx, cudaEventRecord(j.ev_staged, ctx->hd));
         CK(ctx, cudaStreamWaitEvent(ctx->main, j.ev_staged, 0));
+        ctx->main_fenced.store(1);
     }
 
     // GPU: the whole range, persistent dispatcher (C8)
@@ -804,7 +972,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     c.barrier_next = ctx->dbar + 32 * ((j.slot + 1) % kSlots);
     c.merge_ctr = ctx->dmctr + j.slot;
     c.merge_ctr_next = ctx->dmctr + (j.slot + 1) % kSlots;
-    c.exit_word = ctx->exit_dptr;
+    c.exit_word = ctx->exit_dptr + j.slot;
     c.mg = DevMergeList{};
     c.mg.n = 0;
 
@@ -840,7 +1008,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         M.epoch = j.epoch;
         M.hi = L.hi;
         M.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot + 2 : nullptr;
-        M.exit_word = ctx->exit_dptr;
+        M.exit_word = ctx->exit_dptr + j.slot;
     }
     M.wm_word = ctx->dwm;
     M.epoch = j.epoch;
@@ -856,19 +1024,25 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
         if (j.lite) {
             const int nx = (j.slot + 1) % kSlots;
             SlotReset r{ctx->dclaim + nx, ctx->stats ? ctx->dtasks + nx : nullptr, ctx->dmctr + nx, ctx->dbar + 32 * nx,
-                        ctx->dbar + 32 * j.slot, ctx->exit_dptr, j.epoch};
-            if (gpu_launch_plain(L.a, L.g, j.t0, j.t1, ctx->main, &r) < 0)
+                        ctx->dbar + 32 * j.slot, ctx->lite_exit_word ? ctx->exit_dptr + j.slot : nullptr, j.epoch,
+                        plain_stamp(ctx)};
+            if (gpu_launch_plain(L.a, L.g, j.t0, j.t1, ctx->main, &r, pdl_mode(ctx, L)) < 0)
                 return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
-        } else if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0) {
-            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        } else {
+            if (gpu_launch_coop(L.a, L.g, c, ctx->num_sms, ctx->main) < 0)
+                return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+            ctx->pdl_chain.clear();   // an ordinary launch that never triggers early: the next
+            ctx->pdl_chain_grids = 0;
+                                      // grid starts after it (and everything before it) completed
         }
         ctx->tr.add("A_launched", j.epoch);
+        if (timing) CK(ctx, cudaEventRecord(j.ev_t1, ctx->main));
         CK(ctx, cudaEventRecord(j.ev_k1, ctx->main));
         ctx->tr.add("A_k1", j.epoch);
         // GPU exit signal for the host executor (L18.s19): the fused tail (or, lite, the plain
         // grid's last CTA) stores the epoch to mapped host memory; unfused, a bare memop does it.
         if (!c.fused && !j.lite) {
-            fcl_status xs = stream_store(ctx, ctx->exit_dptr, (unsigned long long)j.epoch, ctx->main, false, &info);
+            fcl_status xs = stream_store(ctx, ctx->exit_dptr + j.slot, (unsigned long long)j.epoch, ctx->main, false, &info);
             if (xs != FCL_SUCCESS) return xs;
         }
         ctx->slot_used[j.slot] = true;
@@ -890,6 +1064,10 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
             return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
         info.gpu_launches += 1;
     }
+    // Small pure-OUT outputs of a free-running launch return lazily (the device copy is
+    // complete once the grid -- with its fused merge -- is; the return copies the whole span,
+    // so host words an abandoned chunk of this launch wrote are overwritten with the same bits)
+    if (j.eager && lazy_return(ctx, L, info)) { j.eager = false; j.lazy = true; }
     if (j.eager) {
         cudaEvent_t mark = j.ev_k1;
         if (!c.fused && !j.lite) { CK(ctx, cudaEventRecord(j.ev_ret, ctx->main)); mark = j.ev_ret; }
@@ -910,7 +1088,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     // host copies of every argument must be current (pending returns of earlier launches)
     for (int k = 0; k < L.a.nbuf; ++k) {
         fcl_buffer b = L.bufs[k];
-        if (b->d2h_pending && !(j.eager && (L.acc[k] & 2))) {
+        if (d2h_busy(ctx, b) && !((j.eager || j.lazy) && (L.acc[k] & 2))) {
             CK(ctx, cudaEventSynchronize(b->d2h_ev));
         }
     }
@@ -923,7 +1101,20 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     int nch = 0;
     bool in_flight = false, gpu_done = !j.gpu_launched, cpu_all = false, staged_any = false, hd_joined = false;
     int64_t cur_lo = 0, cur_hi = 0, cur_size = 0, cpu_done_wgs = 0;
-    quiesce(ctx);   // an earlier launch's abandoned chunk must have stopped before ours starts
+    // The GPU may finish before the host side can start (a launch queued behind a busy
+    // coordinator, or the pool still stopping an earlier launch's abandoned chunk -- which can
+    // take a scheduler quantum when a worker thread has been preempted): then no chunk is
+    // started at all, and the abandoned chunk is left to stop on its own.
+    auto gpu_exited = [&]() {
+        return !j.forced && j.gpu_launched &&
+               (__atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch ||
+                (j.lite && !ctx->lite_exit_word && cudaEventQuery(j.ev_k1) == cudaSuccess));
+    };
+    bool exited_before = gpu_exited();
+    while (!exited_before && !quiesce_try(ctx)) {   // the pool must be idle before ours starts
+        for (int k = 0; k < ctx->exit_poll_pauses; ++k) _mm_pause();
+        exited_before = gpu_exited();
+    }
 
     auto start_chunk = [&]() {
         int64_t size = ceil_pct(pct, nwg);
@@ -945,6 +1136,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             info.published_watermark = clo;
             return FCL_SUCCESS;
         }
+        ctx->hd_used.store(1, std::memory_order_relaxed);
         if (!hd_joined) {
             CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
             hd_joined = true;
@@ -969,17 +1161,28 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     };
 
     info.published_watermark = L.hi;
-    if (hi_cur > lo_cpu) start_chunk();
-    else cpu_all = true;
+    if (exited_before) {
+        gpu_done = true;
+        ctx->tr.add("gpu_exit_seen", j.epoch);
+    } else if (hi_cur > lo_cpu) {
+        start_chunk();
+    } else {
+        cpu_all = true;
+    }
     unsigned spin = 0;
     while (in_flight) {
-        if (!j.forced && !gpu_done && __atomic_load_n(ctx->exit_host, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch) {
+        if (!j.forced && !gpu_done && __atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch) {
             gpu_done = true;   // GPU exit (L18.s19)
             ctx->tr.add("gpu_exit_seen", j.epoch);
             break;
         }
-        if ((++spin & 0xFFFF) == 0 && j.gpu_launched) {   // a failed dispatcher never signals
+        if ((++spin & ctx->exit_query_mask) == 0 && j.gpu_launched) {   // a failed dispatcher never signals
             const cudaError_t q = cudaEventQuery(j.ev_k1);
+            if (q == cudaSuccess && j.lite && !ctx->lite_exit_word) {   // (no exit word: the event is the signal)
+                gpu_done = true;
+                ctx->tr.add("gpu_exit_seen", j.epoch);
+                break;
+            }
             if (q != cudaSuccess && q != cudaErrorNotReady) { ex.abort_flag = 1; ex.wait(); return cuda_fail(ctx, q, "dispatcher"); }
         }
         if (ex.finished()) {
@@ -1022,11 +1225,12 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     };
     // (only for exact spans: a piece of work-groups must map to its own bytes, not to a
     // conservative cover such as CORR's row-plus-column symmat footprint)
-    const bool race = gpu_done && !j.forced && (j.dev_merge || j.lite) && !j.eager && !ctx->no_race && j.exact_spans &&
+    const bool race = gpu_done && !j.forced && (j.dev_merge || j.lite) && !j.eager && !j.lazy && !ctx->no_race && j.exact_spans &&
                       hi_cur > L.lo && out_bytes(L.lo, hi_cur) >= ctx->race_min_bytes;
     if (race) {
         ctx->tr.add("race_begin", j.epoch);
         info.race = 1;
+        ctx->dh_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaStreamWaitEvent(ctx->dh, j.ev_k1, 0));
         const size_t unit_b = std::max<size_t>(1, out_bytes(L.lo, std::min<int64_t>(L.lo + j.unit, L.hi)));
         const int64_t piece = j.unit * std::max<int64_t>(1, (int64_t)(ctx->race_piece_bytes / unit_b));
@@ -1089,10 +1293,10 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         for (int q = 0; q < L.nout; ++q) {   // the buffers' return events follow the last piece
             fcl_buffer ob = L.bufs[L.out_idx[q]];
             CK(ctx, cudaEventRecord(ob->d2h_ev, ctx->dh));
-            ob->d2h_pending = true;
+            ob->d2h_pending = true; ob->d2h_on_main = false; ob->d2h_gen = ctx->finish_gen.load();
         }
         ctx->tr.add("race_end", j.epoch);
-    } else if (in_flight && j.eager && gpu_done) {
+    } else if (in_flight && (j.eager || j.lazy) && gpu_done) {
         // GPU finished first and the (pure-OUT) result is already on its way back: abandon the
         // chunk without waiting for it (L18.s19).  Its workers only write words bit-identical to
         // the returned ones; whatever could change what they read or write waits in quiesce().
@@ -1118,7 +1322,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         // the merge is already queued (or, lite, cannot be needed); only the precise return
         // of large outputs is left
         if (gpu_done) {
-            if (!j.eager && !race) {
+            if (!j.eager && !j.lazy && !race) {
                 // The host copy already holds every published chunk, and the GPU acted on some
                 // watermark >= the lowest one published, so returning the device copy (merged
                 // by the fused tail) below the host's own published watermark is complete --
@@ -1152,7 +1356,10 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         info.gpu_watermark = merge_lo;
         if (merge_lo < L.hi) {
             info.merged = 1;
-            if (wait_staged) CK(ctx, cudaStreamWaitEvent(ctx->main, j.ev_staged, 0));
+            if (wait_staged) {
+                CK(ctx, cudaStreamWaitEvent(ctx->main, j.ev_staged, 0));
+                ctx->main_fenced.store(1);
+            }
             st = enqueue_merges(ctx, j, merge_lo, L.hi);
             if (st != FCL_SUCCESS) return st;
         }
@@ -1273,13 +1480,17 @@ fcl_status run_gpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     const int64_t t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo), t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
     const bool timing = ctx->ktiming || (L.o.flags & FCL_LAUNCH_TIMING);
     if (timing) CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
-    if (gpu_launch_plain(L.a, L.g, t0, t1, ctx->main) < 0)
+    SlotReset r{};
+    r.tstamp = plain_stamp(ctx);
+    if (gpu_launch_plain(L.a, L.g, t0, t1, ctx->main, &r, pdl_mode(ctx, L)) < 0)
         return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+    if (timing) CK(ctx, cudaEventRecord(ctx->ev_t1, ctx->main));
     CK(ctx, cudaEventRecord(ctx->ev_k1, ctx->main));
     ctx->sync_have_k = timing;
     info.gpu_launches += 1;
     info.gpu_path = FCL_GPU_PATH_PLAIN;
     info.gpu_tasks = info.gpu_tasks_total = t1 - t0;
+    if (lazy_return(ctx, L, info)) return FCL_SUCCESS;
     return enqueue_d2h(ctx, L, L.lo, L.hi, info, ctx->ev_k1);
 }
 
@@ -1390,8 +1601,8 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocPortable)) != cudaSuccess) return fail(e, "pinned scratch");
     std::memset(hp, 0, 64);
     ctx->wm_host = (unsigned long long *)hp;
-    if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "exit word");
-    std::memset(hp, 0, 64);
+    if ((e = cudaHostAlloc(&hp, 8 * fcl_context_st::kSlots, cudaHostAllocMapped | cudaHostAllocPortable)) != cudaSuccess) return fail(e, "exit word");
+    std::memset(hp, 0, 8 * fcl_context_st::kSlots);
     ctx->exit_host = (unsigned long long *)hp;
     if ((e = cudaHostGetDevicePointer(&dp, hp, 0)) != cudaSuccess) return fail(e, "exit word mapping");
     ctx->exit_dptr = (unsigned long long *)dp;
@@ -1416,9 +1627,14 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->dstamp = ctx->dwm + 2;
     ctx->dmctr = ctx->dstamp + 4 * fcl_context_st::kSlots;
     ctx->dbar = (unsigned int *)(ctx->dmctr + fcl_context_st::kSlots);
-    for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_k1})
+    if (getenv("FCL_STATS") && atoi(getenv("FCL_STATS")) != 0) {
+        if ((e = cudaMalloc(&dp, 16 * fcl_context_st::kPlainStamps)) != cudaSuccess) return fail(e, "stamps");
+        cudaMemset(dp, 0, 16 * fcl_context_st::kPlainStamps);
+        ctx->dpstamp = (unsigned long long *)dp;
+    }
+    for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_t1})
         if ((e = cudaEventCreate(pe)) != cudaSuccess) return fail(e, "events");
-    for (cudaEvent_t *pe : {&ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h, &ctx->race_ev[0], &ctx->race_ev[1],
+    for (cudaEvent_t *pe : {&ctx->ev_k1, &ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h, &ctx->race_ev[0], &ctx->race_ev[1],
                             &ctx->race_ev[2], &ctx->race_ev[3]})
         if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
     // stream memory operations for publication (driver entry point; fall back to a kernel store)
@@ -1435,6 +1651,9 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_EAGER_RETURN_BYTES")) ctx->eager_return_bytes = (size_t)atoll(getenv("FCL_EAGER_RETURN_BYTES"));
     ctx->stats = getenv("FCL_STATS") && atoi(getenv("FCL_STATS")) != 0;
     ctx->tr.on = getenv("FCL_TRACE") && atoi(getenv("FCL_TRACE")) != 0;
+    ctx->pdl = !(getenv("FCL_NO_PDL") && atoi(getenv("FCL_NO_PDL")) != 0);
+    if (getenv("FCL_LITE_EXIT") && atoi(getenv("FCL_LITE_EXIT")) == 0) { ctx->lite_exit_word = false; ctx->exit_query_mask = 0x3F; }
+    if (getenv("FCL_LAZY_BYTES")) ctx->lazy_max_bytes = (size_t)atoll(getenv("FCL_LAZY_BYTES"));
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
     ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
     ctx->no_lite = getenv("FCL_NO_LITE") && atoi(getenv("FCL_NO_LITE")) != 0;
@@ -1481,17 +1700,17 @@ fcl_status fcl_release_context(fcl_context ctx) {
     ctx->ex.shutdown();
     for (auto &pe : ctx->pool) cudaFree(pe.p);
     for (Job *j : ctx->free_jobs) {
-        for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
+        for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_t1, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
             if (e) cudaEventDestroy(e);
         delete j;
     }
     if (ctx->last && ctx->last->done.load()) {
         Job *j = ctx->last;
-        for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
+        for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_t1, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
             if (e) cudaEventDestroy(e);
         delete j;
     }
-    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_k1, ctx->ev_mark, ctx->ev_hd_release, ctx->ev_gd2h, ctx->race_ev[0],
+    for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_t1, ctx->ev_k1, ctx->ev_mark, ctx->ev_hd_release, ctx->ev_gd2h, ctx->race_ev[0],
                           ctx->race_ev[1], ctx->race_ev[2], ctx->race_ev[3]})
         if (e) cudaEventDestroy(e);
     if (ctx->status_host) cudaFreeHost(ctx->status_host);
@@ -1526,7 +1745,7 @@ static fcl_status create_buffer_impl(fcl_context ctx, uint32_t flags, size_t byt
     }
     if (flags & FCL_MEM_USE_HOST_PTR) { b->host = host_ptr; b->own_host = false; }
     else {
-        if ((e = cudaHostAlloc(&b->host, bytes, cudaHostAllocPortable)) != cudaSuccess) {
+        if ((e = cudaHostAlloc(&b->host, bytes, cudaHostAllocPortable | cudaHostAllocMapped)) != cudaSuccess) {
             cudaGetLastError();
             if (b->own_dev) cudaFree(b->dev);
             delete b;
@@ -1535,6 +1754,13 @@ static fcl_status create_buffer_impl(fcl_context ctx, uint32_t flags, size_t byt
         b->own_host = true;
     }
     if ((e = cudaEventCreateWithFlags(&b->d2h_ev, cudaEventDisableTiming)) != cudaSuccess) { delete b; return cuda_fail(ctx, e, "event"); }
+    // device-visible address of the host mirror (write-through returns); caller memory that is
+    // not pinned and mapped has none
+    {
+        void *dp = nullptr;
+        if (cudaHostGetDevicePointer(&dp, b->host, 0) == cudaSuccess) b->host_dptr = dp;
+        else { cudaGetLastError(); b->host_dptr = nullptr; }
+    }
     const bool ext_host = (flags & FCL_MEM_USE_HOST_PTR) != 0, ext_dev = (flags & FCL_MEM_USE_DEVICE_PTR) != 0;
     if (host_init) {
         std::memcpy(b->host, host_init, bytes);
@@ -1572,6 +1798,10 @@ fcl_status fcl_release_buffer(fcl_buffer b) {
     cudaSetDevice(ctx->device);
     drain(ctx);
     quiesce(ctx);   // no abandoned chunk may still touch the mirror being freed
+    if (b->ret_lazy) {   // its pending return is dropped with it
+        b->ret_lazy = false;
+        ctx->lazy.erase(std::remove(ctx->lazy.begin(), ctx->lazy.end(), b), ctx->lazy.end());
+    }
     cudaStreamSynchronize(ctx->main);
     cudaStreamSynchronize(ctx->hd);
     cudaStreamSynchronize(ctx->dh);
@@ -1594,7 +1824,8 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
     if (!src || offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "write range");
     drain(ctx);
     quiesce(ctx);   // an abandoned chunk may still read or write this mirror
-    if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
+    if (b->ret_lazy && (s = flush_returns(ctx, false)) != FCL_SUCCESS) return s;
+    if (d2h_busy(ctx, b)) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
     char *h = (char *)b->host + offset;
     if (n < b->bytes) {
         s = make_valid(ctx, b, true, true, nullptr);
@@ -1617,7 +1848,8 @@ fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t 
     (void)blocking;
     drain(ctx);
     quiesce(ctx);
-    if (b->d2h_pending) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
+    if (b->ret_lazy && (s = flush_returns(ctx, false)) != FCL_SUCCESS) return s;
+    if (d2h_busy(ctx, b)) { CK(ctx, cudaEventSynchronize(b->d2h_ev)); b->d2h_pending = false; }
     if (b->host_valid) {   // location tracking (L20.s31-33): no transfer when the host is current
         const char *h = (const char *)b->host + offset;
         if (dst != h) std::memcpy(dst, h, n);
@@ -1819,6 +2051,15 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         return s;
     }
 
+    // lazy returns of buffers whose host copy this launch's host side reads (or that a
+    // host-decided merge may change) are queued first; phase B waits for them
+    for (int k = 0; k < L.a.nbuf; ++k)
+        if (L.bufs[k]->ret_lazy && ((L.acc[k] & 1) || L.o.defer_merge || L.o.forced_split >= 0)) {
+            s = flush_returns(ctx, false);
+            if (s != FCL_SUCCESS) return s;
+            break;
+        }
+
     // cooperative launch: both copies of every argument must be current
     Job *j = job_alloc(ctx);
     if (!j) return set_err(ctx, FCL_OUT_OF_RESOURCES, "job allocation");
@@ -1837,8 +2078,9 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         // A pending return copy of a buffer this launch writes still reads its device copy:
         // order the overwrite behind it on the device; the host side of the hazard is
         // resolved in phase B.
-        if (b->d2h_pending && (L.acc[k] & 2)) {
+        if (d2h_busy(ctx, b) && (L.acc[k] & 2) && !b->d2h_on_main) {
             const cudaError_t e = cudaStreamWaitEvent(ctx->main, b->d2h_ev, 0);
+            ctx->main_fenced.store(1);
             if (e != cudaSuccess) { s = cuda_fail(ctx, e, "stream wait"); break; }
         }
     }
@@ -1884,11 +2126,12 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
     CK(ctx, cudaEventRecord(ctx->ev_mark, ctx->main));
     CK(ctx, cudaStreamWaitEvent(ctx->hd, ctx->ev_mark, 0));   // pool reuse is ordered after the merge
     if (b->r_b1 > b->r_b0) {
+        ctx->dh_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaStreamWaitEvent(ctx->dh, ctx->ev_mark, 0));
         CK(ctx, cudaMemcpyAsync((char *)b->host + b->r_b0, (char *)b->dev + b->r_b0, b->r_b1 - b->r_b0,
                                 cudaMemcpyDeviceToHost, ctx->dh));
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
-        b->d2h_pending = true;
+        b->d2h_pending = true; b->d2h_on_main = false; b->d2h_gen = ctx->finish_gen.load();
     }
     b->r_b0 = b->r_b1 = 0;
     if (b->twin) pool_put(ctx, b->twin, false);
@@ -1913,18 +2156,31 @@ fcl_status fcl_finish(fcl_context ctx) {
     if (!ctx) return FCL_INVALID_CONTEXT;
     cudaSetDevice(ctx->device);
     ctx->tr.add("finish_begin", ctx->epoch);
+    // one batched copy of every lazy return, queued on main right behind the last grid (before
+    // the host sides are drained: the device copies it reads are final in stream order, and a
+    // host chunk still running only writes the same bits)
+    {
+        fcl_status f = flush_returns(ctx, true);
+        if (f != FCL_SUCCESS) return f;
+    }
     drain(ctx);
     ctx->tr.add("finish_drained", ctx->epoch);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
     // dh first: its return copies are ordered behind the kernels, so by the time it is done
     // main and hd usually are too and their syncs are cheap checks
-    CK(ctx, cudaStreamSynchronize(ctx->dh));
+    if (ctx->dh_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->dh));
+    ctx->finish_gen.fetch_add(1, std::memory_order_acq_rel);   // every queued return copy is done
     ctx->tr.add("finish_dh", ctx->epoch);
     CK(ctx, cudaStreamSynchronize(ctx->main));
+    ctx->pdl_chain.clear();   // every grid on main has completed
+    ctx->pdl_chain_grids = 0;
     ctx->tr.add("finish_main", ctx->epoch);
-    CK(ctx, cudaStreamSynchronize(ctx->hd));
+    if (ctx->hd_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->hd));
     ctx->tr.add("finish_hd", ctx->epoch);
-    quiesce(ctx);   // abandoned host chunks have stopped (usually long ago)
+    // An abandoned chunk of a free-running launch may still be stopping: it only writes words
+    // identical to the returned ones, so every host copy is already coherent.  Whatever could
+    // change what it reads or writes (buffer I/O, a conflicting or host-side launch, release)
+    // waits for it (quiesce); fcl_finish does not.
     CK(ctx, cudaGetLastError());
     ctx->tr.add("finish_end", ctx->epoch);
     if (ctx->tr.on && ctx->stats) {
@@ -1937,6 +2193,19 @@ fcl_status fcl_finish(fcl_context ctx) {
                     if (st[4 * k + q] && st[4 * k + q] != ~0ull)
                         ctx->tr.recs.push_back({(double)(st[4 * k + q] % 1000000000000ull) * 1e-6, names[q], (uint32_t)k});
             }
+        }
+        if (ctx->dpstamp && ctx->pst_n > 0) {
+            std::vector<unsigned long long> ps(2 * (size_t)ctx->pst_n);
+            if (cudaMemcpy(ps.data(), ctx->dpstamp, 16 * (size_t)ctx->pst_n, cudaMemcpyDeviceToHost) == cudaSuccess) {
+                std::lock_guard<std::mutex> lk(ctx->tr.mu);
+                for (int k = 0; k < ctx->pst_n; ++k) {
+                    ctx->tr.recs.push_back({(double)(ps[2 * k] % 1000000000000ull) * 1e-6, "gpu_plain_start_ns", (uint32_t)k});
+                    ctx->tr.recs.push_back({(double)(ps[2 * k + 1] % 1000000000000ull) * 1e-6, "gpu_plain_end_ns", (uint32_t)k});
+                }
+            }
+            cudaMemset(ctx->dpstamp, 0, 16 * (size_t)ctx->pst_n);
+            cudaDeviceSynchronize();
+            ctx->pst_n = 0;
         }
     }
     return FCL_SUCCESS;
@@ -1951,7 +2220,7 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info) {
     if (!j) {   // the last launch was a single-device one
         if (ctx->sync_have_k) {
             float ms = 0.f;
-            if (cudaEventSynchronize(ctx->ev_k1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_k0, ctx->ev_k1) == cudaSuccess)
+            if (cudaEventSynchronize(ctx->ev_t1) == cudaSuccess && cudaEventElapsedTime(&ms, ctx->ev_k0, ctx->ev_t1) == cudaSuccess)
                 ctx->sync_info.t_gpu_kernel_ms = ms;
         }
         cudaGetLastError();
@@ -1960,7 +2229,7 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info) {
     }
     if (j->have_k) {
         float ms = 0.f;
-        if (cudaEventSynchronize(j->ev_k1) == cudaSuccess && cudaEventElapsedTime(&ms, j->ev_k0, j->ev_k1) == cudaSuccess)
+        if (cudaEventSynchronize(j->ev_t1) == cudaSuccess && cudaEventElapsedTime(&ms, j->ev_k0, j->ev_t1) == cudaSuccess)
             j->info.t_gpu_kernel_ms = ms;
         // the watermark of a cooperative launch whose host side did not need it (valid while
         // no later dispatcher has run: this is the most recent launch and the queue is drained)

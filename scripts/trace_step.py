@@ -22,7 +22,15 @@ bufs = [H.create_buffers(ctx, P) for P in Ps]
 for dl, db, sl, sb in meta.get("shared", []):
     bufs[dl][db] = bufs[sl][sb]
 launches = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode) for P, b in zip(Ps, bufs)]
+flush = None
+if os.environ.get("TRACE_FLUSH"):   # bench-like: L2 flushed and the GPU idle before each step
+    import torch
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    sweep = torch.ones(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
 for rep in range(30):
+    if flush is not None:
+        flush.fill_(1.0); sweep.sum()
+        torch.cuda.synchronize()
     for L in launches:
         L()
     ctx.finish()
