@@ -342,3 +342,99 @@ def test_blocking_launch_reports_complete_info(ctx):
     ctx.finish()
     for b in bufs:
         b.release()
+
+
+def _atax_chain(ctx, n, seed):
+    P1 = W.make("atax_tmp", n, n, seed=seed, lws1d=64)
+    P2 = W.make("atax_y", n, n, seed=seed + 1, lws1d=64)
+    A, x, tmp = (ctx.buffer_from_array(b) for b in P1.bufs)
+    y = ctx.buffer_from_array(P2.bufs[2])
+    x2 = ctx.buffer_from_array((P1.bufs[1] * -0.5 + 0.25).astype(np.float32))
+    Pg = W.make("gesummv", 256, seed=seed + 2, lws1d=64)
+    g = [ctx.buffer_from_array(b) for b in Pg.bufs]
+    return (P1, P2, Pg), (A, x, tmp, y, x2), g
+
+
+def _run_sequence(ctx, P, B, g, modes, sync_each):
+    (P1, P2, Pg), (A, x, tmp, y, x2) = P, B
+    n = P1.n0
+    seq = [
+        ("atax_tmp_f32", P1, [A, x, tmp, n, n]),      # tmp = A x
+        ("gesummv_f32", Pg, H.make_args(ctx, Pg, g)),  # independent
+        ("atax_y_f32", P2, [A, tmp, y, n, n]),        # RAW on tmp
+        ("atax_tmp_f32", P1, [A, x2, tmp, n, n]),     # WAR on tmp (read just above), WAW on tmp
+        ("gesummv_f32", Pg, H.make_args(ctx, Pg, g)),  # WAW on its own outputs
+        ("atax_y_f32", P2, [A, tmp, y, n, n]),        # RAW on the new tmp, WAW on y
+    ]
+    for k, (name, Pk, args) in enumerate(seq):
+        ctx.enqueue_ndrange(name, Pk.gws, Pk.lws, args, mode=modes[k % len(modes)])
+        if sync_each:
+            ctx.finish()
+    ctx.finish()
+    return [b.read_array(np.float32) for b in (tmp, y, g[3], g[4])], \
+           [H.device_array(b, np.float32) for b in (tmp, y, g[3], g[4])]
+
+
+@pytest.mark.parametrize("modes", [("gpu",), ("coop",), ("gpu", "coop"), ("coop", "gpu", "gpu")], ids=lambda m: "-".join(m))
+def test_dependent_launch_chains_without_sync(ctx, modes):
+    """Back-to-back launches with RAW / WAR / WAW dependencies and independent ones, no finish
+    in between (programmatic dependent launch decides per grid whether to wait in-kernel, and
+    small outputs return lazily): host and device copies equal the fully synchronised run."""
+    P, B, g = _atax_chain(ctx, 320, seed=30)
+    want_h, want_d = _run_sequence(ctx, P, B, g, ("gpu",), sync_each=True)
+    for rep in range(3):
+        got_h, got_d = _run_sequence(ctx, P, B, g, modes, sync_each=False)
+        for k in range(4):
+            assert_bits(got_h[k], want_h[k], f"host output {k}, rep {rep}")
+            assert_bits(got_d[k], want_d[k], f"device output {k}, rep {rep}")
+    for b in list(B) + g:
+        b.release()
+
+
+def test_many_independent_plain_grids_then_dependent(ctx):
+    """More independent plain grids in a row than one PDL chain may hold (8), then a grid that
+    reads all their outputs' producers' inputs: every result equals the single-launch one."""
+    probs = [W.make("bicg_q", 384, 257, seed=40 + k, lws1d=64) for k in range(11)]
+    refs = [H.run(ctx, P, mode="gpu")[0][2] for P in probs]
+    bufs = [H.create_buffers(ctx, P) for P in probs]
+    for P, b in zip(probs, bufs):
+        ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode="gpu")
+    # WAW on the first launch's output, then RAW through the host (CPU-only reads nothing of it,
+    # but must see coherent host copies of everything)
+    P0 = probs[0]
+    ctx.enqueue_ndrange(H.kernel_name(P0), P0.gws, P0.lws, H.make_args(ctx, P0, bufs[0]), mode="coop")
+    for P, b, r in zip(probs, bufs, refs):
+        assert_bits(b[2].read_array(np.float32), r, f"{P.kernel} read before finish")
+    ctx.finish()
+    for P, b, r in zip(probs, bufs, refs):
+        assert_bits(H.device_array(b[2], np.float32), r, f"{P.kernel} device")
+    for bl in bufs:
+        for b in bl:
+            b.release()
+
+
+def test_lazy_return_consumers(ctx, oracle_mod):
+    """A GPU-only launch's small output returns lazily: a read before fcl_finish, a CPU-only
+    launch reading it on the host, and a cooperative launch whose host chunks read it must all
+    see the GPU's values."""
+    n = 320
+    P1 = W.make("atax_tmp", n, n, seed=50, lws1d=64)
+    P2 = W.make("atax_y", n, n, seed=51, lws1d=64)
+    A, x, tmp = (ctx.buffer_from_array(b) for b in P1.bufs)
+    y = ctx.buffer_from_array(P2.bufs[2])
+    R1 = oracle_outputs(oracle_mod, P1)[2]
+    L2 = oracle_mod.Launch("atax_y", False, n, n, list(P2.gws), list(P2.lws),
+                           [P1.bufs[0].astype(np.float64), R1.copy(), np.zeros(n)])
+    oracle_mod.run_range(L2, 0, L2.num_groups())
+    # read before finish
+    ctx.enqueue_ndrange("atax_tmp_f32", P1.gws, P1.lws, [A, x, tmp, n, n], mode="gpu")
+    assert_parity(tmp.read_array(np.float32), R1, False, "lazy tmp read before finish")
+    # host-side consumers of a lazily returned output
+    for m2, opts in [("cpu", {}), ("coop", {"forced_split": 0}), ("coop", {"host_delay_us": 0})]:
+        tmp.write_array(np.full(n, 7.0, np.float32))
+        ctx.enqueue_ndrange("atax_tmp_f32", P1.gws, P1.lws, [A, x, tmp, n, n], mode="gpu")
+        ctx.enqueue_ndrange("atax_y_f32", P2.gws, P2.lws, [A, tmp, y, n, n], mode=m2, **opts)
+        ctx.finish()
+        assert_parity(y.read_array(np.float32), L2.bufs[2], False, f"gpu -> {m2} {opts}")
+    for b in (A, x, tmp, y):
+        b.release()
