@@ -141,6 +141,11 @@ fcl_status fcl_get_kernel(fcl_context ctx, const char *name, fcl_kernel *out);
 /* Writes a '\0'-terminated signature such as "A:in x:in tmp:out n0:i n1:i"
  * into buf (at most len bytes). */
 fcl_status fcl_kernel_signature(fcl_kernel k, char *buf, size_t len);
+/* Alternate host bodies of a kernel (C26, L22.s4-11): *n (>= 1) variants; names[v] for v < *n
+ * is "cpu" (the CPU-oriented body, variant 0) or "wi" (the kernel as written for the GPU, run
+ * work-item by work-item).  All variants of a kernel produce bit-identical outputs.
+ * names may be NULL. */
+fcl_status fcl_kernel_host_variants(fcl_kernel k, int32_t *n, const char **names, int32_t max_names);
 
 #define FCL_ARG_BUFFER 0
 #define FCL_ARG_INT    1
@@ -180,6 +185,11 @@ typedef struct {
     int32_t blocking;        /* 1 = return only when the launch's host side is done (the paper's
                                 blocking calls, L22.s14); 0 (default) = OpenCL-style enqueue */
     int32_t flags;           /* FCL_LAUNCH_* bits */
+    int32_t host_variant;    /* host body variant (C26 online profiling, L22.s4-11): -1 (default) =
+                                profile -- when the kernel has alternate host bodies, the first
+                                host chunks try each on a small allocation and the fastest per
+                                work-group runs the rest (and later launches of the same kernel
+                                and shape); >= 0 = always this one (fcl_kernel_host_variants) */
 } fcl_launch_opts;
 
 /* opts.flags: record CUDA events around the GPU kernel (info.t_gpu_kernel_ms); off by default
@@ -216,6 +226,10 @@ typedef struct {
     int32_t chunk_sizes[64];     /* first chunk sizes (C11 trace) */
     int32_t gpu_path;            /* FCL_GPU_PATH_*: how the GPU side of the launch ran */
     int32_t race;                /* 1 = large output returned by the return race */
+    int32_t host_variant;        /* host body variant used after profiling (-1: the host ran nothing) */
+    int32_t n_host_variants;     /* alternate host bodies the kernel has */
+    double  profile_ms_per_wg[4];/* online-profiling time per work-group of each variant (0 = not
+                                    measured in this launch) */
 } fcl_launch_info;
 
 /* Launch `kernel` over the NDRange (work_dim in 1..3, gws[k] % lws[k] == 0,

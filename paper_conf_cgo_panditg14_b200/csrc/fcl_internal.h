@@ -42,6 +42,7 @@ struct KArgs {
     int nbuf;
     void *dev[6];
     void *host[6];
+    int host_variant;      // host body variant (C26): 0 = CPU-oriented (default), 1 = work-item order
     int64_t n0, n1;        // rows / columns of the row-major input (SYRK/SYR2K: N, M)
     float alpha, beta, eps;
     int32_t ialpha, ibeta;
@@ -153,6 +154,9 @@ const char *gpu_last_error_string();
 // storing an incomplete value (write-once).
 void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts,
                   const volatile int *abort_flag);
+// Alternate host bodies (C26): how many a kernel has and their names ("cpu", "wi").
+int host_num_variants(int kernel);
+const char *host_variant_name(int kernel, int v);
 // Work-groups per executor claim (host_exec_range) and the range executor itself.
 int64_t host_batch(const KArgs &a, const Geom &g);
 void host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *abort_flag);

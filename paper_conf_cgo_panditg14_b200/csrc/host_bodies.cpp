@@ -332,9 +332,142 @@ void wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
     }
 }
 
+// ---------------------------------------------------------------- work-item-order variants
+// Alternate host bodies (C26, L22.s4-11): the kernel as written for the GPU, run work-item by
+// work-item -- each output element computed on its own with the canonical chain, walking the
+// input in the device kernel's (coalescing) order, which strides through host memory.  They
+// stand for the unmodified OpenCL kernel a CPU runtime would execute; the bodies above are the
+// CPU-oriented versions with interchanged loops (the paper's hand-written CORR kernel, L26.s5-7).
+// Both produce bit-identical outputs: loop interchange leaves every output's chain unchanged.
+
+// col-dot: work-item j walks its column, partition by partition
+template <typename T, int MODE>
+void wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+    const int64_t lws = g.lws[0];
+    const int64_t nrows = a.n0, ncols = a.n1;
+    const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, ncols);
+    if (c0 >= c1) return;
+    int64_t lo, hi;
+    part_range(c1 - c0, part, nparts, lo, hi);
+    const T *A = (const T *)a.host[0];
+    const T *v = (MODE == COL_DOT) ? (const T *)a.host[1] : nullptr;
+    const T *mean = (MODE == COL_SQDEV) ? (const T *)a.host[1] : nullptr;
+    T *out = (T *)a.host[(MODE == COL_SUM) ? 1 : 2];
+    for (int64_t j = c0 + lo; j < c0 + hi; ++j) {
+        if (aborted(ab)) return;
+        const T mj = (MODE == COL_SQDEV) ? mean[j] : T(0);
+        T tot = 0;
+        for (int q = 0; q < kColPartitions; ++q) {
+            T acc = 0;
+            for (int64_t i = q; i < nrows; i += kColPartitions) {
+                const T x = A[i * ncols + j];
+                if (MODE == COL_DOT) acc = op_fma(x, v[i], acc);
+                else if (MODE == COL_SUM) acc = op_add(acc, x);
+                else { const T c = op_add(x, -mj); acc = op_fma(c, c, acc); }
+            }
+            tot = (q == 0) ? acc : op_add(tot, acc);
+        }
+        if (MODE == COL_DOT) out[j] = tot;
+        else if (MODE == COL_SUM) out[j] = (T)((float)tot / (float)nrows);
+        else {
+            const float s = std::sqrt((float)tot / (float)nrows);
+            out[j] = (T)((s <= a.eps) ? 1.0f : s);
+        }
+    }
+}
+
+// SYRK / SYR2K: work-item (i, j) runs its k-chain
+template <typename T, bool TWO>
+void wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+    const int64_t n = a.n0, m = a.n1;
+    Wg2D w = wg2d(g, fgid, n, n);
+    if (w.r0 >= w.r1 || w.c0 >= w.c1) return;
+    const int64_t nc = w.c1 - w.c0, nitems = (w.r1 - w.r0) * nc;
+    int64_t lo, hi;
+    part_range(nitems, part, nparts, lo, hi);
+    const T *A = (const T *)a.host[0];
+    const T *B = TWO ? (const T *)a.host[1] : nullptr;
+    T *C = (T *)a.host[TWO ? 2 : 1];
+    const T alpha = a.integer ? (T)(uint32_t)a.ialpha : (T)a.alpha;
+    const T beta = a.integer ? (T)(uint32_t)a.ibeta : (T)a.beta;
+    for (int64_t it = lo; it < hi; ++it) {
+        if ((it & 15) == 0 && aborted(ab)) return;
+        const int64_t i = w.r0 + it / nc, j = w.c0 + it % nc;
+        const T *ai = A + i * m, *aj = A + j * m;
+        const T *bi = TWO ? B + i * m : nullptr, *bj = TWO ? B + j * m : nullptr;
+        T acc = 0;
+        for (int64_t k = 0; k < m; ++k) {
+            if (TWO) {
+                acc = op_fma(ai[k], bj[k], acc);   // A[i][k] * B[j][k]
+                acc = op_fma(bi[k], aj[k], acc);   // B[i][k] * A[j][k]
+            } else {
+                acc = op_fma(ai[k], aj[k], acc);
+            }
+        }
+        C[i * n + j] = op_fma(alpha, acc, op_mul(beta, C[i * n + j]));
+    }
+}
+
+// CORR symmat: work-item j1 computes its row, each j2 > j1 down the two columns
+void wg_corr_corr_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+    const int64_t n = a.n0, m = a.n1;
+    const int64_t lws = g.lws[0];
+    const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, m);
+    if (c0 >= c1) return;
+    int64_t lo, hi;
+    part_range(c1 - c0, part, nparts, lo, hi);
+    const float *d = (const float *)a.host[0];
+    float *sym = (float *)a.host[1];
+    for (int64_t j1 = c0 + lo; j1 < c0 + hi; ++j1) {
+        sym[j1 * m + j1] = 1.0f;
+        for (int64_t j2 = j1 + 1; j2 < m; ++j2) {
+            if ((j2 & 15) == 0 && aborted(ab)) return;
+            float acc = 0.0f;
+            for (int64_t i = 0; i < n; ++i) acc = std::fmaf(d[i * m + j1], d[i * m + j2], acc);
+            sym[j1 * m + j2] = acc;
+            sym[j2 * m + j1] = acc;
+        }
+    }
+}
+
 }  // namespace
 
+int host_num_variants(int kernel) {
+    switch (kernel) {
+    case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD:
+    case K_SYRK: case K_SYR2K: case K_CORR_CORR:
+        return 2;
+    default:
+        return 1;   // the work-item order is already the CPU-friendly one
+    }
+}
+
+const char *host_variant_name(int kernel, int v) {
+    if (host_num_variants(kernel) == 1) return "wi";
+    return v == 0 ? "cpu" : "wi";
+}
+
 void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *abort_flag) {
+    if (a.host_variant == 1 && host_num_variants(a.kernel) > 1) {
+        switch (a.kernel) {
+        case K_ATAX_Y: case K_BICG_S:
+            if (a.integer) wg_coldot_wi<uint32_t, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
+            else wg_coldot_wi<float, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
+            return;
+        case K_CORR_MEAN: wg_coldot_wi<float, COL_SUM>(a, g, fgid, part, nparts, abort_flag); return;
+        case K_CORR_STD: wg_coldot_wi<float, COL_SQDEV>(a, g, fgid, part, nparts, abort_flag); return;
+        case K_SYRK:
+            if (a.integer) wg_syrk_wi<uint32_t, false>(a, g, fgid, part, nparts, abort_flag);
+            else wg_syrk_wi<float, false>(a, g, fgid, part, nparts, abort_flag);
+            return;
+        case K_SYR2K:
+            if (a.integer) wg_syrk_wi<uint32_t, true>(a, g, fgid, part, nparts, abort_flag);
+            else wg_syrk_wi<float, true>(a, g, fgid, part, nparts, abort_flag);
+            return;
+        case K_CORR_CORR: wg_corr_corr_wi(a, g, fgid, part, nparts, abort_flag); return;
+        default: break;
+        }
+    }
     switch (a.kernel) {
     case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV:
         if (a.integer) wg_rowdot<uint32_t>(a, g, fgid, part, nparts, abort_flag);

@@ -32,6 +32,8 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <array>
 #include <mutex>
 #include <string>
 #include <thread>
@@ -401,6 +403,10 @@ struct fcl_context_st {
     // 0 = off).  At that point the device copy is authoritative for every registered span.
     size_t lazy_max_bytes = 1u << 20;
     std::vector<fcl_buffer> lazy;
+    // Online profiling of alternate host bodies (C26): the winner per kernel and shape, so that
+    // only the first launch of a shape pays for trying the slower variants
+    std::mutex var_mu;
+    std::map<std::array<int64_t, 6>, int> variant_cache;
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
@@ -777,6 +783,60 @@ fcl_status flush_returns(fcl_context ctx, bool at_finish) {
     return FCL_SUCCESS;
 }
 
+// ---- online profiling of alternate host bodies (C26, L22.s4-11) ----
+// "It starts by running each kernel version for a small allocation size and measuring time
+// taken for its completion.  The best performing kernel version is picked for the remaining
+// subkernels."  The allocation is one host chunk per variant (the C11 chunk of that moment);
+// the comparison is per work-group.
+struct VariantPick {
+    int nvar = 1, var = 0, next = 0;
+    bool profiling = false;
+    double ms_per_wg[4] = {0, 0, 0, 0};
+};
+
+std::array<int64_t, 6> variant_key(const Launch &L) {
+    return {L.a.kernel, L.a.integer ? 1 : 0, L.a.n0, L.a.n1, L.g.lws[0], L.g.work_dim > 1 ? L.g.lws[1] : 1};
+}
+
+VariantPick pick_variant(fcl_context ctx, const Launch &L) {
+    VariantPick vp;
+    vp.nvar = host_num_variants(L.a.kernel);
+    if (L.o.host_variant >= 0) { vp.var = std::min(L.o.host_variant, vp.nvar - 1); return vp; }
+    if (vp.nvar == 1) return vp;
+    std::lock_guard<std::mutex> lk(ctx->var_mu);
+    auto it = ctx->variant_cache.find(variant_key(L));
+    if (it != ctx->variant_cache.end()) vp.var = it->second;
+    else vp.profiling = true;
+    return vp;
+}
+
+// Variant for the next host chunk.
+int chunk_variant(VariantPick &vp) {
+    if (vp.profiling && vp.next < vp.nvar) return vp.next++;
+    return vp.var;
+}
+
+// A chunk of `wgs` work-groups run with variant v took dt ms.
+void variant_measured(fcl_context ctx, const Launch &L, VariantPick &vp, int v, double dt, int64_t wgs) {
+    if (!vp.profiling || wgs <= 0 || v < 0 || v >= 4) return;
+    vp.ms_per_wg[v] = dt / (double)wgs;
+    for (int k = 0; k < vp.nvar; ++k)
+        if (vp.ms_per_wg[k] <= 0) return;
+    int best = 0;
+    for (int k = 1; k < vp.nvar; ++k)
+        if (vp.ms_per_wg[k] < vp.ms_per_wg[best]) best = k;
+    vp.var = best;
+    vp.profiling = false;
+    std::lock_guard<std::mutex> lk(ctx->var_mu);
+    ctx->variant_cache[variant_key(L)] = best;
+}
+
+void variant_info(const VariantPick &vp, fcl_launch_info &info) {
+    info.host_variant = vp.var;
+    info.n_host_variants = vp.nvar;
+    for (int k = 0; k < 4; ++k) info.profile_ms_per_wg[k] = vp.ms_per_wg[k];
+}
+
 // Stats mode: stamp pair for the next plain grid (read and cleared by fcl_finish).
 unsigned long long *plain_stamp(fcl_context ctx) {
     if (!ctx->dpstamp || ctx->pst_n >= fcl_context_st::kPlainStamps) return nullptr;
@@ -1099,6 +1159,8 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     int pct = std::max(1, L.o.init_chunk_pct);
     double prev_avg = -1.0, t_start = 0.0, busy = 0.0;
     int nch = 0;
+    VariantPick vp = pick_variant(ctx, L);
+    int cur_var = vp.var;
     bool in_flight = false, gpu_done = !j.gpu_launched, cpu_all = false, staged_any = false, hd_joined = false;
     int64_t cur_lo = 0, cur_hi = 0, cur_size = 0, cpu_done_wgs = 0;
     // The GPU may finish before the host side can start (a launch queued behind a busy
@@ -1128,7 +1190,9 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         if (nch < 64) info.chunk_sizes[nch] = (int32_t)size;
         ++nch;
         t_start = now_ms();
-        ex.submit(L.a, L.g, cur_lo, cur_hi, parts, nact);
+        KArgs ka = L.a;
+        ka.host_variant = cur_var = chunk_variant(vp);
+        ex.submit(ka, L.g, cur_lo, cur_hi, parts, nact);
         in_flight = true;
     };
     auto stage_chunk = [&](int64_t clo, int64_t chi) -> fcl_status {
@@ -1190,6 +1254,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             busy += dt;
             in_flight = false;
             cpu_done_wgs += cur_size;
+            variant_measured(ctx, L, vp, cur_var, dt, cur_size);
             const double avg = dt / (double)cur_size;
             if (nch == 1 || avg < prev_avg) pct += std::max(0, L.o.step_pct);   // C11
             prev_avg = avg;
@@ -1248,7 +1313,9 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             if (nch < 64) info.chunk_sizes[nch] = (int32_t)size;
             ++nch;
             t_start = now_ms();
-            ex.submit(L.a, L.g, cur_lo, cur_hi, 1, nact);
+            KArgs ka = L.a;
+            ka.host_variant = cur_var = chunk_variant(vp);
+            ex.submit(ka, L.g, cur_lo, cur_hi, 1, nact);
             in_flight = true;
         };
         for (;;) {
@@ -1314,6 +1381,8 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     }
     info.t_host_ms = busy;
     info.n_chunks = nch;
+    variant_info(vp, info);
+    if (nch == 0) info.host_variant = -1;
     info.cpu_wgs = cpu_done_wgs;
     info.gpu_watermark = L.hi;
     fcl_status st = FCL_SUCCESS;
@@ -1501,12 +1570,44 @@ fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     const int parts = (L.o.cpu_wg_split && nwg < nact) ? (int)((nact + nwg - 1) / nwg) : 1;
     const double t0 = now_ms();
     quiesce(ctx);
-    ex.submit(L.a, L.g, L.lo, L.hi, parts, nact);
-    ex.wait();
+    VariantPick vp = pick_variant(ctx, L);
+    int64_t hi = L.hi;
+    int nch = 0;
+    if (vp.profiling) {   // wake the pool first: no variant's sample pays for sleeping workers
+        ex.submit(L.a, L.g, L.lo, L.lo, 1, nact);
+        ex.wait();
+    }
+    // online profiling: one small allocation per variant, from the top, then the winner
+    while (vp.profiling && vp.next < vp.nvar && hi > L.lo) {
+        const int v = chunk_variant(vp);
+        const int64_t size = std::min<int64_t>(hi - L.lo, std::max<int64_t>(L.o.cpu_wg_split ? 1 : nact,
+                                                                           ceil_pct(std::max(1, L.o.init_chunk_pct), nwg)));
+        const int p = (L.o.cpu_wg_split && size < nact) ? (int)((nact + size - 1) / size) : 1;
+        KArgs ka = L.a;
+        ka.host_variant = v;
+        const double tc = now_ms();
+        ex.submit(ka, L.g, hi - size, hi, p, nact);
+        ex.wait();
+        variant_measured(ctx, L, vp, v, now_ms() - tc, size);
+        if (nch < 64) info.chunk_sizes[nch] = (int32_t)size;
+        ++nch;
+        hi -= size;
+    }
+    if (hi > L.lo) {
+        KArgs ka = L.a;
+        ka.host_variant = vp.var;
+        const int64_t rest = hi - L.lo;
+        const int p = (L.o.cpu_wg_split && rest < nact) ? (int)((nact + rest - 1) / rest) : 1;
+        ex.submit(ka, L.g, L.lo, hi, p, nact);
+        ex.wait();
+        if (nch < 64) info.chunk_sizes[nch] = (int32_t)rest;
+        ++nch;
+    }
+    (void)parts;
+    variant_info(vp, info);
     info.t_host_ms = now_ms() - t0;
     info.cpu_wgs = nwg;
-    info.n_chunks = 1;
-    info.chunk_sizes[0] = (int32_t)nwg;
+    info.n_chunks = nch;
     info.cpu_did_all = 1;
     info.published_watermark = L.lo;
     for (int q = 0; q < L.nout; ++q) L.bufs[L.out_idx[q]]->dev_valid = false;   // lazy H2D on next GPU use
@@ -1563,6 +1664,7 @@ fcl_status fcl_default_launch_opts(fcl_launch_opts *o) {
     o->wg_lo = 0;
     o->wg_hi = 0;
     o->blocking = 0;
+    o->host_variant = -1;
     return FCL_SUCCESS;
 }
 
@@ -1885,6 +1987,16 @@ fcl_status fcl_get_kernel(fcl_context ctx, const char *name, fcl_kernel *out) {
     return FCL_INVALID_KERNEL_NAME;
 }
 
+fcl_status fcl_kernel_host_variants(fcl_kernel k, int32_t *n, const char **names, int32_t max_names) {
+    if (!k || !k->def) return FCL_INVALID_KERNEL;
+    if (!n) return FCL_INVALID_VALUE;
+    const int kid = k->def->id;
+    *n = host_num_variants(kid);
+    if (names)
+        for (int v = 0; v < *n && v < max_names; ++v) names[v] = host_variant_name(kid, v);
+    return FCL_SUCCESS;
+}
+
 fcl_status fcl_kernel_signature(fcl_kernel k, char *buf, size_t len) {
     if (!k || !buf || len == 0) return FCL_INVALID_VALUE;
     std::string s;
@@ -1985,6 +2097,8 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
     fcl_default_launch_opts(&o);
     if (opts) o = *opts;
     if (o.mode < FCL_MODE_COOP || o.mode > FCL_MODE_CPU_ONLY) return set_err(ctx, FCL_INVALID_VALUE, "mode");
+    if (o.host_variant >= host_num_variants(a.kernel))
+        return set_err(ctx, FCL_INVALID_VALUE, "host_variant %d: %s has %d", o.host_variant, kd->name, host_num_variants(a.kernel));
     int64_t lo = o.wg_lo, hi = o.wg_hi > 0 ? o.wg_hi : g.n_wg;
     if (lo < 0 || hi > g.n_wg || lo >= hi) return set_err(ctx, FCL_INVALID_VALUE, "wg range [%lld, %lld)", (long long)lo, (long long)hi);
     const int64_t al = gpu_slice_align(a, g);

@@ -33,7 +33,8 @@ MODES = {"coop": MODE_COOP, "gpu": MODE_GPU_ONLY, "gpu_only": MODE_GPU_ONLY,
 EXPORTED = [
     "fcl_create_context", "fcl_release_context", "fcl_create_buffer", "fcl_create_buffer_ext",
     "fcl_release_buffer", "fcl_write_buffer", "fcl_read_buffer", "fcl_buffer_info",
-    "fcl_get_kernel", "fcl_kernel_signature", "fcl_default_launch_opts", "fcl_enqueue_ndrange",
+    "fcl_get_kernel", "fcl_kernel_signature", "fcl_kernel_host_variants", "fcl_default_launch_opts",
+    "fcl_enqueue_ndrange",
     "fcl_merge", "fcl_merge_raw", "fcl_finish", "fcl_get_launch_info", "fcl_slice_range",
     "fcl_status_string", "fcl_last_error", "fcl_version",
 ]
@@ -58,7 +59,7 @@ class LaunchOpts(ctypes.Structure):
                 ("defer_merge", ctypes.c_int32), ("n_host_threads", ctypes.c_int32),
                 ("host_delay_us", ctypes.c_int32), ("drop_publish", ctypes.c_int32),
                 ("wg_lo", ctypes.c_int64), ("wg_hi", ctypes.c_int64),
-                ("blocking", ctypes.c_int32), ("flags", ctypes.c_int32)]
+                ("blocking", ctypes.c_int32), ("flags", ctypes.c_int32), ("host_variant", ctypes.c_int32)]
 
 
 class LaunchInfo(ctypes.Structure):
@@ -71,11 +72,14 @@ class LaunchInfo(ctypes.Structure):
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64),
                 ("t_call_ms", ctypes.c_double), ("t_gpu_kernel_ms", ctypes.c_double),
                 ("t_merge_ms", ctypes.c_double), ("t_host_ms", ctypes.c_double),
-                ("chunk_sizes", ctypes.c_int32 * 64), ("gpu_path", ctypes.c_int32), ("race", ctypes.c_int32)]
+                ("chunk_sizes", ctypes.c_int32 * 64), ("gpu_path", ctypes.c_int32), ("race", ctypes.c_int32),
+                ("host_variant", ctypes.c_int32), ("n_host_variants", ctypes.c_int32),
+                ("profile_ms_per_wg", ctypes.c_double * 4)]
 
     def as_dict(self) -> dict:
-        d = {k: getattr(self, k) for k, _ in self._fields_ if k != "chunk_sizes"}
+        d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("chunk_sizes", "profile_ms_per_wg")}
         d["chunk_sizes"] = [int(v) for v in self.chunk_sizes[: min(64, max(0, self.n_chunks))]]
+        d["profile_ms_per_wg"] = [float(v) for v in self.profile_ms_per_wg[: max(0, self.n_host_variants)]]
         return d
 
 
@@ -103,6 +107,7 @@ def load() -> ctypes.CDLL:
                              ctypes.POINTER(ctypes.c_uint32)], i32),
         "fcl_get_kernel": ([vp, ctypes.c_char_p, ctypes.POINTER(vp)], i32),
         "fcl_kernel_signature": ([vp, ctypes.c_char_p, sz], i32),
+        "fcl_kernel_host_variants": ([vp, ctypes.POINTER(i32), ctypes.POINTER(ctypes.c_char_p), i32], i32),
         "fcl_default_launch_opts": ([ctypes.POINTER(LaunchOpts)], i32),
         "fcl_enqueue_ndrange": ([vp, vp, ctypes.c_uint32, ctypes.POINTER(sz), ctypes.POINTER(sz),
                                  ctypes.POINTER(Arg), ctypes.c_uint32, ctypes.POINTER(LaunchOpts),
@@ -208,11 +213,15 @@ class Kernel:
         _check(load().fcl_kernel_signature(self.handle, buf, 256), "fcl_kernel_signature")
         self.signature = buf.value.decode()
         self.params = [tuple(p.split(":")) for p in self.signature.split()]
+        n = ctypes.c_int32()
+        names = (ctypes.c_char_p * 4)()
+        _check(load().fcl_kernel_host_variants(self.handle, ctypes.byref(n), names, 4), "fcl_kernel_host_variants")
+        self.host_variants = [names[v].decode() for v in range(min(4, n.value))]
 
 
 def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg_split=1,
               abort_period=0, defer_merge=0, n_host_threads=0, host_delay_us=0, drop_publish=0,
-              wg_lo=0, wg_hi=0, blocking=0, timing=0) -> LaunchOpts:
+              wg_lo=0, wg_hi=0, blocking=0, timing=0, host_variant=-1) -> LaunchOpts:
     o = LaunchOpts()
     load().fcl_default_launch_opts(ctypes.byref(o))
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
@@ -223,6 +232,7 @@ def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg
     o.wg_lo, o.wg_hi = int(wg_lo), int(wg_hi)
     o.blocking = int(blocking)
     o.flags = LAUNCH_TIMING if timing else 0
+    o.host_variant = int(host_variant)
     return o
 
 

@@ -48,12 +48,33 @@ def test_default_opts(lib):
     assert lib.fcl_default_launch_opts(None) == -30
 
 
-def test_struct_layouts_match_header():
-    # offsets the C compiler uses for the public structs (x86-64 SysV)
-    assert ctypes.sizeof(fcl.ContextDesc) == 40
-    assert ctypes.sizeof(fcl.Arg) == 32
-    assert fcl.LaunchOpts.forced_split.offset == 8 and ctypes.sizeof(fcl.LaunchOpts) == 72
-    assert fcl.LaunchInfo.t_call_ms.offset == 104 and ctypes.sizeof(fcl.LaunchInfo) == 400
+def test_struct_layouts_match_header(tmp_path):
+    """Every field offset and struct size of the ctypes mirrors equals what the C compiler
+    gives for include/fcl.h (a probe program compiled with gcc prints them)."""
+    import subprocess
+    structs = {"fcl_context_desc": fcl.ContextDesc, "fcl_arg": fcl.Arg,
+               "fcl_launch_opts": fcl.LaunchOpts, "fcl_launch_info": fcl.LaunchInfo}
+    src = ['#include <stdio.h>', '#include <stddef.h>', '#include "fcl.h"', "int main(void) {"]
+    for cname, py in structs.items():
+        src.append(f'printf("{cname} sizeof %zu\\n", sizeof({cname}));')
+        for fname, _ in py._fields_:
+            src.append(f'printf("{cname} {fname} %zu\\n", offsetof({cname}, {fname}));')
+    src.append("return 0; }")
+    c = tmp_path / "probe.c"
+    c.write_text("\n".join(src))
+    exe = tmp_path / "probe"
+    inc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include")
+    subprocess.run(["gcc", "-I", inc, str(c), "-o", str(exe)], check=True)
+    out = subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split("\n")
+    got = {}
+    for line in out:
+        if line:
+            cname, field, v = line.split()
+            got[(cname, field)] = int(v)
+    for cname, py in structs.items():
+        assert got[(cname, "sizeof")] == ctypes.sizeof(py), cname
+        for fname, _ in py._fields_:
+            assert got[(cname, fname)] == getattr(py, fname).offset, (cname, fname)
 
 
 def test_kernel_table_and_signatures(lib):

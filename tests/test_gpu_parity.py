@@ -438,3 +438,53 @@ def test_lazy_return_consumers(ctx, oracle_mod):
         assert_parity(y.read_array(np.float32), L2.bufs[2], False, f"gpu -> {m2} {opts}")
     for b in (A, x, tmp, y):
         b.release()
+
+
+VARIANT_CASES = [c for c in CASES if c[0] in ("atax_y", "bicg_s", "corr_mean", "corr_std", "syrk", "syr2k", "corr_corr")]
+
+
+@pytest.mark.parametrize("case", VARIANT_CASES, ids=_ids)
+def test_host_variants_bit_identical(ctx, case):
+    """Every alternate host body (C26: "cpu" loop-interchanged, "wi" work-item order as written
+    for the GPU) gives the GPU-only result bit for bit, alone and in a cooperative split."""
+    P = _problem(case, seed=21)
+    k = ctx.kernel(H.kernel_name(P))
+    assert k.host_variants == ["cpu", "wi"]
+    ref, _ = H.run(ctx, P, mode="gpu")
+    for v in (0, 1):
+        for mode, opts in [("cpu", {}), ("coop", {"forced_split": P.num_groups // 3})]:
+            out, info = H.run(ctx, P, mode=mode, host_variant=v, **opts)
+            assert info["host_variant"] == v and info["n_host_variants"] == 2
+            for i in P.out_indices:
+                assert_bits(out[i], ref[i], f"{P.kernel} variant {v} {mode}")
+
+
+@pytest.mark.parametrize("kernel,n0,n1,lws,must_win", [("bicg_s", 2048, 2048, 64, None),
+                                                       ("corr_corr", 256, 512, 64, 0)])
+def test_online_profiling_picks_the_faster_body(kernel, n0, n1, lws, must_win):
+    """CPU-only launches with profiling on (the default): the first launch of a shape times each
+    host body on one small allocation and keeps the fastest per work-group; later launches of
+    the shape reuse the choice without profiling (L22.s4-11).  CORR's symmat is the paper's
+    case (L26.s5-7): the work-item order walks two columns per output and loses clearly."""
+    from paper_conf_cgo_panditg14_b200 import fcl
+    c = fcl.Context(0)
+    try:
+        P = W.make(kernel, n0, n1, seed=22, lws1d=lws)
+        o = P.out_indices[0]
+        ref, _ = H.run(c, P, mode="gpu")
+        out, info = H.run(c, P, mode="cpu")
+        assert info["n_host_variants"] == 2
+        t = info["profile_ms_per_wg"]
+        assert t[0] > 0 and t[1] > 0, info
+        assert info["host_variant"] == (0 if t[0] <= t[1] else 1)
+        if must_win is not None:
+            assert info["host_variant"] == must_win, f"per-work-group times {t}"
+        assert_bits(out[o], ref[o], "profiled CPU-only")
+        out, info2 = H.run(c, P, mode="cpu")
+        assert info2["host_variant"] == info["host_variant"] and info2["profile_ms_per_wg"] == [0.0, 0.0]
+        assert_bits(out[o], ref[o], "cached choice")
+        # a forced variant bypasses the profiler
+        _, info3 = H.run(c, P, mode="cpu", host_variant=1)
+        assert info3["host_variant"] == 1 and info3["profile_ms_per_wg"] == [0.0, 0.0]
+    finally:
+        c.release()
