@@ -4,6 +4,7 @@ share statistics.  One JSON line per configuration (written to stdout).
 
 Usage: python scripts/bench_configs.py [config ...]   (default: all)
 """
+import gc
 import json
 import os
 import statistics
@@ -42,8 +43,8 @@ def cfg_problems(name):
         return [W.make("syr2k", 2048, 2048, seed=0)], {}
     if name == "conv2d16384":
         return [W.make("conv2d", 16384, 16384, seed=0, out_init="zero")], {}
-    if name == "corr4096":
-        n = m = 4096
+    if name.startswith("corr"):
+        n = m = int(name[4:])
         data = W.corr_chain_inputs(n, m, seed=0)
         Ps = []
         for k in ("corr_mean", "corr_std", "corr_reduce", "corr_corr"):
@@ -101,11 +102,23 @@ def run_config(name, steps, cpu_steps, modes):
     # dominant kernel: the one with the most algorithmic work
     dom = max(range(len(Ps)), key=lambda k: algorithmic(Ps[k])[1] / (HBM * 1e9 if algorithmic(Ps[k])[0] == "hbm" else FP32_TFLOPS * 1e12))
     out = {"config": name, "launches": [H.kernel_name(P) for P in Ps], "dominant": H.kernel_name(Ps[dom])}
-    for mode in modes:
-        prepared = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, timing=(k == dom))
+    for mode_spec in modes:
+        # "mode" or "mode:vK" (host body variant K forced; default: online profiling, C26)
+        mode, _, var = mode_spec.partition(":v")
+        hv = int(var) if var else -1
+        # timed steps without CUDA timing events (they would keep consecutive grids from
+        # overlapping); the per-launch detail step below times the dominant kernel
+        # (a forced variant applies to the kernels that have it; the others run their only body)
+        hvs = [hv if hv < len(ctx.kernel(H.kernel_name(P)).host_variants) else -1 for P in Ps]
+        prepared = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, host_variant=hvs[k])
                     for k, (P, b) in enumerate(zip(Ps, bufsets))]
+        prepared_t = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, host_variant=hvs[k],
+                                  timing=(k == dom)) for k, (P, b) in enumerate(zip(Ps, bufsets))]
         nsteps = cpu_steps if mode == "cpu" else steps
         ts, kms, infos = [], [], []
+        first_ms = None
+        gc.collect()
+        gc.disable()   # no cyclic collection inside the timed steps
         for rep in range(nsteps + 2):
             for li in reset:     # in-place kernels: restore their input (outside the timed region)
                 bufsets[li][0].write_array(originals[li])
@@ -120,18 +133,21 @@ def run_config(name, steps, cpu_steps, modes):
             ctx.finish()
             e1.record(stream)
             e1.synchronize()
+            if rep == 0:
+                first_ms = e0.elapsed_time(e1)
             if rep >= 2:
                 ts.append(e0.elapsed_time(e1))
+        gc.enable()
         # one extra instrumented step for per-launch detail
         for li in reset:
             bufsets[li][0].write_array(originals[li])
         ctx.finish()
-        for k, L in enumerate(prepared):
+        for k, L in enumerate(prepared_t):
             L()
             ctx.finish()
             infos.append(ctx.launch_info())
         res = {"step_ms_mean": round(statistics.mean(ts), 4), "step_ms_median": round(statistics.median(ts), 4),
-               "steps": len(ts)}
+               "steps": len(ts), "first_step_ms": round(first_ms, 4)}
         di = infos[dom]
         if mode != "cpu" and di["t_gpu_kernel_ms"] > 0:
             bound, amt = algorithmic(Ps[dom])
@@ -146,8 +162,8 @@ def run_config(name, steps, cpu_steps, modes):
                                    "unit": "TFLOP/s", "frac": round(ach / FP32_TFLOPS, 4), "kernel_ms": round(kms, 4)}
         res["launch_info"] = [{k: i[k] for k in ("gpu_watermark", "published_watermark", "n_wg", "cpu_wgs", "n_chunks",
                                                  "merged", "cpu_did_all", "gpu_launches", "h2d_bytes", "d2h_bytes",
-                                                 "chunk_sizes")} for i in infos]
-        out[mode] = res
+                                                 "chunk_sizes", "host_variant", "profile_ms_per_wg")} for i in infos]
+        out[mode_spec] = res
     if "gpu" in out and "cpu" in out and "coop" in out:
         g, c, p = out["gpu"]["step_ms_mean"], out["cpu"]["step_ms_mean"], out["coop"]["step_ms_mean"]
         ideal = 1.0 / (1.0 / g + 1.0 / c)
@@ -164,12 +180,17 @@ def run_config(name, steps, cpu_steps, modes):
 
 
 def main():
-    names = sys.argv[1:] or ["atax256", "gesummv_bicg4096", "syrk2048", "syr2k2048", "conv2d16384", "corr4096"]
+    args = sys.argv[1:]
+    modes = ["gpu", "coop", "cpu"]
+    if args and args[0].startswith("--modes="):
+        modes = args[0].split("=", 1)[1].split(",")
+        args = args[1:]
+    names = args or ["atax256", "gesummv_bicg4096", "syrk2048", "syr2k2048", "conv2d16384", "corr4096"]
     for name in names:
         steps = 30 if name not in ("conv2d16384", "corr4096") else 6
-        cpu_steps = 3 if name in ("conv2d16384", "syrk2048", "syr2k2048") else (1 if name == "corr4096" else 10)
+        cpu_steps = 3 if name in ("conv2d16384", "syrk2048", "syr2k2048") else (1 if name in ("corr4096", "corr1024") else 10)
         t0 = time.time()
-        res = run_config(name, steps, cpu_steps, ["gpu", "coop", "cpu"])
+        res = run_config(name, steps, cpu_steps, modes)
         res["wall_s"] = round(time.time() - t0, 1)
         print(json.dumps(res), flush=True)
 

@@ -39,13 +39,24 @@ def q(ts):
 
 for T in thr:
     ctx = fcl.Context(0, n_host_threads=T, streams=(stream.cuda_stream, None, None))
-    Ps = bench.problems(0)
-    bufs = [H.create_buffers(ctx, Ps[0])]
-    b2 = H.create_buffers(ctx, Ps[1])
-    b3 = H.create_buffers(ctx, Ps[2])
-    b3[0].release()
-    b3[0] = b2[0]
-    bufs += [b2, b3]
+    cfg = os.environ.get("CFG")
+    if cfg:   # any scripts/bench_configs.py configuration
+        sys.path.insert(0, os.path.join(ROOT, "scripts"))
+        from bench_configs import cfg_problems
+        Ps, meta = cfg_problems(cfg)
+        bufs = [H.create_buffers(ctx, P) for P in Ps]
+        for dl, db, sl, sb in meta.get("shared", []):
+            if bufs[dl][db] is not bufs[sl][sb]:
+                bufs[dl][db].release()
+                bufs[dl][db] = bufs[sl][sb]
+    else:
+        Ps = bench.problems(0)
+        bufs = [H.create_buffers(ctx, Ps[0])]
+        b2 = H.create_buffers(ctx, Ps[1])
+        b3 = H.create_buffers(ctx, Ps[2])
+        b3[0].release()
+        b3[0] = b2[0]
+        bufs += [b2, b3]
     prepared = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m)
                     for P, b in zip(Ps, bufs)] for m in ("coop", "gpu")}
 
@@ -71,6 +82,8 @@ for T in thr:
             e1.record(stream)
             e1.synchronize()
             ts.append(e0.elapsed_time(e1))
+        if os.environ.get("SHOW_SLOW"):
+            print(m, "slow steps:", [(k, round(t, 3)) for k, t in enumerate(ts) if t > 3 * sorted(ts)[len(ts) // 2]], flush=True)
         gc.enable()
         res.setdefault(m, []).append(q(ts))
     print(f"threads={T}", res, flush=True)
