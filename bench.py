@@ -226,6 +226,9 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     bufs += [b2, b3]
     prepared = {m: [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=m)
                     for P, b in zip(Ps, bufs)] for m in ("coop", "gpu", "cpu")}
+    # the method without device selection: every launch runs cooperatively
+    prepared["coop_always"] = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode="coop",
+                                           select=-1) for P, b in zip(Ps, bufs)]
     # per-launch detail steps only: CUDA timing events around the dominant kernel (GESUMMV).
     # Not in the timed steps -- a timing event between two grids keeps the second from
     # starting under the first's tail (programmatic dependent launch) and costs ~3 us itself.
@@ -244,24 +247,36 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
                 infos.append(ctx.launch_info())
         ctx.finish()
 
+    def one_step(mode: str, infos=None, idle=True) -> float:
+        with torch.cuda.stream(stream):
+            flush.fill_(1.0); sweep.sum()          # L2 flush (outside the timed interval)
+        # idle GPU at e0: host-side work (the CPU-only leg, the host share of a cooperative
+        # launch, launch submission) cannot hide under the flush.  The per-launch detail
+        # steps (idle=False) instead queue behind the flush, so that the kernel-only events
+        # see device time and not the host's submission latency.
+        if idle:
+            stream.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        step(mode, infos)
+        e1.record(stream)
+        e1.synchronize()
+        return e0.elapsed_time(e1)
+
     def timed(mode: str, k: int, collect=False, idle=True):
         ts, infos = [], []
         for _ in range(k):
-            with torch.cuda.stream(stream):
-                flush.fill_(1.0); sweep.sum()          # L2 flush (outside the timed interval)
-            # idle GPU at e0: host-side work (the CPU-only leg, the host share of a cooperative
-            # launch, launch submission) cannot hide under the flush.  The per-launch detail
-            # steps (idle=False) instead queue behind the flush, so that the kernel-only events
-            # see device time and not the host's submission latency.
-            if idle:
-                stream.synchronize()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            step(mode, infos if collect else None)
-            e1.record(stream)
-            e1.synchronize()
-            ts.append(e0.elapsed_time(e1))
+            ts.append(one_step(mode, infos if collect else None, idle))
         return ts, infos
+
+    def timed_interleaved(modes, k: int):
+        # the baselines step by step next to the measured mode: slow drifts of the host (PCIe,
+        # clocks, the hypervisor) hit every mode alike
+        ts = {m: [] for m in modes}
+        for _ in range(k):
+            for m in modes:
+                ts[m].append(one_step(m))
+        return ts
 
     def max_over_ranks(x: float) -> float:
         if dist is None:
@@ -271,7 +286,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         return float(t.item())
 
     # warm-up (all modes), then the timed COOP steps
-    for m in ("gpu", "cpu", "coop"):
+    for m in ("gpu", "cpu", "coop_always", "coop"):
         for _ in range(max(1, args.warmup)):
             step(m)
     if dist is not None:
@@ -287,12 +302,15 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         torch.cuda.synchronize()
         gc.collect()
         gc.disable()   # as timeit does: no cyclic collection inside the timed region
+        c0 = ctx.counters()
         t_wall0 = time.perf_counter()
-        coop_ts, _ = timed("coop", args.steps)
+        # the timed COOP steps, each followed by a GPU-only step and a COOP step without device
+        # selection (baselines under the same conditions: sampler running, gc off)
+        tsm = timed_interleaved(("coop", "gpu", "coop_always"), args.steps)
         torch.cuda.synchronize()
         t_wall = time.perf_counter() - t_wall0
-        # the GPU-only baseline under the same conditions (sampler running, gc off), right after
-        gpu_ts, _ = timed("gpu", args.steps)
+        c1 = ctx.counters()
+        coop_ts, gpu_ts, always_ts = tsm["coop"], tsm["gpu"], tsm["coop_always"]
         gc.enable()
         if dist is not None:
             dist.barrier()
@@ -302,6 +320,12 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         while len(clk.lines) < 5 and time.perf_counter() - t_s < 3.0:
             step("coop")
     coop_ms = max_over_ranks(sum(coop_ts) / len(coop_ts))
+    always_ms = max_over_ranks(sum(always_ts) / len(always_ts))
+    # how the timed COOP launches ran (device selection); the coop_always steps
+    # add only cooperative non-probe launches, the GPU-only steps only gpu_only
+    dc = {k: c1[k] - c0[k] for k in c0}
+    selection = {"launches": 3 * args.steps, "probes_cooperative": dc["probe"], "gpu_alone": dc["sel_gpu"],
+                 "host_alone": dc["sel_cpu"], "select_period": 16}
     if os.environ.get("FCL_BENCH_DEBUG"):
         print("coop step ms:", [round(t, 3) for t in coop_ts], file=sys.stderr)
 
@@ -314,14 +338,16 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     cpu_ms = max_over_ranks(statistics.mean(cpu_ts))
     ideal_ms = 1.0 / (1.0 / gpu_ms + 1.0 / cpu_ms)
 
-    # dominant kernel: the GESUMMV dispatcher (2 N^2 floats); CUDA-event duration on main
+    # dominant kernel: GESUMMV (2 N^2 floats); CUDA-event duration on main
     ges = infos[0::3]   # launch order per step: gesummv, bicg_s, bicg_q
     k_ms = statistics.mean(i["t_gpu_kernel_ms"] for i in ges if i["t_gpu_kernel_ms"] > 0)
-    # which GPU path the cooperative GESUMMV launches took (FCL_GPU_PATH_*): a single wave
-    # without in-task polls runs as the lite plain grid, else the persistent dispatcher
+    # which GPU path the COOP GESUMMV launches took (FCL_GPU_PATH_*): the GPU alone after device
+    # selection (plain grid), the lite plain grid of a single-wave cooperative launch, or the
+    # persistent dispatcher -- the first two run the same kernel
     paths = {i.get("gpu_path", 1) for i in ges}
-    gesummv_kernel = ("plain_kernel<RowDotBody<float,2>> (GESUMMV, lite cooperative launch)" if paths == {2}
-                      else "coop_kernel<RowDotBody<float,2>> (GESUMMV dispatcher)")
+    gesummv_kernel = ("coop_kernel<RowDotBody<float,2>> (GESUMMV dispatcher)" if 1 in paths
+                      else "plain_kernel<RowDotBody<float,2>> (GESUMMV; COOP launch: lite grid or GPU alone "
+                           "by device selection)")
     peaks = measured_peaks()
     achieved = algorithmic_bytes(N)["gesummv"] / (k_ms * 1e-3) / 1e9
     launches_per_step = statistics.mean(
@@ -395,7 +421,9 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
             "config": {"workload": "gesummv_bicg4096", "n": N, "kernels": ["gesummv", "bicg_s", "bicg_q"],
                        "mode": "coop", "lws": 256, "work_groups_per_kernel": 16, "host_threads": host_threads,
                        "l2": "flushed between steps (256 MiB write + 256 MiB read sweep)", "parallelism": f"replicas{world}"},
-            "coop_ms": round(coop_ms, 4), "gpu_only_ms": round(gpu_ms, 4), "cpu_only_ms": round(cpu_ms, 4),
+            "coop_ms": round(coop_ms, 4), "coop_always_ms": round(always_ms, 4),
+            "gpu_only_ms": round(gpu_ms, 4), "cpu_only_ms": round(cpu_ms, 4),
+            "selection": selection,
             "ideal_coop_ms": round(ideal_ms, 4), "frac_of_ideal": round(ideal_ms / coop_ms, 4),
             "coop_vs_best_single": round(min(gpu_ms, cpu_ms) / coop_ms, 4),
             "wall_ms_per_step": round(t_wall * 1e3 / args.steps, 4),

@@ -190,7 +190,21 @@ typedef struct {
                                 host chunks try each on a small allocation and the fastest per
                                 work-group runs the rest (and later launches of the same kernel
                                 and shape); >= 0 = always this one (fcl_kernel_host_variants) */
+    int32_t select;          /* COOP device selection from online profiles:
+                                FCL_SELECT_DEFAULT (0) = the context's setting (on unless the
+                                environment sets FCL_SELECT=0), FCL_SELECT_ON (1), FCL_SELECT_OFF (-1:
+                                always the cooperative path).  When on, a free-running COOP launch of a
+                                kernel and shape whose last cooperative probe showed that one device
+                                cannot contribute runs on the other alone: GPU-only if the host
+                                finished no work-group before the GPU exited, CPU-only if the host
+                                covered the whole range first; every FCL_SELECT_PERIOD-th (16) launch
+                                of the shape probes cooperatively again.  Forced splits, deferred
+                                merges and fault injection are never redirected. */
 } fcl_launch_opts;
+
+#define FCL_SELECT_OFF     (-1)
+#define FCL_SELECT_DEFAULT 0
+#define FCL_SELECT_ON      1
 
 /* opts.flags: record CUDA events around the GPU kernel (info.t_gpu_kernel_ms); off by default
  * because each event costs host time on the launch path. */
@@ -230,7 +244,14 @@ typedef struct {
     int32_t n_host_variants;     /* alternate host bodies the kernel has */
     double  profile_ms_per_wg[4];/* online-profiling time per work-group of each variant (0 = not
                                     measured in this launch) */
+    int32_t selected;            /* FCL_SELECTED_*: what a COOP launch ran as (opts.select) */
+    int32_t probe;               /* 1 = this cooperative launch refreshes the selection profile */
 } fcl_launch_info;
+
+/* info.selected */
+#define FCL_SELECTED_COOP 0  /* both devices (the method) */
+#define FCL_SELECTED_GPU  1  /* GPU alone: the host could not finish a work-group before the GPU */
+#define FCL_SELECTED_CPU  2  /* host alone: it covered the whole range before the GPU exited */
 
 /* Launch `kernel` over the NDRange (work_dim in 1..3, gws[k] % lws[k] == 0,
  * prod(lws) <= 1024) with args in the kernel's signature order.
@@ -270,6 +291,19 @@ fcl_status fcl_finish(fcl_context ctx);
 /* Info of the most recent fcl_enqueue_ndrange, with event timings resolved
  * (call after fcl_finish). */
 fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info);
+
+/* Cumulative launch counters of the context since its creation (diagnostics; how COOP launches
+ * ran under device selection).  counts[FCL_COUNT_*] for k < n are written; n
+ * larger than FCL_COUNT_N writes FCL_COUNT_N entries.  Thread-compatible like every call on the
+ * context.  Errors: FCL_INVALID_CONTEXT, FCL_INVALID_VALUE (counts NULL or n < 0). */
+#define FCL_COUNT_COOP       0  /* COOP launches that ran cooperatively (probes included) */
+#define FCL_COUNT_PROBE      1  /* ... of which device-selection probes */
+#define FCL_COUNT_SEL_GPU    2  /* COOP launches run on the GPU alone by device selection */
+#define FCL_COUNT_SEL_CPU    3  /* COOP launches run on the host alone by device selection */
+#define FCL_COUNT_GPU_ONLY   4  /* GPU_ONLY-mode launches */
+#define FCL_COUNT_CPU_ONLY   5  /* CPU_ONLY-mode launches */
+#define FCL_COUNT_N          6
+fcl_status fcl_get_counters(fcl_context ctx, int64_t *counts, int32_t n);
 
 /* Multi-GPU slicing helper: a contiguous flattened-id range for
  * rank `rank` of `nranks`, balanced and aligned to the kernel's GPU task

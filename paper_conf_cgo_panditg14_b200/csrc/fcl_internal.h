@@ -126,6 +126,7 @@ struct SlotReset {
     unsigned long long *exit_word;
     unsigned int epoch;
     unsigned long long *tstamp;   // optional (stats): [block-0 start, last CTA end] %globaltimer
+    unsigned long long delay_ns;  // test hook (FCL_TEST_GPU_DELAY_US): block 0 idles this long first
 };
 // pdl: PDL_OFF = ordinary launch; PDL_NOWAIT = programmatic stream serialization, the grid may
 // start while the previous plain grid drains and does not wait for it (the runtime found no

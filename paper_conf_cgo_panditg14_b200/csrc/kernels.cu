@@ -494,6 +494,10 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
         __syncthreads();
     }
     pdl_trigger();
+    if (r.delay_ns && blockIdx.x == 0) {   // test hook: a slow GPU (tests/test_gpu_select.py)
+        const unsigned long long t0 = globaltimer();
+        while (globaltimer() - t0 < r.delay_ns) __nanosleep(1000);
+    }
     __shared__ __align__(16) typename Body::Smem smem;
     __shared__ long long s_key;
     TaskCtx tc;

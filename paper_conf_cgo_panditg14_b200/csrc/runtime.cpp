@@ -345,6 +345,9 @@ struct Job {
     fcl_launch_info info{};
     fcl_status status = FCL_SUCCESS;
     std::atomic<int> done{0};
+    bool probe = false;                  // refreshes the device-selection profile of its shape
+    bool probe_gpu_idle = false;         // the GPU had nothing queued when the probe was enqueued
+    std::array<int64_t, 8> sel_key{};
 };
 
 }  // namespace
@@ -407,14 +410,31 @@ struct fcl_context_st {
     // only the first launch of a shape pays for trying the slower variants
     std::mutex var_mu;
     std::map<std::array<int64_t, 6>, int> variant_cache;
+    // Device selection from online profiles: per kernel and shape, what the
+    // last cooperative probe showed (FCL_SELECTED_*) and how many launches the shape has had.
+    struct SelectEnt { int64_t launches = 0; int choice = FCL_SELECTED_COOP; };
+    std::mutex sel_mu;
+    std::map<std::array<int64_t, 8>, SelectEnt> sel;
+    bool select_on = true;                       // FCL_SELECT=0: off unless a launch asks for it
+    int64_t counts[FCL_COUNT_N] = {};            // fcl_get_counters (calling thread only)
+    int select_period = 16;                      // FCL_SELECT_PERIOD: every n-th launch of a shape probes
+    uint32_t pool_keep = 256;                    // FCL_POOL_KEEP: launches an unused pool buffer survives
+    size_t pool_cap = 16ull << 30;               // FCL_POOL_CAP_MB: unused buffers beyond this are freed
+    unsigned long long test_gpu_delay_ns = 0;    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
     bool memop_nobarrier_ok = true;              // cleared when the driver rejects NO_MEMORY_BARRIER
     int exit_poll_pauses = 8;                    // pause instructions between exit-word polls (FCL_EXIT_POLL_PAUSES)
-    bool lite_exit_word = true;                  // FCL_LITE_EXIT=0: lite grids store no exit word, the
-                                                 // coordinator polls their completion event instead
+    // Lite grids store no exit word by default (FCL_LITE_EXIT=1 restores it): the last-CTA
+    // arrival it needs costs ~2 us of grid tail per launch.  The coordinator learns that a lite
+    // grid finished from fcl_finish's main-stream synchronisation (main_done_epoch) or, between
+    // finishes, from its completion event polled every exit_query_mask+1 iterations.
+    bool lite_exit_word = false;
     unsigned exit_query_mask = 0xFFFF;           // event polls every mask+1 exit-word polls
+    unsigned lite_query_mask = 0x3F;             // the same for lite grids without an exit word
+    // every grid queued on main up to this epoch has completed (set by fcl_finish)
+    std::atomic<uint32_t> main_done_epoch{0};
     // Deferred quiescence: an abandoned chunk of an eagerly returned launch may
     // still be running; its launch's buffers are kept here until quiesce() has waited for it.
     std::mutex qz_mu;
@@ -501,7 +521,10 @@ void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait) {
     int best = -1;
     for (size_t k = 0; k < ctx->pool.size(); ++k) {
         const PoolEnt &e = ctx->pool[k];
-        if (!e.used && e.bytes >= bytes && (best < 0 || e.bytes < ctx->pool[(size_t)best].bytes)) best = (int)k;
+        // best fit, but never a buffer much larger than asked for (a 16 KB stage must not take
+        // the 64 MB one the next launch of the step needs)
+        const bool fits = e.bytes >= bytes && e.bytes <= std::max(2 * bytes, bytes + ((size_t)1 << 20));
+        if (!e.used && fits && (best < 0 || e.bytes < ctx->pool[(size_t)best].bytes)) best = (int)k;
     }
     if (best >= 0) {
         PoolEnt &e = ctx->pool[(size_t)best];
@@ -530,11 +553,18 @@ void pool_put(fcl_context ctx, void *p, bool hd_pending) {
         if (e.p == p) { e.used = false; e.hd_pending = e.hd_pending || hd_pending; e.last_epoch = ctx->epoch; }
 }
 
-// "At the end of each kernel execution, older unused buffers are freed" (L20.s29).
+// "At the end of each kernel execution, older unused buffers are freed" (L20.s29).  "Older" on a
+// 180 GB device: unused for pool_keep cooperative launches, or beyond pool_cap bytes in total.
+// (A short horizon made a kernel that runs cooperatively only now and then -- a device-selection
+// probe, DESIGN.md §6.6 -- pay cudaMalloc/cudaFree, and cudaFree synchronises the device.)
 void pool_trim(fcl_context ctx) {
     std::lock_guard<std::mutex> lk(ctx->pool_mu);
+    size_t total = 0;
+    for (const auto &e : ctx->pool) total += e.bytes;
     for (auto it = ctx->pool.begin(); it != ctx->pool.end();) {
-        if (!it->used && !it->hd_pending && it->last_epoch + 16 < ctx->epoch) {
+        const bool old = it->last_epoch + ctx->pool_keep < ctx->epoch || total > ctx->pool_cap;
+        if (!it->used && !it->hd_pending && old) {
+            total -= it->bytes;
             cudaFree(it->p);
             it = ctx->pool.erase(it);
         } else {
@@ -838,6 +868,43 @@ void variant_info(const VariantPick &vp, fcl_launch_info &info) {
 }
 
 // Stats mode: stamp pair for the next plain grid (read and cleared by fcl_finish).
+// ---- device selection from online profiles ----
+// A free-running cooperative launch whose kernel and shape showed, in the last cooperative
+// probe, that one device cannot contribute -- the host finished no work-group before the GPU
+// exited, or it covered the whole range before the GPU did -- runs on the other device alone.
+// Every select_period-th launch of the shape is a cooperative probe again.
+std::array<int64_t, 8> select_key(const Launch &L) {
+    return {L.a.kernel, L.a.integer ? 1 : 0, L.a.n0, L.a.n1, L.g.lws[0], L.g.work_dim > 1 ? L.g.lws[1] : 1, L.lo, L.hi};
+}
+
+bool select_eligible(fcl_context ctx, const Launch &L) {
+    const bool on = L.o.select == FCL_SELECT_ON || (L.o.select == FCL_SELECT_DEFAULT && ctx->select_on);
+    return on && ctx->select_period > 0 && L.o.mode == FCL_MODE_COOP && L.o.forced_split < 0 && !L.o.defer_merge &&
+           L.o.host_delay_us == 0 && !L.o.drop_publish && L.hi > L.lo;
+}
+
+// Returns FCL_SELECTED_* for this launch; *probe: it runs cooperatively to refresh the profile.
+int select_device(fcl_context ctx, const Launch &L, bool *probe) {
+    std::lock_guard<std::mutex> lk(ctx->sel_mu);
+    auto &e = ctx->sel[select_key(L)];
+    const int64_t n = e.launches++;
+    *probe = (n % ctx->select_period) == 0 || e.choice == FCL_SELECTED_COOP;
+    return *probe ? FCL_SELECTED_COOP : e.choice;
+}
+
+void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
+    int c = FCL_SELECTED_COOP;
+    // A lite launch (single wave, no polls) computes every work-group on the GPU: partial host
+    // work can only shorten a host-bounded return copy, never with an eager or lazy return.
+    const bool host_work_useless = j.lite && (j.eager || j.lazy);
+    // The host covering the whole range first only shows it is the faster device when the probe's
+    // grid did not have to wait for earlier GPU work (in a chain of kernels it always does).
+    if (!gpu_done) c = j.probe_gpu_idle ? FCL_SELECTED_CPU : FCL_SELECTED_COOP;
+    else if (gpu_done && (j.info.cpu_wgs == 0 || host_work_useless)) c = FCL_SELECTED_GPU;   // nothing in time
+    std::lock_guard<std::mutex> lk(ctx->sel_mu);
+    ctx->sel[j.sel_key].choice = c;
+}
+
 unsigned long long *plain_stamp(fcl_context ctx) {
     if (!ctx->dpstamp || ctx->pst_n >= fcl_context_st::kPlainStamps) return nullptr;
     return ctx->dpstamp + 2 * ctx->pst_n++;
@@ -926,7 +993,8 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     if (ctx->slot_used[j.slot]) {
         // the dispatcher that used this status slot 16 launches ago must have finished
         const uint32_t prev = j.epoch - kSlots;
-        while (__atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) < prev) {
+        while (__atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) < prev &&
+               ctx->main_done_epoch.load(std::memory_order_acquire) - prev >= 0x80000000u) {
             const cudaError_t q = cudaStreamQuery(ctx->main);
             if (q == cudaSuccess) break;
             if (q != cudaErrorNotReady) return cuda_fail(ctx, q, "slot reuse");
@@ -1085,7 +1153,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
             const int nx = (j.slot + 1) % kSlots;
             SlotReset r{ctx->dclaim + nx, ctx->stats ? ctx->dtasks + nx : nullptr, ctx->dmctr + nx, ctx->dbar + 32 * nx,
                         ctx->dbar + 32 * j.slot, ctx->lite_exit_word ? ctx->exit_dptr + j.slot : nullptr, j.epoch,
-                        plain_stamp(ctx)};
+                        plain_stamp(ctx), ctx->test_gpu_delay_ns};
             if (gpu_launch_plain(L.a, L.g, j.t0, j.t1, ctx->main, &r, pdl_mode(ctx, L)) < 0)
                 return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
         } else {
@@ -1105,7 +1173,9 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
             fcl_status xs = stream_store(ctx, ctx->exit_dptr + j.slot, (unsigned long long)j.epoch, ctx->main, false, &info);
             if (xs != FCL_SUCCESS) return xs;
         }
-        ctx->slot_used[j.slot] = true;
+        // (a lite grid without an exit word uses nothing of its slot; a later launch of the
+        // slot must not wait for a word it never stores)
+        ctx->slot_used[j.slot] = !j.lite || ctx->lite_exit_word;
         ctx->main_tail = j.ev_k1;
         info.gpu_path = j.lite ? FCL_GPU_PATH_LITE : FCL_GPU_PATH_DISPATCHER;
         j.have_k = timing;
@@ -1167,10 +1237,16 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     // coordinator, or the pool still stopping an earlier launch's abandoned chunk -- which can
     // take a scheduler quantum when a worker thread has been preempted): then no chunk is
     // started at all, and the abandoned chunk is left to stop on its own.
+    const bool event_exit = j.lite && !ctx->lite_exit_word;   // no exit word: the event (or finish) tells
+    const unsigned qmask = event_exit ? ctx->lite_query_mask : ctx->exit_query_mask;
+    auto exit_word_seen = [&]() {
+        return __atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch ||
+               ctx->main_done_epoch.load(std::memory_order_acquire) - j.epoch < 0x80000000u;
+    };
+    unsigned spin = 0;
     auto gpu_exited = [&]() {
         return !j.forced && j.gpu_launched &&
-               (__atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch ||
-                (j.lite && !ctx->lite_exit_word && cudaEventQuery(j.ev_k1) == cudaSuccess));
+               (exit_word_seen() || (event_exit && (++spin & qmask) == 0 && cudaEventQuery(j.ev_k1) == cudaSuccess));
     };
     bool exited_before = gpu_exited();
     while (!exited_before && !quiesce_try(ctx)) {   // the pool must be idle before ours starts
@@ -1233,16 +1309,15 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     } else {
         cpu_all = true;
     }
-    unsigned spin = 0;
     while (in_flight) {
-        if (!j.forced && !gpu_done && __atomic_load_n(ctx->exit_host + j.slot, __ATOMIC_ACQUIRE) >= (unsigned long long)j.epoch) {
+        if (!j.forced && !gpu_done && j.gpu_launched && exit_word_seen()) {
             gpu_done = true;   // GPU exit (L18.s19)
             ctx->tr.add("gpu_exit_seen", j.epoch);
             break;
         }
-        if ((++spin & ctx->exit_query_mask) == 0 && j.gpu_launched) {   // a failed dispatcher never signals
+        if ((++spin & qmask) == 0 && j.gpu_launched) {   // a failed dispatcher never signals
             const cudaError_t q = cudaEventQuery(j.ev_k1);
-            if (q == cudaSuccess && j.lite && !ctx->lite_exit_word) {   // (no exit word: the event is the signal)
+            if (q == cudaSuccess && event_exit) {   // (no exit word: the event is the signal)
                 gpu_done = true;
                 ctx->tr.add("gpu_exit_seen", j.epoch);
                 break;
@@ -1386,6 +1461,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     info.cpu_wgs = cpu_done_wgs;
     info.gpu_watermark = L.hi;
     fcl_status st = FCL_SUCCESS;
+    if (j.probe) select_update(ctx, j, gpu_done);
 
     if (j.dev_merge || j.lite) {
         // the merge is already queued (or, lite, cannot be needed); only the precise return
@@ -1754,7 +1830,12 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->stats = getenv("FCL_STATS") && atoi(getenv("FCL_STATS")) != 0;
     ctx->tr.on = getenv("FCL_TRACE") && atoi(getenv("FCL_TRACE")) != 0;
     ctx->pdl = !(getenv("FCL_NO_PDL") && atoi(getenv("FCL_NO_PDL")) != 0);
-    if (getenv("FCL_LITE_EXIT") && atoi(getenv("FCL_LITE_EXIT")) == 0) { ctx->lite_exit_word = false; ctx->exit_query_mask = 0x3F; }
+    if (getenv("FCL_LITE_EXIT")) ctx->lite_exit_word = atoi(getenv("FCL_LITE_EXIT")) != 0;
+    if (getenv("FCL_POOL_KEEP")) ctx->pool_keep = (uint32_t)std::max(0, atoi(getenv("FCL_POOL_KEEP")));
+    if (getenv("FCL_POOL_CAP_MB")) ctx->pool_cap = (size_t)atoll(getenv("FCL_POOL_CAP_MB")) << 20;
+    if (getenv("FCL_SELECT")) ctx->select_on = atoi(getenv("FCL_SELECT")) != 0;
+    if (getenv("FCL_TEST_GPU_DELAY_US")) ctx->test_gpu_delay_ns = 1000ull * (unsigned long long)atoll(getenv("FCL_TEST_GPU_DELAY_US"));
+    if (getenv("FCL_SELECT_PERIOD")) ctx->select_period = std::max(0, atoi(getenv("FCL_SELECT_PERIOD")));
     if (getenv("FCL_LAZY_BYTES")) ctx->lazy_max_bytes = (size_t)atoll(getenv("FCL_LAZY_BYTES"));
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
     ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
@@ -2121,6 +2202,13 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         drain(ctx);
         if (!ctx->defer_list.empty()) return set_err(ctx, FCL_INVALID_VALUE, "a deferred merge is pending (call fcl_merge)");
     }
+    int selected = FCL_SELECTED_COOP;
+    bool probe = false;
+    if (select_eligible(ctx, L)) {
+        selected = select_device(ctx, L, &probe);
+        if (selected == FCL_SELECTED_GPU) L.o.mode = FCL_MODE_GPU_ONLY;
+        else if (selected == FCL_SELECTED_CPU) L.o.mode = FCL_MODE_CPU_ONLY;
+    }
     const bool coop = L.o.mode == FCL_MODE_COOP;
     ctx->tr.add("enq_begin", ctx->epoch + 1);
     // The single-device modes and any launch that conflicts with a pending one wait for the
@@ -2128,8 +2216,11 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     // tracking resolves, L20.s1-9; here conservatively by draining).
     bool host_needed = false;
     for (int k = 0; k < L.a.nbuf; ++k) host_needed |= !L.bufs[k]->host_valid || !L.bufs[k]->dev_valid;
-    if (!coop || host_needed || L.o.blocking || conflicts_with_pending(ctx, L)) drain(ctx);
-    if (!coop || conflicts_with_quiescing(ctx, L)) quiesce(ctx);
+    // A launch redirected to the GPU alone (device selection) is ordered like a cooperative one:
+    // on main behind every pending grid, waiting only for host sides it conflicts with.
+    const bool gpu_sel = selected == FCL_SELECTED_GPU;
+    if ((!coop && !gpu_sel) || host_needed || L.o.blocking || conflicts_with_pending(ctx, L)) drain(ctx);
+    if ((!coop && !gpu_sel) || conflicts_with_quiescing(ctx, L)) quiesce(ctx);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
 
     if (!coop) {
@@ -2155,6 +2246,10 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
             }
         }
         s = (L.o.mode == FCL_MODE_GPU_ONLY) ? run_gpu_only(ctx, L, info) : run_cpu_only(ctx, L, info);
+        info.selected = selected;
+        ctx->counts[selected == FCL_SELECTED_GPU ? FCL_COUNT_SEL_GPU
+                    : selected == FCL_SELECTED_CPU ? FCL_COUNT_SEL_CPU
+                    : L.o.mode == FCL_MODE_GPU_ONLY ? FCL_COUNT_GPU_ONLY : FCL_COUNT_CPU_ONLY] += 1;
         info.t_call_ms = now_ms() - t_call;
         {
             std::lock_guard<std::mutex> lk(ctx->q_mu);
@@ -2178,7 +2273,17 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     Job *j = job_alloc(ctx);
     if (!j) return set_err(ctx, FCL_OUT_OF_RESOURCES, "job allocation");
     j->L = L;
+    j->probe = probe;
+    j->probe_gpu_idle = false;
+    ctx->counts[FCL_COUNT_COOP] += 1;
+    if (probe) ctx->counts[FCL_COUNT_PROBE] += 1;
+    if (probe) {
+        j->sel_key = select_key(L);
+        j->probe_gpu_idle = cudaStreamQuery(ctx->main) == cudaSuccess;
+    }
     fcl_launch_info &info = j->info;
+    info.selected = FCL_SELECTED_COOP;
+    info.probe = probe ? 1 : 0;
     info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
     info.gpu_watermark = info.published_watermark = L.hi;
     for (int k = 0; k < L.a.nbuf; ++k) {
@@ -2277,6 +2382,19 @@ fcl_status fcl_finish(fcl_context ctx) {
         fcl_status f = flush_returns(ctx, true);
         if (f != FCL_SUCCESS) return f;
     }
+    // Host sides of lite launches never queue work on main and end when their grid has: with
+    // only those pending, main is synchronised first and its completion handed to the
+    // coordinator (main_done_epoch), which is how they learn it without an exit word.
+    bool all_lite = true;
+    {
+        std::lock_guard<std::mutex> lk(ctx->q_mu);
+        for (Job *p : ctx->queue) all_lite = all_lite && p->lite;
+    }
+    if (all_lite) {
+        CK(ctx, cudaStreamSynchronize(ctx->main));
+        ctx->main_done_epoch.store(ctx->epoch, std::memory_order_release);
+        ctx->tr.add("finish_main_first", ctx->epoch);
+    }
     drain(ctx);
     ctx->tr.add("finish_drained", ctx->epoch);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
@@ -2285,7 +2403,10 @@ fcl_status fcl_finish(fcl_context ctx) {
     if (ctx->dh_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->dh));
     ctx->finish_gen.fetch_add(1, std::memory_order_acq_rel);   // every queued return copy is done
     ctx->tr.add("finish_dh", ctx->epoch);
-    CK(ctx, cudaStreamSynchronize(ctx->main));
+    if (!all_lite) {
+        CK(ctx, cudaStreamSynchronize(ctx->main));
+        ctx->main_done_epoch.store(ctx->epoch, std::memory_order_release);
+    }
     ctx->pdl_chain.clear();   // every grid on main has completed
     ctx->pdl_chain_grids = 0;
     ctx->tr.add("finish_main", ctx->epoch);
@@ -2322,6 +2443,13 @@ fcl_status fcl_finish(fcl_context ctx) {
             ctx->pst_n = 0;
         }
     }
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_get_counters(fcl_context ctx, int64_t *counts, int32_t n) {
+    if (!ctx) return FCL_INVALID_CONTEXT;
+    if (!counts || n < 0) return FCL_INVALID_VALUE;
+    for (int32_t k = 0; k < n && k < FCL_COUNT_N; ++k) counts[k] = ctx->counts[k];
     return FCL_SUCCESS;
 }
 

@@ -35,7 +35,7 @@ EXPORTED = [
     "fcl_release_buffer", "fcl_write_buffer", "fcl_read_buffer", "fcl_buffer_info",
     "fcl_get_kernel", "fcl_kernel_signature", "fcl_kernel_host_variants", "fcl_default_launch_opts",
     "fcl_enqueue_ndrange",
-    "fcl_merge", "fcl_merge_raw", "fcl_finish", "fcl_get_launch_info", "fcl_slice_range",
+    "fcl_merge", "fcl_merge_raw", "fcl_finish", "fcl_get_launch_info", "fcl_get_counters", "fcl_slice_range",
     "fcl_status_string", "fcl_last_error", "fcl_version",
 ]
 
@@ -59,7 +59,8 @@ class LaunchOpts(ctypes.Structure):
                 ("defer_merge", ctypes.c_int32), ("n_host_threads", ctypes.c_int32),
                 ("host_delay_us", ctypes.c_int32), ("drop_publish", ctypes.c_int32),
                 ("wg_lo", ctypes.c_int64), ("wg_hi", ctypes.c_int64),
-                ("blocking", ctypes.c_int32), ("flags", ctypes.c_int32), ("host_variant", ctypes.c_int32)]
+                ("blocking", ctypes.c_int32), ("flags", ctypes.c_int32), ("host_variant", ctypes.c_int32),
+                ("select", ctypes.c_int32)]
 
 
 class LaunchInfo(ctypes.Structure):
@@ -74,7 +75,7 @@ class LaunchInfo(ctypes.Structure):
                 ("t_merge_ms", ctypes.c_double), ("t_host_ms", ctypes.c_double),
                 ("chunk_sizes", ctypes.c_int32 * 64), ("gpu_path", ctypes.c_int32), ("race", ctypes.c_int32),
                 ("host_variant", ctypes.c_int32), ("n_host_variants", ctypes.c_int32),
-                ("profile_ms_per_wg", ctypes.c_double * 4)]
+                ("profile_ms_per_wg", ctypes.c_double * 4), ("selected", ctypes.c_int32), ("probe", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("chunk_sizes", "profile_ms_per_wg")}
@@ -116,6 +117,7 @@ def load() -> ctypes.CDLL:
         "fcl_merge_raw": ([vp, vp, vp, sz, ctypes.c_uint32, vp], i32),
         "fcl_finish": ([vp], i32),
         "fcl_get_launch_info": ([vp, ctypes.POINTER(LaunchInfo)], i32),
+        "fcl_get_counters": ([vp, ctypes.POINTER(i64), i32], i32),
         "fcl_slice_range": ([vp, ctypes.c_uint32, ctypes.POINTER(sz), ctypes.POINTER(sz), i32, i32,
                              ctypes.POINTER(i64), ctypes.POINTER(i64)], i32),
         "fcl_status_string": ([i32], ctypes.c_char_p),
@@ -221,7 +223,7 @@ class Kernel:
 
 def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg_split=1,
               abort_period=0, defer_merge=0, n_host_threads=0, host_delay_us=0, drop_publish=0,
-              wg_lo=0, wg_hi=0, blocking=0, timing=0, host_variant=-1) -> LaunchOpts:
+              wg_lo=0, wg_hi=0, blocking=0, timing=0, host_variant=-1, select=0) -> LaunchOpts:
     o = LaunchOpts()
     load().fcl_default_launch_opts(ctypes.byref(o))
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
@@ -233,6 +235,7 @@ def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg
     o.blocking = int(blocking)
     o.flags = LAUNCH_TIMING if timing else 0
     o.host_variant = int(host_variant)
+    o.select = int(select)
     return o
 
 
@@ -323,6 +326,14 @@ class Context:
         info = LaunchInfo()
         _check(load().fcl_get_launch_info(self.handle, ctypes.byref(info)), "fcl_get_launch_info", self.handle)
         return info.as_dict()
+
+    COUNTERS = ("coop", "probe", "sel_gpu", "sel_cpu", "gpu_only", "cpu_only")
+
+    def counters(self) -> dict:
+        """Cumulative launch counters (fcl_get_counters): how COOP launches ran under device selection."""
+        c = (ctypes.c_int64 * len(self.COUNTERS))()
+        _check(load().fcl_get_counters(self.handle, c, len(self.COUNTERS)), "fcl_get_counters", self.handle)
+        return {k: int(c[i]) for i, k in enumerate(self.COUNTERS)}
 
     def slice_range(self, kernel, gws, lws, rank: int, nranks: int):
         k = self.kernel(kernel) if isinstance(kernel, str) else kernel

@@ -43,7 +43,10 @@ for t, tag, e in host:
     cur.append((t, tag, e))
     if tag == "finish_end":
         steps.append(cur); cur = []
-for st in steps[-3:]:
+show = steps[-3:]
+if os.environ.get("TRACE_SLOWEST"):   # the slowest steps instead of the last ones
+    show = sorted(steps, key=lambda st: st[-1][0] - st[0][0])[-int(os.environ["TRACE_SLOWEST"]):]
+for st in show:
     t0 = st[0][0]
     print(" | ".join(f"{tag}:{e}@{(t - t0) * 1000:.1f}" for t, tag, e in st))
 gpu = sorted((float(t), tag, int(e)) for t, tag, e in recs if tag.startswith("gpu_"))

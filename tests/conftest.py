@@ -25,3 +25,9 @@ def oracle_mod():
     import oracle
     oracle.build()
     return oracle
+
+
+# Device selection from online profiles redirects repeated COOP launches of a
+# shape to one device; the parity tests exercise the cooperative path itself, so contexts
+# created by the tests default to it off (tests/test_gpu_select.py turns it on per launch).
+os.environ.setdefault("FCL_SELECT", "0")

@@ -460,7 +460,7 @@ def test_host_variants_bit_identical(ctx, case):
 
 
 @pytest.mark.parametrize("kernel,n0,n1,lws,must_win", [("bicg_s", 2048, 2048, 64, None),
-                                                       ("corr_corr", 256, 512, 64, 0)])
+                                                       ("corr_corr", 1024, 1024, 64, 0)])
 def test_online_profiling_picks_the_faster_body(kernel, n0, n1, lws, must_win):
     """CPU-only launches with profiling on (the default): the first launch of a shape times each
     host body on one small allocation and keeps the fastest per work-group; later launches of

@@ -1,0 +1,114 @@
+"""Device selection from online profiles (opts.select): a COOP launch of a shape
+whose last cooperative probe showed that one device cannot contribute runs on the other alone,
+with every FCL_SELECT_PERIOD-th launch (16) of the shape probing cooperatively again.  Whatever
+runs, the result is the single-device result bit for bit."""
+import numpy as np
+import pytest
+
+import fcl_harness as H
+import workloads as W
+from _util import assert_bits
+
+pytestmark = pytest.mark.gpu
+
+SEL_COOP, SEL_GPU, SEL_CPU = 0, 1, 2
+PATH_NONE, PATH_PLAIN = 0, 3
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    from paper_conf_cgo_panditg14_b200 import _build, fcl
+    _build.build()
+    c = fcl.Context(0)
+    yield c
+    c.release()
+
+
+def test_gpu_favoured_shape_runs_on_the_gpu_alone(ctx):
+    """SYRK 512: the GPU finishes long before the host's first 2 % chunk (21 work-groups), so the
+    probe records "host finished nothing" and the next 15 launches are GPU-only plain grids."""
+    P = W.make("syrk", 512, 512, seed=5)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    c0 = ctx.counters()
+    seen = []
+    for i in range(18):
+        out, info = H.run(ctx, P, mode="coop", select=1)
+        seen.append((info["probe"], info["selected"]))
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], f"launch {i}")
+        if info["probe"]:
+            assert info["selected"] == SEL_COOP and info["gpu_path"] in (1, 2)
+        else:
+            assert info["selected"] == SEL_GPU, seen
+            assert info["gpu_path"] == PATH_PLAIN and info["cpu_wgs"] == 0
+    assert seen[0] == (1, SEL_COOP) and seen[16] == (1, SEL_COOP), seen
+    assert all(s == (0, SEL_GPU) for s in seen[1:16]), seen
+    c1 = ctx.counters()
+    assert c1["sel_gpu"] - c0["sel_gpu"] == 16 and c1["probe"] - c0["probe"] == 2, (c0, c1)
+    assert c1["coop"] - c0["coop"] == 2 and c1["gpu_only"] - c0["gpu_only"] == 0, (c0, c1)
+
+
+def test_host_favoured_shape_runs_on_the_host_alone(ctx, monkeypatch):
+    """The host covers a small ATAX range before the GPU exits (L16.s21) in a probe started on an
+    idle GPU -- made slow here by a fault-injection sleep in front of the grid -- so the next
+    launch of the shape runs on the host alone and leaves the device copy stale (refreshed on
+    the next GPU use).  A probe whose grid waits behind earlier GPU work proves nothing: a GPU
+    busy with a long SYRK does not make the host the faster device."""
+    from paper_conf_cgo_panditg14_b200 import fcl
+    P = W.make("atax_tmp", 64, 64, seed=7, lws1d=16)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    # a GPU busy with earlier work: the probe proves nothing, the shape stays cooperative
+    big = W.make("syrk", 2048, 2048, seed=6)
+    bb = H.create_buffers(ctx, big)
+    ctx.enqueue_ndrange(H.kernel_name(big), big.gws, big.lws, H.make_args(ctx, big, bb), mode="gpu")
+    out, info = H.run(ctx, P, mode="coop", select=1)
+    assert info["probe"] == 1
+    _, info = H.run(ctx, P, mode="coop", select=1)
+    assert info["selected"] == SEL_COOP, info
+    for b in bb:
+        b.release()
+    # an idle but slow GPU (its grid idles 20 ms first): the host covers the range, the shape
+    # moves to the host
+    monkeypatch.setenv("FCL_TEST_GPU_DELAY_US", "20000")
+    c2 = fcl.Context(0)
+    try:
+        out, info = H.run(c2, P, mode="coop", select=1)
+        assert info["probe"] == 1 and info["cpu_did_all"] == 1, info
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], "probe")
+        bufs = H.create_buffers(c2, P)
+        out, info = H.run(c2, P, mode="coop", select=1, bufs=bufs)
+        assert info["selected"] == SEL_CPU and info["gpu_path"] == PATH_NONE and info["d2h_bytes"] == 0, info
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], "host alone")
+    # the stale device copy is refreshed before a GPU launch reads it
+        Q = W.make("atax_y", 64, 64, seed=7, lws1d=16)
+        Q.bufs[0] = P.bufs[0]
+        Q.bufs[1] = out[2].copy()
+        refq, _ = H.run(c2, Q, mode="cpu")
+        yb = c2.buffer_from_array(Q.bufs[2])
+        outq, _ = H.run(c2, Q, mode="gpu", bufs=[bufs[0], bufs[2], yb])
+        for k in Q.out_indices:
+            assert_bits(outq[k], refq[k], "GPU after a host-alone launch")
+        for b in bufs + [yb]:
+            b.release()
+    finally:
+        c2.release()
+
+
+def test_selection_off_always_cooperative(ctx):
+    P = W.make("syrk", 256, 256, seed=8)
+    for _ in range(4):
+        _, info = H.run(ctx, P, mode="coop", select=-1)
+        assert info["selected"] == SEL_COOP and info["probe"] == 0 and info["gpu_path"] in (1, 2)
+
+
+def test_test_hooks_are_never_redirected(ctx):
+    P = W.make("syrk", 256, 256, seed=9)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    for _ in range(3):
+        H.run(ctx, P, mode="coop", select=1)
+    out, info = H.run(ctx, P, mode="coop", select=1, forced_split=P.num_groups // 2)
+    assert info["selected"] == SEL_COOP and info["cpu_wgs"] == P.num_groups - P.num_groups // 2
+    for k in P.out_indices:
+        assert_bits(out[k], ref[k], "forced split")
