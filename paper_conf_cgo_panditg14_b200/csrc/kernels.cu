@@ -927,11 +927,12 @@ struct GemmBody {
         long long ntile;  // tiles per dimension
         long long ngx, lws0, lws1, lws;  // work-group geometry for keys
         int vec4;
+        int sym;          // SYRK: upper-triangle tiles, each also writes its mirror (KArgs::sym)
     };
     struct Smem { T s[2][2][GBK][GBM + GPAD]; };   // [stage][A|B][k'][m]
 
     __device__ static void tile_of(const Params &p, long long t, long long &bi, long long &bj) {
-        if (OP == G_CORR) {  // upper triangle, row-major over (b1 <= b2)
+        if (OP == G_CORR || (OP == G_SYRK && p.sym)) {  // upper triangle, row-major over (b1 <= b2)
             long long b1 = 0, rem = t;
             while (rem >= p.ntile - b1) { rem -= p.ntile - b1; ++b1; }
             bi = b1; bj = b1 + rem;
@@ -967,9 +968,41 @@ struct GemmBody {
         }
     }
 
-    // One k'-tile into registers: 8 elements of each operand tile per thread.
+    // 4 consecutive elements, no bounds checks (interior tiles: every index in range, vec4)
+    __device__ static void ld4(const T *q, T *r) {
+        const T4 v = ld_cached4(q);
+        r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
+    }
+    // One k'-tile into registers: 8 elements of each operand tile per thread.  IN: the tile and
+    // the k'-range are interior (no bounds checks).
+    template <bool IN>
     __device__ static void gload(const Params &p, long long i0, long long j0, long long kt, T ra[8], T rb[8]) {
         const int tid = threadIdx.x;
+        if (IN) {
+            if (OP == G_CORR) {
+                const int kk = tid >> 4, c = (tid & 15) * 8;
+                const T *row = p.A + (kt * GBK + kk) * p.ld;
+                ld4(row + i0 + c, ra); ld4(row + i0 + c + 4, ra + 4);
+                ld4(row + j0 + c, rb); ld4(row + j0 + c + 4, rb + 4);
+            } else if (OP == G_SYRK) {
+                const int row = tid >> 1;
+                const long long k = kt * GBK + (tid & 1) * 8;
+                const T *xa = p.A + (i0 + row) * p.ld + k, *xb = p.A + (j0 + row) * p.ld + k;
+                ld4(xa, ra); ld4(xa + 4, ra + 4);
+                ld4(xb, rb); ld4(xb + 4, rb + 4);
+            } else {
+                const int row = tid >> 1;
+                const long long k = kt * (GBK / 2) + (tid & 1) * 4;
+                T x[4], y[4];
+                ld4(p.A + (i0 + row) * p.ld + k, x); ld4(p.B + (i0 + row) * p.ld + k, y);
+#pragma unroll
+                for (int q = 0; q < 4; ++q) { ra[2 * q] = x[q]; ra[2 * q + 1] = y[q]; }
+                ld4(p.B + (j0 + row) * p.ld + k, x); ld4(p.A + (j0 + row) * p.ld + k, y);
+#pragma unroll
+                for (int q = 0; q < 4; ++q) { rb[2 * q] = x[q]; rb[2 * q + 1] = y[q]; }
+            }
+            return;
+        }
         if (OP == G_CORR) {
             const int kk = tid >> 4, c = (tid & 15) * 8;
             const long long k = kt * GBK + kk;
@@ -1016,21 +1049,14 @@ struct GemmBody {
         b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w; b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
     }
 
-    __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &sm) {
-        long long bi, bj;
-        tile_of(p, t, bi, bj);
-        const long long i0 = bi * GBM, j0 = bj * GBM;
+    // The k'-loop (ascending k' per output, one fma per term).  Returns true on an abort.
+    template <bool IN>
+    __device__ static bool mainloop(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][8]) {
         const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
-        T acc[8][8];
-#pragma unroll
-        for (int r = 0; r < 8; ++r)
-#pragma unroll
-            for (int c = 0; c < 8; ++c) acc[r][c] = 0;
-
         const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;   // K'
         const long long nkt = (kdim + GBK - 1) / GBK;
         T ra[8], rb[8];
-        gload(p, i0, j0, 0, ra, rb);
+        gload<IN>(p, i0, j0, 0, ra, rb);
         sstore(sm, 0, ra, rb);
         __syncthreads();
         const long long per = tc.period();
@@ -1038,7 +1064,7 @@ struct GemmBody {
             const long long kend = (nkt - kb < per) ? nkt : kb + per;
             for (long long kt = kb; kt < kend; ++kt) {
                 const int st = (int)(kt & 1);
-                if (kt + 1 < nkt) gload(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
+                if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
                 T a[2][8], b[2][8];
                 frag(sm, st, 0, tx, ty, a[0], b[0]);
 #pragma unroll
@@ -1054,7 +1080,52 @@ struct GemmBody {
             }
             if (kend < nkt && tc.check()) return true;   // abort check every abort_period k'-tiles (Fig 12)
         }
+        return false;
+    }
+
+    __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &sm) {
+        long long bi, bj;
+        tile_of(p, t, bi, bj);
+        const long long i0 = bi * GBM, j0 = bj * GBM;
+        const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+        T acc[8][8];
+#pragma unroll
+        for (int r = 0; r < 8; ++r)
+#pragma unroll
+            for (int c = 0; c < 8; ++c) acc[r][c] = 0;
+        const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;
+        const bool interior = p.vec4 && i0 + GBM <= p.n && j0 + GBM <= p.n && kdim % GBK == 0 &&
+                              (OP != G_SYR2K || p.m % 4 == 0);
+        if (interior ? mainloop<true>(p, i0, j0, tc, sm, acc) : mainloop<false>(p, i0, j0, tc, sm, acc)) return true;
         // epilogue: write-once stores
+        if (OP == G_SYRK && p.sym && bi != bj) {
+            // mirror block: C[j][i] from acc(i, j) (bit-identical to acc(j, i)); the four rows
+            // r of a thread's half are four consecutive columns of the mirror row
+#pragma unroll
+            for (int c = 0; c < 8; ++c) {
+                const long long j = j0 + ((c < 4) ? tx * 4 + c : 64 + tx * 4 + (c - 4));
+                if (j >= p.n) continue;
+                T *crow = p.C + j * p.n;
+#pragma unroll
+                for (int half = 0; half < 2; ++half) {
+                    const long long ib = i0 + half * 64 + ty * 4;
+                    if (p.vec4 && ib + 3 < p.n) {
+                        T4 cv = *reinterpret_cast<T4 *>(crow + ib);
+                        cv.x = op_fma(p.alpha, acc[half * 4 + 0][c], op_mul(p.beta, cv.x));
+                        cv.y = op_fma(p.alpha, acc[half * 4 + 1][c], op_mul(p.beta, cv.y));
+                        cv.z = op_fma(p.alpha, acc[half * 4 + 2][c], op_mul(p.beta, cv.z));
+                        cv.w = op_fma(p.alpha, acc[half * 4 + 3][c], op_mul(p.beta, cv.w));
+                        *reinterpret_cast<T4 *>(crow + ib) = cv;
+                    } else {
+#pragma unroll
+                        for (int r = 0; r < 4; ++r) {
+                            const long long i = ib + r;
+                            if (i < p.n) crow[i] = op_fma(p.alpha, acc[half * 4 + r][c], op_mul(p.beta, crow[i]));
+                        }
+                    }
+                }
+            }
+        }
 #pragma unroll
         for (int r = 0; r < 8; ++r) {
             const long long i = i0 + ((r < 4) ? ty * 4 + r : 64 + ty * 4 + (r - 4));
@@ -1227,6 +1298,7 @@ static typename GemmBody<T, OP>::Params gemm_params(const KArgs &a, const Geom &
     p.ngx = g.ng[0]; p.lws0 = g.lws[0]; p.lws1 = g.work_dim > 1 ? g.lws[1] : 1; p.lws = g.lws[0];
     p.vec4 = (p.ld % 4 == 0) && (p.n % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.C) &&
              (OP != G_SYR2K || is_aligned16(p.B));
+    p.sym = (OP == G_SYRK && a.sym) ? 1 : 0;
     return p;
 }
 
@@ -1311,7 +1383,8 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
     }
     case K_SYRK: case K_SYR2K: {
         const long long nt = (a.n0 + GBM - 1) / GBM;
-        ts.ntasks = nt * nt; ts.threads = 256; break;
+        ts.ntasks = (a.kernel == K_SYRK && a.sym) ? nt * (nt + 1) / 2 : nt * nt;
+        ts.threads = 256; break;
     }
     case K_CORR_CORR: {
         const long long nt = (a.n1 + GBM - 1) / GBM;
@@ -1336,7 +1409,13 @@ int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t) {
     }
     case K_SYRK: case K_SYR2K: {
         const long long nt = (a.n0 + GBM - 1) / GBM;
-        const long long bi = t / nt, bj = t % nt;
+        long long bi = t / nt, bj = t % nt;
+        if (a.kernel == K_SYRK && a.sym) {   // upper triangle; the key is the direct block's
+            long long rem = t;
+            bi = 0;
+            while (rem >= nt - bi) { rem -= nt - bi; ++bi; }
+            bj = bi + rem;
+        }
         return (bj * GBM) / g.lws[0] + g.ng[0] * ((bi * GBM) / g.lws[1]);
     }
     case K_CORR_CORR: {

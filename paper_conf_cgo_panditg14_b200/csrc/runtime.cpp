@@ -392,6 +392,7 @@ struct fcl_context_st {
     unsigned long long *dmctr = nullptr;         // fused-merge chunk counters, one per slot
     bool unfused = false;                        // FCL_UNFUSED_MERGE=1: merge as a separate kernel
     bool no_lite = false;                        // FCL_NO_LITE=1: always the full dispatcher
+    bool no_sym = false;                         // FCL_NO_SYM=1: SYRK runs every tile (no mirrored writes)
     bool ktiming = false;                        // CUDA events around every kernel (FCL_KTIMING=1)
     cudaEvent_t main_tail = nullptr;             // ev_k1 of the last cooperative dispatcher
     uint32_t epoch = 0;
@@ -1840,6 +1841,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
     ctx->unfused = getenv("FCL_UNFUSED_MERGE") && atoi(getenv("FCL_UNFUSED_MERGE")) != 0;
     ctx->no_lite = getenv("FCL_NO_LITE") && atoi(getenv("FCL_NO_LITE")) != 0;
+    ctx->no_sym = getenv("FCL_NO_SYM") && atoi(getenv("FCL_NO_SYM")) != 0;
     ctx->no_race = getenv("FCL_NO_RACE") && atoi(getenv("FCL_NO_RACE")) != 0;
     if (getenv("FCL_ABORT_PERIOD")) ctx->env_abort_period = atoi(getenv("FCL_ABORT_PERIOD"));
     if (getenv("FCL_EXIT_POLL_PAUSES")) ctx->exit_poll_pauses = std::max(1, atoi(getenv("FCL_EXIT_POLL_PAUSES")));
@@ -2185,6 +2187,7 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
     const int64_t al = gpu_slice_align(a, g);
     if ((lo % al) || (hi % al && hi != g.n_wg))
         return set_err(ctx, FCL_INVALID_VALUE, "wg range must be aligned to %lld work-groups (fcl_slice_range)", (long long)al);
+    a.sym = a.kernel == K_SYRK && lo == 0 && !ctx->no_sym;
     L.ctx = ctx; L.kd = kd; L.a = a; L.g = g; L.lo = lo; L.hi = hi; L.o = o;
     return FCL_SUCCESS;
 }

@@ -102,52 +102,84 @@ def run_config(name, steps, cpu_steps, modes):
     # dominant kernel: the one with the most algorithmic work
     dom = max(range(len(Ps)), key=lambda k: algorithmic(Ps[k])[1] / (HBM * 1e9 if algorithmic(Ps[k])[0] == "hbm" else FP32_TFLOPS * 1e12))
     out = {"config": name, "launches": [H.kernel_name(P) for P in Ps], "dominant": H.kernel_name(Ps[dom])}
-    for mode_spec in modes:
-        # "mode" or "mode:vK" (host body variant K forced; default: online profiling, C26)
-        mode, _, var = mode_spec.partition(":v")
+    # "mode" or "mode:vK" (host body variant K forced; default: online profiling, C26);
+    # "coop_always": COOP without device selection
+    def parse(spec):
+        mode, _, var = spec.partition(":v")
         hv = int(var) if var else -1
+        sel = 0
+        if mode == "coop_always":
+            mode, sel = "coop", -1
+        # a forced variant applies to the kernels that have it; the others run their only body
+        hvs = [hv if hv < len(ctx.kernel(H.kernel_name(P)).host_variants) else -1 for P in Ps]
+        return mode, hvs, sel
+
+    prepared, prepared_t = {}, {}
+    for spec in modes:
+        mode, hvs, sel = parse(spec)
         # timed steps without CUDA timing events (they would keep consecutive grids from
         # overlapping); the per-launch detail step below times the dominant kernel
-        # (a forced variant applies to the kernels that have it; the others run their only body)
-        hvs = [hv if hv < len(ctx.kernel(H.kernel_name(P)).host_variants) else -1 for P in Ps]
-        prepared = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, host_variant=hvs[k])
-                    for k, (P, b) in enumerate(zip(Ps, bufsets))]
-        prepared_t = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, host_variant=hvs[k],
-                                  timing=(k == dom)) for k, (P, b) in enumerate(zip(Ps, bufsets))]
-        nsteps = cpu_steps if mode == "cpu" else steps
-        ts, kms, infos = [], [], []
-        first_ms = None
-        gc.collect()
-        gc.disable()   # no cyclic collection inside the timed steps
-        for rep in range(nsteps + 2):
-            for li in reset:     # in-place kernels: restore their input (outside the timed region)
-                bufsets[li][0].write_array(originals[li])
-            ctx.finish()
-            with torch.cuda.stream(stream):
-                flush.fill_(1.0); sweep.sum()
-            stream.synchronize()   # idle GPU at e0: host work cannot hide under the flush
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            for k, L in enumerate(prepared):
-                L()
-            ctx.finish()
-            e1.record(stream)
-            e1.synchronize()
+        prepared[spec] = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode,
+                                      host_variant=hvs[k], select=sel) for k, (P, b) in enumerate(zip(Ps, bufsets))]
+        prepared_t[spec] = [ctx.prepare(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode,
+                                        host_variant=hvs[k], select=sel, timing=(k == dom))
+                            for k, (P, b) in enumerate(zip(Ps, bufsets))]
+
+    def one_step(spec):
+        for li in reset:     # in-place kernels: restore their input (outside the timed region)
+            bufsets[li][0].write_array(originals[li])
+        ctx.finish()
+        with torch.cuda.stream(stream):
+            flush.fill_(1.0); sweep.sum()
+        stream.synchronize()   # idle GPU at e0: host work cannot hide under the flush
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for L in prepared[spec]:
+            L()
+        ctx.finish()
+        e1.record(stream)
+        e1.synchronize()
+        return e0.elapsed_time(e1)
+
+    # GPU-side modes interleaved step by step (slow host/PCIe drifts hit every mode alike); the
+    # CPU-only leg separately, with fewer steps
+    ts = {spec: [] for spec in modes}
+    first = {}
+    gc.collect()
+    gc.disable()   # no cyclic collection inside the timed steps
+    fast = [m for m in modes if parse(m)[0] != "cpu"]
+    for rep in range(steps + 2):
+        for spec in fast:
+            t = one_step(spec)
             if rep == 0:
-                first_ms = e0.elapsed_time(e1)
+                first[spec] = t
             if rep >= 2:
-                ts.append(e0.elapsed_time(e1))
-        gc.enable()
+                ts[spec].append(t)
+    for spec in modes:
+        if spec in fast:
+            continue
+        for rep in range(cpu_steps + 1):
+            t = one_step(spec)
+            if rep == 0:
+                first[spec] = t
+            else:
+                ts[spec].append(t)
+    gc.enable()
+    for spec in modes:
+        mode = parse(spec)[0]
+        c0 = ctx.counters()
         # one extra instrumented step for per-launch detail
         for li in reset:
             bufsets[li][0].write_array(originals[li])
         ctx.finish()
-        for k, L in enumerate(prepared_t):
+        infos = []
+        for L in prepared_t[spec]:
             L()
             ctx.finish()
             infos.append(ctx.launch_info())
-        res = {"step_ms_mean": round(statistics.mean(ts), 4), "step_ms_median": round(statistics.median(ts), 4),
-               "steps": len(ts), "first_step_ms": round(first_ms, 4)}
+        v = ts[spec]
+        res = {"step_ms_mean": round(statistics.mean(v), 4), "step_ms_median": round(statistics.median(v), 4),
+               "steps": len(v), "first_step_ms": round(first[spec], 4)}
         di = infos[dom]
         if mode != "cpu" and di["t_gpu_kernel_ms"] > 0:
             bound, amt = algorithmic(Ps[dom])
@@ -162,13 +194,18 @@ def run_config(name, steps, cpu_steps, modes):
                                    "unit": "TFLOP/s", "frac": round(ach / FP32_TFLOPS, 4), "kernel_ms": round(kms, 4)}
         res["launch_info"] = [{k: i[k] for k in ("gpu_watermark", "published_watermark", "n_wg", "cpu_wgs", "n_chunks",
                                                  "merged", "cpu_did_all", "gpu_launches", "h2d_bytes", "d2h_bytes",
-                                                 "chunk_sizes", "host_variant", "profile_ms_per_wg")} for i in infos]
-        out[mode_spec] = res
+                                                 "chunk_sizes", "host_variant", "profile_ms_per_wg", "gpu_path",
+                                                 "selected", "probe")} for i in infos]
+        out[spec] = res
     if "gpu" in out and "cpu" in out and "coop" in out:
         g, c, p = out["gpu"]["step_ms_mean"], out["cpu"]["step_ms_mean"], out["coop"]["step_ms_mean"]
         ideal = 1.0 / (1.0 / g + 1.0 / c)
         out["summary"] = {"gpu_ms": g, "cpu_ms": c, "coop_ms": p, "ideal_ms": round(ideal, 4),
                           "coop_vs_best_single": round(min(g, c) / p, 4), "frac_of_ideal": round(ideal / p, 4)}
+        if "coop_always" in out:
+            a = out["coop_always"]["step_ms_mean"]
+            out["summary"].update({"coop_always_ms": a, "coop_always_vs_best_single": round(min(g, c) / a, 4)})
+    out["counters"] = ctx.counters()
     done = set()
     for bl in bufsets:
         for b in bl:
@@ -181,13 +218,13 @@ def run_config(name, steps, cpu_steps, modes):
 
 def main():
     args = sys.argv[1:]
-    modes = ["gpu", "coop", "cpu"]
+    modes = ["gpu", "coop", "coop_always", "cpu"]
     if args and args[0].startswith("--modes="):
         modes = args[0].split("=", 1)[1].split(",")
         args = args[1:]
     names = args or ["atax256", "gesummv_bicg4096", "syrk2048", "syr2k2048", "conv2d16384", "corr4096"]
     for name in names:
-        steps = 30 if name not in ("conv2d16384", "corr4096") else 6
+        steps = 40 if name not in ("conv2d16384", "corr4096") else 20
         cpu_steps = 3 if name in ("conv2d16384", "syrk2048", "syr2k2048") else (1 if name in ("corr4096", "corr1024") else 10)
         t0 = time.time()
         res = run_config(name, steps, cpu_steps, modes)
