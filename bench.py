@@ -62,8 +62,8 @@ class ClockSampler:
     its pipe: a reader thread competing for the GIL with the launching thread stalled
     cooperative steps by milliseconds."""
 
-    def __init__(self, index: int):
-        self.index, self.proc, self.path = index, None, None
+    def __init__(self, index: int, cores=None):
+        self.index, self.proc, self.path, self.cores = index, None, None, cores
 
     def __enter__(self):
         if os.environ.get("FCL_NO_CLOCKS"):
@@ -75,9 +75,12 @@ class ClockSampler:
         try:
             fd, self.path = tempfile.mkstemp(prefix="fcl_clocks_", suffix=".csv")
             self.out = os.fdopen(fd, "w")
+            cores = self.cores
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}", "--format=csv,noheader,nounits",
                                           "-i", str(self.index), "-lms", "100"],
-                                         stdout=self.out, stderr=subprocess.DEVNULL, text=True)
+                                         stdout=self.out, stderr=subprocess.DEVNULL, text=True,
+                                         # on the core(s) no host-executor thread spins on
+                                         preexec_fn=(lambda: os.sched_setaffinity(0, cores)) if cores else None)
         except Exception:
             self.proc = None
         return self
@@ -214,6 +217,10 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     # spinning thread stalls the launch path by milliseconds)
     host_threads = max(1, cores - 3)
     ctx = fcl.Context(local_rank, n_host_threads=host_threads, streams=(stream.cuda_stream, None, None))
+    # the launching thread on the core the runtime leaves for it; the clock sampler on the one
+    # left free (coordinator, caller and workers take the others)
+    slice_cores = H.pin_caller()
+    free_cores = set(slice_cores[2 + host_threads:]) if slice_cores else None
 
     Ps = problems(1000 * rank)
     step_bytes = sum(algorithmic_bytes(N).values())
@@ -293,7 +300,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         dist.barrier()
     torch.cuda.synchronize()
     import gc
-    with ClockSampler(local_rank) as clk:
+    with ClockSampler(local_rank, free_cores or None) as clk:
         clk.wait_started()
         for _ in range(max(1, args.warmup)):   # re-warm after the sampler's start-up
             step("coop")

@@ -14,6 +14,36 @@ from paper_conf_cgo_panditg14_b200 import fcl
 import workloads as W
 
 
+def pin_caller() -> list:
+    """Pin the calling (launching) thread to the core the runtime leaves for it.
+
+    The context pins its coordinator to the first core of the process affinity and its workers
+    from the third on (csrc/runtime.cpp, Executor::start); the second is the caller's.  Left
+    floating, the caller can be placed on a core where a worker spins and lose a scheduler
+    quantum (~1 ms) in the middle of a launch or fcl_finish.  Returns the cores left over after
+    the workers (for helper processes), possibly empty."""
+    import os
+    global _CALLER_CORES
+    if _CALLER_CORES is None:
+        _CALLER_CORES = sorted(os.sched_getaffinity(0))
+    cores = _CALLER_CORES
+    if len(cores) < 3:
+        return []
+    os.sched_setaffinity(0, {cores[1]})
+    return cores
+
+
+def unpin_caller() -> None:
+    """Restore the affinity pin_caller() narrowed (before creating another context: the runtime
+    lays its threads out over the creating thread's affinity)."""
+    import os
+    if _CALLER_CORES is not None:
+        os.sched_setaffinity(0, set(_CALLER_CORES))
+
+
+_CALLER_CORES = None
+
+
 def kernel_name(P: W.Problem) -> str:
     return f"{P.kernel}_{'i32' if P.integer else 'f32'}"
 

@@ -196,8 +196,9 @@ typedef struct {
                                 always the cooperative path).  When on, a free-running COOP launch of a
                                 kernel and shape whose last cooperative probe showed that one device
                                 cannot contribute runs on the other alone: GPU-only if the host
-                                finished no work-group before the GPU exited, CPU-only if the host
-                                covered the whole range first; every FCL_SELECT_PERIOD-th (16) launch
+                                finished less than FCL_SELECT_MIN_SHARE (10 %) of the work-groups
+                                before the GPU exited, CPU-only if the host covered the whole range
+                                first on an idle GPU; every FCL_SELECT_PERIOD-th (16) launch
                                 of the shape probes cooperatively again.  Forced splits, deferred
                                 merges and fault injection are never redirected. */
 } fcl_launch_opts;

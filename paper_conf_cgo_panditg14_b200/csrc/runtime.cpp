@@ -18,6 +18,9 @@
 //   * stager/publisher: after each chunk, its output span goes host->device on `hd` and a stream
 //     memory operation then stores {epoch, lo} -- status follows data (C13, L16.s11/s.15-18);
 //   * merge launcher (C15, Fig 9) and the device->host return of the GPU's part (C17, L16.s36-38).
+#include <execinfo.h>
+#include <csignal>
+#include <unistd.h>
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <immintrin.h>
@@ -291,6 +294,7 @@ struct fcl_buffer_st {
     bool d2h_pending;
     bool d2h_on_main;      // the pending return copy is queued on main (a lazy return): later
                            // grids on main are ordered behind it without a cross-stream wait
+    bool d2h_on_race;      // ... queued on the race stream (a later return on dh waits for it)
     bool ret_lazy;         // a lazy return of [ret_b0, ret_b1) is registered, not yet queued
     size_t ret_b0, ret_b1;
     uint64_t d2h_gen;      // ctx->finish_gen when the pending return was queued
@@ -358,6 +362,11 @@ struct fcl_context_st {
     cudaStream_t main = nullptr, hd = nullptr, dh = nullptr;
     bool own_main = false, own_hd = false, own_dh = false;
     cudaStream_t xs = nullptr;   // exit-signal memops of lite launches (never carries data)
+    // Return-race pieces (DESIGN.md §6.4 item 8) go on their own stream: on dh they would queue
+    // behind a later launch's return that waits for its (long) kernel, and stop returning while
+    // that kernel runs.  A later return of the same buffer waits for the race's d2h_ev.
+    cudaStream_t dr = nullptr;
+    std::atomic<int> dr_used{0};
     int status_location = FCL_STATUS_DEVICE;
     // One 64-bit status word per launch slot (epoch % kSlots): a dispatcher that is still
     // running after its host side returned never sees a later launch's watermark.
@@ -419,6 +428,7 @@ struct fcl_context_st {
     bool select_on = true;                       // FCL_SELECT=0: off unless a launch asks for it
     int64_t counts[FCL_COUNT_N] = {};            // fcl_get_counters (calling thread only)
     int select_period = 16;                      // FCL_SELECT_PERIOD: every n-th launch of a shape probes
+    double select_min_share = 0.10;              // FCL_SELECT_MIN_SHARE: host share a probe must reach
     uint32_t pool_keep = 256;                    // FCL_POOL_KEEP: launches an unused pool buffer survives
     size_t pool_cap = 16ull << 30;               // FCL_POOL_CAP_MB: unused buffers beyond this are freed
     unsigned long long test_gpu_delay_ns = 0;    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
@@ -666,10 +676,11 @@ fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, fcl
         out_span(L.a, L.g, L.out_idx[q], wlo, whi, &b0, &b1);
         if (b1 <= b0) continue;
         ctx->dh_used.store(1, std::memory_order_relaxed);
+        if (d2h_busy(ctx, b) && b->d2h_on_race) CK(ctx, cudaStreamWaitEvent(ctx->dh, b->d2h_ev, 0));
         CK(ctx, cudaMemcpyAsync((char *)b->host + b0, (char *)b->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
         info.d2h_bytes += (int64_t)(b1 - b0);
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
-        b->d2h_pending = true; b->d2h_on_main = false; b->d2h_gen = ctx->finish_gen.load();
+        b->d2h_pending = true; b->d2h_on_main = false; b->d2h_on_race = false; b->d2h_gen = ctx->finish_gen.load();
     }
     return FCL_SUCCESS;
 }
@@ -807,7 +818,7 @@ fcl_status flush_returns(fcl_context ctx, bool at_finish) {
         b->ret_lazy = false;
         if (!at_finish) {
             CK(ctx, cudaEventRecord(b->d2h_ev, ctx->main));
-            b->d2h_pending = true; b->d2h_on_main = true; b->d2h_gen = ctx->finish_gen.load();
+            b->d2h_pending = true; b->d2h_on_main = true; b->d2h_on_race = false; b->d2h_gen = ctx->finish_gen.load();
         }
     }
     ctx->lazy.clear();
@@ -901,7 +912,11 @@ void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
     // The host covering the whole range first only shows it is the faster device when the probe's
     // grid did not have to wait for earlier GPU work (in a chain of kernels it always does).
     if (!gpu_done) c = j.probe_gpu_idle ? FCL_SELECTED_CPU : FCL_SELECTED_COOP;
-    else if (gpu_done && (j.info.cpu_wgs == 0 || host_work_useless)) c = FCL_SELECTED_GPU;   // nothing in time
+    // The host's share must also pay for the cooperative path's fixed costs (host side, chunk
+    // bookkeeping, a piecewise return): below min_share of the range it does not (CORR 1024's
+    // reduce: 7 % of the work-groups, 0.39 vs 0.26 ms GPU-only).
+    else if (gpu_done && (host_work_useless || (double)j.info.cpu_wgs < ctx->select_min_share * (double)(j.L.hi - j.L.lo)))
+        c = FCL_SELECTED_GPU;
     std::lock_guard<std::mutex> lk(ctx->sel_mu);
     ctx->sel[j.sel_key].choice = c;
 }
@@ -1371,8 +1386,12 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     if (race) {
         ctx->tr.add("race_begin", j.epoch);
         info.race = 1;
-        ctx->dh_used.store(1, std::memory_order_relaxed);
-        CK(ctx, cudaStreamWaitEvent(ctx->dh, j.ev_k1, 0));
+        ctx->dr_used.store(1, std::memory_order_relaxed);
+        CK(ctx, cudaStreamWaitEvent(ctx->dr, j.ev_k1, 0));
+        for (int q = 0; q < L.nout; ++q) {   // behind any earlier return of the same buffers
+            fcl_buffer ob = L.bufs[L.out_idx[q]];
+            if (d2h_busy(ctx, ob) && !ob->d2h_on_main) CK(ctx, cudaStreamWaitEvent(ctx->dr, ob->d2h_ev, 0));
+        }
         const size_t unit_b = std::max<size_t>(1, out_bytes(L.lo, std::min<int64_t>(L.lo + j.unit, L.hi)));
         const int64_t piece = j.unit * std::max<int64_t>(1, (int64_t)(ctx->race_piece_bytes / unit_b));
         int64_t F = L.lo;   // end of the prefix whose return is queued
@@ -1420,10 +1439,10 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
                     size_t b0, b1;
                     out_span(L.a, L.g, L.out_idx[q], F, b, &b0, &b1);
                     if (b1 <= b0) continue;
-                    CK(ctx, cudaMemcpyAsync((char *)ob->host + b0, (char *)ob->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
+                    CK(ctx, cudaMemcpyAsync((char *)ob->host + b0, (char *)ob->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dr));
                     info.d2h_bytes += (int64_t)(b1 - b0);
                 }
-                CK(ctx, cudaEventRecord(ctx->race_ev[(qh + qn) & 3], ctx->dh));
+                CK(ctx, cudaEventRecord(ctx->race_ev[(qh + qn) & 3], ctx->dr));
                 ++qn;
                 F = b;
             } else {
@@ -1435,8 +1454,8 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         }
         for (int q = 0; q < L.nout; ++q) {   // the buffers' return events follow the last piece
             fcl_buffer ob = L.bufs[L.out_idx[q]];
-            CK(ctx, cudaEventRecord(ob->d2h_ev, ctx->dh));
-            ob->d2h_pending = true; ob->d2h_on_main = false; ob->d2h_gen = ctx->finish_gen.load();
+            CK(ctx, cudaEventRecord(ob->d2h_ev, ctx->dr));
+            ob->d2h_pending = true; ob->d2h_on_main = false; ob->d2h_on_race = true; ob->d2h_gen = ctx->finish_gen.load();
         }
         ctx->tr.add("race_end", j.epoch);
     } else if (in_flight && (j.eager || j.lazy) && gpu_done) {
@@ -1745,7 +1764,24 @@ fcl_status fcl_default_launch_opts(fcl_launch_opts *o) {
     return FCL_SUCCESS;
 }
 
+// FCL_SEGV_TRACE=1: a native backtrace on SIGSEGV/SIGBUS/SIGABRT (diagnostics on the GPU box)
+static void segv_trace(int sig) {
+    void *frames[64];
+    const int n = backtrace(frames, 64);
+    char msg[64];
+    const int len = snprintf(msg, sizeof msg, "fcl: signal %d, native backtrace:\n", sig);
+    if (len > 0) { ssize_t w = write(2, msg, (size_t)len); (void)w; }
+    backtrace_symbols_fd(frames, n, 2);
+    signal(sig, SIG_DFL);
+    raise(sig);
+}
+
 fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
+    if (getenv("FCL_SEGV_TRACE") && atoi(getenv("FCL_SEGV_TRACE")) != 0) {
+        signal(SIGSEGV, segv_trace);
+        signal(SIGBUS, segv_trace);
+        signal(SIGABRT, segv_trace);
+    }
     if (!out) return FCL_INVALID_VALUE;
     *out = nullptr;
     fcl_context_desc d{};
@@ -1775,6 +1811,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if ((e = mk(d.hd_stream, &ctx->hd, &ctx->own_hd)) != cudaSuccess) return fail(e, "hd stream");
     if ((e = mk(d.dh_stream, &ctx->dh, &ctx->own_dh)) != cudaSuccess) return fail(e, "dh stream");
     if ((e = cudaStreamCreateWithFlags(&ctx->xs, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "exit-signal stream");
+    if ((e = cudaStreamCreateWithFlags(&ctx->dr, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "race stream");
     // status words (one per launch slot), GPU-exit word, pinned copy of the wm word
     void *hp = nullptr, *dp = nullptr;
     if ((e = cudaHostAlloc(&hp, 64, cudaHostAllocPortable)) != cudaSuccess) return fail(e, "pinned scratch");
@@ -1836,6 +1873,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_POOL_CAP_MB")) ctx->pool_cap = (size_t)atoll(getenv("FCL_POOL_CAP_MB")) << 20;
     if (getenv("FCL_SELECT")) ctx->select_on = atoi(getenv("FCL_SELECT")) != 0;
     if (getenv("FCL_TEST_GPU_DELAY_US")) ctx->test_gpu_delay_ns = 1000ull * (unsigned long long)atoll(getenv("FCL_TEST_GPU_DELAY_US"));
+    if (getenv("FCL_SELECT_MIN_SHARE")) ctx->select_min_share = atof(getenv("FCL_SELECT_MIN_SHARE"));
     if (getenv("FCL_SELECT_PERIOD")) ctx->select_period = std::max(0, atoi(getenv("FCL_SELECT_PERIOD")));
     if (getenv("FCL_LAZY_BYTES")) ctx->lazy_max_bytes = (size_t)atoll(getenv("FCL_LAZY_BYTES"));
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
@@ -1907,6 +1945,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
     if (ctx->own_dh) cudaStreamDestroy(ctx->dh);
     if (ctx->xs) cudaStreamDestroy(ctx->xs);
+    if (ctx->dr) cudaStreamDestroy(ctx->dr);
     delete ctx;
     return FCL_SUCCESS;
 }
@@ -1990,6 +2029,7 @@ fcl_status fcl_release_buffer(fcl_buffer b) {
     cudaStreamSynchronize(ctx->main);
     cudaStreamSynchronize(ctx->hd);
     cudaStreamSynchronize(ctx->dh);
+    cudaStreamSynchronize(ctx->dr);
     if (b->merge_pending) {
         if (b->twin) pool_put(ctx, b->twin, false);
         if (b->stage) pool_put(ctx, b->stage, false);
@@ -2350,10 +2390,11 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
     if (b->r_b1 > b->r_b0) {
         ctx->dh_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaStreamWaitEvent(ctx->dh, ctx->ev_mark, 0));
+        if (d2h_busy(ctx, b) && b->d2h_on_race) CK(ctx, cudaStreamWaitEvent(ctx->dh, b->d2h_ev, 0));
         CK(ctx, cudaMemcpyAsync((char *)b->host + b->r_b0, (char *)b->dev + b->r_b0, b->r_b1 - b->r_b0,
                                 cudaMemcpyDeviceToHost, ctx->dh));
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
-        b->d2h_pending = true; b->d2h_on_main = false; b->d2h_gen = ctx->finish_gen.load();
+        b->d2h_pending = true; b->d2h_on_main = false; b->d2h_on_race = false; b->d2h_gen = ctx->finish_gen.load();
     }
     b->r_b0 = b->r_b1 = 0;
     if (b->twin) pool_put(ctx, b->twin, false);
@@ -2404,6 +2445,7 @@ fcl_status fcl_finish(fcl_context ctx) {
     // dh first: its return copies are ordered behind the kernels, so by the time it is done
     // main and hd usually are too and their syncs are cheap checks
     if (ctx->dh_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->dh));
+    if (ctx->dr_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->dr));
     ctx->finish_gen.fetch_add(1, std::memory_order_acq_rel);   // every queued return copy is done
     ctx->tr.add("finish_dh", ctx->epoch);
     if (!all_lite) {

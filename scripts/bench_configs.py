@@ -87,7 +87,9 @@ def algorithmic(P):
 def run_config(name, steps, cpu_steps, modes):
     Ps, meta = cfg_problems(name)
     stream = torch.cuda.Stream()
+    H.unpin_caller()   # the runtime lays its threads out over the creating thread's affinity
     ctx = fcl.Context(0, streams=(stream.cuda_stream, None, None))
+    H.pin_caller()
     bufsets = [H.create_buffers(ctx, P) for P in Ps]
     for (dl, db, sl, sb) in meta.get("shared", []):
         if bufsets[dl][db] is not bufsets[sl][sb]:

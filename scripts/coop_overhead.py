@@ -27,6 +27,7 @@ def main():
     Ps, meta = cfg_problems(name)
     stream = torch.cuda.Stream()
     ctx = fcl.Context(0, n_host_threads=nthr, streams=(stream.cuda_stream, None, None))
+    H.pin_caller()
     bufs = [H.create_buffers(ctx, P) for P in Ps]
     for dl, db, sl, sb in meta.get("shared", []):
         bufs[dl][db] = bufs[sl][sb]

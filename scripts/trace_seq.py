@@ -18,6 +18,7 @@ seq = (sys.argv[1] if len(sys.argv) > 1 else "gpu,coop,coop_always").split(",")
 which = sys.argv[2] if len(sys.argv) > 2 else "gesummv_bicg4096"
 stream = torch.cuda.Stream()
 ctx = fcl.Context(0, n_host_threads=13, streams=(stream.cuda_stream, None, None))
+H.pin_caller()
 Ps, meta = cfg_problems(which)
 bufs = [H.create_buffers(ctx, P) for P in Ps]
 for dl, db, sl, sb in meta.get("shared", []):
