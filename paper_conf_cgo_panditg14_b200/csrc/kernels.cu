@@ -909,13 +909,20 @@ struct Conv2DBody {
 enum { G_SYRK = 0, G_SYR2K = 1, G_CORR = 2 };
 constexpr int GBM = 128, GBK = 16, GPAD = 4;
 
-template <typename T, int OP>
+// TN: outputs per thread along the tile's columns.  TN = 8: 256 threads, 8 x 8 outputs each,
+// two CTAs per SM.  TN = 4: 512 threads, 8 x 4 each, one CTA per SM -- for SYRK's upper-triangle
+// grid (136 tiles at N = 2048, one per SM), where 16 warps hide the k'-tile loads that 8 cannot.
+template <typename T, int OP, int TN = 8>
 struct GemmBody {
-    static constexpr int kThreads = 256;
+    static_assert(TN == 8 || (TN == 4 && OP == G_SYRK), "TN = 4 is the SYRK upper-triangle variant");
+    static constexpr int kThreads = TN == 8 ? 256 : 512;
 #ifndef FCL_GEMM_MINB
 #define FCL_GEMM_MINB 2
 #endif
-    static constexpr int kMinBlocks = FCL_GEMM_MINB;
+    static constexpr int kMinBlocks = TN == 8 ? FCL_GEMM_MINB : 1;
+    static constexpr int TXN = GBM / TN;                 // threads along the columns
+    static constexpr int NB = TN / 4;                    // float4 column groups per thread
+    static constexpr int LD = GBM * GBK / kThreads;      // elements of each operand a thread loads per k'-tile
     static constexpr bool kLateClaim = true;   // tasks of ~0.1-1 ms: an exposed claim costs nothing
     typedef typename V4<T>::type T4;
     struct Params {
@@ -976,7 +983,7 @@ struct GemmBody {
     // One k'-tile into registers: 8 elements of each operand tile per thread.  IN: the tile and
     // the k'-range are interior (no bounds checks).
     template <bool IN>
-    __device__ static void gload(const Params &p, long long i0, long long j0, long long kt, T ra[8], T rb[8]) {
+    __device__ static void gload(const Params &p, long long i0, long long j0, long long kt, T ra[LD], T rb[LD]) {
         const int tid = threadIdx.x;
         if (IN) {
             if (OP == G_CORR) {
@@ -985,11 +992,11 @@ struct GemmBody {
                 ld4(row + i0 + c, ra); ld4(row + i0 + c + 4, ra + 4);
                 ld4(row + j0 + c, rb); ld4(row + j0 + c + 4, rb + 4);
             } else if (OP == G_SYRK) {
-                const int row = tid >> 1;
-                const long long k = kt * GBK + (tid & 1) * 8;
+                const int row = tid / (GBK / LD);
+                const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
                 const T *xa = p.A + (i0 + row) * p.ld + k, *xb = p.A + (j0 + row) * p.ld + k;
-                ld4(xa, ra); ld4(xa + 4, ra + 4);
-                ld4(xb, rb); ld4(xb + 4, rb + 4);
+                ld4(xa, ra); ld4(xb, rb);
+                if (LD == 8) { ld4(xa + 4, ra + 4); ld4(xb + 4, rb + 4); }
             } else {
                 const int row = tid >> 1;
                 const long long k = kt * (GBK / 2) + (tid & 1) * 4;
@@ -1009,10 +1016,10 @@ struct GemmBody {
             load4_row(p, p.A, k, i0 + c, ra); load4_row(p, p.A, k, i0 + c + 4, ra + 4);
             load4_row(p, p.A, k, j0 + c, rb); load4_row(p, p.A, k, j0 + c + 4, rb + 4);
         } else if (OP == G_SYRK) {
-            const int row = tid >> 1;
-            const long long k = kt * GBK + (tid & 1) * 8;
-            load4_k(p, p.A, i0 + row, k, ra); load4_k(p, p.A, i0 + row, k + 4, ra + 4);
-            load4_k(p, p.A, j0 + row, k, rb); load4_k(p, p.A, j0 + row, k + 4, rb + 4);
+            const int row = tid / (GBK / LD);
+            const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
+            load4_k(p, p.A, i0 + row, k, ra); load4_k(p, p.A, j0 + row, k, rb);
+            if (LD == 8) { load4_k(p, p.A, i0 + row, k + 4, ra + 4); load4_k(p, p.A, j0 + row, k + 4, rb + 4); }
         } else {   // SYR2K: this k'-tile covers k in [kt*GBK/2, (kt+1)*GBK/2)
             const int row = tid >> 1;
             const long long k = kt * (GBK / 2) + (tid & 1) * 4;
@@ -1026,7 +1033,7 @@ struct GemmBody {
         }
     }
     __device__ static T4 mk4(T a, T b, T c, T d) { T4 v; v.x = a; v.y = b; v.z = c; v.w = d; return v; }
-    __device__ static void sstore(Smem &sm, int st, const T ra[8], const T rb[8]) {
+    __device__ static void sstore(Smem &sm, int st, const T ra[LD], const T rb[LD]) {
         const int tid = threadIdx.x;
         if (OP == G_CORR) {
             const int kk = tid >> 4, c = (tid & 15) * 8;
@@ -1035,27 +1042,29 @@ struct GemmBody {
             *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c]) = mk4(rb[0], rb[1], rb[2], rb[3]);
             *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c + 4]) = mk4(rb[4], rb[5], rb[6], rb[7]);
         } else {
-            const int row = tid >> 1, kq = (tid & 1) * 8;
+            const int row = tid / (GBK / LD), kq = (tid % (GBK / LD)) * LD;
 #pragma unroll
-            for (int q = 0; q < 8; ++q) { sm.s[st][0][kq + q][row] = ra[q]; sm.s[st][1][kq + q][row] = rb[q]; }
+            for (int q = 0; q < LD; ++q) { sm.s[st][0][kq + q][row] = ra[q]; sm.s[st][1][kq + q][row] = rb[q]; }
         }
     }
-    __device__ static void frag(const Smem &sm, int st, int kk, int tx, int ty, T a[8], T b[8]) {
+    __device__ static void frag(const Smem &sm, int st, int kk, int tx, int ty, T a[8], T b[TN]) {
         const T4 a0 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][ty * 4]);
         const T4 a1 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][64 + ty * 4]);
-        const T4 b0 = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][tx * 4]);
-        const T4 b1 = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][64 + tx * 4]);
         a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w; a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
-        b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w; b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
+#pragma unroll
+        for (int h = 0; h < NB; ++h) {
+            const T4 bv = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][h * 64 + tx * 4]);
+            b[4 * h] = bv.x; b[4 * h + 1] = bv.y; b[4 * h + 2] = bv.z; b[4 * h + 3] = bv.w;
+        }
     }
 
     // The k'-loop (ascending k' per output, one fma per term).  Returns true on an abort.
     template <bool IN>
-    __device__ static bool mainloop(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][8]) {
-        const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+    __device__ static bool mainloop(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][TN]) {
+        const int tx = threadIdx.x % TXN, ty = threadIdx.x / TXN;
         const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;   // K'
         const long long nkt = (kdim + GBK - 1) / GBK;
-        T ra[8], rb[8];
+        T ra[LD], rb[LD];
         gload<IN>(p, i0, j0, 0, ra, rb);
         sstore(sm, 0, ra, rb);
         __syncthreads();
@@ -1065,7 +1074,7 @@ struct GemmBody {
             for (long long kt = kb; kt < kend; ++kt) {
                 const int st = (int)(kt & 1);
                 if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
-                T a[2][8], b[2][8];
+                T a[2][8], b[2][TN];
                 frag(sm, st, 0, tx, ty, a[0], b[0]);
 #pragma unroll
                 for (int kk = 0; kk < GBK; ++kk) {
@@ -1073,7 +1082,7 @@ struct GemmBody {
 #pragma unroll
                     for (int r = 0; r < 8; ++r)
 #pragma unroll
-                        for (int c = 0; c < 8; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+                        for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
                 }
                 if (kt + 1 < nkt) sstore(sm, st ^ 1, ra, rb);
                 __syncthreads();
@@ -1087,12 +1096,12 @@ struct GemmBody {
         long long bi, bj;
         tile_of(p, t, bi, bj);
         const long long i0 = bi * GBM, j0 = bj * GBM;
-        const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
-        T acc[8][8];
+        const int tx = threadIdx.x % TXN, ty = threadIdx.x / TXN;
+        T acc[8][TN];
 #pragma unroll
         for (int r = 0; r < 8; ++r)
 #pragma unroll
-            for (int c = 0; c < 8; ++c) acc[r][c] = 0;
+            for (int c = 0; c < TN; ++c) acc[r][c] = 0;
         const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;
         const bool interior = p.vec4 && i0 + GBM <= p.n && j0 + GBM <= p.n && kdim % GBK == 0 &&
                               (OP != G_SYR2K || p.m % 4 == 0);
@@ -1102,8 +1111,8 @@ struct GemmBody {
             // mirror block: C[j][i] from acc(i, j) (bit-identical to acc(j, i)); the four rows
             // r of a thread's half are four consecutive columns of the mirror row
 #pragma unroll
-            for (int c = 0; c < 8; ++c) {
-                const long long j = j0 + ((c < 4) ? tx * 4 + c : 64 + tx * 4 + (c - 4));
+            for (int c = 0; c < TN; ++c) {
+                const long long j = j0 + (c / 4) * 64 + tx * 4 + (c % 4);
                 if (j >= p.n) continue;
                 T *crow = p.C + j * p.n;
 #pragma unroll
@@ -1130,7 +1139,7 @@ struct GemmBody {
         for (int r = 0; r < 8; ++r) {
             const long long i = i0 + ((r < 4) ? ty * 4 + r : 64 + ty * 4 + (r - 4));
 #pragma unroll
-            for (int half = 0; half < 2; ++half) {
+            for (int half = 0; half < NB; ++half) {
                 const long long jb = j0 + half * 64 + tx * 4;
                 if (OP == G_CORR) {
 #pragma unroll
@@ -1284,9 +1293,9 @@ static typename ColDotBody<T, MODE>::Params coldot_params(const KArgs &a, const 
     return p;
 }
 
-template <typename T, int OP>
-static typename GemmBody<T, OP>::Params gemm_params(const KArgs &a, const Geom &g) {
-    typename GemmBody<T, OP>::Params p;
+template <typename T, int OP, int TN = 8>
+static typename GemmBody<T, OP, TN>::Params gemm_params(const KArgs &a, const Geom &g) {
+    typename GemmBody<T, OP, TN>::Params p;
     p.A = (const T *)a.dev[0];
     if (OP == G_SYR2K) { p.B = (const T *)a.dev[1]; p.C = (T *)a.dev[2]; }
     else { p.B = nullptr; p.C = (T *)a.dev[1]; }
@@ -1347,6 +1356,10 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
         return f.template go<Conv2DBody<float>>(p);
     }
     case K_SYRK:
+        if (a.sym) {   // upper-triangle grid: one 512-thread CTA per SM
+            if (a.integer) return f.template go<GemmBody<int32_t, G_SYRK, 4>>(gemm_params<int32_t, G_SYRK, 4>(a, g));
+            return f.template go<GemmBody<float, G_SYRK, 4>>(gemm_params<float, G_SYRK, 4>(a, g));
+        }
         if (a.integer) return f.template go<GemmBody<int32_t, G_SYRK>>(gemm_params<int32_t, G_SYRK>(a, g));
         return f.template go<GemmBody<float, G_SYRK>>(gemm_params<float, G_SYRK>(a, g));
     case K_SYR2K:
@@ -1384,7 +1397,7 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
     case K_SYRK: case K_SYR2K: {
         const long long nt = (a.n0 + GBM - 1) / GBM;
         ts.ntasks = (a.kernel == K_SYRK && a.sym) ? nt * (nt + 1) / 2 : nt * nt;
-        ts.threads = 256; break;
+        ts.threads = (a.kernel == K_SYRK && a.sym) ? 512 : 256; break;
     }
     case K_CORR_CORR: {
         const long long nt = (a.n1 + GBM - 1) / GBM;

@@ -230,14 +230,22 @@ struct Executor {
             }
         }
     }
-    // Submit work-groups [lo_, hi_) split `parts` ways; returns immediately.
+    // Submit work-groups [lo_, hi_) split `parts` ways; returns immediately.  The previous job
+    // must be finished (every claimed item executed or skipped): callers quiesce first.
     void submit(const KArgs &a_, const Geom &g_, int64_t lo_, int64_t hi_, int parts, int nact) {
+        wait();   // (defensive: a straggler's done increment must not count for the new job)
+        const uint64_t g1 = gen.load(std::memory_order_relaxed) + 1;
+        // Close the claim word first (new generation, no item claimable): a worker still looping
+        // on the previous job -- e.g. one that woke for an empty job -- may have loaded the old
+        // word and be about to compare-and-swap it; with the word changed its CAS fails, so it
+        // can never claim an "item" of the old job while the fields below already describe the
+        // new one (that executed a work-group twice: in-place kernels applied twice).
+        next.store(((g1 & 0xFFFFFFu) << 40) | ((1ull << 40) - 1), std::memory_order_seq_cst);
         a = a_; g = g_; lo = lo_; hi = hi_; nparts = parts;
         batch = parts > 1 ? 1 : std::max<int64_t>(1, host_batch(a_, g_));
         total = parts > 1 ? (hi_ - lo_) * parts : (hi_ - lo_ + batch - 1) / batch;
         active = std::max(1, std::min(nact, T));
         done.store(0, std::memory_order_relaxed);
-        const uint64_t g1 = gen.load(std::memory_order_relaxed) + 1;
         next.store((g1 & 0xFFFFFFu) << 40, std::memory_order_release);
         gen.store(g1, std::memory_order_release);
         if (sleepers.load() > 0) {
@@ -1397,6 +1405,9 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         int64_t F = L.lo;   // end of the prefix whose return is queued
         int qh = 0, qn = 0;
         auto race_chunk = [&]() {
+            // never while an abandoned chunk of an earlier launch may still run (the GPU may have
+            // finished before this host side started, so the pool was never quiesced)
+            if (!quiesce_try(ctx)) return;
             const double per_wg = cpu_done_wgs > 0 ? busy / (double)cpu_done_wgs : -1.0;
             int64_t size = per_wg > 0 ? (int64_t)(ctx->race_chunk_ms / per_wg) : ceil_pct(pct, nwg);
             size = std::max<int64_t>(size, nact);

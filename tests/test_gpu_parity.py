@@ -488,3 +488,17 @@ def test_online_profiling_picks_the_faster_body(kernel, n0, n1, lws, must_win):
         assert info3["host_variant"] == 1 and info3["profile_ms_per_wg"] == [0.0, 0.0]
     finally:
         c.release()
+
+
+def test_executor_back_to_back_jobs_in_place(ctx):
+    """Regression: a worker that woke for an empty job could claim an 'item' of it while the next
+    job's fields were being written and run that job's work-group a second time -- an in-place
+    (INOUT) kernel then applied twice.  CPU-only launches of new shapes (each profiles its host
+    bodies behind an empty wake-up job, then runs more jobs back to back) must equal GPU-only."""
+    for k, n in enumerate(range(160, 320, 8)):
+        P = W.make("syrk", n, 70, seed=40 + k)
+        ref, _ = H.run(ctx, P, mode="gpu")
+        out, info = H.run(ctx, P, mode="cpu")
+        assert info["cpu_did_all"] == 1
+        for i in P.out_indices:
+            assert_bits(out[i], ref[i], f"syrk {n}x70 cpu-only")
