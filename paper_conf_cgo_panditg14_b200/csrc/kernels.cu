@@ -914,7 +914,7 @@ constexpr int GBM = 128, GBK = 16, GPAD = 4;
 // grid (136 tiles at N = 2048, one per SM), where 16 warps hide the k'-tile loads that 8 cannot.
 template <typename T, int OP, int TN = 8>
 struct GemmBody {
-    static_assert(TN == 8 || (TN == 4 && OP == G_SYRK), "TN = 4 is the SYRK upper-triangle variant");
+    static_assert(TN == 8 || (TN == 4 && OP != G_SYR2K), "TN = 4: SYRK upper triangle, CORR symmat");
     static constexpr int kThreads = TN == 8 ? 256 : 512;
 #ifndef FCL_GEMM_MINB
 #define FCL_GEMM_MINB 2
@@ -987,10 +987,10 @@ struct GemmBody {
         const int tid = threadIdx.x;
         if (IN) {
             if (OP == G_CORR) {
-                const int kk = tid >> 4, c = (tid & 15) * 8;
+                const int kk = tid / (GBM / LD), c = (tid % (GBM / LD)) * LD;
                 const T *row = p.A + (kt * GBK + kk) * p.ld;
-                ld4(row + i0 + c, ra); ld4(row + i0 + c + 4, ra + 4);
-                ld4(row + j0 + c, rb); ld4(row + j0 + c + 4, rb + 4);
+                ld4(row + i0 + c, ra); ld4(row + j0 + c, rb);
+                if (LD == 8) { ld4(row + i0 + c + 4, ra + 4); ld4(row + j0 + c + 4, rb + 4); }
             } else if (OP == G_SYRK) {
                 const int row = tid / (GBK / LD);
                 const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
@@ -1011,10 +1011,10 @@ struct GemmBody {
             return;
         }
         if (OP == G_CORR) {
-            const int kk = tid >> 4, c = (tid & 15) * 8;
+            const int kk = tid / (GBM / LD), c = (tid % (GBM / LD)) * LD;
             const long long k = kt * GBK + kk;
-            load4_row(p, p.A, k, i0 + c, ra); load4_row(p, p.A, k, i0 + c + 4, ra + 4);
-            load4_row(p, p.A, k, j0 + c, rb); load4_row(p, p.A, k, j0 + c + 4, rb + 4);
+            load4_row(p, p.A, k, i0 + c, ra); load4_row(p, p.A, k, j0 + c, rb);
+            if (LD == 8) { load4_row(p, p.A, k, i0 + c + 4, ra + 4); load4_row(p, p.A, k, j0 + c + 4, rb + 4); }
         } else if (OP == G_SYRK) {
             const int row = tid / (GBK / LD);
             const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
@@ -1036,11 +1036,13 @@ struct GemmBody {
     __device__ static void sstore(Smem &sm, int st, const T ra[LD], const T rb[LD]) {
         const int tid = threadIdx.x;
         if (OP == G_CORR) {
-            const int kk = tid >> 4, c = (tid & 15) * 8;
+            const int kk = tid / (GBM / LD), c = (tid % (GBM / LD)) * LD;
             *reinterpret_cast<T4 *>(&sm.s[st][0][kk][c]) = mk4(ra[0], ra[1], ra[2], ra[3]);
-            *reinterpret_cast<T4 *>(&sm.s[st][0][kk][c + 4]) = mk4(ra[4], ra[5], ra[6], ra[7]);
             *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c]) = mk4(rb[0], rb[1], rb[2], rb[3]);
-            *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c + 4]) = mk4(rb[4], rb[5], rb[6], rb[7]);
+            if (LD == 8) {
+                *reinterpret_cast<T4 *>(&sm.s[st][0][kk][c + 4]) = mk4(ra[4], ra[5], ra[6], ra[7]);
+                *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c + 4]) = mk4(rb[4], rb[5], rb[6], rb[7]);
+            }
         } else {
             const int row = tid / (GBK / LD), kq = (tid % (GBK / LD)) * LD;
 #pragma unroll
@@ -1365,7 +1367,11 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
     case K_SYR2K:
         if (a.integer) return f.template go<GemmBody<int32_t, G_SYR2K>>(gemm_params<int32_t, G_SYR2K>(a, g));
         return f.template go<GemmBody<float, G_SYR2K>>(gemm_params<float, G_SYR2K>(a, g));
-    case K_CORR_CORR: return f.template go<GemmBody<float, G_CORR>>(gemm_params<float, G_CORR>(a, g));
+    case K_CORR_CORR:
+#ifndef FCL_CORR_TN
+#define FCL_CORR_TN 8   // (TN = 4, one 512-thread CTA per SM: 1.62 vs 1.55 ms at M = N = 4096)
+#endif
+        return f.template go<GemmBody<float, G_CORR, FCL_CORR_TN>>(gemm_params<float, G_CORR, FCL_CORR_TN>(a, g));
     default: return -1;
     }
 }
@@ -1401,7 +1407,7 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
     }
     case K_CORR_CORR: {
         const long long nt = (a.n1 + GBM - 1) / GBM;
-        ts.ntasks = nt * (nt + 1) / 2; ts.threads = 256; break;
+        ts.ntasks = nt * (nt + 1) / 2; ts.threads = FCL_CORR_TN == 4 ? 512 : 256; break;
     }
     default: break;
     }
