@@ -822,6 +822,41 @@ struct Conv2DBody {
         return s;
     }
 
+    // A warp's 128 x 8 block away from every border (input rows ib-1 .. ib+8 and columns
+    // j-1 .. j+4 exist for all lanes, no output on the border): no per-row or per-column
+    // checks, one pointer walking the rows, and the halo columns loaded by the two edge lanes
+    // for every row up front, so that no shuffle sits under a divergent branch.
+    __device__ static void run_interior(const Params &p, long long ib, long long j, int lane) {
+        typedef typename V4<T>::type T4;
+        const long long nj = p.tl.ncols;
+        const T *src = p.A + (ib - 1) * nj + j;
+        const bool l0 = lane == 0, l31 = lane == 31;
+        const T *edge = src + (l0 ? -1 : 4);
+        T4 v[10];
+        T lh[10], rh[10];
+#pragma unroll
+        for (int q = 0; q < 10; ++q) v[q] = ld_cached4(src + q * nj);
+#pragma unroll
+        for (int q = 0; q < 10; ++q) lh[q] = (l0 || l31) ? __ldg(edge + q * nj) : T(0);
+#pragma unroll
+        for (int q = 0; q < 10; ++q) {
+            const T up = __shfl_up_sync(0xffffffffu, v[q].w, 1);
+            const T dn = __shfl_down_sync(0xffffffffu, v[q].x, 1);
+            rh[q] = l31 ? lh[q] : dn;
+            lh[q] = l0 ? lh[q] : up;
+        }
+        T *dst = p.B + ib * nj + j;
+#pragma unroll
+        for (int q = 1; q <= 8; ++q) {
+            T4 o;
+            o.x = tap9(p, lh[q - 1], lh[q], lh[q + 1], v[q - 1].x, v[q].x, v[q + 1].x, v[q - 1].y, v[q].y, v[q + 1].y);
+            o.y = tap9(p, v[q - 1].x, v[q].x, v[q + 1].x, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z);
+            o.z = tap9(p, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w);
+            o.w = tap9(p, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w, rh[q - 1], rh[q], rh[q + 1]);
+            __stcs(reinterpret_cast<T4 *>(dst + (q - 1) * nj), o);
+        }
+    }
+
     __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
         const Tile2D &tl = p.tl;
         const long long tx = t % tl.ntx, ty = t / tl.ntx;
@@ -834,6 +869,11 @@ struct Conv2DBody {
             const int rg = warp >> 1;                // which 8-row group
             const long long j = c0 + cg * 128 + lane * 4;   // first of this thread's 4 columns
             const long long ib = r0 + rg * 8;        // first output row of the group
+            const long long wj0 = c0 + cg * 128;     // the warp's first column (warp-uniform test)
+            if (ib >= 1 && ib + 8 <= ni - 1 && wj0 >= 1 && wj0 + 128 <= nj - 1) {
+                run_interior(p, ib, j, lane);
+                return false;
+            }
             if (ib >= ni) return false;
             const bool colok = j < nj;               // nj % 4 == 0 on this path
             typename V4<T>::type v[10];
