@@ -19,11 +19,11 @@ ncu --set full --clock-control none --import-source on --kernel-name-base demang
 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:merge_kernel' -s 2 -c 1 \
     -o gpurun_out/${TAG}_merge python scripts/merge_one.py > /dev/null 2>&1
 # compute-bound dispatcher: SYRK 2048 and the 2DCONV stencil
-FCL_SELECT=0 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:coop_kernel.*GemmBody<float, .*0>' -s 1 -c 1 \
+FCL_SELECT=0 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:coop_kernel.*GemmBody<float, (\(int\))?0' -s 1 -c 1 \
     -o gpurun_out/${TAG}_syrk python scripts/profile_step.py coop 2 syrk:2048 > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*GemmBody<float, .*0>' -s 1 -c 1 \
+ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*GemmBody<float, (\(int\))?0' -s 1 -c 1 \
     -o gpurun_out/${TAG}_syrk_plain python scripts/profile_step.py gpu 2 syrk:2048 > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*GemmBody<float, .*1>' -s 1 -c 1 \
+ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*GemmBody<float, (\(int\))?1' -s 1 -c 1 \
     -o gpurun_out/${TAG}_syr2k_plain python scripts/profile_step.py gpu 2 syr2k:2048 > /dev/null 2>&1
 FCL_SELECT=0 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:coop_kernel.*Conv2DBody<float>' -s 1 -c 1 \
     -o gpurun_out/${TAG}_conv2d python scripts/profile_step.py coop 2 conv2d:16384 > /dev/null 2>&1
