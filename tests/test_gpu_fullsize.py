@@ -104,3 +104,21 @@ def test_config4_corr_4096_chain(ctx, oracle_mod):
     assert_parity(np.where(mask, got_sym, 0.0), np.where(mask, L.bufs[1], 0.0), False, "corr symmat sampled")
     for b in (d, mean, std, sym):
         b.release()
+
+
+@pytest.mark.parametrize("kernel,n0,n1", [("gesummv", 4096, 4096), ("bicg_s", 4096, 4096), ("syrk", 2048, 2048)])
+def test_device_selection_full_size(ctx, oracle_mod, kernel, n0, n1):
+    """The bench's launch configuration: COOP with device selection on.  The
+    probe runs cooperatively, the next launches of the shape on the GPU alone; every result is
+    the GPU-only result bit for bit and matches the oracle on sampled work-groups."""
+    P = W.make(kernel, n0, n1, seed=23, lws1d=256)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    n = P.num_groups
+    seen = []
+    for i in range(3):
+        out, info = H.run(ctx, P, mode="coop", select=1)
+        seen.append((info["probe"], info["selected"]))
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], f"{kernel} launch {i} {seen[-1]}")
+    assert seen[0] == (1, 0) and seen[1][0] == 0, seen
+    _check_sampled(oracle_mod, P, out, [0, n // 2, n - 1])
