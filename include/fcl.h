@@ -115,9 +115,13 @@ fcl_status fcl_release_buffer(fcl_buffer buf);
 /* Write [offset, offset+n) of buf from host memory src to both copies
  * (clEnqueueWriteBuffer -> writes to both devices, L16.s1).  src may be the
  * buffer's own host mirror (then only the device copy is updated).  With
- * blocking == 0 the host->device copy is asynchronous on the main stream;
- * src may be reused as soon as the call returns (it is copied to the pinned
- * mirror first).  Errors: FCL_INVALID_VALUE (range), FCL_CONTEXT_LOST. */
+ * blocking == 1 the host->device copy is made before the call returns.  With
+ * blocking == 0 a partial write copies asynchronously on the main stream, and
+ * a write of the whole buffer refreshes the device copy lazily: when a launch
+ * first needs it on the GPU (never, if the data is consumed on the host alone
+ * under device selection).  src may be reused as soon as the
+ * call returns (it is copied to the pinned mirror first).
+ * Errors: FCL_INVALID_VALUE (range), FCL_CONTEXT_LOST. */
 fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer buf, size_t offset, size_t n,
                             const void *src, int32_t blocking);
 
@@ -303,7 +307,9 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info);
 #define FCL_COUNT_SEL_CPU    3  /* COOP launches run on the host alone by device selection */
 #define FCL_COUNT_GPU_ONLY   4  /* GPU_ONLY-mode launches */
 #define FCL_COUNT_CPU_ONLY   5  /* CPU_ONLY-mode launches */
-#define FCL_COUNT_N          6
+#define FCL_COUNT_H2D_BYTES  6  /* bytes copied host -> device (writes, refreshes, staged chunks) */
+#define FCL_COUNT_D2H_BYTES  7  /* bytes copied device -> host (returns, reads) */
+#define FCL_COUNT_N          8
 fcl_status fcl_get_counters(fcl_context ctx, int64_t *counts, int32_t n);
 
 /* Multi-GPU slicing helper: a contiguous flattened-id range for

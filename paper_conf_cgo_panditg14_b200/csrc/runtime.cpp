@@ -359,7 +359,7 @@ struct Job {
     std::atomic<int> done{0};
     bool probe = false;                  // refreshes the device-selection profile of its shape
     bool probe_gpu_idle = false;         // the GPU had nothing queued when the probe was enqueued
-    std::array<int64_t, 8> sel_key{};
+    std::array<int64_t, 9> sel_key{};
 };
 
 }  // namespace
@@ -432,9 +432,9 @@ struct fcl_context_st {
     // last cooperative probe showed (FCL_SELECTED_*) and how many launches the shape has had.
     struct SelectEnt { int64_t launches = 0; int choice = FCL_SELECTED_COOP; };
     std::mutex sel_mu;
-    std::map<std::array<int64_t, 8>, SelectEnt> sel;
+    std::map<std::array<int64_t, 9>, SelectEnt> sel;
     bool select_on = true;                       // FCL_SELECT=0: off unless a launch asks for it
-    int64_t counts[FCL_COUNT_N] = {};            // fcl_get_counters (calling thread only)
+    std::atomic<int64_t> counts[FCL_COUNT_N] = {};   // fcl_get_counters (launch counts, bytes moved)
     int select_period = 16;                      // FCL_SELECT_PERIOD: every n-th launch of a shape probes
     double select_min_share = 0.10;              // FCL_SELECT_MIN_SHARE: host share a probe must reach
     uint32_t pool_keep = 256;                    // FCL_POOL_KEEP: launches an unused pool buffer survives
@@ -647,11 +647,13 @@ fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_d
     if (need_dev && !b->dev_valid) {
         ctx->main_fenced.store(1);
         CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
+        ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)b->bytes;
         b->dev_valid = true;
         if (info) info->h2d_bytes += (int64_t)b->bytes;
     }
     if (need_host && !b->host_valid) {
         CK(ctx, cudaMemcpyAsync(b->host, b->dev, b->bytes, cudaMemcpyDeviceToHost, ctx->main));
+        ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)b->bytes;
         CK(ctx, cudaStreamSynchronize(ctx->main));
         b->host_valid = true;
         if (info) info->d2h_bytes += (int64_t)b->bytes;
@@ -686,6 +688,7 @@ fcl_status enqueue_d2h(fcl_context ctx, Launch &L, int64_t wlo, int64_t whi, fcl
         ctx->dh_used.store(1, std::memory_order_relaxed);
         if (d2h_busy(ctx, b) && b->d2h_on_race) CK(ctx, cudaStreamWaitEvent(ctx->dh, b->d2h_ev, 0));
         CK(ctx, cudaMemcpyAsync((char *)b->host + b0, (char *)b->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dh));
+        ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)(b1 - b0);
         info.d2h_bytes += (int64_t)(b1 - b0);
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));
         b->d2h_pending = true; b->d2h_on_main = false; b->d2h_on_race = false; b->d2h_gen = ctx->finish_gen.load();
@@ -816,6 +819,7 @@ fcl_status flush_returns(fcl_context ctx, bool at_finish) {
     at.srcLocHint.type = cudaMemLocationTypeDevice; at.srcLocHint.id = ctx->device;
     at.dstLocHint.type = cudaMemLocationTypeHost; at.dstLocHint.id = 0;
     size_t aidx = 0, fail = 0;
+    for (size_t k = 0; k < n; ++k) ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)sz[k];
     if (n == 1 || cudaMemcpyBatchAsync(dst.data(), src.data(), sz.data(), n, &at, &aidx, 1, &fail, ctx->main) != cudaSuccess) {
         cudaGetLastError();   // (a driver without batched copies: one copy per buffer)
         for (size_t k = 0; k < n; ++k)
@@ -893,8 +897,12 @@ void variant_info(const VariantPick &vp, fcl_launch_info &info) {
 // probe, that one device cannot contribute -- the host finished no work-group before the GPU
 // exited, or it covered the whole range before the GPU did -- runs on the other device alone.
 // Every select_period-th launch of the shape is a cooperative probe again.
-std::array<int64_t, 8> select_key(const Launch &L) {
-    return {L.a.kernel, L.a.integer ? 1 : 0, L.a.n0, L.a.n1, L.g.lws[0], L.g.work_dim > 1 ? L.g.lws[1] : 1, L.lo, L.hi};
+// The shape, and whether an input has to reach the GPU first (a stale device copy, e.g. after a
+// lazy non-blocking write): the same kernel is host- or GPU-favoured depending on that transfer.
+std::array<int64_t, 9> select_key(const Launch &L) {
+    int64_t stale = 0;
+    for (int k = 0; k < L.a.nbuf; ++k) stale |= ((L.acc[k] & 1) && !L.bufs[k]->dev_valid) ? 1 : 0;
+    return {L.a.kernel, L.a.integer ? 1 : 0, L.a.n0, L.a.n1, L.g.lws[0], L.g.work_dim > 1 ? L.g.lws[1] : 1, L.lo, L.hi, stale};
 }
 
 bool select_eligible(fcl_context ctx, const Launch &L) {
@@ -1311,6 +1319,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             out_span(L.a, L.g, L.out_idx[q], clo, chi, &b0, &b1);
             if (b1 > b0) {
                 CK(ctx, cudaMemcpyAsync((char *)j.stage[q] + b0, (char *)b->host + b0, b1 - b0, cudaMemcpyHostToDevice, ctx->hd));
+                ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)(b1 - b0);
                 info.h2d_bytes += (int64_t)(b1 - b0);
             }
         }
@@ -1451,6 +1460,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
                     out_span(L.a, L.g, L.out_idx[q], F, b, &b0, &b1);
                     if (b1 <= b0) continue;
                     CK(ctx, cudaMemcpyAsync((char *)ob->host + b0, (char *)ob->dev + b0, b1 - b0, cudaMemcpyDeviceToHost, ctx->dr));
+                    ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)(b1 - b0);
                     info.d2h_bytes += (int64_t)(b1 - b0);
                 }
                 CK(ctx, cudaEventRecord(ctx->race_ev[(qh + qn) & 3], ctx->dr));
@@ -2070,7 +2080,16 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
     // overwriting the pinned mirror: no queued copy may still read its old contents
     if (src != h) CK(ctx, cudaStreamSynchronize(ctx->main));
     if (src != h) std::memcpy(h, src, n);
+    if (!blocking && n == b->bytes) {
+        // a non-blocking write of the whole buffer refreshes the device copy lazily, when a
+        // launch first needs it on the GPU -- never, if the data is consumed on the host alone
+        // (device selection)
+        b->host_valid = true;
+        b->dev_valid = false;
+        return FCL_SUCCESS;
+    }
     CK(ctx, cudaMemcpyAsync((char *)b->dev + offset, h, n, cudaMemcpyHostToDevice, ctx->main));
+    ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)n;
     b->host_valid = b->dev_valid = true;
     if (blocking) CK(ctx, cudaStreamSynchronize(ctx->main));
     return FCL_SUCCESS;
@@ -2402,6 +2421,7 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer b) {
         ctx->dh_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaStreamWaitEvent(ctx->dh, ctx->ev_mark, 0));
         if (d2h_busy(ctx, b) && b->d2h_on_race) CK(ctx, cudaStreamWaitEvent(ctx->dh, b->d2h_ev, 0));
+        ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)(b->r_b1 - b->r_b0);
         CK(ctx, cudaMemcpyAsync((char *)b->host + b->r_b0, (char *)b->dev + b->r_b0, b->r_b1 - b->r_b0,
                                 cudaMemcpyDeviceToHost, ctx->dh));
         CK(ctx, cudaEventRecord(b->d2h_ev, ctx->dh));

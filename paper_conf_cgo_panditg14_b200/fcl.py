@@ -327,7 +327,7 @@ class Context:
         _check(load().fcl_get_launch_info(self.handle, ctypes.byref(info)), "fcl_get_launch_info", self.handle)
         return info.as_dict()
 
-    COUNTERS = ("coop", "probe", "sel_gpu", "sel_cpu", "gpu_only", "cpu_only")
+    COUNTERS = ("coop", "probe", "sel_gpu", "sel_cpu", "gpu_only", "cpu_only", "h2d_bytes", "d2h_bytes")
 
     def counters(self) -> dict:
         """Cumulative launch counters (fcl_get_counters): how COOP launches ran under device selection."""
