@@ -112,3 +112,28 @@ def test_test_hooks_are_never_redirected(ctx):
     assert info["selected"] == SEL_COOP and info["cpu_wgs"] == P.num_groups - P.num_groups // 2
     for k in P.out_indices:
         assert_bits(out[k], ref[k], "forced split")
+
+
+def test_lazy_write_refresh_and_host_alone(ctx):
+    """A non-blocking write of a whole buffer leaves the device copy stale (include/fcl.h): a
+    GPU launch refreshes it first (the bytes show in fcl_get_counters), a CPU-only launch moves
+    nothing, and both give the reference result."""
+    P = W.make("gesummv", 512, seed=31, lws1d=64)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    bufs = H.create_buffers(ctx, P)
+    ins = [bufs[k] for k in range(len(P.bufs)) if k not in P.out_indices]
+    for mode, moves in (("gpu", True), ("cpu", False)):
+        for b in ins:
+            b.write(b.host_ptr, blocking=False)
+        c0 = ctx.counters()
+        out, _ = H.run(ctx, P, mode=mode, bufs=bufs)
+        c1 = ctx.counters()
+        moved = c1["h2d_bytes"] - c0["h2d_bytes"]
+        if moves:
+            assert moved >= sum(b.nbytes for b in ins), (moved, mode)
+        else:
+            assert moved == 0, (moved, mode)
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], f"after lazy write, {mode}")
+    for b in bufs:
+        b.release()
