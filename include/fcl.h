@@ -251,6 +251,8 @@ typedef struct {
                                     measured in this launch) */
     int32_t selected;            /* FCL_SELECTED_*: what a COOP launch ran as (opts.select) */
     int32_t probe;               /* 1 = this cooperative launch refreshes the selection profile */
+    int64_t streamed_wgs;        /* work-groups whose stale input rows were streamed to the GPU in
+                                    pieces while the host computed */
 } fcl_launch_info;
 
 /* info.selected */

@@ -91,6 +91,11 @@ struct CoopCtl {
     unsigned long long *merge_ctr_next; // the next launch's chunk counter (reset here)
     unsigned long long *exit_word;      // mapped host word set to `epoch` after the barrier
     DevMergeList mg;                    // merge list (mg.n == 0: nothing to merge in-kernel)
+    // Streamed inputs: {epoch:32 | front:32}, device word written by stream
+    // memops behind the H2D pieces -- work-groups [0, front) have their input rows on the
+    // device.  nullptr: every input is resident.  A task waits for its rows or for the host to
+    // cover it.
+    const unsigned long long *arrival;
 };
 
 // Decode the dispatcher's wm word: the lowest watermark launch `epoch` acted on, or

@@ -384,6 +384,30 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
             if (threadIdx.x == 0) { record_wm(c, w); marked = true; }
             break;
         }
+        if (c.arrival) {
+            // streamed inputs: wait until this task's rows arrived, or the host covers it (then
+            // every later task is covered too); a stalled stream is a bug -- trap, never hang
+            if (threadIdx.x == 0) {
+                int covered = 0;
+                const unsigned long long t0 = globaltimer();
+                unsigned int ns = 128;
+                for (;;) {
+                    const unsigned long long a = ld_status(c.arrival);
+                    const unsigned int front = ((unsigned int)(a >> 32) == c.epoch) ? (unsigned int)a : 0u;
+                    if ((unsigned long long)key < (unsigned long long)front) break;
+                    const unsigned int wv = decode_w(ld_status(c.status), c);
+                    if ((unsigned long long)key >= (unsigned long long)wv) { record_wm(c, wv); marked = true; covered = 1; break; }
+                    if (globaltimer() - t0 > 5000000000ull) __trap();
+                    __nanosleep(ns);
+                    if (ns < 2048) ns *= 2;
+                }
+                s_flag = covered;
+            }
+            __syncthreads();
+            const int covered = s_flag;
+            __syncthreads();
+            if (covered) break;
+        }
         if (threadIdx.x == 0) s_key = key;   // read back by thread 0 only
         // claim the next task while this one runs (no claim at all when the grid already
         // covers every task: no contention on the counter)

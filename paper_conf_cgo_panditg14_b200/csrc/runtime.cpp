@@ -357,6 +357,8 @@ struct Job {
     fcl_launch_info info{};
     fcl_status status = FCL_SUCCESS;
     std::atomic<int> done{0};
+    bool stream = false;                 // inputs streamed to the device in row pieces (§6.7)
+    int nstream = 0, sbuf[6] = {0};      // streamed buffers (argument indices)
     bool probe = false;                  // refreshes the device-selection profile of its shape
     bool probe_gpu_idle = false;         // the GPU had nothing queued when the probe was enqueued
     std::array<int64_t, 9> sel_key{};
@@ -439,7 +441,12 @@ struct fcl_context_st {
     double select_min_share = 0.10;              // FCL_SELECT_MIN_SHARE: host share a probe must reach
     uint32_t pool_keep = 256;                    // FCL_POOL_KEEP: launches an unused pool buffer survives
     size_t pool_cap = 16ull << 30;               // FCL_POOL_CAP_MB: unused buffers beyond this are freed
-    unsigned long long test_gpu_delay_ns = 0;    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
+    unsigned long long test_gpu_delay_ns = 0;
+    // Streamed inputs: arrival fronts, one per launch slot, and the piece events
+    bool stream_on = true;                       // FCL_NO_STREAM=1: stale inputs are copied whole first
+    unsigned long long *darrival = nullptr;
+    cudaEvent_t stream_ev[4] = {};
+    size_t stream_piece_bytes = 8u << 20;        // FCL_STREAM_PIECE_BYTES    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
@@ -988,6 +995,8 @@ Job *job_alloc(fcl_context ctx) {
     j->have_k = j->have_m = j->wm_pending = false;
     j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = j->lite = j->exact_spans = false;
     j->lazy = false;
+    j->stream = false;
+    j->nstream = 0;
     j->unit = 1;
     std::memset(&j->info, 0, sizeof j->info);
     for (int q = 0; q < 6; ++q) j->twin[q] = j->stage[q] = nullptr;
@@ -1069,7 +1078,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     int opt_period = L.o.abort_period;
     if (opt_period == 0 && ctx->env_abort_period != 0) opt_period = ctx->env_abort_period;   // FCL_ABORT_PERIOD
     const int abort_period = opt_period > 0 ? opt_period : (opt_period < 0 ? 0 : gpu_default_abort_period(L.a));
-    j.lite = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && abort_period == 0 && !ctx->no_lite &&
+    j.lite = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && abort_period == 0 && !ctx->no_lite && !j.stream &&
              (j.t1 - j.t0) <= gpu_coop_capacity(L.a, L.g, ctx->num_sms);
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
     const void *srcs[6];
@@ -1133,6 +1142,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     c.merge_ctr = ctx->dmctr + j.slot;
     c.merge_ctr_next = ctx->dmctr + (j.slot + 1) % kSlots;
     c.exit_word = ctx->exit_dptr + j.slot;
+    c.arrival = j.stream ? ctx->darrival + j.slot : nullptr;
     c.mg = DevMergeList{};
     c.mg.n = 0;
 
@@ -1333,6 +1343,56 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         return FCL_SUCCESS;
     };
 
+    // Streamed inputs (§6.7): row pieces of the stale matrices in ascending work-group order on
+    // hd, each followed by the arrival front (a stream memop), never beyond the host's frontier
+    // (the work-groups it has taken), at most two pieces outstanding.
+    int64_t s_sent = L.lo;
+    int s_head = 0, s_out = 0;
+    unsigned s_spin = 0;
+    int64_t s_piece = 1;
+    if (j.stream) {
+        size_t per_wg = 0;
+        for (int q = 0; q < j.nstream; ++q) per_wg += (size_t)L.g.lws[0] * (size_t)L.a.n1 * L.bufs[j.sbuf[q]]->elem_size;
+        s_piece = std::max<int64_t>(1, (int64_t)(ctx->stream_piece_bytes / std::max<size_t>(1, per_wg)));
+    }
+    auto pump = [&]() -> fcl_status {
+        if (!j.stream || gpu_done) return FCL_SUCCESS;
+        if (s_out > 0 && ((++s_spin & 15) == 0 || s_out >= 2)) {
+            while (s_out > 0) {
+                const cudaError_t q = cudaEventQuery(ctx->stream_ev[s_head & 3]);
+                if (q == cudaErrorNotReady) break;
+                if (q != cudaSuccess) return cuda_fail(ctx, q, "stream piece");
+                ++s_head; --s_out;
+            }
+        }
+        const int64_t frontier = in_flight ? cur_lo : hi_cur;
+        while (s_out < 2 && s_sent < frontier) {
+            const int64_t hi = std::min<int64_t>(s_sent + s_piece, frontier);
+            ctx->hd_used.store(1, std::memory_order_relaxed);
+            if (!hd_joined) {   // behind every earlier kernel that may still read the old device copy
+                CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
+                hd_joined = true;
+            }
+            const int64_t r0 = s_sent * L.g.lws[0], r1 = std::min<int64_t>(hi * L.g.lws[0], L.a.n0);
+            for (int q = 0; q < j.nstream && r1 > r0; ++q) {
+                fcl_buffer b = L.bufs[j.sbuf[q]];
+                const size_t rb = (size_t)L.a.n1 * b->elem_size;
+                CK(ctx, cudaMemcpyAsync((char *)b->dev + (size_t)r0 * rb, (char *)b->host + (size_t)r0 * rb,
+                                        (size_t)(r1 - r0) * rb, cudaMemcpyHostToDevice, ctx->hd));
+                ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)((size_t)(r1 - r0) * rb);
+                info.h2d_bytes += (int64_t)((size_t)(r1 - r0) * rb);
+            }
+            fcl_status st = stream_store(ctx, ctx->darrival + j.slot, ((unsigned long long)j.epoch << 32) | (uint32_t)hi,
+                                         ctx->hd, true, &info);
+            if (st != FCL_SUCCESS) return st;
+            CK(ctx, cudaEventRecord(ctx->stream_ev[(s_head + s_out) & 3], ctx->hd));
+            ++s_out;
+            s_sent = hi;
+            info.streamed_wgs = s_sent - L.lo;
+        }
+        return FCL_SUCCESS;
+    };
+
     info.published_watermark = L.hi;
     if (exited_before) {
         gpu_done = true;
@@ -1342,7 +1402,15 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     } else {
         cpu_all = true;
     }
+    {
+        fcl_status st = pump();
+        if (st != FCL_SUCCESS) { ex.abort_flag = 1; ex.wait(); return st; }
+    }
     while (in_flight) {
+        {
+            fcl_status st = pump();
+            if (st != FCL_SUCCESS) { ex.abort_flag = 1; ex.wait(); return st; }
+        }
         if (!j.forced && !gpu_done && j.gpu_launched && exit_word_seen()) {
             gpu_done = true;   // GPU exit (L18.s19)
             ctx->tr.add("gpu_exit_seen", j.epoch);
@@ -1871,8 +1939,12 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     }
     for (cudaEvent_t *pe : {&ctx->ev_k0, &ctx->ev_t1})
         if ((e = cudaEventCreate(pe)) != cudaSuccess) return fail(e, "events");
+    if ((e = cudaMalloc(&dp, 8 * fcl_context_st::kSlots)) != cudaSuccess) return fail(e, "arrival words");
+    cudaMemset(dp, 0, 8 * fcl_context_st::kSlots);
+    ctx->darrival = (unsigned long long *)dp;
     for (cudaEvent_t *pe : {&ctx->ev_k1, &ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h, &ctx->race_ev[0], &ctx->race_ev[1],
-                            &ctx->race_ev[2], &ctx->race_ev[3]})
+                            &ctx->race_ev[2], &ctx->race_ev[3], &ctx->stream_ev[0], &ctx->stream_ev[1], &ctx->stream_ev[2],
+                            &ctx->stream_ev[3]})
         if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
     // stream memory operations for publication (driver entry point; fall back to a kernel store)
     {
@@ -1892,6 +1964,8 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_LITE_EXIT")) ctx->lite_exit_word = atoi(getenv("FCL_LITE_EXIT")) != 0;
     if (getenv("FCL_POOL_KEEP")) ctx->pool_keep = (uint32_t)std::max(0, atoi(getenv("FCL_POOL_KEEP")));
     if (getenv("FCL_POOL_CAP_MB")) ctx->pool_cap = (size_t)atoll(getenv("FCL_POOL_CAP_MB")) << 20;
+    ctx->stream_on = !(getenv("FCL_NO_STREAM") && atoi(getenv("FCL_NO_STREAM")) != 0);
+    if (getenv("FCL_STREAM_PIECE_BYTES")) ctx->stream_piece_bytes = std::max<size_t>(1 << 16, (size_t)atoll(getenv("FCL_STREAM_PIECE_BYTES")));
     if (getenv("FCL_SELECT")) ctx->select_on = atoi(getenv("FCL_SELECT")) != 0;
     if (getenv("FCL_TEST_GPU_DELAY_US")) ctx->test_gpu_delay_ns = 1000ull * (unsigned long long)atoll(getenv("FCL_TEST_GPU_DELAY_US"));
     if (getenv("FCL_SELECT_MIN_SHARE")) ctx->select_min_share = atof(getenv("FCL_SELECT_MIN_SHARE"));
@@ -1962,6 +2036,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->wm_host) cudaFreeHost(ctx->wm_host);
     if (ctx->exit_host) cudaFreeHost(ctx->exit_host);
     if (ctx->dclaim) cudaFree(ctx->dclaim);
+    if (ctx->darrival) cudaFree(ctx->darrival);
     if (ctx->own_main) cudaStreamDestroy(ctx->main);
     if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
     if (ctx->own_dh) cudaStreamDestroy(ctx->dh);
@@ -2359,11 +2434,25 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     info.probe = probe ? 1 : 0;
     info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
     info.gpu_watermark = info.published_watermark = L.hi;
+    // Streamed inputs (§6.7): the row-partitioned matrices of a row-dot kernel whose device copy
+    // is stale go to the GPU in ascending row pieces while the host computes from the top.
+    if (ctx->stream_on && (L.a.kernel == K_GESUMMV || L.a.kernel == K_ATAX_TMP || L.a.kernel == K_BICG_Q) &&
+        L.g.work_dim == 1 && L.g.lws[0] % 4 == 0 && L.o.forced_split < 0 && !L.o.defer_merge) {
+        for (int k = 0; k < L.a.nbuf; ++k) {
+            fcl_buffer b = L.bufs[k];
+            if (L.acc[k] == 1 && !b->dev_valid && required_elems(L.a.kernel, k, L.a.n0, L.a.n1) == L.a.n0 * L.a.n1 &&
+                L.a.n1 > 1)
+                j->sbuf[j->nstream++] = k;
+        }
+        j->stream = j->nstream > 0;
+    }
     for (int k = 0; k < L.a.nbuf; ++k) {
         fcl_buffer b = L.bufs[k];
+        bool streamed = false;
+        for (int q = 0; q < j->nstream; ++q) streamed |= j->sbuf[q] == k;
         // A device copy left stale by a CPU-only launch is refreshed first (lazy H2D; the
         // queue is drained above whenever a copy is stale).
-        if (!b->dev_valid) {
+        if (!b->dev_valid && !streamed) {
             s = make_valid(ctx, b, false, true, &info);
             if (s != FCL_SUCCESS) break;
         }

@@ -75,7 +75,8 @@ class LaunchInfo(ctypes.Structure):
                 ("t_merge_ms", ctypes.c_double), ("t_host_ms", ctypes.c_double),
                 ("chunk_sizes", ctypes.c_int32 * 64), ("gpu_path", ctypes.c_int32), ("race", ctypes.c_int32),
                 ("host_variant", ctypes.c_int32), ("n_host_variants", ctypes.c_int32),
-                ("profile_ms_per_wg", ctypes.c_double * 4), ("selected", ctypes.c_int32), ("probe", ctypes.c_int32)]
+                ("profile_ms_per_wg", ctypes.c_double * 4), ("selected", ctypes.c_int32), ("probe", ctypes.c_int32),
+                ("streamed_wgs", ctypes.c_int64)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("chunk_sizes", "profile_ms_per_wg")}

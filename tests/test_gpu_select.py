@@ -137,3 +137,27 @@ def test_lazy_write_refresh_and_host_alone(ctx):
             assert_bits(out[k], ref[k], f"after lazy write, {mode}")
     for b in bufs:
         b.release()
+
+
+@pytest.mark.parametrize("kernel,integer,lws", [("gesummv", False, 64), ("gesummv", True, 64),
+                                                ("atax_tmp", False, 32), ("bicg_q", False, 128)])
+def test_streamed_inputs(ctx, kernel, integer, lws):
+    """Stale input matrices (a non-blocking whole-buffer write) of a row-dot kernel stream to the
+    GPU in row pieces while the host computes from the top; GPU work-groups
+    wait for their rows or for the host to cover them.  The result is the GPU-only one bit for
+    bit, with the host slowed down (the GPU then takes most pieces) and at full speed."""
+    P = W.make(kernel, 2048, 2048, integer=integer, seed=33, lws1d=lws)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    for kw in (dict(host_delay_us=300), dict()):
+        bufs = H.create_buffers(ctx, P)
+        for k in range(len(P.bufs)):
+            if k not in P.out_indices:
+                bufs[k].write(bufs[k].host_ptr, blocking=False)
+        out, info = H.run(ctx, P, mode="coop", bufs=bufs, select=-1, **kw)
+        assert info["streamed_wgs"] > 0 or info["cpu_did_all"] == 1, info
+        if kw:
+            assert info["streamed_wgs"] > 0, info
+        for k in P.out_indices:
+            assert_bits(out[k], ref[k], f"{kernel} streamed {kw}")
+        for b in bufs:
+            b.release()
