@@ -1124,6 +1124,65 @@ struct GemmBody {
         }
     }
 
+    // CORR's operand is K-major already (data[k][col]): interior tiles stream it with cp.async
+    // straight into shared memory, NSA stages of GBKA k-rows (three tiles in flight, no register
+    // staging), in the same bytes as Smem.
+    static constexpr int GBKA = 8, NSA = 4;
+    struct SmemA { T s[NSA][2][GBKA][GBM + GPAD]; };
+    __device__ static void cp_async16(void *dst, const void *src) {
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
+    }
+    __device__ static bool mainloop_async(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][TN]) {
+        static_assert(sizeof(SmemA) <= sizeof(Smem), "async stages must fit the static smem");
+        static_assert(kThreads == 256 && TN == 8, "one 16-byte copy per operand and thread");
+        SmemA &sa = *reinterpret_cast<SmemA *>(&sm);
+        const int tid = threadIdx.x, tx = tid % TXN, ty = tid / TXN;
+        const int lr = tid >> 5, lc = (tid & 31) * 4;
+        const long long nkt = p.m / GBKA;
+        auto issue = [&](long long kt) {
+            if (kt < nkt) {
+                const int st = (int)(kt % NSA);
+                const T *row = p.A + (kt * GBKA + lr) * p.ld;
+                cp_async16(&sa.s[st][0][lr][lc], row + i0 + lc);
+                cp_async16(&sa.s[st][1][lr][lc], row + j0 + lc);
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        };
+#pragma unroll
+        for (int q = 0; q < NSA - 1; ++q) issue(q);
+        const long long per = 2 * tc.period();   // polls every `per` GBKA-tiles (= period GBK-tiles)
+        for (long long kt = 0; kt < nkt; ++kt) {
+            asm volatile("cp.async.wait_group %0;" ::"n"(NSA - 2) : "memory");
+            __syncthreads();   // tile kt landed for every thread; stage (kt-1) % NSA is free
+            issue(kt + NSA - 1);
+            const int st = (int)(kt % NSA);
+            T a[2][8], b[2][TN];
+            auto fr = [&](int kk, T *fa, T *fb) {
+                const T4 a0 = *reinterpret_cast<const T4 *>(&sa.s[st][0][kk][ty * 4]);
+                const T4 a1 = *reinterpret_cast<const T4 *>(&sa.s[st][0][kk][64 + ty * 4]);
+                const T4 b0 = *reinterpret_cast<const T4 *>(&sa.s[st][1][kk][tx * 4]);
+                const T4 b1 = *reinterpret_cast<const T4 *>(&sa.s[st][1][kk][64 + tx * 4]);
+                fa[0] = a0.x; fa[1] = a0.y; fa[2] = a0.z; fa[3] = a0.w; fa[4] = a1.x; fa[5] = a1.y; fa[6] = a1.z; fa[7] = a1.w;
+                fb[0] = b0.x; fb[1] = b0.y; fb[2] = b0.z; fb[3] = b0.w; fb[4] = b1.x; fb[5] = b1.y; fb[6] = b1.z; fb[7] = b1.w;
+            };
+            fr(0, a[0], b[0]);
+#pragma unroll
+            for (int kk = 0; kk < GBKA; ++kk) {
+                if (kk + 1 < GBKA) fr(kk + 1, a[(kk + 1) & 1], b[(kk + 1) & 1]);
+#pragma unroll
+                for (int r = 0; r < 8; ++r)
+#pragma unroll
+                    for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+            }
+            if ((kt + 1) % per == 0 && kt + 1 < nkt && tc.check()) {   // abort check (Fig 12)
+                asm volatile("cp.async.wait_all;" ::: "memory");
+                return true;
+            }
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        return false;
+    }
+
     // The k'-loop (ascending k' per output, one fma per term).  Returns true on an abort.
     template <bool IN>
     __device__ static bool mainloop(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][TN]) {
@@ -1171,7 +1230,18 @@ struct GemmBody {
         const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;
         const bool interior = p.vec4 && i0 + GBM <= p.n && j0 + GBM <= p.n && kdim % GBK == 0 &&
                               (OP != G_SYR2K || p.m % 4 == 0);
-        if (interior ? mainloop<true>(p, i0, j0, tc, sm, acc) : mainloop<false>(p, i0, j0, tc, sm, acc)) return true;
+#ifndef FCL_CORR_ASYNC
+#define FCL_CORR_ASYNC 1
+#endif
+        bool done_async = false;
+        if constexpr (OP == G_CORR && TN == 8 && FCL_CORR_ASYNC) {
+            if (interior && p.m % GBKA == 0) {
+                if (mainloop_async(p, i0, j0, tc, sm, acc)) return true;
+                done_async = true;
+            }
+        }
+        if (!done_async && (interior ? mainloop<true>(p, i0, j0, tc, sm, acc) : mainloop<false>(p, i0, j0, tc, sm, acc)))
+            return true;
         // epilogue: write-once stores
         if (OP == G_SYRK && p.sym && bi != bj) {
             // mirror block: C[j][i] from acc(i, j) (bit-identical to acc(j, i)); the four rows
