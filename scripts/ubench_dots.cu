@@ -87,6 +87,102 @@ __global__ void __launch_bounds__(128, MINB) rowdot(const __grid_constant__ RP p
     }
 }
 
+// ---- row-dot with register double buffering: the next U blocks' loads are issued before the
+// current ones are consumed (continuous loads per warp); RW rows per warp interleaved (RW
+// independent streams per warp).  Same canonical order as rowdot.
+template <int NMAT, int U, int RW, int MINB>
+__global__ void __launch_bounds__(128, MINB) rowdot_db(const __grid_constant__ RP p) {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const long long i0 = ((long long)blockIdx.x * 4 + warp) * RW;
+    if (i0 >= p.n) return;
+    const int nfull = p.n / 128;
+    float acc[RW][2][4];
+#pragma unroll
+    for (int r = 0; r < RW; ++r)
+#pragma unroll
+        for (int m = 0; m < 2; ++m)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) acc[r][m][q] = 0.f;
+    const float *pa[RW], *pb[RW];
+#pragma unroll
+    for (int r = 0; r < RW; ++r) { pa[r] = p.A + (i0 + r) * p.n + 4 * lane; pb[r] = p.B + (i0 + r) * p.n + 4 * lane; }
+    const float *px = p.x + 4 * lane;
+    float4 cur[RW][2][U], nxt[RW][2][U];
+#pragma unroll
+    for (int r = 0; r < RW; ++r)
+#pragma unroll
+        for (int u = 0; u < U; ++u) { cur[r][0][u] = ld_stream4(pa[r] + u * 128); if (NMAT == 2) cur[r][1][u] = ld_stream4(pb[r] + u * 128); }
+    for (int k = 0; k < nfull; k += U) {
+        const bool more = k + U < nfull;
+        if (more) {
+#pragma unroll
+            for (int r = 0; r < RW; ++r)
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    nxt[r][0][u] = ld_stream4(pa[r] + (k + U + u) * 128);
+                    if (NMAT == 2) nxt[r][1][u] = ld_stream4(pb[r] + (k + U + u) * 128);
+                }
+        }
+        float4 xv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) xv[u] = ld_cached4(px + (k + u) * 128);
+#pragma unroll
+        for (int r = 0; r < RW; ++r)
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+#pragma unroll
+                for (int m = 0; m < NMAT; ++m) {
+                    acc[r][m][0] = __fmaf_rn(cur[r][m][u].x, xv[u].x, acc[r][m][0]);
+                    acc[r][m][1] = __fmaf_rn(cur[r][m][u].y, xv[u].y, acc[r][m][1]);
+                    acc[r][m][2] = __fmaf_rn(cur[r][m][u].z, xv[u].z, acc[r][m][2]);
+                    acc[r][m][3] = __fmaf_rn(cur[r][m][u].w, xv[u].w, acc[r][m][3]);
+                }
+        if (more) {
+#pragma unroll
+            for (int r = 0; r < RW; ++r)
+#pragma unroll
+                for (int m = 0; m < 2; ++m)
+#pragma unroll
+                    for (int u = 0; u < U; ++u) cur[r][m][u] = nxt[r][m][u];
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < RW; ++r) {
+        const float va = fold4(acc[r][0][0], acc[r][0][1], acc[r][0][2], acc[r][0][3]);
+        if (NMAT == 1) { if (lane == 0) p.o0[i0 + r] = va; }
+        else {
+            const float vb = fold4(acc[r][1][0], acc[r][1][1], acc[r][1][2], acc[r][1][3]);
+            if (lane == 0) { p.o0[i0 + r] = va; p.o1[i0 + r] = __fadd_rn(__fmul_rn(p.alpha, va), __fmul_rn(p.beta, vb)); }
+        }
+    }
+}
+
+// plain copy (read + write) of the same byte count: 8 independent 16-byte loads per thread
+__global__ void __launch_bounds__(256) copy8_kernel(const float4 *__restrict__ s, float4 *__restrict__ d, size_t n) {
+    const size_t st = (size_t)gridDim.x * blockDim.x * 8;
+    for (size_t i = (size_t)blockIdx.x * blockDim.x * 8 + threadIdx.x; i < n; i += st) {
+        float4 v[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) if (i + q * blockDim.x < n) v[q] = __ldcs(s + i + q * blockDim.x);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) if (i + q * blockDim.x < n) __stcs(d + i + q * blockDim.x, v[q]);
+    }
+}
+// read-only, 8 independent 16-byte loads per thread in flight
+__global__ void __launch_bounds__(256) read8_kernel(const float4 *__restrict__ s, size_t n, float *sink) {
+    const size_t st = (size_t)gridDim.x * blockDim.x * 8;
+    float acc = 0.f;
+    for (size_t i = (size_t)blockIdx.x * blockDim.x * 8 + threadIdx.x; i < n; i += st) {
+        float4 v[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) v[q] = (i + q * blockDim.x < n) ? __ldcs(s + i + q * blockDim.x) : make_float4(0, 0, 0, 0);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc += v[q].x;
+    }
+    if (acc == 12345.0f) *sink = acc;
+}
+
 // ---- row-dot through shared memory: TMA bulk copies (cp.async.bulk) of each warp's row
 // into a per-CTA ring of NS stages; stage = 4 rows x SB columns x NMAT matrices.
 __device__ __forceinline__ void mbar_init(uint64_t *b, unsigned cnt) {
@@ -337,6 +433,21 @@ int main(int argc, char **argv) {
     ROWV("gesummv R1 U2 whole-row L2 prefetch", rowdot<2, 2, 1, 8>)
     ROWV("gesummv R2 U2 windowed L2 prefetch", rowdot<2, 2, 2, 8>)
     ROWV("gesummv U4 minb7", rowdot<2, 4, 0, 7>)
+    {   // ceilings for 134 MB at this size
+        for (int bpsm : {2, 4, 8}) {
+            char nm[64]; snprintf(nm, 64, "copy 64 MiB (134 MB moved), %d CTA/SM", bpsm);
+            float ms = time_it([&] { copy8_kernel<<<148 * bpsm, 256>>>((const float4 *)A, (float4 *)B, nn / 4); });
+            report(nm, ms, 2.0 * nn * 4, true);
+            snprintf(nm, 64, "read 2 x 64 MiB, 8 loads in flight, %d CTA/SM", bpsm);
+            ms = time_it([&] { read8_kernel<<<148 * bpsm, 256>>>((const float4 *)A, nn / 4, g_sink); read8_kernel<<<148 * bpsm, 256>>>((const float4 *)B, nn / 4, g_sink); });
+            report(nm, ms, 2.0 * nn * 4, true);
+        }
+        CK(cudaMemcpy(B, hB.data(), nn * 4, cudaMemcpyHostToDevice));
+    }
+    ROWV("gesummv double-buffered U2 RW1", (rowdot_db<2, 2, 1, 7>))
+    ROWV("gesummv double-buffered U2 RW1 minb4", (rowdot_db<2, 2, 1, 4>))
+    ROWV("gesummv double-buffered U1 RW2", (rowdot_db<2, 1, 2, 4>))
+    ROWV("gesummv double-buffered U4 RW1 minb4", (rowdot_db<2, 4, 1, 4>))
     ROWV("gesummv U4 minb7 whole-row prefetch", rowdot<2, 4, 1, 7>)
     ROWV("gesummv U1 whole-row prefetch", rowdot<2, 1, 1, 8>)
 #define ROWT(NAME, NMAT_, NS, SBc, MINB) { CK(cudaMemset(o0, 0, n * 4)); CK(cudaMemset(o1, 0, n * 4)); \
