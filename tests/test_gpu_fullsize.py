@@ -122,3 +122,24 @@ def test_device_selection_full_size(ctx, oracle_mod, kernel, n0, n1):
             assert_bits(out[k], ref[k], f"{kernel} launch {i} {seen[-1]}")
     assert seen[0] == (1, 0) and seen[1][0] == 0, seen
     _check_sampled(oracle_mod, P, out, [0, n // 2, n - 1])
+
+
+@pytest.mark.parametrize("kernel", ["gesummv", "bicg_q"])
+def test_streamed_inputs_full_size(ctx, oracle_mod, kernel):
+    """The bench's e2e configuration at full size: inputs written non-blocking (device copies
+    stale), the row-dot matrices streamed to the GPU in row pieces while the host computes from
+    the top.  Bits equal GPU-only; sampled work-groups match the oracle."""
+    P = W.make(kernel, 4096, 4096, seed=24, lws1d=256)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    bufs = H.create_buffers(ctx, P)
+    for k in range(len(P.bufs)):
+        if k not in P.out_indices:
+            bufs[k].write(bufs[k].host_ptr, blocking=False)
+    out, info = H.run(ctx, P, mode="coop", bufs=bufs, select=-1)
+    assert info["streamed_wgs"] > 0 or info["cpu_did_all"] == 1, info
+    for k in P.out_indices:
+        assert_bits(out[k], ref[k], f"{kernel} streamed")
+    n = P.num_groups
+    _check_sampled(oracle_mod, P, out, [0, n // 2, n - 1])
+    for b in bufs:
+        b.release()
