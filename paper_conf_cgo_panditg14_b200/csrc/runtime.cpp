@@ -2437,7 +2437,8 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     // Streamed inputs (§6.7): the row-partitioned matrices of a row-dot kernel whose device copy
     // is stale go to the GPU in ascending row pieces while the host computes from the top.
     if (ctx->stream_on && (L.a.kernel == K_GESUMMV || L.a.kernel == K_ATAX_TMP || L.a.kernel == K_BICG_Q) &&
-        L.g.work_dim == 1 && L.g.lws[0] % 4 == 0 && L.o.forced_split < 0 && !L.o.defer_merge) {
+        L.g.work_dim == 1 && L.g.lws[0] % 4 == 0 && L.o.forced_split < 0 && !L.o.defer_merge &&
+        !L.o.drop_publish) {   // (the GPU waits for pieces or for the watermark: both must come)
         for (int k = 0; k < L.a.nbuf; ++k) {
             fcl_buffer b = L.bufs[k];
             if (L.acc[k] == 1 && !b->dev_valid && required_elems(L.a.kernel, k, L.a.n0, L.a.n1) == L.a.n0 * L.a.n1 &&
