@@ -25,6 +25,8 @@ ncu --set full --clock-control none --import-source on --kernel-name-base demang
     -o gpurun_out/${TAG}_syrk_plain python scripts/profile_step.py gpu 2 syrk:2048 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*GemmBody<float, (\(int\))?1' -s 1 -c 1 \
     -o gpurun_out/${TAG}_syr2k_plain python scripts/profile_step.py gpu 2 syr2k:2048 > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:plain_kernel.*GemmBody<float, (\(int\))?2' -s 1 -c 1 \
+    -o gpurun_out/${TAG}_corr_plain python scripts/profile_step.py gpu 2 corr_corr:4096 > /dev/null 2>&1
 FCL_SELECT=0 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k 'regex:coop_kernel.*Conv2DBody<float>' -s 1 -c 1 \
     -o gpurun_out/${TAG}_conv2d python scripts/profile_step.py coop 2 conv2d:16384 > /dev/null 2>&1
 ls -la gpurun_out/

@@ -59,6 +59,7 @@ for name, rep in [("gesummv, cooperative launch (lite plain grid when single-wav
                   ("merge_kernel 1 GiB, scatter 10 %", "merge"), ("SYRK 2048 dispatcher", "syrk"),
                   ("SYRK 2048 plain grid (GPU-only; upper-triangle tiles + mirrors)", "syrk_plain"),
                   ("SYR2K 2048 plain grid (GPU-only)", "syr2k_plain"),
+                  ("CORR symmat 4096 plain grid (GPU-only; cp.async pipeline)", "corr_plain"),
                   ("2DCONV 16384^2 dispatcher", "conv2d")]:
     p = os.path.join(SRC, f"{TAG}_{rep}.ncu-rep")
     if not os.path.exists(p):
@@ -74,7 +75,8 @@ for name, rep in [("gesummv, cooperative launch (lite plain grid when single-wav
         if "dram_read" in d and "dram_write" in d:
             tb = to_bytes(d["dram_read_raw"], d["dram_read"]) + to_bytes(d["dram_write_raw"], d["dram_write"])
             key = {"gesummv_coop": "gesummv", "merge": "merge_kernel", "syrk": "syrk", "conv2d": "conv2d",
-                   "gesummv_plain": "gesummv_plain", "syrk_plain": "syrk_plain", "syr2k_plain": "syr2k_plain"}[rep]
+                   "gesummv_plain": "gesummv_plain", "syrk_plain": "syrk_plain", "syr2k_plain": "syr2k_plain",
+                   "corr_plain": "corr_plain"}[rep]
             traffic[key] = int(tb)
             lines.append(f"  - dram traffic (read+write): {tb / 1e6:.1f} MB")
     lines.append("")
