@@ -441,12 +441,12 @@ struct fcl_context_st {
     double select_min_share = 0.10;              // FCL_SELECT_MIN_SHARE: host share a probe must reach
     uint32_t pool_keep = 256;                    // FCL_POOL_KEEP: launches an unused pool buffer survives
     size_t pool_cap = 16ull << 30;               // FCL_POOL_CAP_MB: unused buffers beyond this are freed
-    unsigned long long test_gpu_delay_ns = 0;
+    unsigned long long test_gpu_delay_ns = 0;    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
     // Streamed inputs: arrival fronts, one per launch slot, and the piece events
     bool stream_on = true;                       // FCL_NO_STREAM=1: stale inputs are copied whole first
     unsigned long long *darrival = nullptr;
     cudaEvent_t stream_ev[4] = {};
-    size_t stream_piece_bytes = 8u << 20;        // FCL_STREAM_PIECE_BYTES    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
+    size_t stream_piece_bytes = 8u << 20;        // FCL_STREAM_PIECE_BYTES
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
     bool no_race = false;                        // FCL_NO_RACE=1
