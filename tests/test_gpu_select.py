@@ -161,3 +161,32 @@ def test_streamed_inputs(ctx, kernel, integer, lws):
             assert_bits(out[k], ref[k], f"{kernel} streamed {kw}")
         for b in bufs:
             b.release()
+
+
+def test_e2e_loop_selection_and_streaming(ctx):
+    """The bench's e2e loop at a reduced size: every step writes the inputs (non-blocking, device
+    copies stale), runs GESUMMV + BICG s/q as COOP launches with device selection, reads the
+    outputs.  Probes, streamed launches, host-alone and GPU-alone launches interleave over 20
+    steps; every step's results equal the GPU-only ones bit for bit."""
+    Ps = [W.make("gesummv", 1024, seed=41, lws1d=64),
+          W.make("bicg_s", 1024, 1024, seed=42, lws1d=64),
+          W.make("bicg_q", 1024, 1024, seed=43, lws1d=64)]
+    refs = [H.run(ctx, P, mode="gpu")[0] for P in Ps]
+    bufs = [H.create_buffers(ctx, P) for P in Ps]
+    c0 = ctx.counters()
+    for step in range(20):
+        for P, bl in zip(Ps, bufs):
+            for k in range(len(P.bufs)):
+                if k not in P.out_indices:
+                    bl[k].write(bl[k].host_ptr, blocking=False)
+        for P, bl in zip(Ps, bufs):
+            ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, bl), mode="coop", select=1)
+        ctx.finish()
+        for P, bl, ref in zip(Ps, bufs, refs):
+            for k in P.out_indices:
+                assert_bits(bl[k].read_array(np.float32), ref[k], f"{P.kernel} step {step}")
+    c1 = ctx.counters()
+    assert c1["probe"] > c0["probe"]
+    for bl in bufs:
+        for b in bl:
+            b.release()
