@@ -148,6 +148,9 @@ int gpu_launch_plain(const KArgs &a, const Geom &g, int64_t task_lo, int64_t tas
 // CTAs of the persistent dispatcher resident at once (occupancy x SMs): a launch with no more
 // tasks than this runs in a single wave, every CTA's only task unchecked.
 int64_t gpu_coop_capacity(const KArgs &a, const Geom &g, int num_sms);
+// Load every kernel of the library now (CUDA lazy loading would load a kernel at its first
+// launch, which may wait for the device -- see kernels.cu).  0 on success.
+int gpu_preload_kernels();
 // Fig 9 diff-merge on [0, bytes) of three device buffers.
 int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes, int elem_size,
                      int num_sms, void *stream);

@@ -1711,3 +1711,44 @@ int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void 
 }
 
 }  // namespace fcl
+
+// ------------------------------------------------------------------------------------------
+// Eager loading of every kernel of the library.  With CUDA's lazy module loading a kernel is
+// loaded at its first launch, and loading may wait for the device: a first-time launch queued
+// while a cooperative grid waits for host-driven copies (streamed inputs) can
+// then stall the host thread that issues those copies -- a deadlock.  The context loads
+// everything once, at creation.
+// ------------------------------------------------------------------------------------------
+namespace fcl {
+template <class Body>
+static int preload_body() {
+    cudaFuncAttributes at;
+    int bad = 0;
+    bad |= cudaFuncGetAttributes(&at, coop_kernel<Body>) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, plain_kernel<Body>) != cudaSuccess;
+    return bad;
+}
+int gpu_preload_kernels() {
+    int bad = 0;
+    bad |= preload_body<RowDotBody<float, 1>>() | preload_body<RowDotBody<int32_t, 1>>();
+    bad |= preload_body<RowDotBody<float, 2>>() | preload_body<RowDotBody<int32_t, 2>>();
+    bad |= preload_body<ColDotBody<float, COL_DOT>>() | preload_body<ColDotBody<int32_t, COL_DOT>>();
+    bad |= preload_body<ColDotBody<float, COL_SUM>>() | preload_body<ColDotBody<float, COL_SQDEV>>();
+    bad |= preload_body<CorrReduceBody>();
+    bad |= preload_body<Conv2DBody<float>>() | preload_body<Conv2DBody<int32_t>>();
+    bad |= preload_body<GemmBody<float, G_SYRK>>() | preload_body<GemmBody<int32_t, G_SYRK>>();
+    bad |= preload_body<GemmBody<float, G_SYRK, 4>>() | preload_body<GemmBody<int32_t, G_SYRK, 4>>();
+    bad |= preload_body<GemmBody<float, G_SYR2K>>() | preload_body<GemmBody<int32_t, G_SYR2K>>();
+    bad |= preload_body<GemmBody<float, G_CORR, FCL_CORR_TN>>();
+    cudaFuncAttributes at;
+    bad |= cudaFuncGetAttributes(&at, merge_kernel<1>) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, merge_kernel<2>) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, merge_kernel<4>) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, merge_kernel<8>) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, merge_dev_kernel) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, copies_kernel) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, store64_kernel) != cudaSuccess;
+    if (bad) { cudaGetLastError(); return seterr(cudaErrorInvalidDeviceFunction, "kernel preload"); }
+    return 0;
+}
+}  // namespace fcl

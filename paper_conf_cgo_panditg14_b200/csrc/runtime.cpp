@@ -1042,15 +1042,14 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
             _mm_pause();
         }
     }
-    // main-stream position before this launch: this job's first staging copy waits for it,
-    // so no pool buffer is overwritten while an earlier merge still reads it.  The previous
-    // launch's end-of-dispatcher event (its merge is fused into the dispatcher) serves.
-    if (ctx->main_tail && !ctx->unfused) {
-        j.main_before = ctx->main_tail;
-    } else {
-        CK(ctx, cudaEventRecord(j.ev_start, ctx->main));
-        j.main_before = j.ev_start;
-    }
+    // main-stream position before this launch: this job's first staging copy (and the pieces
+    // of streamed inputs) wait for it, so no pool buffer or input is overwritten while an
+    // earlier kernel still reads it.  Always this job's own event: the previous dispatcher's
+    // end event (used here before) belongs to a job that can be recycled and re-recorded --
+    // behind this launch's own grid, or a later one -- while this launch still waits on it;
+    // with streamed inputs that made the grid wait for pieces that waited for the grid.
+    CK(ctx, cudaEventRecord(j.ev_start, ctx->main));
+    j.main_before = j.ev_start;
 
     // Host chunk boundaries are aligned to the output span unit (1 work-group for 1-D kernels,
     // one work-group row for 2-D row-major ones).  The staged spans are then exactly the host's
@@ -1983,6 +1982,9 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_RACE_CHUNK_MS")) ctx->race_chunk_ms = atof(getenv("FCL_RACE_CHUNK_MS"));
     if (getenv("FCL_KTIMING")) ctx->ktiming = atoi(getenv("FCL_KTIMING")) != 0;
     if ((e = cudaDeviceSynchronize()) != cudaSuccess) return fail(e, "init sync");
+    // (FCL_NO_PRELOAD=1: keep CUDA's lazy loading -- only to show what the preload prevents)
+    if (!(getenv("FCL_NO_PRELOAD") && atoi(getenv("FCL_NO_PRELOAD")) != 0) && gpu_preload_kernels() != 0)
+        return fail(cudaErrorInvalidDeviceFunction, "kernel preload");
     const char *pin = getenv("FCL_PIN_THREADS");
     const bool do_pin = d.pin_threads ? true : (pin ? atoi(pin) != 0 : true);
     int nthr = d.n_host_threads;

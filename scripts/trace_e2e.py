@@ -28,21 +28,39 @@ in_bufs = [bufs[0][0], bufs[0][1], bufs[0][2], bufs[1][0], bufs[1][1], bufs[2][1
 out_bufs = [bufs[0][3], bufs[0][4], bufs[1][2], bufs[2][2]]
 outs = [np.empty(b.nbytes // 4, np.float32) for b in out_bufs]
 ts = []
+import traceback
+failed = False
 for r in range(40):
-    stream.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for b in in_bufs:
-        b.write(b.host_ptr, blocking=False)
-    for l in L:
-        l()
-    ctx.finish()
-    for b, o in zip(out_bufs, outs):
-        b.read(o.ctypes.data)
-    e1.record(stream)
-    e1.synchronize()
-    ts.append(e0.elapsed_time(e1))
+  try:
+      stream.synchronize()
+      e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+      e0.record(stream)
+      for b in in_bufs:
+          b.write(b.host_ptr, blocking=False)
+      for l in L:
+          l()
+      ctx.finish()
+      for b, o in zip(out_bufs, outs):
+          b.read(o.ctypes.data)
+      e1.record(stream)
+      e1.synchronize()
+      ts.append(e0.elapsed_time(e1))
+  except Exception:
+    traceback.print_exc()
+    print("FAILED at step", r)
+    failed = True
+    break
 print("step ms", [round(t, 3) for t in ts[-12:]])
+if failed:
+    try:
+        ctx.release()
+    except Exception:
+        pass
+    recs = [l.split() for l in open(os.environ["FCL_TRACE_FILE"])]
+    host = [(float(t), tag, int(e)) for t, tag, e in recs if not tag.startswith("gpu_")]
+    t0 = host[-60][0] if len(host) > 60 else host[0][0]
+    print(" | ".join(f"{tag}:{e}@{(t - t0) * 1000:.0f}" for t, tag, e in host[-60:]))
+    sys.exit(1)
 for b in in_bufs:
     b.write(b.host_ptr, blocking=False)
 for l, P in zip(L, Ps):

@@ -190,3 +190,42 @@ def test_e2e_loop_selection_and_streaming(ctx):
     for bl in bufs:
         for b in bl:
             b.release()
+
+
+_FIRST_LAUNCH_SCRIPT = r'''
+import sys
+sys.path.insert(0, sys.argv[1])
+import numpy as np
+import fcl_harness as H
+import workloads as W
+from paper_conf_cgo_panditg14_b200 import fcl
+ctx = fcl.Context(0)
+P = W.make("gesummv", 2048, seed=51, lws1d=64)
+Q = W.make("conv2d", 512, 512, seed=52)
+bp, bq = H.create_buffers(ctx, P), H.create_buffers(ctx, Q)
+for k in range(len(P.bufs)):
+    if k not in P.out_indices:
+        bp[k].write(bp[k].host_ptr, blocking=False)
+# a streamed launch (its grid waits for host-driven copies), then kernels this process has never
+# launched, queued behind it without a drain
+ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, bp), mode="coop", select=-1, host_delay_us=200)
+ctx.enqueue_ndrange(H.kernel_name(Q), Q.gws, Q.lws, H.make_args(ctx, Q, bq), mode="coop", select=-1)
+ctx.finish()
+print("ok")
+'''
+
+
+def test_first_launch_of_a_kernel_behind_a_streamed_grid(tmp_path):
+    """Regression: with CUDA's lazy module loading a kernel was loaded at its first launch, which
+    could wait for a cooperative grid that itself waited for host-driven copies of streamed inputs
+    (a deadlock, caught by the 5 s guard as a launch failure).  The context now loads every
+    kernel at creation; a fresh process launching a new kernel behind a streamed one must finish."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "first_launch.py"
+    script.write_text(_FIRST_LAUNCH_SCRIPT)
+    env = dict(os.environ, FCL_SELECT="0")
+    r = subprocess.run([sys.executable, str(script), root], capture_output=True, text=True, timeout=120, env=env)
+    assert r.returncode == 0 and "ok" in r.stdout, (r.stdout[-2000:], r.stderr[-2000:])
