@@ -81,7 +81,9 @@ typedef struct {
 
 /* Create a context on desc->device (desc may be NULL: device 0, defaults).
  * Owns: streams it creates, the pinned status words, device counters, the
- * twin/stage pool and the host executor threads.  Errors: FCL_INVALID_VALUE,
+ * twin/stage pool and the host executor threads.  Loads every kernel of the
+ * library (no lazy loading at a first launch, which can wait for the device
+ * while a grid waits for host-driven copies).  Errors: FCL_INVALID_VALUE,
  * FCL_DEVICE_NOT_AVAILABLE, FCL_OUT_OF_RESOURCES, FCL_CUDA_ERROR. */
 fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out);
 fcl_status fcl_release_context(fcl_context ctx);
