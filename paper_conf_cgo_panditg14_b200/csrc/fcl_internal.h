@@ -46,10 +46,10 @@ struct KArgs {
     int64_t n0, n1;        // rows / columns of the row-major input (SYRK/SYR2K: N, M)
     float alpha, beta, eps;
     int32_t ialpha, ibeta;
-    // SYRK over a range that starts at work-group 0: the GPU runs only the upper-triangle tiles
-    // and writes each one's mirror too -- fma(A_i, A_j, acc) == fma(A_j, A_i, acc) bit for bit,
-    // so C's accumulator is symmetric; a slice that starts higher needs its
-    // lower-left blocks, whose mirrors lie below the slice, and runs every tile
+    // SYRK over the whole range: the GPU runs only the upper-triangle tiles and writes each
+    // one's mirror too -- fma(A_i, A_j, acc) == fma(A_j, A_i, acc) bit for bit, so C's
+    // accumulator is symmetric; a slice runs every tile of its rows (its
+    // lower-left blocks' mirrors lie outside it, and its own mirrors would land outside it)
     bool sym;
 };
 

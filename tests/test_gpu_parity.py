@@ -502,3 +502,25 @@ def test_executor_back_to_back_jobs_in_place(ctx):
         assert info["cpu_did_all"] == 1
         for i in P.out_indices:
             assert_bits(out[i], ref[i], f"syrk {n}x70 cpu-only")
+
+
+def test_syrk_slices_same_buffer(ctx):
+    """SYRK (C in place) run as consecutive slices on the SAME buffers, each slice cooperative:
+    every element of C is updated exactly once (a slice must not touch C's device copy outside
+    its rows -- the upper-triangle grid's mirror blocks would), and the result is the GPU-only one."""
+    P = W.make("syrk", 384, 96, seed=61)
+    ref, _ = H.run(ctx, P, mode="gpu")
+    k = ctx.kernel(H.kernel_name(P))
+    for nranks in (2, 3):
+        bufs = H.create_buffers(ctx, P)
+        for r in range(nranks):
+            lo, hi = ctx.slice_range(k, P.gws, P.lws, r, nranks)
+            ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, bufs), mode="coop",
+                                wg_lo=lo, wg_hi=hi)
+            ctx.finish()
+        out = bufs[1].read_array(np.float32)
+        assert_bits(out, ref[1], f"syrk {nranks} slices on one buffer")
+        dev = H.device_array(bufs[1], np.float32)
+        assert_bits(dev, ref[1], f"syrk {nranks} slices, device copy")
+        for b in bufs:
+            b.release()
