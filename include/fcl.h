@@ -186,8 +186,9 @@ typedef struct {
     int32_t n_host_threads;  /* 0 = context default; else use at most this many */
     int32_t host_delay_us;   /* fault injection: sleep before each host chunk */
     int32_t drop_publish;    /* fault injection: stage chunks but never publish the watermark */
-    int64_t wg_lo, wg_hi;    /* execute only flattened ids [wg_lo, wg_hi) (multi-GPU slice);
-                                wg_hi <= 0 means the whole NDRange */
+    int64_t wg_lo, wg_hi;    /* execute only flattened ids [wg_lo, wg_hi) (multi-GPU slice, SURVEY
+                                §8e); wg_hi < 0 (default) = the whole NDRange; wg_lo == wg_hi = an
+                                empty slice: the call returns FCL_SUCCESS and runs nothing */
     int32_t blocking;        /* 1 = return only when the launch's host side is done (the paper's
                                 blocking calls, L22.s14); 0 (default) = OpenCL-style enqueue */
     int32_t flags;           /* FCL_LAUNCH_* bits */

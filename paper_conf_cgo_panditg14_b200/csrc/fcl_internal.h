@@ -51,6 +51,9 @@ struct KArgs {
     // accumulator is symmetric; a slice runs every tile of its rows (its
     // lower-left blocks' mirrors lie outside it, and its own mirrors would land outside it)
     bool sym;
+    // Row-dot inputs streamed to the device in pieces while the grid runs: the
+    // body loads them through L2 only
+    bool streamed;
 };
 
 // Device-side merge of a cooperative launch's output buffers (domain read from wm_word).
@@ -155,7 +158,9 @@ int gpu_preload_kernels();
 int gpu_launch_merge(void *gpu, const void *cpu, const void *twin, size_t bytes, int elem_size,
                      int num_sms, void *stream);
 int gpu_launch_merge_dev(const DevMergeList &L, size_t max_bytes, int num_sms, void *stream);
-// Copy up to 6 (dst, src, bytes) device regions in one launch (16-byte aligned pointers).
+// Copy up to 6 (dst, src, bytes) regions in one launch (16-byte aligned pointers; dst may be the
+// device-visible address of mapped host memory).  1 = launched, 0 = nothing to copy, -2 = a
+// pointer is not 16-byte aligned (nothing launched), -1 = launch failure.
 int gpu_launch_copies(int n, void *const *dst, const void *const *src, const size_t *bytes, int num_sms,
                       void *stream);
 // One-thread kernel that stores `value` to `addr` (status publication fallback).

@@ -52,6 +52,13 @@ __device__ __forceinline__ typename V4<T>::type ld_stream4(const T *p) {
                  : "l"(p));
     return v;
 }
+// 128-bit load through L2 only (.cg): for input rows that H2D copies may still be writing while
+// the kernel runs (streamed inputs) -- never served from a stale L1 line or the
+// non-coherent path.
+template <typename T>
+__device__ __forceinline__ typename V4<T>::type ld_cg4(const T *p) {
+    return __ldcg(reinterpret_cast<const typename V4<T>::type *>(p));
+}
 template <typename T>
 __device__ __forceinline__ typename V4<T>::type ld_cached4(const T *p) {
     return __ldg(reinterpret_cast<const typename V4<T>::type *>(p));
@@ -63,6 +70,14 @@ __device__ __forceinline__ typename V4<T>::type ld_cached4(const T *p) {
 __device__ __forceinline__ unsigned long long ld_status(const unsigned long long *p) {
     unsigned long long v;
     asm volatile("ld.relaxed.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+// System-scope acquire: data published before the word (H2D pieces ahead of the arrival-front
+// memop on the same stream) is visible to this thread's later loads, and -- through the CTA
+// barrier that follows -- to the CTA's.
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ unsigned long long globaltimer() {
@@ -392,7 +407,7 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
                 const unsigned long long t0 = globaltimer();
                 unsigned int ns = 128;
                 for (;;) {
-                    const unsigned long long a = ld_status(c.arrival);
+                    const unsigned long long a = ld_acquire_sys(c.arrival);
                     const unsigned int front = ((unsigned int)(a >> 32) == c.epoch) ? (unsigned int)a : 0u;
                     if ((unsigned long long)key < (unsigned long long)front) break;
                     const unsigned int wv = decode_w(ld_status(c.status), c);
@@ -588,10 +603,15 @@ struct RowDotBody {
     struct Params {
         const T *A; const T *B; const T *x; T *out0; T *out1;
         long long nrows, ncols, lws; int R; T alpha, beta; int vec4;
+        int streamed;   // A/B rows arrive by H2D pieces during the kernel: loads through L2 only
     };
     typedef EmptySmem Smem;
 
     __device__ static long long key(const Params &p, long long t) { return (t * p.R) / p.lws; }
+    template <bool CG>
+    __device__ static typename V4<T>::type ldm4(const T *q) { return CG ? ld_cg4(q) : ld_stream4(q); }
+    template <bool CG>
+    __device__ static T ldm(const T *q) { return CG ? __ldcg(q) : *q; }
 
     __device__ static T warp_fold(T p0, T p1, T p2, T p3) {
         T v = op_add(op_add(op_add(p0, p1), p2), p3);
@@ -600,7 +620,11 @@ struct RowDotBody {
         return v;
     }
 
-    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
+    __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &sm) {
+        return p.streamed ? run_t<true>(p, t, tc, sm) : run_t<false>(p, t, tc, sm);
+    }
+    template <bool CG>
+    __device__ static bool run_t(const Params &p, long long t, TaskCtx &, Smem &) {
         const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
         for (int r = warp; r < p.R; r += kWarps) {
             const long long i = t * p.R + r;
@@ -618,8 +642,8 @@ struct RowDotBody {
                     typename V4<T>::type av[U], bv[U], xv[U];
 #pragma unroll
                     for (int u = 0; u < U; ++u) {
-                        av[u] = ld_stream4(pa + u * 128);
-                        if (NMAT == 2) bv[u] = ld_stream4(pb + u * 128);
+                        av[u] = ldm4<CG>(pa + u * 128);
+                        if (NMAT == 2) bv[u] = ldm4<CG>(pb + u * 128);
                     }
                     if (NMAT == 2) pb += U * 128;
 #pragma unroll
@@ -636,11 +660,11 @@ struct RowDotBody {
                 }
                 for (; k < nfull; ++k) {
                     const long long j = k * 128 + 4 * lane;
-                    typename V4<T>::type av = ld_stream4(Ar + j), xv = ld_cached4(p.x + j);
+                    typename V4<T>::type av = ldm4<CG>(Ar + j), xv = ld_cached4(p.x + j);
                     a0 = op_fma(av.x, xv.x, a0); a1 = op_fma(av.y, xv.y, a1);
                     a2 = op_fma(av.z, xv.z, a2); a3 = op_fma(av.w, xv.w, a3);
                     if (NMAT == 2) {
-                        typename V4<T>::type bv = ld_stream4(Br + j);
+                        typename V4<T>::type bv = ldm4<CG>(Br + j);
                         b0 = op_fma(bv.x, xv.x, b0); b1 = op_fma(bv.y, xv.y, b1);
                         b2 = op_fma(bv.z, xv.z, b2); b3 = op_fma(bv.w, xv.w, b3);
                     }
@@ -652,8 +676,8 @@ struct RowDotBody {
 #define FCL_ROWDOT_TAIL(C, AC, BC)                                             \
                 if (j + C < p.ncols) {                                         \
                     const T xv = p.x[j + C];                                   \
-                    AC = op_fma(Ar[j + C], xv, AC);                            \
-                    if (NMAT == 2) BC = op_fma(Br[j + C], xv, BC);             \
+                    AC = op_fma(ldm<CG>(Ar + j + C), xv, AC);                  \
+                    if (NMAT == 2) BC = op_fma(ldm<CG>(Br + j + C), xv, BC);   \
                 }
                 FCL_ROWDOT_TAIL(0, a0, b0)
                 FCL_ROWDOT_TAIL(1, a1, b1)
@@ -1411,6 +1435,7 @@ static typename RowDotBody<T, NMAT>::Params rowdot_params(const KArgs &a, const 
     if (a.integer) { p.alpha = (T)a.ialpha; p.beta = (T)a.ibeta; }
     else { p.alpha = (T)a.alpha; p.beta = (T)a.beta; }
     p.vec4 = (p.ncols % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.x) && (NMAT == 1 || is_aligned16(p.B));
+    p.streamed = a.streamed ? 1 : 0;
     return p;
 }
 
@@ -1689,7 +1714,7 @@ int gpu_launch_copies(int n, void *const *dst, const void *const *src, const siz
     size_t total = 0;
     L.n = n;
     for (int b = 0; b < n && b < 6; ++b) {
-        if ((reinterpret_cast<uintptr_t>(dst[b]) | reinterpret_cast<uintptr_t>(src[b])) & 15u) return -1;
+        if ((reinterpret_cast<uintptr_t>(dst[b]) | reinterpret_cast<uintptr_t>(src[b])) & 15u) return -2;
         L.dst[b] = (uint8_t *)dst[b]; L.src[b] = (const uint8_t *)src[b]; L.bytes[b] = bytes[b];
         total += bytes[b];
     }

@@ -446,6 +446,11 @@ struct fcl_context_st {
     bool stream_on = true;                       // FCL_NO_STREAM=1: stale inputs are copied whole first
     unsigned long long *darrival = nullptr;
     cudaEvent_t stream_ev[4] = {};
+    // hd position after the last piece of the last streamed launch: pieces still in flight read
+    // the pinned mirror and write the device copy, so a later write of the mirror
+    // (fcl_write_buffer) or a refresh of the device copy (make_valid) waits for it
+    cudaEvent_t ev_stream_done = nullptr;
+    bool stream_pending = false;                 // set by phase B, read after drain()
     size_t stream_piece_bytes = 8u << 20;        // FCL_STREAM_PIECE_BYTES
     // Return race: when the GPU finishes first and a large output is still to come
     // back, it is returned in ascending pieces while the host keeps computing from the top.
@@ -652,6 +657,9 @@ fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_d
         }
     }
     if (need_dev && !b->dev_valid) {
+        if (ctx->stream_pending) {   // pieces of a streamed launch may still write this device copy
+            CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_stream_done, 0));
+        }
         ctx->main_fenced.store(1);
         CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
         ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)b->bytes;
@@ -821,17 +829,29 @@ fcl_status flush_returns(fcl_context ctx, bool at_finish) {
         sz[k] = b->ret_b1 - b->ret_b0;
     }
     ctx->main_fenced.store(1);   // a copy between grids on main: the next grid is ordinary
-    cudaMemcpyAttributes at = {};
-    at.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-    at.srcLocHint.type = cudaMemLocationTypeDevice; at.srcLocHint.id = ctx->device;
-    at.dstLocHint.type = cudaMemLocationTypeHost; at.dstLocHint.id = 0;
-    size_t aidx = 0, fail = 0;
     for (size_t k = 0; k < n; ++k) ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)sz[k];
-    if (n == 1 || cudaMemcpyBatchAsync(dst.data(), src.data(), sz.data(), n, &at, &aidx, 1, &fail, ctx->main) != cudaSuccess) {
-        cudaGetLastError();   // (a driver without batched copies: one copy per buffer)
+    // One gather kernel stores every span through the mapped host mirrors (16-byte SM stores
+    // over PCIe, posted): one launch instead of one copy-engine transfer per buffer.  Spans that
+    // are not 16-byte aligned, buffers without a mapping, or more than 6 spans: one
+    // cudaMemcpyAsync per span.
+    bool gathered = false;
+    if (n <= 6) {
+        std::vector<void *> hdst(n);
+        bool ok = true;
+        for (size_t k = 0; k < n && ok; ++k) {
+            fcl_buffer b = ctx->lazy[k];
+            ok = b->host_dptr != nullptr;
+            if (ok) hdst[k] = (char *)b->host_dptr + b->ret_b0;
+        }
+        if (ok) {
+            const int r = gpu_launch_copies((int)n, hdst.data(), (const void *const *)src.data(), sz.data(), ctx->num_sms, ctx->main);
+            if (r == -1) return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+            gathered = r >= 0;   // (-2: a span is not 16-byte aligned)
+        }
+    }
+    if (!gathered)
         for (size_t k = 0; k < n; ++k)
             CK(ctx, cudaMemcpyAsync(dst[k], src[k], sz[k], cudaMemcpyDeviceToHost, ctx->main));
-    }
     for (size_t k = 0; k < n; ++k) {
         fcl_buffer b = ctx->lazy[k];
         b->ret_lazy = false;
@@ -1562,6 +1582,10 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         busy += now_ms() - t_start;
         ex.abort_flag = 0;
     }
+    if (j.stream && s_sent > L.lo) {   // up to two pieces may still be in flight on hd
+        CK(ctx, cudaEventRecord(ctx->ev_stream_done, ctx->hd));
+        ctx->stream_pending = true;
+    }
     info.t_host_ms = busy;
     info.n_chunks = nch;
     variant_info(vp, info);
@@ -1846,7 +1870,7 @@ fcl_status fcl_default_launch_opts(fcl_launch_opts *o) {
     o->cpu_wg_split = 1;
     o->abort_period = 0;
     o->wg_lo = 0;
-    o->wg_hi = 0;
+    o->wg_hi = -1;
     o->blocking = 0;
     o->host_variant = -1;
     return FCL_SUCCESS;
@@ -1943,7 +1967,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     ctx->darrival = (unsigned long long *)dp;
     for (cudaEvent_t *pe : {&ctx->ev_k1, &ctx->ev_mark, &ctx->ev_hd_release, &ctx->ev_gd2h, &ctx->race_ev[0], &ctx->race_ev[1],
                             &ctx->race_ev[2], &ctx->race_ev[3], &ctx->stream_ev[0], &ctx->stream_ev[1], &ctx->stream_ev[2],
-                            &ctx->stream_ev[3]})
+                            &ctx->stream_ev[3], &ctx->ev_stream_done})
         if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess) return fail(e, "events");
     // stream memory operations for publication (driver entry point; fall back to a kernel store)
     {
@@ -2031,7 +2055,8 @@ fcl_status fcl_release_context(fcl_context ctx) {
         delete j;
     }
     for (cudaEvent_t e : {ctx->ev_k0, ctx->ev_t1, ctx->ev_k1, ctx->ev_mark, ctx->ev_hd_release, ctx->ev_gd2h, ctx->race_ev[0],
-                          ctx->race_ev[1], ctx->race_ev[2], ctx->race_ev[3]})
+                          ctx->race_ev[1], ctx->race_ev[2], ctx->race_ev[3], ctx->stream_ev[0], ctx->stream_ev[1],
+                          ctx->stream_ev[2], ctx->stream_ev[3], ctx->ev_stream_done})
         if (e) cudaEventDestroy(e);
     if (ctx->status_host) cudaFreeHost(ctx->status_host);
     else if (ctx->status_dptr) cudaFree(ctx->status_dptr);
@@ -2154,8 +2179,13 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
         s = make_valid(ctx, b, true, true, nullptr);
         if (s != FCL_SUCCESS) return s;
     }
-    // overwriting the pinned mirror: no queued copy may still read its old contents
+    // overwriting the pinned mirror: no queued copy may still read its old contents (main, and
+    // the pieces of a streamed launch on hd)
     if (src != h) CK(ctx, cudaStreamSynchronize(ctx->main));
+    if (ctx->stream_pending) {
+        CK(ctx, cudaEventSynchronize(ctx->ev_stream_done));
+        ctx->stream_pending = false;
+    }
     if (src != h) std::memcpy(h, src, n);
     if (!blocking && n == b->bytes) {
         // a non-blocking write of the whole buffer refreshes the device copy lazily, when a
@@ -2329,8 +2359,9 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
     if (o.mode < FCL_MODE_COOP || o.mode > FCL_MODE_CPU_ONLY) return set_err(ctx, FCL_INVALID_VALUE, "mode");
     if (o.host_variant >= host_num_variants(a.kernel))
         return set_err(ctx, FCL_INVALID_VALUE, "host_variant %d: %s has %d", o.host_variant, kd->name, host_num_variants(a.kernel));
-    int64_t lo = o.wg_lo, hi = o.wg_hi > 0 ? o.wg_hi : g.n_wg;
-    if (lo < 0 || hi > g.n_wg || lo >= hi) return set_err(ctx, FCL_INVALID_VALUE, "wg range [%lld, %lld)", (long long)lo, (long long)hi);
+    // wg_hi < 0: the whole NDRange; wg_lo == wg_hi: an empty slice (nothing runs)
+    int64_t lo = o.wg_lo, hi = o.wg_hi >= 0 ? o.wg_hi : g.n_wg;
+    if (lo < 0 || hi > g.n_wg || lo > hi) return set_err(ctx, FCL_INVALID_VALUE, "wg range [%lld, %lld)", (long long)lo, (long long)hi);
     const int64_t al = gpu_slice_align(a, g);
     if ((lo % al) || (hi % al && hi != g.n_wg))
         return set_err(ctx, FCL_INVALID_VALUE, "wg range must be aligned to %lld work-groups (fcl_slice_range)", (long long)al);
@@ -2350,6 +2381,14 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     Launch L{};
     s = build_launch(ctx, kernel, work_dim, gws, lws, args, n_args, opts, L);
     if (s != FCL_SUCCESS) return s;
+    if (L.hi == L.lo) {   // an empty slice (a rank with no work-groups): nothing to run
+        if (info_out) {
+            std::memset(info_out, 0, sizeof *info_out);
+            info_out->wg_lo = info_out->wg_hi = info_out->gpu_watermark = info_out->published_watermark = L.lo;
+            info_out->host_variant = -1;
+        }
+        return FCL_SUCCESS;
+    }
     if (!ctx->defer_list.empty()) {
         drain(ctx);
         if (!ctx->defer_list.empty()) return set_err(ctx, FCL_INVALID_VALUE, "a deferred merge is pending (call fcl_merge)");
@@ -2440,7 +2479,9 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     info.gpu_watermark = info.published_watermark = L.hi;
     // Streamed inputs (§6.7): the row-partitioned matrices of a row-dot kernel whose device copy
     // is stale go to the GPU in ascending row pieces while the host computes from the top.
-    if (ctx->stream_on && (L.a.kernel == K_GESUMMV || L.a.kernel == K_ATAX_TMP || L.a.kernel == K_BICG_Q) &&
+    // (the arrival front must be a stream memop: a store kernel could wait for an SM the
+    // grid it signals occupies)
+    if (ctx->stream_on && ctx->write64 && (L.a.kernel == K_GESUMMV || L.a.kernel == K_ATAX_TMP || L.a.kernel == K_BICG_Q) &&
         L.g.work_dim == 1 && L.g.lws[0] % 4 == 0 && L.o.forced_split < 0 && !L.o.defer_merge &&
         !L.o.drop_publish) {   // (the GPU waits for pieces or for the watermark: both must come)
         for (int k = 0; k < L.a.nbuf; ++k) {
@@ -2450,6 +2491,7 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
                 j->sbuf[j->nstream++] = k;
         }
         j->stream = j->nstream > 0;
+        j->L.a.streamed = j->stream;
     }
     for (int k = 0; k < L.a.nbuf; ++k) {
         fcl_buffer b = L.bufs[k];
@@ -2479,6 +2521,9 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         ctx->free_jobs.push_back(j);
         return s;
     }
+    // what is known at return, copied before the coordinator may start writing the job's info
+    info.t_call_ms = now_ms() - t_call;
+    if (info_out && !L.o.blocking) *info_out = info;
     {
         std::lock_guard<std::mutex> lk(ctx->q_mu);
         if (ctx->last && ctx->last != j && ctx->last->done.load()) ctx->free_jobs.push_back(ctx->last);
@@ -2491,9 +2536,9 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     if (L.o.blocking) {
         drain(ctx);
         s = j->status;
+        info.t_call_ms = now_ms() - t_call;
+        if (info_out) *info_out = info;   // (complete: the host side is done)
     }
-    info.t_call_ms = now_ms() - t_call;
-    if (info_out) *info_out = info;
     return s;
 }
 
@@ -2643,22 +2688,23 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info) {
         float ms = 0.f;
         if (cudaEventSynchronize(j->ev_t1) == cudaSuccess && cudaEventElapsedTime(&ms, j->ev_k0, j->ev_t1) == cudaSuccess)
             j->info.t_gpu_kernel_ms = ms;
-        // the watermark of a cooperative launch whose host side did not need it (valid while
-        // no later dispatcher has run: this is the most recent launch and the queue is drained)
-        if (j->wm_pending) {
-            int64_t wm = j->L.hi;
-            if (read_gpu_watermark(ctx, *j, &wm) == FCL_SUCCESS) {
-                j->info.gpu_watermark = wm;
-                j->info.merged = wm < j->L.hi;
-                if (wm <= j->L.lo) j->info.cpu_did_all = 1;
-            }
-            j->wm_pending = false;
+    }
+    // the watermark of a cooperative launch whose host side did not need it (valid while no
+    // later dispatcher has run: this is the most recent launch and the queue is drained) --
+    // resolved for every launch, timed or not
+    if (j->wm_pending) {
+        int64_t wm = j->L.hi;
+        if (read_gpu_watermark(ctx, *j, &wm) == FCL_SUCCESS) {
+            j->info.gpu_watermark = wm;
+            j->info.merged = wm < j->L.hi;
+            if (wm <= j->L.lo) j->info.cpu_did_all = 1;
         }
-        if (ctx->stats && j->info.gpu_tasks < 0) {
-            unsigned long long nt = 0;
-            if (cudaMemcpy(&nt, ctx->dtasks + j->slot, 8, cudaMemcpyDeviceToHost) == cudaSuccess)
-                j->info.gpu_tasks = (int64_t)nt;
-        }
+        j->wm_pending = false;
+    }
+    if (ctx->stats && j->gpu_launched && j->info.gpu_tasks < 0) {
+        unsigned long long nt = 0;
+        if (cudaMemcpy(&nt, ctx->dtasks + j->slot, 8, cudaMemcpyDeviceToHost) == cudaSuccess)
+            j->info.gpu_tasks = (int64_t)nt;
     }
     if (j->have_m) {
         float ms = 0.f;

@@ -224,7 +224,7 @@ class Kernel:
 
 def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg_split=1,
               abort_period=0, defer_merge=0, n_host_threads=0, host_delay_us=0, drop_publish=0,
-              wg_lo=0, wg_hi=0, blocking=0, timing=0, host_variant=-1, select=0) -> LaunchOpts:
+              wg_lo=0, wg_hi=-1, blocking=0, timing=0, host_variant=-1, select=0) -> LaunchOpts:
     o = LaunchOpts()
     load().fcl_default_launch_opts(ctypes.byref(o))
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)

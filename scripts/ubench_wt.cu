@@ -52,34 +52,6 @@ int main() {
         printf("  3 x cudaMemcpyAsync D2H (1/3 each) %7.2f us\n", time_it([&] {
             for (int k = 0; k < 3; ++k) CK(cudaMemcpyAsync((char *)h + k * bytes / 3, (char *)d + k * bytes / 3, bytes / 3, cudaMemcpyDeviceToHost, 0));
         }));
-        {
-            void *dsts[3], *srcs[3]; size_t sizes[3];
-            for (int k = 0; k < 3; ++k) { dsts[k] = (char *)h + k * bytes / 3; srcs[k] = (char *)d + k * bytes / 3; sizes[k] = bytes / 3; }
-            cudaMemcpyAttributes at = {};
-            at.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-            at.srcLocHint.type = cudaMemLocationTypeDevice; at.srcLocHint.id = 0;
-            at.dstLocHint.type = cudaMemLocationTypeHost; at.dstLocHint.id = 0;
-            size_t aidx = 0, fail = 0;
-            cudaStream_t st; CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
-            cudaError_t e = cudaMemcpyBatchAsync(dsts, srcs, sizes, 3, &at, &aidx, 1, &fail, st);
-            CK(cudaStreamSynchronize(st));
-            if (e != cudaSuccess) { printf("  batch: %s\n", cudaGetErrorString(e)); cudaGetLastError(); }
-            else {
-                cudaEvent_t e0, e1; CK(cudaEventCreate(&e0)); CK(cudaEventCreate(&e1));
-                std::vector<float> ts;
-                for (int r = 0; r < 55; ++r) {
-                    CK(cudaStreamSynchronize(st));
-                    CK(cudaEventRecord(e0, st));
-                    CK(cudaMemcpyBatchAsync(dsts, srcs, sizes, 3, &at, &aidx, 1, &fail, st));
-                    CK(cudaEventRecord(e1, st));
-                    CK(cudaEventSynchronize(e1));
-                    float ms; CK(cudaEventElapsedTime(&ms, e0, e1));
-                    if (r >= 5) ts.push_back(ms * 1e3f);
-                }
-                std::sort(ts.begin(), ts.end());
-                printf("  cudaMemcpyBatchAsync 3 pieces      %7.2f us\n", ts[ts.size() / 2]);
-            }
-        }
         CK(cudaFree(d)); CK(cudaFreeHost(h));
     }
     return 0;
