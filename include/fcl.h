@@ -208,6 +208,12 @@ typedef struct {
                                 first on an idle GPU; every FCL_SELECT_PERIOD-th (16) launch
                                 of the shape probes cooperatively again.  Forced splits, deferred
                                 merges and fault injection are never redirected. */
+    int32_t gpu_delay_us;        /* fault injection: in a COOP launch every GPU task starts this many us
+                                    late (a slow GPU, so that the host covers part of the range in a
+                                    free-running race); such a launch runs the persistent dispatcher */
+    int32_t record_exec_counts;  /* test hook (1 = on): count, per work-group, how often each device
+                                    executed it to completion -- read with fcl_get_exec_counts after
+                                    fcl_finish.  The launch first waits for pending launches. */
 } fcl_launch_opts;
 
 #define FCL_SELECT_OFF     (-1)
@@ -256,6 +262,10 @@ typedef struct {
     int32_t probe;               /* 1 = this cooperative launch refreshes the selection profile */
     int64_t streamed_wgs;        /* work-groups whose stale input rows were streamed to the GPU in
                                     pieces while the host computed */
+    double  chunk_ms[64];        /* host time of each started chunk (chunk_sizes order) that completed;
+                                    0 = abandoned.  The first n_c11_chunks are the C11 chunks, timed
+                                    exactly as the heuristic saw them (L18.s23-32) */
+    int32_t n_c11_chunks;        /* chunks sized by C11; the rest of n_chunks are return-race chunks */
 } fcl_launch_info;
 
 /* info.selected */
@@ -316,6 +326,20 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info);
 #define FCL_COUNT_D2H_BYTES  7  /* bytes copied device -> host (returns, reads) */
 #define FCL_COUNT_N          8
 fcl_status fcl_get_counters(fcl_context ctx, int64_t *counts, int32_t n);
+
+/* Per-work-group execution counts of the most recent launch made with opts.record_exec_counts
+ * (test hook; north_star's invariant "every output word is written by exactly one
+ * device", L16.s9 "non-overlapping parts").  Arrays of n >= the NDRange's work-group count,
+ * indexed by flattened id (Fig 5); entries outside the launch's [wg_lo, wg_hi) are 0.
+ *   gpu_done[f]  : completed GPU task fragments that stored work-group f's outputs
+ *   gpu_frags[f] : GPU task fragments covering f (a tile task spans several work-groups, a
+ *                  row/column-dot task is a part of one: f ran completely on the GPU iff
+ *                  gpu_done[f] == gpu_frags[f], and not at all iff gpu_done[f] == 0)
+ *   cpu_done[f]  : host executions of f that completed (all its parts stored)
+ * Any pointer may be NULL.  Waits for the context (like fcl_finish).
+ * Errors: FCL_INVALID_CONTEXT; FCL_INVALID_VALUE (no recorded launch, n too small). */
+fcl_status fcl_get_exec_counts(fcl_context ctx, int64_t n, int32_t *gpu_done, int32_t *gpu_frags,
+                               int32_t *cpu_done);
 
 /* Multi-GPU slicing helper: a contiguous flattened-id range for
  * rank `rank` of `nranks`, balanced and aligned to the kernel's GPU task

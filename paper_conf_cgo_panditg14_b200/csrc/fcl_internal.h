@@ -13,6 +13,7 @@
 #pragma once
 #include <cstddef>
 #include <cstdint>
+#include <vector>
 
 typedef struct CUstream_st *cudaStream_t_fwd;
 
@@ -54,6 +55,9 @@ struct KArgs {
     // Row-dot inputs streamed to the device in pieces while the grid runs: the
     // body loads them through L2 only
     bool streamed;
+    // Test hook (opts.record_exec_counts): per work-group host completions, counted by the
+    // executor (rec_parts: parts of a split work-group done so far).  nullptr = off.
+    int32_t *rec_cpu_done, *rec_cpu_parts;
 };
 
 // Device-side merge of a cooperative launch's output buffers (domain read from wm_word).
@@ -99,6 +103,9 @@ struct CoopCtl {
     // device.  nullptr: every input is resident.  A task waits for its rows or for the host to
     // cover it.
     const unsigned long long *arrival;
+    unsigned long long task_delay_ns;   // fault injection (opts.gpu_delay_us): every task starts late
+    unsigned int *exec_cnt;             // test hook: per task (index - task_lo) completions, or nullptr
+    unsigned int *exec_w;               // ... and the work-group mask the task ran with
 };
 
 // Decode the dispatcher's wm word: the lowest watermark launch `epoch` acted on, or
@@ -120,6 +127,9 @@ struct TaskSpace {
 };
 TaskSpace gpu_task_space(const KArgs &a, const Geom &g);
 int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t);   // min fgid of task t
+// Work-groups task t writes outputs of (a tile spans several; row/column dot tasks are part of
+// one; SYRK's upper-triangle tiles also their mirror block), appended to `out`.
+void gpu_task_wgs(const KArgs &a, const Geom &g, int64_t t, std::vector<int64_t> &out);
 bool gpu_geometry_ok(const KArgs &a, const Geom &g, const char **why);
 int gpu_default_abort_period(const KArgs &a);
 // Slice boundaries (multi-GPU / wg_lo, wg_hi) must be multiples of this many work-groups
@@ -140,6 +150,7 @@ struct SlotReset {
     unsigned int epoch;
     unsigned long long *tstamp;   // optional (stats): [block-0 start, last CTA end] %globaltimer
     unsigned long long delay_ns;  // test hook (FCL_TEST_GPU_DELAY_US): block 0 idles this long first
+    unsigned int *exec_cnt;       // test hook: per block completions (opts.record_exec_counts), or nullptr
 };
 // pdl: PDL_OFF = ordinary launch; PDL_NOWAIT = programmatic stream serialization, the grid may
 // start while the previous plain grid drains and does not wait for it (the runtime found no
@@ -171,14 +182,15 @@ const char *gpu_last_error_string();
 // Execute part `part` of `nparts` of work-group `fgid` on host memory (C9 / C23).
 // `abort_flag` is polled inside long bodies; a body that sees it set stops before
 // storing an incomplete value (write-once).
-void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts,
+// Returns true when the part completed (every output stored), false when the abort flag stopped it.
+bool host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts,
                   const volatile int *abort_flag);
 // Alternate host bodies (C26): how many a kernel has and their names ("cpu", "wi").
 int host_num_variants(int kernel);
 const char *host_variant_name(int kernel, int v);
 // Work-groups per executor claim (host_exec_range) and the range executor itself.
 int64_t host_batch(const KArgs &a, const Geom &g);
-void host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *abort_flag);
+bool host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *abort_flag);
 
 // Conservative contiguous byte span [*b0, *b1) of output buffer `buf_index` written by
 // work-groups [lo, hi) (superset of the exact footprint; the diff-merge tolerates it).

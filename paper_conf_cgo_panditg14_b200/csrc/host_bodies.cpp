@@ -61,12 +61,12 @@ bool rowdot(const T *Ar, const T *x, int64_t ncols, const volatile int *ab, T *r
 }
 
 template <typename T>
-void wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t lws = g.lws[0];
     const bool ges = (a.kernel == K_GESUMMV);
     const int64_t nrows = a.n0, ncols = ges ? a.n0 : a.n1;
     const int64_t r0 = fgid * lws, r1 = std::min<int64_t>(r0 + lws, nrows);
-    if (r0 >= r1) return;
+    if (r0 >= r1) return true;
     int64_t lo, hi;
     part_range(r1 - r0, part, nparts, lo, hi);
     const T *A = (const T *)a.host[0];
@@ -75,7 +75,7 @@ void wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
         T *out = (T *)a.host[2];
         for (int64_t i = r0 + lo; i < r0 + hi; ++i) {
             T v;
-            if (!rowdot<T>(A + i * ncols, x, ncols, ab, &v)) return;
+            if (!rowdot<T>(A + i * ncols, x, ncols, ab, &v)) return false;
             out[i] = v;
         }
     } else {
@@ -86,11 +86,12 @@ void wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
         const T beta = a.integer ? (T)(uint32_t)a.ibeta : (T)a.beta;
         for (int64_t i = r0 + lo; i < r0 + hi; ++i) {
             T va, vb;
-            if (!rowdot<T>(A + i * ncols, x, ncols, ab, &va) || !rowdot<T>(B + i * ncols, x, ncols, ab, &vb)) return;
+            if (!rowdot<T>(A + i * ncols, x, ncols, ab, &va) || !rowdot<T>(B + i * ncols, x, ncols, ab, &vb)) return false;
             tmp[i] = va;
             y[i] = op_add(op_mul(alpha, va), op_mul(beta, vb));
         }
     }
+    return true;
 }
 
 // ---------------------------------------------------------------- col-dot (ATAX k2, BICG k1, CORR mean/std)
@@ -99,14 +100,14 @@ void wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
 enum { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
 
 template <typename T, int MODE>
-void wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t lws = g.lws[0];
     const int64_t nrows = a.n0, ncols = a.n1;
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, ncols);
-    if (c0 >= c1) return;
+    if (c0 >= c1) return true;
     int64_t lo, hi;
     part_range(c1 - c0, part, nparts, lo, hi);
-    if (lo >= hi) return;
+    if (lo >= hi) return true;
     const int64_t pc0 = c0 + lo, w = hi - lo;
     const T *A = (const T *)a.host[0];
     const T *v = (MODE == COL_DOT) ? (const T *)a.host[1] : nullptr;
@@ -115,7 +116,7 @@ void wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
     thread_local std::vector<T> P;
     P.assign((size_t)kColPartitions * (size_t)w, T(0));
     for (int64_t i = 0; i < nrows; ++i) {
-        if ((i & 31) == 0 && aborted(ab)) return;
+        if ((i & 31) == 0 && aborted(ab)) return false;
         T *pq = P.data() + (size_t)(i & (kColPartitions - 1)) * (size_t)w;
         const T *ar = A + i * ncols + pc0;
         if (MODE == COL_DOT) {
@@ -143,6 +144,7 @@ void wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
             out[pc0 + jj] = (T)((s <= a.eps) ? 1.0f : s);
         }
     }
+    return true;
 }
 
 // ---------------------------------------------------------------- 2-D work-group geometry helpers
@@ -158,32 +160,33 @@ inline Wg2D wg2d(const Geom &g, int64_t fgid, int64_t nrows, int64_t ncols) {
 // ---------------------------------------------------------------- CORR reduce (in place)
 // Rectangle [r0, r1) x [c0, c1) of the output (a work-group, or a batch of work-groups of one
 // work-group row: wide rows stream and vectorize).
-void corr_reduce_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
+bool corr_reduce_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
     float *d = (float *)a.host[0];
     const float *mean = (const float *)a.host[1], *sd = (const float *)a.host[2];
     const float sqrtn = std::sqrt((float)n);
     for (int64_t i = r0; i < r1; ++i) {
-        if (aborted(ab)) return;
+        if (aborted(ab)) return false;
         for (int64_t j = c0; j < c1; ++j) {
             const float den = sqrtn * sd[j];
             d[i * m + j] = (d[i * m + j] + (-mean[j])) / den;
         }
     }
+    return true;
 }
 
-void wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     Wg2D w = wg2d(g, fgid, a.n0, a.n1);
-    if (w.r0 >= w.r1 || w.c0 >= w.c1) return;
+    if (w.r0 >= w.r1 || w.c0 >= w.c1) return true;
     int64_t lo, hi;
     part_range(w.r1 - w.r0, part, nparts, lo, hi);
-    corr_reduce_rect(a, w.r0 + lo, w.r0 + hi, w.c0, w.c1, ab);
+    return corr_reduce_rect(a, w.r0 + lo, w.r0 + hi, w.c0, w.c1, ab);
 }
 
 // ---------------------------------------------------------------- 2DCONV
 // Rectangle [r0, r1) x [c0, c1) of the output, border excluded by the caller.
 template <typename T>
-void conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
+bool conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
     const int64_t nj = a.n1;
     const T *A = (const T *)a.host[0];
     T *B = (T *)a.host[1];
@@ -196,7 +199,7 @@ void conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1,
         for (int q = 0; q < 9; ++q) c[q] = (T)cf[q];
     }
     for (int64_t i = r0; i < r1; ++i) {
-        if (aborted(ab)) return;
+        if (aborted(ab)) return false;
         const T *um = A + (i - 1) * nj, *u0 = A + i * nj, *up = A + (i + 1) * nj;
         for (int64_t j = c0; j < c1; ++j) {
             T s = op_mul(c[0], um[j - 1]);
@@ -211,38 +214,39 @@ void conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1,
             B[i * nj + j] = s;
         }
     }
+    return true;
 }
 
 template <typename T>
-void wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t ni = a.n0, nj = a.n1;
     Wg2D w = wg2d(g, fgid, ni, nj);
     const int64_t r0 = std::max<int64_t>(w.r0, 1), r1 = std::min<int64_t>(w.r1, ni - 1);
     const int64_t c0 = std::max<int64_t>(w.c0, 1), c1 = std::min<int64_t>(w.c1, nj - 1);
-    if (r0 >= r1 || c0 >= c1) return;
+    if (r0 >= r1 || c0 >= c1) return true;
     int64_t lo, hi;
     part_range(r1 - r0, part, nparts, lo, hi);
-    conv2d_rect<T>(a, r0 + lo, r0 + hi, c0, c1, ab);
+    return conv2d_rect<T>(a, r0 + lo, r0 + hi, c0, c1, ab);
 }
 
 // ---------------------------------------------------------------- SYRK / SYR2K
 // Each output accumulates its k-chain in ascending k, one fma per term (SYR2K: A_i*B_j then
 // B_i*A_j for each k), then C = fma(alpha, acc, beta * C).  Mirrors GemmBody in kernels.cu.
 template <typename T, bool TWO>
-void wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
     Wg2D w = wg2d(g, fgid, n, n);
-    if (w.r0 >= w.r1 || w.c0 >= w.c1) return;
+    if (w.r0 >= w.r1 || w.c0 >= w.c1) return true;
     const int64_t nr = w.r1 - w.r0, nc = w.c1 - w.c0;
     // split the work-group's outputs into (row group x column group) parts
     const int nrg = (int)std::min<int64_t>(nparts, nr);
     const int ncg = (int)std::max<int64_t>(1, std::min<int64_t>(nparts / nrg, (nc + 7) / 8));
-    if (part >= nrg * ncg) return;
+    if (part >= nrg * ncg) return true;
     int64_t rlo, rhi, clo, chi;
     part_range(nr, part / ncg, nrg, rlo, rhi);
     part_range(nc, part % ncg, ncg, clo, chi);
     const int64_t j0 = w.c0 + clo, wc = chi - clo;
-    if (rlo >= rhi || wc <= 0) return;
+    if (rlo >= rhi || wc <= 0) return true;
     const T *A = (const T *)a.host[0];
     const T *B = TWO ? (const T *)a.host[1] : nullptr;
     T *C = (T *)a.host[TWO ? 2 : 1];
@@ -252,25 +256,25 @@ void wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, 
     thread_local std::vector<T> At, Bt, acc;
     At.resize((size_t)m * (size_t)wc);
     for (int64_t jj = 0; jj < wc; ++jj) {
-        if (aborted(ab)) return;
+        if (aborted(ab)) return false;
         for (int64_t k = 0; k < m; ++k) At[(size_t)(k * wc + jj)] = A[(j0 + jj) * m + k];
     }
     if (TWO) {
         Bt.resize((size_t)m * (size_t)wc);
         for (int64_t jj = 0; jj < wc; ++jj) {
-            if (aborted(ab)) return;
+            if (aborted(ab)) return false;
             for (int64_t k = 0; k < m; ++k) Bt[(size_t)(k * wc + jj)] = B[(j0 + jj) * m + k];
         }
     }
     acc.resize((size_t)wc);
     for (int64_t i = w.r0 + rlo; i < w.r0 + rhi; ++i) {
-        if (aborted(ab)) return;
+        if (aborted(ab)) return false;
         std::fill(acc.begin(), acc.end(), T(0));
         T *ac = acc.data();
         const T *ai = A + i * m;
         const T *bi = TWO ? B + i * m : nullptr;
         for (int64_t k = 0; k < m; ++k) {
-            if ((k & 511) == 511 && aborted(ab)) return;   // write-once: nothing stored yet
+            if ((k & 511) == 511 && aborted(ab)) return false;   // write-once: nothing stored yet
             const T aik = ai[k];
             if (TWO) {
                 const T bik = bi[k];
@@ -287,16 +291,17 @@ void wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, 
         T *ci = C + i * n + j0;
         for (int64_t jj = 0; jj < wc; ++jj) ci[jj] = op_fma(alpha, ac[jj], op_mul(beta, ci[jj]));
     }
+    return true;
 }
 
 // ---------------------------------------------------------------- CORR symmat
 // symmat[j1][j2] = symmat[j2][j1] = sum_i d[i][j1] * d[i][j2] (j2 > j1, ascending i, fma
 // chain); symmat[j1][j1] = 1.  Work-items j1 processed in blocks of 8 for row reuse.
-void wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
     const int64_t lws = g.lws[0];
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, m);
-    if (c0 >= c1) return;
+    if (c0 >= c1) return true;
     int64_t lo, hi;
     part_range(c1 - c0, part, nparts, lo, hi);
     const float *d = (const float *)a.host[0];
@@ -310,7 +315,7 @@ void wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
         if (width > 0) {
             acc.assign((size_t)nb * (size_t)width, 0.0f);
             for (int64_t i = 0; i < n; ++i) {
-                if ((i & 63) == 0 && aborted(ab)) return;
+                if ((i & 63) == 0 && aborted(ab)) return false;
                 const float *row = d + i * m;
                 for (int b = 0; b < nb; ++b) {
                     const int64_t j1 = jb + b;
@@ -330,6 +335,7 @@ void wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
             }
         }
     }
+    return true;
 }
 
 // ---------------------------------------------------------------- work-item-order variants
@@ -342,11 +348,11 @@ void wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
 
 // col-dot: work-item j walks its column, partition by partition
 template <typename T, int MODE>
-void wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t lws = g.lws[0];
     const int64_t nrows = a.n0, ncols = a.n1;
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, ncols);
-    if (c0 >= c1) return;
+    if (c0 >= c1) return true;
     int64_t lo, hi;
     part_range(c1 - c0, part, nparts, lo, hi);
     const T *A = (const T *)a.host[0];
@@ -354,7 +360,7 @@ void wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
     const T *mean = (MODE == COL_SQDEV) ? (const T *)a.host[1] : nullptr;
     T *out = (T *)a.host[(MODE == COL_SUM) ? 1 : 2];
     for (int64_t j = c0 + lo; j < c0 + hi; ++j) {
-        if (aborted(ab)) return;
+        if (aborted(ab)) return false;
         const T mj = (MODE == COL_SQDEV) ? mean[j] : T(0);
         T tot = 0;
         for (int q = 0; q < kColPartitions; ++q) {
@@ -374,14 +380,15 @@ void wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
             out[j] = (T)((s <= a.eps) ? 1.0f : s);
         }
     }
+    return true;
 }
 
 // SYRK / SYR2K: work-item (i, j) runs its k-chain
 template <typename T, bool TWO>
-void wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
     Wg2D w = wg2d(g, fgid, n, n);
-    if (w.r0 >= w.r1 || w.c0 >= w.c1) return;
+    if (w.r0 >= w.r1 || w.c0 >= w.c1) return true;
     const int64_t nc = w.c1 - w.c0, nitems = (w.r1 - w.r0) * nc;
     int64_t lo, hi;
     part_range(nitems, part, nparts, lo, hi);
@@ -391,7 +398,7 @@ void wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npart
     const T alpha = a.integer ? (T)(uint32_t)a.ialpha : (T)a.alpha;
     const T beta = a.integer ? (T)(uint32_t)a.ibeta : (T)a.beta;
     for (int64_t it = lo; it < hi; ++it) {
-        if ((it & 15) == 0 && aborted(ab)) return;
+        if ((it & 15) == 0 && aborted(ab)) return false;
         const int64_t i = w.r0 + it / nc, j = w.c0 + it % nc;
         const T *ai = A + i * m, *aj = A + j * m;
         const T *bi = TWO ? B + i * m : nullptr, *bj = TWO ? B + j * m : nullptr;
@@ -406,14 +413,15 @@ void wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npart
         }
         C[i * n + j] = op_fma(alpha, acc, op_mul(beta, C[i * n + j]));
     }
+    return true;
 }
 
 // CORR symmat: work-item j1 computes its row, each j2 > j1 down the two columns
-void wg_corr_corr_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_corr_corr_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
     const int64_t lws = g.lws[0];
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, m);
-    if (c0 >= c1) return;
+    if (c0 >= c1) return true;
     int64_t lo, hi;
     part_range(c1 - c0, part, nparts, lo, hi);
     const float *d = (const float *)a.host[0];
@@ -421,13 +429,14 @@ void wg_corr_corr_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int 
     for (int64_t j1 = c0 + lo; j1 < c0 + hi; ++j1) {
         sym[j1 * m + j1] = 1.0f;
         for (int64_t j2 = j1 + 1; j2 < m; ++j2) {
-            if ((j2 & 15) == 0 && aborted(ab)) return;
+            if ((j2 & 15) == 0 && aborted(ab)) return false;
             float acc = 0.0f;
             for (int64_t i = 0; i < n; ++i) acc = std::fmaf(d[i * m + j1], d[i * m + j2], acc);
             sym[j1 * m + j2] = acc;
             sym[j2 * m + j1] = acc;
         }
     }
+    return true;
 }
 
 }  // namespace
@@ -447,53 +456,45 @@ const char *host_variant_name(int kernel, int v) {
     return v == 0 ? "cpu" : "wi";
 }
 
-void host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *abort_flag) {
+bool host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *abort_flag) {
     if (a.host_variant == 1 && host_num_variants(a.kernel) > 1) {
         switch (a.kernel) {
         case K_ATAX_Y: case K_BICG_S:
-            if (a.integer) wg_coldot_wi<uint32_t, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
-            else wg_coldot_wi<float, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
-            return;
-        case K_CORR_MEAN: wg_coldot_wi<float, COL_SUM>(a, g, fgid, part, nparts, abort_flag); return;
-        case K_CORR_STD: wg_coldot_wi<float, COL_SQDEV>(a, g, fgid, part, nparts, abort_flag); return;
+            if (a.integer) return wg_coldot_wi<uint32_t, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
+            return wg_coldot_wi<float, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
+        case K_CORR_MEAN: return wg_coldot_wi<float, COL_SUM>(a, g, fgid, part, nparts, abort_flag);
+        case K_CORR_STD: return wg_coldot_wi<float, COL_SQDEV>(a, g, fgid, part, nparts, abort_flag);
         case K_SYRK:
-            if (a.integer) wg_syrk_wi<uint32_t, false>(a, g, fgid, part, nparts, abort_flag);
-            else wg_syrk_wi<float, false>(a, g, fgid, part, nparts, abort_flag);
-            return;
+            if (a.integer) return wg_syrk_wi<uint32_t, false>(a, g, fgid, part, nparts, abort_flag);
+            return wg_syrk_wi<float, false>(a, g, fgid, part, nparts, abort_flag);
         case K_SYR2K:
-            if (a.integer) wg_syrk_wi<uint32_t, true>(a, g, fgid, part, nparts, abort_flag);
-            else wg_syrk_wi<float, true>(a, g, fgid, part, nparts, abort_flag);
-            return;
-        case K_CORR_CORR: wg_corr_corr_wi(a, g, fgid, part, nparts, abort_flag); return;
+            if (a.integer) return wg_syrk_wi<uint32_t, true>(a, g, fgid, part, nparts, abort_flag);
+            return wg_syrk_wi<float, true>(a, g, fgid, part, nparts, abort_flag);
+        case K_CORR_CORR: return wg_corr_corr_wi(a, g, fgid, part, nparts, abort_flag);
         default: break;
         }
     }
     switch (a.kernel) {
     case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV:
-        if (a.integer) wg_rowdot<uint32_t>(a, g, fgid, part, nparts, abort_flag);
-        else wg_rowdot<float>(a, g, fgid, part, nparts, abort_flag);
-        break;
+        if (a.integer) return wg_rowdot<uint32_t>(a, g, fgid, part, nparts, abort_flag);
+        return wg_rowdot<float>(a, g, fgid, part, nparts, abort_flag);
     case K_ATAX_Y: case K_BICG_S:
-        if (a.integer) wg_coldot<uint32_t, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
-        else wg_coldot<float, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
-        break;
-    case K_CORR_MEAN: wg_coldot<float, COL_SUM>(a, g, fgid, part, nparts, abort_flag); break;
-    case K_CORR_STD: wg_coldot<float, COL_SQDEV>(a, g, fgid, part, nparts, abort_flag); break;
-    case K_CORR_REDUCE: wg_corr_reduce(a, g, fgid, part, nparts, abort_flag); break;
-    case K_CORR_CORR: wg_corr_corr(a, g, fgid, part, nparts, abort_flag); break;
+        if (a.integer) return wg_coldot<uint32_t, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
+        return wg_coldot<float, COL_DOT>(a, g, fgid, part, nparts, abort_flag);
+    case K_CORR_MEAN: return wg_coldot<float, COL_SUM>(a, g, fgid, part, nparts, abort_flag);
+    case K_CORR_STD: return wg_coldot<float, COL_SQDEV>(a, g, fgid, part, nparts, abort_flag);
+    case K_CORR_REDUCE: return wg_corr_reduce(a, g, fgid, part, nparts, abort_flag);
+    case K_CORR_CORR: return wg_corr_corr(a, g, fgid, part, nparts, abort_flag);
     case K_CONV2D:
-        if (a.integer) wg_conv2d<uint32_t>(a, g, fgid, part, nparts, abort_flag);
-        else wg_conv2d<float>(a, g, fgid, part, nparts, abort_flag);
-        break;
+        if (a.integer) return wg_conv2d<uint32_t>(a, g, fgid, part, nparts, abort_flag);
+        return wg_conv2d<float>(a, g, fgid, part, nparts, abort_flag);
     case K_SYRK:
-        if (a.integer) wg_syrk<uint32_t, false>(a, g, fgid, part, nparts, abort_flag);
-        else wg_syrk<float, false>(a, g, fgid, part, nparts, abort_flag);
-        break;
+        if (a.integer) return wg_syrk<uint32_t, false>(a, g, fgid, part, nparts, abort_flag);
+        return wg_syrk<float, false>(a, g, fgid, part, nparts, abort_flag);
     case K_SYR2K:
-        if (a.integer) wg_syrk<uint32_t, true>(a, g, fgid, part, nparts, abort_flag);
-        else wg_syrk<float, true>(a, g, fgid, part, nparts, abort_flag);
-        break;
-    default: break;
+        if (a.integer) return wg_syrk<uint32_t, true>(a, g, fgid, part, nparts, abort_flag);
+        return wg_syrk<float, true>(a, g, fgid, part, nparts, abort_flag);
+    default: return true;
     }
 }
 
@@ -506,7 +507,8 @@ int64_t host_batch(const KArgs &a, const Geom &g) {
 }
 
 // Work-groups [f_lo, f_hi) (any order is valid: every work-group writes only its own outputs).
-void host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *ab) {
+// Returns true when every one of them completed (false: the abort flag stopped the run).
+bool host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *ab) {
     if ((a.kernel == K_CONV2D || a.kernel == K_CORR_REDUCE) && g.work_dim == 2) {
         const int64_t ngx = g.ng[0];
         for (int64_t f = f_lo; f < f_hi;) {   // one segment per work-group row
@@ -514,25 +516,27 @@ void host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, 
             const int64_t gx1 = std::min<int64_t>(ngx, gx0 + (f_hi - f));
             Wg2D w0 = wg2d(g, f, a.n0, a.n1);
             const int64_t c1 = std::min<int64_t>(gx1 * g.lws[0], a.n1);
+            bool ok = true;
             if (a.kernel == K_CORR_REDUCE) {
-                corr_reduce_rect(a, w0.r0, w0.r1, w0.c0, c1, ab);
+                ok = corr_reduce_rect(a, w0.r0, w0.r1, w0.c0, c1, ab);
             } else {
                 const int64_t r0 = std::max<int64_t>(w0.r0, 1), r1 = std::min<int64_t>(w0.r1, a.n0 - 1);
                 const int64_t c0 = std::max<int64_t>(w0.c0, 1), cc1 = std::min<int64_t>(c1, a.n1 - 1);
                 if (r0 < r1 && c0 < cc1) {
-                    if (a.integer) conv2d_rect<uint32_t>(a, r0, r1, c0, cc1, ab);
-                    else conv2d_rect<float>(a, r0, r1, c0, cc1, ab);
+                    if (a.integer) ok = conv2d_rect<uint32_t>(a, r0, r1, c0, cc1, ab);
+                    else ok = conv2d_rect<float>(a, r0, r1, c0, cc1, ab);
                 }
             }
-            if (aborted(ab)) return;
+            if (!ok) return false;
             f = gy * ngx + gx1;
         }
-        return;
+        return true;
     }
     for (int64_t f = f_hi - 1; f >= f_lo; --f) {
-        if (aborted(ab)) return;
-        host_exec_wg(a, g, f, 0, 1, ab);
+        if (aborted(ab)) return false;
+        if (!host_exec_wg(a, g, f, 0, 1, ab)) return false;
     }
+    return true;
 }
 
 // Conservative contiguous output span of work-groups [lo, hi) (see fcl_internal.h).

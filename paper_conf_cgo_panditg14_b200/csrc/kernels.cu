@@ -115,6 +115,11 @@ struct TaskCtx {
     unsigned long long *s_st;    // shared, 16-byte aligned: status pair prefetched by thread 0
     long long *s_key;            // shared: key of the running task
     int *s_flag;                 // shared broadcast slot (D2: the local 'completedatcpu'); w + 1 after an abort
+    // The watermark this task was checked against: work-groups with flattened id >= wmask are
+    // the host's, so a task spanning several work-groups (tiles) stores none of their outputs --
+    // at a fixed split every output word is then written by exactly one device (north_star's
+    // invariant, L16.s9 "non-overlapping parts").  0xFFFFFFFF: no mask (plain grids, first tasks).
+    unsigned int wmask;
 
     // In-task poll period in body iterations (a huge value when there is none): bodies run
     // their inner loop in blocks of this many iterations and call check() between blocks, so
@@ -387,14 +392,28 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     }
     const bool claims = c.task_lo + (long long)gridDim.x < c.task_hi;
     TaskCtx tc;
-    tc.c = &c; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.s_st = s_st;
+    tc.c = &c; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.s_st = s_st; tc.wmask = 0xFFFFFFFFu;
     // the status is needed only by in-task polls and by the check before a claimed task
     const bool need_status = claims || c.abort_period > 0;
     if (threadIdx.x == 0 && need_status) status_prefetch(c, s_st);
     bool marked = false;   // thread 0: this CTA recorded a watermark (skip or abort)
+    unsigned int rec_w = c.w_default;   // thread 0: lowest mask watermark recorded so far
     for (;;) {
         if (t >= c.task_hi) break;
         const long long key = Body::key(bp, t);
+        if (c.task_delay_ns) {
+            // fault injection (opts.gpu_delay_us): the GPU reaches this task late -- and, as a
+            // work-group that starts late (Fig 8), checks the status when it does
+            if (threadIdx.x == 0) {
+                const unsigned long long t0 = globaltimer();
+                while (globaltimer() - t0 < c.task_delay_ns) __nanosleep(1000);
+                s_w = decode_w(ld_status(c.status), c);
+            }
+            __syncthreads();
+            w = s_w;
+            checked = true;
+            __syncthreads();
+        }
         if (checked && (unsigned long long)key >= (unsigned long long)w) {   // covered by the host
             if (threadIdx.x == 0) { record_wm(c, w); marked = true; }
             break;
@@ -429,6 +448,14 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
         long long t_next = c.task_hi;
         if (!Body::kLateClaim && threadIdx.x == 0 && claims)
             t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
+        // a task that may span work-groups the host covers stores only those below w (the
+        // watermark acted on: the merge domain starts at or below it)
+        tc.wmask = (Body::kMasks && checked) ? w : 0xFFFFFFFFu;
+        if (Body::kMasks && checked && w < rec_w && threadIdx.x == 0) {
+            record_wm(c, w);
+            rec_w = w;
+            marked = true;
+        }
         const bool aborted = Body::run(bp, t, tc, smem);
         if (aborted) {
             if (threadIdx.x == 0) { record_wm(c, tc.abort_w()); marked = true; }
@@ -436,6 +463,10 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
         }
         if (threadIdx.x == 0) {
             if (c.tasks) atomicAdd(c.tasks, 1ull);
+            if (c.exec_cnt) {   // test hook (opts.record_exec_counts): completed tasks and their mask
+                atomicAdd(c.exec_cnt + (t - c.task_lo), 1u);
+                c.exec_w[t - c.task_lo] = tc.wmask;
+            }
             // long tasks claim after they finish: nothing of the dispatcher stays in a register
             if (Body::kLateClaim && claims) t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
             s_task = t_next;
@@ -540,8 +571,9 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
     __shared__ __align__(16) typename Body::Smem smem;
     __shared__ long long s_key;
     TaskCtx tc;
-    tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = &s_flag; tc.s_key = &s_key;
+    tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.wmask = 0xFFFFFFFFu;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
+    if (r.exec_cnt && threadIdx.x == 0) atomicAdd(r.exec_cnt + blockIdx.x, 1u);   // test hook
     if (r.tstamp) {
         __syncthreads();
         if (threadIdx.x == 0) atomicMax(r.tstamp + 1, globaltimer());
@@ -597,6 +629,7 @@ struct RowDotBody {
     // still one wave at N = 4096; 0.74 vs 0.71 of HBM with 2 blocks, scripts/ubench_dots.cu).
     static constexpr int kThreads = 128;
     static constexpr int kMinBlocks = (NMAT == 2) ? 7 : 8;
+    static constexpr bool kMasks = false;   // a task is part of one work-group
     static constexpr bool kLateClaim = false;
     static constexpr int kWarps = kThreads / 32;
     static constexpr int U = 4;   // 128-column blocks whose loads are issued together
@@ -717,6 +750,7 @@ template <typename T, int MODE>
 struct ColDotBody {
     static constexpr int kThreads = 256;
     static constexpr int kMinBlocks = 2;
+    static constexpr bool kMasks = false;   // a task is part of one work-group
     static constexpr bool kLateClaim = false;
     static constexpr int U = 16;
     struct Params {
@@ -814,24 +848,35 @@ struct Tile2D {
         const long long tx = t % ntx, ty = t / ntx;
         return tx * tw + ngx * (ty * th);
     }
+    // work-group of output element (i, j), Fig 5 flattening
+    // (32-bit arithmetic: extents and flattened ids are < 2^32, checked at launch)
+    __device__ unsigned int fgid(long long i, long long j) const {
+        return (unsigned int)j / (unsigned int)lws0 + (unsigned int)ngx * ((unsigned int)i / (unsigned int)lws1);
+    }
+    // is output (i, j) below the mask watermark (0xFFFFFFFF: no mask)?
+    __device__ bool keep(unsigned int wm, long long i, long long j) const {
+        return wm == 0xFFFFFFFFu || fgid(i, j) < wm;
+    }
 };
 
 // CORR reduce (in place): d[i][j] = (d[i][j] - mean[j]) / (sqrt(n) * std[j]).
 struct CorrReduceBody {
     static constexpr int kThreads = 256;
     static constexpr int kMinBlocks = 4;
+    static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = false;
     struct Params { float *data; const float *mean; const float *std_; Tile2D tl; float sqrtn; };
     typedef EmptySmem Smem;
     __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
-    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
+    __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &) {
         const Tile2D &tl = p.tl;
         const long long tx = t % tl.ntx, ty = t / tl.ntx;
         const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
         const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
+        const unsigned int wm = tc.wmask;
         for (int e = threadIdx.x; e < tcols * trows; e += kThreads) {
             const long long i = r0 + e / tcols, j = c0 + e % tcols;
-            if (i < tl.nrows && j < tl.ncols) {
+            if (i < tl.nrows && j < tl.ncols && tl.keep(wm, i, j)) {
                 float *q = p.data + i * tl.ncols + j;
                 const float den = __fmul_rn(p.sqrtn, p.std_[j]);
                 *q = __fdiv_rn(__fadd_rn(*q, -p.mean[j]), den);
@@ -852,6 +897,7 @@ template <typename T>
 struct Conv2DBody {
     static constexpr int kThreads = 256;
     static constexpr int kMinBlocks = 2;   // 10 x 16 B of loads in flight per thread needs the registers
+    static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = false;
     struct Params { const T *A; T *B; Tile2D tl; T c[9]; int vec4; };   // c[a*3+b]: row offset a-1, col offset b-1
     typedef EmptySmem Smem;
@@ -874,7 +920,7 @@ struct Conv2DBody {
     // j-1 .. j+4 exist for all lanes, no output on the border): no per-row or per-column
     // checks, one pointer walking the rows, and the halo columns loaded by the two edge lanes
     // for every row up front, so that no shuffle sits under a divergent branch.
-    __device__ static void run_interior(const Params &p, long long ib, long long j, int lane) {
+    __device__ static void run_interior(const Params &p, long long ib, long long j, int lane, unsigned int wm) {
         typedef typename V4<T>::type T4;
         const long long nj = p.tl.ncols;
         const T *src = p.A + (ib - 1) * nj + j;
@@ -901,16 +947,24 @@ struct Conv2DBody {
             o.y = tap9(p, v[q - 1].x, v[q].x, v[q + 1].x, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z);
             o.z = tap9(p, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w);
             o.w = tap9(p, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w, rh[q - 1], rh[q], rh[q + 1]);
-            __stcs(reinterpret_cast<T4 *>(dst + (q - 1) * nj), o);
+            if (wm == 0xFFFFFFFFu || p.tl.keep(wm, ib + q - 1, j + 3)) {   // (fgid grows with j)
+                __stcs(reinterpret_cast<T4 *>(dst + (q - 1) * nj), o);
+            } else {
+                T *d = dst + (q - 1) * nj;
+                if (p.tl.keep(wm, ib + q - 1, j)) __stcs(d, o.x);
+                if (p.tl.keep(wm, ib + q - 1, j + 1)) __stcs(d + 1, o.y);
+                if (p.tl.keep(wm, ib + q - 1, j + 2)) __stcs(d + 2, o.z);
+            }
         }
     }
 
-    __device__ static bool run(const Params &p, long long t, TaskCtx &, Smem &) {
+    __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &) {
         const Tile2D &tl = p.tl;
         const long long tx = t % tl.ntx, ty = t / tl.ntx;
         const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
         const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
         const long long ni = tl.nrows, nj = tl.ncols;
+        const unsigned int wm = tc.wmask;
         if (p.vec4 && tcols == 256 && trows == 32) {
             const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
             const int cg = warp & 1;                 // which 128-column half of the tile
@@ -919,7 +973,7 @@ struct Conv2DBody {
             const long long ib = r0 + rg * 8;        // first output row of the group
             const long long wj0 = c0 + cg * 128;     // the warp's first column (warp-uniform test)
             if (ib >= 1 && ib + 8 <= ni - 1 && wj0 >= 1 && wj0 + 128 <= nj - 1) {
-                run_interior(p, ib, j, lane);
+                run_interior(p, ib, j, lane, wm);
                 return false;
             }
             if (ib >= ni) return false;
@@ -952,13 +1006,13 @@ struct Conv2DBody {
                 o.z = tap9(p, v[q - 1].y, v[q].y, v[q + 1].y, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w);
                 o.w = tap9(p, v[q - 1].z, v[q].z, v[q + 1].z, v[q - 1].w, v[q].w, v[q + 1].w, rh[q - 1], rh[q], rh[q + 1]);
                 T *dst = p.B + i * nj + j;
-                if (j >= 1 && j + 4 <= nj - 1) {
+                if (j >= 1 && j + 4 <= nj - 1 && tl.keep(wm, i, j + 3)) {
                     __stcs(reinterpret_cast<typename V4<T>::type *>(dst), o);
-                } else {   // a border column inside this vector stays untouched
-                    if (j >= 1 && j < nj - 1) __stcs(dst, o.x);
-                    if (j + 1 >= 1 && j + 1 < nj - 1) __stcs(dst + 1, o.y);
-                    if (j + 2 >= 1 && j + 2 < nj - 1) __stcs(dst + 2, o.z);
-                    if (j + 3 >= 1 && j + 3 < nj - 1) __stcs(dst + 3, o.w);
+                } else {   // a border column inside this vector stays untouched (and masked ones)
+                    if (j >= 1 && j < nj - 1 && tl.keep(wm, i, j)) __stcs(dst, o.x);
+                    if (j + 1 >= 1 && j + 1 < nj - 1 && tl.keep(wm, i, j + 1)) __stcs(dst + 1, o.y);
+                    if (j + 2 >= 1 && j + 2 < nj - 1 && tl.keep(wm, i, j + 2)) __stcs(dst + 2, o.z);
+                    if (j + 3 >= 1 && j + 3 < nj - 1 && tl.keep(wm, i, j + 3)) __stcs(dst + 3, o.w);
                 }
             }
             return false;
@@ -977,7 +1031,8 @@ struct Conv2DBody {
             for (; i < iend; ++i) {
 #pragma unroll
                 for (int b = 0; b < 3; ++b) w2[b] = __ldg(a + (i + 1) * nj + b - 1);
-                __stcs(p.B + i * nj + j, tap9(p, w0[0], w1[0], w2[0], w0[1], w1[1], w2[1], w0[2], w1[2], w2[2]));
+                if (tl.keep(wm, i, j))
+                    __stcs(p.B + i * nj + j, tap9(p, w0[0], w1[0], w2[0], w0[1], w1[1], w2[1], w0[2], w1[2], w2[2]));
 #pragma unroll
                 for (int b = 0; b < 3; ++b) { w0[b] = w1[b]; w1[b] = w2[b]; }
             }
@@ -1011,6 +1066,7 @@ struct GemmBody {
     static constexpr int TXN = GBM / TN;                 // threads along the columns
     static constexpr int NB = TN / 4;                    // float4 column groups per thread
     static constexpr int LD = GBM * GBK / kThreads;      // elements of each operand a thread loads per k'-tile
+    static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = true;   // tasks of ~0.1-1 ms: an exposed claim costs nothing
     typedef typename V4<T>::type T4;
     struct Params {
@@ -1266,7 +1322,15 @@ struct GemmBody {
         }
         if (!done_async && (interior ? mainloop<true>(p, i0, j0, tc, sm, acc) : mainloop<false>(p, i0, j0, tc, sm, acc)))
             return true;
-        // epilogue: write-once stores
+        // epilogue: write-once stores, only of outputs whose work-group is below the mask
+        const unsigned int wm = tc.wmask;
+        auto keep = [&](long long i, long long j) -> bool {   // output (i, j): its work-group's id < wm
+            if (wm == 0xFFFFFFFFu) return true;
+            const unsigned int ui = (unsigned int)i, uj = (unsigned int)j;
+            const unsigned int f = (OP == G_CORR) ? ui / (unsigned int)p.lws
+                                                  : uj / (unsigned int)p.lws0 + (unsigned int)p.ngx * (ui / (unsigned int)p.lws1);
+            return f < wm;
+        };
         if (OP == G_SYRK && p.sym && bi != bj) {
             // mirror block: C[j][i] from acc(i, j) (bit-identical to acc(j, i)); the four rows
             // r of a thread's half are four consecutive columns of the mirror row
@@ -1278,7 +1342,7 @@ struct GemmBody {
 #pragma unroll
                 for (int half = 0; half < 2; ++half) {
                     const long long ib = i0 + half * 64 + ty * 4;
-                    if (p.vec4 && ib + 3 < p.n) {
+                    if (p.vec4 && ib + 3 < p.n && keep(j, ib + 3)) {
                         T4 cv = *reinterpret_cast<T4 *>(crow + ib);
                         cv.x = op_fma(p.alpha, acc[half * 4 + 0][c], op_mul(p.beta, cv.x));
                         cv.y = op_fma(p.alpha, acc[half * 4 + 1][c], op_mul(p.beta, cv.y));
@@ -1289,7 +1353,7 @@ struct GemmBody {
 #pragma unroll
                         for (int r = 0; r < 4; ++r) {
                             const long long i = ib + r;
-                            if (i < p.n) crow[i] = op_fma(p.alpha, acc[half * 4 + r][c], op_mul(p.beta, crow[i]));
+                            if (i < p.n && keep(j, i)) crow[i] = op_fma(p.alpha, acc[half * 4 + r][c], op_mul(p.beta, crow[i]));
                         }
                     }
                 }
@@ -1305,7 +1369,7 @@ struct GemmBody {
 #pragma unroll
                     for (int c = 0; c < 4; ++c) {
                         const long long j = jb + c;
-                        if (i < p.n && j < p.n) {
+                        if (i < p.n && j < p.n && keep(i, j)) {   // (row i's work-group writes both)
                             if (j > i) { p.C[i * p.n + j] = acc[r][half * 4 + c]; p.C[j * p.n + i] = acc[r][half * 4 + c]; }
                             else if (j == i) p.C[i * p.n + i] = T(1);
                         }
@@ -1313,7 +1377,7 @@ struct GemmBody {
                 } else {
                     if (i >= p.n) continue;
                     T *crow = p.C + i * p.n;
-                    if (p.vec4 && jb + 3 < p.n) {
+                    if (p.vec4 && jb + 3 < p.n && keep(i, jb + 3)) {
                         T4 cv = *reinterpret_cast<T4 *>(crow + jb);
                         cv.x = op_fma(p.alpha, acc[r][half * 4 + 0], op_mul(p.beta, cv.x));
                         cv.y = op_fma(p.alpha, acc[r][half * 4 + 1], op_mul(p.beta, cv.y));
@@ -1324,7 +1388,7 @@ struct GemmBody {
 #pragma unroll
                         for (int c = 0; c < 4; ++c) {
                             const long long j = jb + c;
-                            if (j < p.n) crow[j] = op_fma(p.alpha, acc[r][half * 4 + c], op_mul(p.beta, crow[j]));
+                            if (j < p.n && keep(i, j)) crow[j] = op_fma(p.alpha, acc[r][half * 4 + c], op_mul(p.beta, crow[j]));
                         }
                     }
                 }
@@ -1603,6 +1667,53 @@ int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t) {
         return (b1 * GBM) / g.lws[0];
     }
     default: return 0;
+    }
+}
+
+void gpu_task_wgs(const KArgs &a, const Geom &g, int64_t t, std::vector<int64_t> &out) {
+    auto rect = [&](int64_t gx0, int64_t gx1, int64_t gy0, int64_t gy1) {
+        gx1 = gx1 < g.ng[0] ? gx1 : g.ng[0];
+        gy1 = gy1 < g.ng[1] ? gy1 : g.ng[1];
+        for (int64_t gy = gy0; gy < gy1; ++gy)
+            for (int64_t gx = gx0; gx < gx1; ++gx) out.push_back(gx + g.ng[0] * gy);
+    };
+    switch (a.kernel) {
+    case K_ATAX_TMP: case K_BICG_Q: case K_GESUMMV:
+    case K_ATAX_Y: case K_BICG_S: case K_CORR_MEAN: case K_CORR_STD:
+        out.push_back(gpu_task_key(a, g, t));   // a task is part of one work-group
+        break;
+    case K_CORR_REDUCE: case K_CONV2D: {
+        int tw, th; tile_shape(g, 256, 32, tw, th);
+        const long long ntx = (g.ng[0] + tw - 1) / tw, tx = t % ntx, ty = t / ntx;
+        rect(tx * tw, tx * tw + tw, ty * th, ty * th + th);
+        break;
+    }
+    case K_SYRK: case K_SYR2K: {
+        const long long nt = (a.n0 + GBM - 1) / GBM;
+        long long bi = t / nt, bj = t % nt;
+        const bool sym = a.kernel == K_SYRK && a.sym;
+        if (sym) {
+            long long rem = t;
+            bi = 0;
+            while (rem >= nt - bi) { rem -= nt - bi; ++bi; }
+            bj = bi + rem;
+        }
+        const long long cx = GBM / g.lws[0], cy = GBM / g.lws[1];
+        rect(bj * cx, bj * cx + cx, bi * cy, bi * cy + cy);
+        if (sym && bi != bj) rect(bi * cx, bi * cx + cx, bj * cy, bj * cy + cy);   // mirror block
+        break;
+    }
+    case K_CORR_CORR: {
+        const long long nt = (a.n1 + GBM - 1) / GBM;
+        long long b1 = 0, rem = t;
+        while (rem >= nt - b1) { rem -= nt - b1; ++b1; }
+        const long long f0 = (b1 * GBM) / g.lws[0];
+        long long f1 = ((b1 + 1) * GBM - 1) / g.lws[0] + 1;
+        if (f1 > g.ng[0]) f1 = g.ng[0];
+        for (long long f = f0; f < f1; ++f) out.push_back(f);
+        break;
+    }
+    default: break;
     }
 }
 

@@ -220,10 +220,18 @@ struct Executor {
                 if (!abort_flag) {
                     if (batch == 1) {
                         const int64_t fgid = hi - 1 - it / nparts;   // descending (L14.s36)
-                        host_exec_wg(a, g, fgid, (int)(it % nparts), nparts, &abort_flag);
+                        const bool ok = host_exec_wg(a, g, fgid, (int)(it % nparts), nparts, &abort_flag);
+                        if (ok && a.rec_cpu_done) {   // test hook: a work-group counts once all its parts completed
+                            if (nparts == 1 || __atomic_add_fetch(a.rec_cpu_parts + fgid, 1, __ATOMIC_ACQ_REL) == nparts) {
+                                if (nparts > 1) __atomic_store_n(a.rec_cpu_parts + fgid, 0, __ATOMIC_RELAXED);
+                                __atomic_add_fetch(a.rec_cpu_done + fgid, 1, __ATOMIC_RELAXED);
+                            }
+                        }
                     } else {   // a run of work-groups, runs claimed in descending order
                         const int64_t fh = hi - it * batch, fl = std::max<int64_t>(lo, fh - batch);
-                        host_exec_range(a, g, fl, fh, &abort_flag);
+                        const bool ok = host_exec_range(a, g, fl, fh, &abort_flag);
+                        if (ok && a.rec_cpu_done)
+                            for (int64_t f = fl; f < fh; ++f) __atomic_add_fetch(a.rec_cpu_done + f, 1, __ATOMIC_RELAXED);
                     }
                 }
                 done.fetch_add(1, std::memory_order_acq_rel);
@@ -507,6 +515,18 @@ struct fcl_context_st {
     cudaEvent_t ev_gd2h = nullptr;               // completion of single-device / deferred returns (on dh)
     fcl_launch_info sync_info{};
     bool sync_have_k = false;
+    // Test hook (opts.record_exec_counts): per-task GPU completions (with the
+    // work-group mask each task ran with) and per-work-group host completions of the last
+    // launch that asked for them -- fcl_get_exec_counts turns them into per-work-group counts.
+    struct ExecRec {
+        bool valid = false;
+        KArgs a{};
+        Geom g{};
+        int64_t lo = 0, hi = 0, t0 = 0, t1 = 0;
+        std::vector<int32_t> cpu_done, cpu_parts;
+        unsigned int *d_cnt = nullptr, *d_w = nullptr;   // [t1 - t0] each
+        size_t d_cap = 0;
+    } rec;
     std::vector<fcl_buffer> defer_list;
     Tracer tr;
 };
@@ -935,7 +955,7 @@ std::array<int64_t, 9> select_key(const Launch &L) {
 bool select_eligible(fcl_context ctx, const Launch &L) {
     const bool on = L.o.select == FCL_SELECT_ON || (L.o.select == FCL_SELECT_DEFAULT && ctx->select_on);
     return on && ctx->select_period > 0 && L.o.mode == FCL_MODE_COOP && L.o.forced_split < 0 && !L.o.defer_merge &&
-           L.o.host_delay_us == 0 && !L.o.drop_publish && L.hi > L.lo;
+           L.o.host_delay_us == 0 && L.o.gpu_delay_us <= 0 && !L.o.record_exec_counts && !L.o.drop_publish && L.hi > L.lo;
 }
 
 // Returns FCL_SELECTED_* for this launch; *probe: it runs cooperatively to refresh the profile.
@@ -1098,6 +1118,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     if (opt_period == 0 && ctx->env_abort_period != 0) opt_period = ctx->env_abort_period;   // FCL_ABORT_PERIOD
     const int abort_period = opt_period > 0 ? opt_period : (opt_period < 0 ? 0 : gpu_default_abort_period(L.a));
     j.lite = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && abort_period == 0 && !ctx->no_lite && !j.stream &&
+             L.o.gpu_delay_us <= 0 &&
              (j.t1 - j.t0) <= gpu_coop_capacity(L.a, L.g, ctx->num_sms);
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
     const void *srcs[6];
@@ -1162,6 +1183,9 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     c.merge_ctr_next = ctx->dmctr + (j.slot + 1) % kSlots;
     c.exit_word = ctx->exit_dptr + j.slot;
     c.arrival = j.stream ? ctx->darrival + j.slot : nullptr;
+    c.task_delay_ns = L.o.gpu_delay_us > 0 ? 1000ull * (unsigned long long)L.o.gpu_delay_us : 0ull;
+    c.exec_cnt = L.o.record_exec_counts ? ctx->rec.d_cnt : nullptr;
+    c.exec_w = L.o.record_exec_counts ? ctx->rec.d_w : nullptr;
     c.mg = DevMergeList{};
     c.mg.n = 0;
 
@@ -1214,7 +1238,8 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
             const int nx = (j.slot + 1) % kSlots;
             SlotReset r{ctx->dclaim + nx, ctx->stats ? ctx->dtasks + nx : nullptr, ctx->dmctr + nx, ctx->dbar + 32 * nx,
                         ctx->dbar + 32 * j.slot, ctx->lite_exit_word ? ctx->exit_dptr + j.slot : nullptr, j.epoch,
-                        plain_stamp(ctx), ctx->test_gpu_delay_ns};
+                        plain_stamp(ctx), ctx->test_gpu_delay_ns,
+                        L.o.record_exec_counts ? ctx->rec.d_cnt : nullptr};
             if (gpu_launch_plain(L.a, L.g, j.t0, j.t1, ctx->main, &r, pdl_mode(ctx, L)) < 0)
                 return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
         } else {
@@ -1447,6 +1472,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         if (ex.finished()) {
             const double dt = now_ms() - t_start;
             busy += dt;
+            if (nch - 1 < 64) info.chunk_ms[nch - 1] = dt;   // (the C11 input, exported for its pin)
             in_flight = false;
             cpu_done_wgs += cur_size;
             variant_measured(ctx, L, vp, cur_var, dt, cur_size);
@@ -1487,6 +1513,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     // conservative cover such as CORR's row-plus-column symmat footprint)
     const bool race = gpu_done && !j.forced && (j.dev_merge || j.lite) && !j.eager && !j.lazy && !ctx->no_race && j.exact_spans &&
                       hi_cur > L.lo && out_bytes(L.lo, hi_cur) >= ctx->race_min_bytes;
+    info.n_c11_chunks = nch;
     if (race) {
         ctx->tr.add("race_begin", j.epoch);
         info.race = 1;
@@ -1523,6 +1550,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         for (;;) {
             if (in_flight && ex.finished()) {
                 busy += now_ms() - t_start;
+                if (nch - 1 < 64) info.chunk_ms[nch - 1] = now_ms() - t_start;
                 in_flight = false;
                 cpu_done_wgs += cur_size;
                 hi_cur = cur_lo;
@@ -1759,6 +1787,7 @@ fcl_status run_gpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     if (timing) CK(ctx, cudaEventRecord(ctx->ev_k0, ctx->main));
     SlotReset r{};
     r.tstamp = plain_stamp(ctx);
+    r.exec_cnt = L.o.record_exec_counts ? ctx->rec.d_cnt : nullptr;
     if (gpu_launch_plain(L.a, L.g, t0, t1, ctx->main, &r, pdl_mode(ctx, L)) < 0)
         return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
     if (timing) CK(ctx, cudaEventRecord(ctx->ev_t1, ctx->main));
@@ -1816,6 +1845,7 @@ fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     info.t_host_ms = now_ms() - t0;
     info.cpu_wgs = nwg;
     info.n_chunks = nch;
+    info.n_c11_chunks = 0;   // (CPU-only: profiling allocations, then the rest in one job)
     info.cpu_did_all = 1;
     info.published_watermark = L.lo;
     for (int q = 0; q < L.nout; ++q) L.bufs[L.out_idx[q]]->dev_valid = false;   // lazy H2D on next GPU use
@@ -2063,6 +2093,8 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->wm_host) cudaFreeHost(ctx->wm_host);
     if (ctx->exit_host) cudaFreeHost(ctx->exit_host);
     if (ctx->dclaim) cudaFree(ctx->dclaim);
+    if (ctx->rec.d_cnt) cudaFree(ctx->rec.d_cnt);
+    if (ctx->rec.d_w) cudaFree(ctx->rec.d_w);
     if (ctx->darrival) cudaFree(ctx->darrival);
     if (ctx->own_main) cudaStreamDestroy(ctx->main);
     if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
@@ -2272,6 +2304,40 @@ fcl_status fcl_kernel_signature(fcl_kernel k, char *buf, size_t len) {
     return s.size() < len ? FCL_SUCCESS : FCL_INVALID_VALUE;
 }
 
+// opts.record_exec_counts: reset the record for launch L (device counters zeroed on main, ahead
+// of L's grid) and point L's host bodies at the per-work-group host counters.
+static fcl_status exec_rec_begin(fcl_context ctx, Launch &L) {
+    auto &r = ctx->rec;
+    const TaskSpace ts = gpu_task_space(L.a, L.g);
+    r.valid = true;
+    r.g = L.g;
+    r.lo = L.lo; r.hi = L.hi;
+    r.t0 = first_task_at(L.a, L.g, ts.ntasks, L.lo);
+    r.t1 = first_task_at(L.a, L.g, ts.ntasks, L.hi);
+    r.cpu_done.assign((size_t)L.g.n_wg, 0);
+    r.cpu_parts.assign((size_t)L.g.n_wg, 0);
+    const size_t need = (size_t)std::max<int64_t>(1, r.t1 - r.t0) * sizeof(unsigned int);
+    if (need > r.d_cap) {
+        if (r.d_cnt) cudaFree(r.d_cnt);
+        if (r.d_w) cudaFree(r.d_w);
+        r.d_cnt = r.d_w = nullptr;
+        r.d_cap = 0;
+        if (cudaMalloc(&r.d_cnt, need) != cudaSuccess || cudaMalloc(&r.d_w, need) != cudaSuccess) {
+            cudaGetLastError();
+            r.valid = false;
+            return set_err(ctx, FCL_OUT_OF_RESOURCES, "exec-count record of %zu bytes", need);
+        }
+        r.d_cap = need;
+    }
+    ctx->main_fenced.store(1);
+    CK(ctx, cudaMemsetAsync(r.d_cnt, 0, need, ctx->main));
+    CK(ctx, cudaMemsetAsync(r.d_w, 0xFF, need, ctx->main));   // plain grids: no mask
+    L.a.rec_cpu_done = r.cpu_done.data();
+    L.a.rec_cpu_parts = r.cpu_parts.data();
+    r.a = L.a;
+    return FCL_SUCCESS;
+}
+
 static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work_dim, const size_t gws[3],
                                const size_t lws[3], const fcl_arg *args, uint32_t n_args, const fcl_launch_opts *opts,
                                Launch &L) {
@@ -2388,6 +2454,12 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
             info_out->host_variant = -1;
         }
         return FCL_SUCCESS;
+    }
+    if (L.o.record_exec_counts) {   // test hook: a fresh record (the previous one's launch must be done)
+        drain(ctx);
+        quiesce(ctx);
+        s = exec_rec_begin(ctx, L);
+        if (s != FCL_SUCCESS) return s;
     }
     if (!ctx->defer_list.empty()) {
         drain(ctx);
@@ -2713,6 +2785,42 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info) {
     }
     cudaGetLastError();
     *info = j->info;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_get_exec_counts(fcl_context ctx, int64_t n, int32_t *gpu_done, int32_t *gpu_frags, int32_t *cpu_done) {
+    if (!ctx) return FCL_INVALID_CONTEXT;
+    cudaSetDevice(ctx->device);
+    drain(ctx);
+    quiesce(ctx);
+    auto &r = ctx->rec;
+    if (!r.valid) return set_err(ctx, FCL_INVALID_VALUE, "no launch recorded execution counts");
+    if (n < r.g.n_wg) return set_err(ctx, FCL_INVALID_VALUE, "n %lld < %lld work-groups", (long long)n, (long long)r.g.n_wg);
+    CK(ctx, cudaStreamSynchronize(ctx->main));
+    const int64_t nt = r.t1 - r.t0;
+    std::vector<unsigned int> cnt((size_t)std::max<int64_t>(0, nt)), wm((size_t)std::max<int64_t>(0, nt));
+    if (nt > 0) {
+        CK(ctx, cudaMemcpy(cnt.data(), r.d_cnt, (size_t)nt * 4, cudaMemcpyDeviceToHost));
+        CK(ctx, cudaMemcpy(wm.data(), r.d_w, (size_t)nt * 4, cudaMemcpyDeviceToHost));
+    }
+    if (gpu_done) std::memset(gpu_done, 0, (size_t)n * 4);
+    if (gpu_frags) std::memset(gpu_frags, 0, (size_t)n * 4);
+    std::vector<int64_t> wgs;
+    for (int64_t t = 0; t < nt; ++t) {
+        wgs.clear();
+        gpu_task_wgs(r.a, r.g, r.t0 + t, wgs);
+        for (int64_t f : wgs) {
+            if (f < 0 || f >= r.g.n_wg) continue;
+            if (gpu_frags) gpu_frags[f] += 1;
+            // a task stores only the work-groups below the watermark it was checked against
+            if (gpu_done && cnt[(size_t)t] && (wm[(size_t)t] == 0xFFFFFFFFu || f < (int64_t)wm[(size_t)t]))
+                gpu_done[f] += (int32_t)cnt[(size_t)t];
+        }
+    }
+    if (cpu_done) {
+        std::memset(cpu_done, 0, (size_t)n * 4);
+        for (int64_t f = 0; f < r.g.n_wg; ++f) cpu_done[f] = __atomic_load_n(&r.cpu_done[(size_t)f], __ATOMIC_RELAXED);
+    }
     return FCL_SUCCESS;
 }
 

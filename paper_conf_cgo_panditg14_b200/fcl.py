@@ -36,6 +36,7 @@ EXPORTED = [
     "fcl_get_kernel", "fcl_kernel_signature", "fcl_kernel_host_variants", "fcl_default_launch_opts",
     "fcl_enqueue_ndrange",
     "fcl_merge", "fcl_merge_raw", "fcl_finish", "fcl_get_launch_info", "fcl_get_counters", "fcl_slice_range",
+    "fcl_get_exec_counts",
     "fcl_status_string", "fcl_last_error", "fcl_version",
 ]
 
@@ -60,7 +61,8 @@ class LaunchOpts(ctypes.Structure):
                 ("host_delay_us", ctypes.c_int32), ("drop_publish", ctypes.c_int32),
                 ("wg_lo", ctypes.c_int64), ("wg_hi", ctypes.c_int64),
                 ("blocking", ctypes.c_int32), ("flags", ctypes.c_int32), ("host_variant", ctypes.c_int32),
-                ("select", ctypes.c_int32)]
+                ("select", ctypes.c_int32), ("gpu_delay_us", ctypes.c_int32),
+                ("record_exec_counts", ctypes.c_int32)]
 
 
 class LaunchInfo(ctypes.Structure):
@@ -76,11 +78,13 @@ class LaunchInfo(ctypes.Structure):
                 ("chunk_sizes", ctypes.c_int32 * 64), ("gpu_path", ctypes.c_int32), ("race", ctypes.c_int32),
                 ("host_variant", ctypes.c_int32), ("n_host_variants", ctypes.c_int32),
                 ("profile_ms_per_wg", ctypes.c_double * 4), ("selected", ctypes.c_int32), ("probe", ctypes.c_int32),
-                ("streamed_wgs", ctypes.c_int64)]
+                ("streamed_wgs", ctypes.c_int64), ("chunk_ms", ctypes.c_double * 64),
+                ("n_c11_chunks", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
-        d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("chunk_sizes", "profile_ms_per_wg")}
+        d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("chunk_sizes", "profile_ms_per_wg", "chunk_ms")}
         d["chunk_sizes"] = [int(v) for v in self.chunk_sizes[: min(64, max(0, self.n_chunks))]]
+        d["chunk_ms"] = [float(v) for v in self.chunk_ms[: min(64, max(0, self.n_chunks))]]
         d["profile_ms_per_wg"] = [float(v) for v in self.profile_ms_per_wg[: max(0, self.n_host_variants)]]
         return d
 
@@ -119,6 +123,7 @@ def load() -> ctypes.CDLL:
         "fcl_finish": ([vp], i32),
         "fcl_get_launch_info": ([vp, ctypes.POINTER(LaunchInfo)], i32),
         "fcl_get_counters": ([vp, ctypes.POINTER(i64), i32], i32),
+        "fcl_get_exec_counts": ([vp, i64, vp, vp, vp], i32),
         "fcl_slice_range": ([vp, ctypes.c_uint32, ctypes.POINTER(sz), ctypes.POINTER(sz), i32, i32,
                              ctypes.POINTER(i64), ctypes.POINTER(i64)], i32),
         "fcl_status_string": ([i32], ctypes.c_char_p),
@@ -224,7 +229,8 @@ class Kernel:
 
 def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg_split=1,
               abort_period=0, defer_merge=0, n_host_threads=0, host_delay_us=0, drop_publish=0,
-              wg_lo=0, wg_hi=-1, blocking=0, timing=0, host_variant=-1, select=0) -> LaunchOpts:
+              wg_lo=0, wg_hi=-1, blocking=0, timing=0, host_variant=-1, select=0, gpu_delay_us=0,
+              record_exec_counts=0) -> LaunchOpts:
     o = LaunchOpts()
     load().fcl_default_launch_opts(ctypes.byref(o))
     o.mode = MODES[mode] if isinstance(mode, str) else int(mode)
@@ -237,6 +243,7 @@ def make_opts(mode="coop", forced_split=-1, init_chunk_pct=2, step_pct=2, cpu_wg
     o.flags = LAUNCH_TIMING if timing else 0
     o.host_variant = int(host_variant)
     o.select = int(select)
+    o.gpu_delay_us, o.record_exec_counts = int(gpu_delay_us), int(record_exec_counts)
     return o
 
 
@@ -335,6 +342,16 @@ class Context:
         c = (ctypes.c_int64 * len(self.COUNTERS))()
         _check(load().fcl_get_counters(self.handle, c, len(self.COUNTERS)), "fcl_get_counters", self.handle)
         return {k: int(c[i]) for i, k in enumerate(self.COUNTERS)}
+
+    def exec_counts(self, n_wg: int) -> dict:
+        """Per-work-group execution counts of the last launch made with record_exec_counts=1
+        (fcl_get_exec_counts): numpy int32 arrays gpu_done, gpu_frags, cpu_done."""
+        import numpy as np
+        out = {k: np.zeros(int(n_wg), np.int32) for k in ("gpu_done", "gpu_frags", "cpu_done")}
+        _check(load().fcl_get_exec_counts(self.handle, int(n_wg), out["gpu_done"].ctypes.data,
+                                          out["gpu_frags"].ctypes.data, out["cpu_done"].ctypes.data),
+               "fcl_get_exec_counts", self.handle)
+        return out
 
     def slice_range(self, kernel, gws, lws, rank: int, nranks: int):
         k = self.kernel(kernel) if isinstance(kernel, str) else kernel
