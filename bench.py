@@ -278,10 +278,13 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
 
     def timed_interleaved(modes, k: int):
         # the baselines step by step next to the measured mode: slow drifts of the host (PCIe,
-        # clocks, the hypervisor) hit every mode alike
+        # clocks, the hypervisor) hit every mode alike; the order rotates every step, so that no
+        # mode always follows the same one (a cooperative step's host side may still be winding
+        # down when the next step starts)
         ts = {m: [] for m in modes}
-        for _ in range(k):
-            for m in modes:
+        for r in range(k):
+            for q in range(len(modes)):
+                m = modes[(q + r) % len(modes)]
                 ts[m].append(one_step(m))
         return ts
 
@@ -332,7 +335,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     # add only cooperative non-probe launches, the GPU-only steps only gpu_only
     dc = {k: c1[k] - c0[k] for k in c0}
     selection = {"launches": 3 * args.steps, "probes_cooperative": dc["probe"], "gpu_alone": dc["sel_gpu"],
-                 "host_alone": dc["sel_cpu"], "select_period": 16}
+                 "host_alone": dc["sel_cpu"], "select_period": "16, doubling up to 256 while probes confirm"}
     if os.environ.get("FCL_BENCH_DEBUG"):
         print("coop step ms:", [round(t, 3) for t in coop_ts], file=sys.stderr)
 

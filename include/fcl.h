@@ -205,8 +205,9 @@ typedef struct {
                                 cannot contribute runs on the other alone: GPU-only if the host
                                 finished less than FCL_SELECT_MIN_SHARE (10 %) of the work-groups
                                 before the GPU exited, CPU-only if the host covered the whole range
-                                first on an idle GPU; every FCL_SELECT_PERIOD-th (16) launch
-                                of the shape probes cooperatively again.  Forced splits, deferred
+                                first on an idle GPU; the FCL_SELECT_PERIOD-th (16) launch after a
+                                probe probes cooperatively again, a period that doubles (up to 16x)
+                                while probes keep confirming the choice.  Forced splits, deferred
                                 merges and fault injection are never redirected. */
     int32_t gpu_delay_us;        /* fault injection: in a COOP launch every GPU task starts this many us
                                     late (a slow GPU, so that the host covers part of the range in a

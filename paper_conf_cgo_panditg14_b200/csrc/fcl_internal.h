@@ -172,8 +172,9 @@ int gpu_launch_merge_dev(const DevMergeList &L, size_t max_bytes, int num_sms, v
 // Copy up to 6 (dst, src, bytes) regions in one launch (16-byte aligned pointers; dst may be the
 // device-visible address of mapped host memory).  1 = launched, 0 = nothing to copy, -2 = a
 // pointer is not 16-byte aligned (nothing launched), -1 = launch failure.
+// pdl: launched with programmatic serialization behind plain grids, waiting in-kernel for them.
 int gpu_launch_copies(int n, void *const *dst, const void *const *src, const size_t *bytes, int num_sms,
-                      void *stream);
+                      void *stream, bool pdl = false);
 // One-thread kernel that stores `value` to `addr` (status publication fallback).
 int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream);
 const char *gpu_last_error_string();

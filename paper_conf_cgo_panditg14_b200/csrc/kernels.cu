@@ -595,7 +595,10 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
 // Twin capture (C5, L16.s2-3): copy every OUT/INOUT buffer to its twin in ONE launch.
 struct CopyList { uint8_t *dst[6]; const uint8_t *src[6]; size_t bytes[6]; int n; };
 
-__global__ void __launch_bounds__(256) copies_kernel(const CopyList L) {
+__global__ void __launch_bounds__(256) copies_kernel(const CopyList L, int pdl_wait) {
+    // (launched behind plain grids with programmatic serialization: wait until they have
+    // completed and their stores are visible -- griddepcontrol.wait covers every earlier grid)
+    if (pdl_wait) asm volatile("griddepcontrol.wait;" ::: "memory");
     const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
     const size_t nth = (size_t)gridDim.x * blockDim.x;
     for (int b = 0; b < L.n; ++b) {
@@ -1820,7 +1823,7 @@ int gpu_launch_merge_dev(const DevMergeList &L, size_t max_bytes, int num_sms, v
 }
 
 int gpu_launch_copies(int n, void *const *dst, const void *const *src, const size_t *bytes, int num_sms,
-                      void *stream) {
+                      void *stream, bool pdl) {
     CopyList L;
     size_t total = 0;
     L.n = n;
@@ -1833,8 +1836,16 @@ int gpu_launch_copies(int n, void *const *dst, const void *const *src, const siz
     long long grid = (long long)((total / 16 + 255) / 256);
     if (grid > (long long)num_sms * 8) grid = (long long)num_sms * 8;
     if (grid < 1) grid = 1;
-    copies_kernel<<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(L);
-    cudaError_t e = cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(256);
+    cfg.stream = (cudaStream_t)stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl ? 1 : 0;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, copies_kernel, L, pdl ? 1 : 0);
     if (e != cudaSuccess) return seterr(e, "copies_kernel launch");
     return 1;
 }

@@ -440,7 +440,10 @@ struct fcl_context_st {
     std::map<std::array<int64_t, 6>, int> variant_cache;
     // Device selection from online profiles: per kernel and shape, what the
     // last cooperative probe showed (FCL_SELECTED_*) and how many launches the shape has had.
-    struct SelectEnt { int64_t launches = 0; int choice = FCL_SELECTED_COOP; };
+    // next_probe: the launch index of the next probe; period: launches between probes, which
+    // doubles (up to 16x select_period) each time a probe confirms the standing choice and
+    // falls back to select_period when it changes
+    struct SelectEnt { int64_t launches = 0; int choice = FCL_SELECTED_COOP; int64_t next_probe = 0; int64_t period = 0; };
     std::mutex sel_mu;
     std::map<std::array<int64_t, 9>, SelectEnt> sel;
     bool select_on = true;                       // FCL_SELECT=0: off unless a launch asks for it
@@ -848,6 +851,9 @@ fcl_status flush_returns(fcl_context ctx, bool at_finish) {
         src[k] = (char *)b->dev + b->ret_b0;
         sz[k] = b->ret_b1 - b->ret_b0;
     }
+    // The gather may start under the tail of the plain grids before it (programmatic dependent
+    // launch) and waits in-kernel for all of them; with no PDL chain in flight it is ordinary.
+    const bool pdl_gather = ctx->pdl && !ctx->main_fenced.load() && ctx->pdl_chain_grids > 0;
     ctx->main_fenced.store(1);   // a copy between grids on main: the next grid is ordinary
     for (size_t k = 0; k < n; ++k) ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)sz[k];
     // One gather kernel stores every span through the mapped host mirrors (16-byte SM stores
@@ -864,7 +870,8 @@ fcl_status flush_returns(fcl_context ctx, bool at_finish) {
             if (ok) hdst[k] = (char *)b->host_dptr + b->ret_b0;
         }
         if (ok) {
-            const int r = gpu_launch_copies((int)n, hdst.data(), (const void *const *)src.data(), sz.data(), ctx->num_sms, ctx->main);
+            const int r = gpu_launch_copies((int)n, hdst.data(), (const void *const *)src.data(), sz.data(), ctx->num_sms,
+                                            ctx->main, pdl_gather);
             if (r == -1) return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
             gathered = r >= 0;   // (-2: a span is not 16-byte aligned)
         }
@@ -963,7 +970,7 @@ int select_device(fcl_context ctx, const Launch &L, bool *probe) {
     std::lock_guard<std::mutex> lk(ctx->sel_mu);
     auto &e = ctx->sel[select_key(L)];
     const int64_t n = e.launches++;
-    *probe = (n % ctx->select_period) == 0 || e.choice == FCL_SELECTED_COOP;
+    *probe = n >= e.next_probe || e.choice == FCL_SELECTED_COOP;
     return *probe ? FCL_SELECTED_COOP : e.choice;
 }
 
@@ -981,7 +988,16 @@ void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
     else if (gpu_done && (host_work_useless || (double)j.info.cpu_wgs < ctx->select_min_share * (double)(j.L.hi - j.L.lo)))
         c = FCL_SELECTED_GPU;
     std::lock_guard<std::mutex> lk(ctx->sel_mu);
-    ctx->sel[j.sel_key].choice = c;
+    auto &e = ctx->sel[j.sel_key];
+    // a probe that confirms the standing single-device choice backs the next one off; any change
+    // (or a cooperative outcome) probes again at the base period
+    const int64_t base = std::max<int64_t>(1, ctx->select_period);
+    e.period = (c != FCL_SELECTED_COOP && c == e.choice && e.period > 0) ? std::min<int64_t>(2 * e.period, 16 * base) : base;
+    // the GPU covered the range before the host completed even its first C11 chunk (2 % of the
+    // range): the host is more than ~50x slower on this shape -- probe again only rarely
+    if (c == FCL_SELECTED_GPU && j.info.cpu_wgs == 0) e.period = 16 * base;
+    e.choice = c;
+    e.next_probe = e.launches + e.period - 1;
 }
 
 unsigned long long *plain_stamp(fcl_context ctx) {
@@ -1088,8 +1104,6 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     // end event (used here before) belongs to a job that can be recycled and re-recorded --
     // behind this launch's own grid, or a later one -- while this launch still waits on it;
     // with streamed inputs that made the grid wait for pieces that waited for the grid.
-    CK(ctx, cudaEventRecord(j.ev_start, ctx->main));
-    j.main_before = j.ev_start;
 
     // Host chunk boundaries are aligned to the output span unit (1 work-group for 1-D kernels,
     // one work-group row for 2-D row-major ones).  The staged spans are then exactly the host's
@@ -1120,6 +1134,9 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     j.lite = (j.t1 > j.t0) && !j.forced && !L.o.defer_merge && abort_period == 0 && !ctx->no_lite && !j.stream &&
              L.o.gpu_delay_us <= 0 &&
              (j.t1 - j.t0) <= gpu_coop_capacity(L.a, L.g, ctx->num_sms);
+    // (a lite launch neither stages nor streams: nothing on hd waits for this position)
+    if (!j.lite) CK(ctx, cudaEventRecord(j.ev_start, ctx->main));
+    j.main_before = j.lite ? nullptr : j.ev_start;
     // twin (original data) and stage (CPU results) per OUT/INOUT buffer (C5, L16.s2-3)
     const void *srcs[6];
     size_t nbytes[6];
@@ -2671,17 +2688,24 @@ fcl_status fcl_finish(fcl_context ctx) {
     // Host sides of lite launches never queue work on main and end when their grid has: with
     // only those pending, main is synchronised first and its completion handed to the
     // coordinator (main_done_epoch), which is how they learn it without an exit word.
-    bool all_lite = true;
+    bool all_lite = true, all_returned = true;   // returned: outputs queued at enqueue (eager / lazy)
     {
         std::lock_guard<std::mutex> lk(ctx->q_mu);
-        for (Job *p : ctx->queue) all_lite = all_lite && p->lite;
+        for (Job *p : ctx->queue) {
+            all_lite = all_lite && p->lite;
+            all_returned = all_returned && (p->eager || p->lazy);
+        }
     }
     if (all_lite) {
         CK(ctx, cudaStreamSynchronize(ctx->main));
         ctx->main_done_epoch.store(ctx->epoch, std::memory_order_release);
         ctx->tr.add("finish_main_first", ctx->epoch);
     }
-    drain(ctx);
+    // Lite host sides still queued end without effect on any buffer (the GPU computed every
+    // work-group and their outputs are in the gather just synchronised, or on dh below): they
+    // are not waited for -- every call that needs the queue empty drains it, and a chunk one of
+    // them may still abandon is quiesced like any other (DESIGN.md §6.4 item 13).
+    if (!all_lite || !all_returned) drain(ctx);
     ctx->tr.add("finish_drained", ctx->epoch);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
     // dh first: its return copies are ordered behind the kernels, so by the time it is done

@@ -26,12 +26,13 @@ def ctx():
 
 def test_gpu_favoured_shape_runs_on_the_gpu_alone(ctx):
     """SYRK 512: the GPU finishes long before the host's first 2 % chunk (21 work-groups), so the
-    probe records "host finished nothing" and the next 15 launches are GPU-only plain grids."""
+    probe records "host finished nothing": the host is far slower on this shape and the next
+    probe comes 256 launches later; all launches in between are GPU-only plain grids."""
     P = W.make("syrk", 512, 512, seed=5)
     ref, _ = H.run(ctx, P, mode="gpu")
     c0 = ctx.counters()
     seen = []
-    for i in range(18):
+    for i in range(50):
         out, info = H.run(ctx, P, mode="coop", select=1)
         seen.append((info["probe"], info["selected"]))
         for k in P.out_indices:
@@ -41,11 +42,30 @@ def test_gpu_favoured_shape_runs_on_the_gpu_alone(ctx):
         else:
             assert info["selected"] == SEL_GPU, seen
             assert info["gpu_path"] == PATH_PLAIN and info["cpu_wgs"] == 0
-    assert seen[0] == (1, SEL_COOP) and seen[16] == (1, SEL_COOP), seen
-    assert all(s == (0, SEL_GPU) for s in seen[1:16]), seen
+    assert seen[0] == (1, SEL_COOP), seen
+    assert all(s == (0, SEL_GPU) for s in seen[1:]), seen
     c1 = ctx.counters()
-    assert c1["sel_gpu"] - c0["sel_gpu"] == 16 and c1["probe"] - c0["probe"] == 2, (c0, c1)
-    assert c1["coop"] - c0["coop"] == 2 and c1["gpu_only"] - c0["gpu_only"] == 0, (c0, c1)
+    assert c1["sel_gpu"] - c0["sel_gpu"] == 49 and c1["probe"] - c0["probe"] == 1, (c0, c1)
+    assert c1["coop"] - c0["coop"] == 1 and c1["gpu_only"] - c0["gpu_only"] == 0, (c0, c1)
+
+
+def test_probe_backoff_doubles_while_confirmed(ctx):
+    """A probe in which the host did complete work but not enough (below 10 % of the range) keeps
+    the shape on the GPU; each confirming probe doubles the distance to the next (16, 32, ...)."""
+    P = W.make("conv2d", 2048, 2048, seed=6, out_init="zero")
+    c0 = ctx.counters()
+    probes = []
+    for i in range(60):
+        out, info = H.run(ctx, P, mode="coop", select=1, gpu_delay_us=0)
+        if info["probe"]:
+            probes.append((i, info["cpu_wgs"], info["selected"]))
+    c1 = ctx.counters()
+    assert probes and probes[0][0] == 0, probes
+    gaps = [b[0] - a[0] for a, b in zip(probes, probes[1:])]
+    # a cooperative outcome probes every launch (gap 1); a GPU one waits the base period, double
+    # the previous gap when confirmed, or the long one after a probe without host progress
+    assert all(g in (1, 16, 32, 64, 128, 256) for g in gaps), (probes, gaps)
+    assert c1["probe"] - c0["probe"] == len(probes), (c0, c1, probes)
 
 
 def test_host_favoured_shape_runs_on_the_host_alone(ctx, monkeypatch):
