@@ -230,8 +230,10 @@ bool wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
 }
 
 // ---------------------------------------------------------------- SYRK / SYR2K
-// Each output accumulates its k-chain in ascending k, one fma per term (SYR2K: A_i*B_j then
-// B_i*A_j for each k), then C = fma(alpha, acc, beta * C).  Mirrors GemmBody in kernels.cu.
+// Each output accumulates its k-chain in ascending k, one fma per term, then
+// C = fma(alpha, acc, beta * C).  SYR2K's per-k pair order is symmetric: for i <= j A_i*B_j then
+// B_i*A_j, for i > j the mirror's B_i*A_j then A_i*B_j -- so acc(i, j) == acc(j, i) bit for bit
+// (DESIGN.md §6.1).  Mirrors GemmBody in kernels.cu.
 template <typename T, bool TWO>
 bool wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
     const int64_t n = a.n0, m = a.n1;
@@ -273,13 +275,19 @@ bool wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, 
         T *ac = acc.data();
         const T *ai = A + i * m;
         const T *bi = TWO ? B + i * m : nullptr;
+        // SYR2K: columns jj < split lie below the diagonal (j < i) and take the mirror's order
+        const int64_t split = TWO ? std::min<int64_t>(std::max<int64_t>(i - j0, 0), wc) : 0;
         for (int64_t k = 0; k < m; ++k) {
             if ((k & 511) == 511 && aborted(ab)) return false;   // write-once: nothing stored yet
             const T aik = ai[k];
             if (TWO) {
                 const T bik = bi[k];
                 const T *bt = Bt.data() + k * wc, *at = At.data() + k * wc;
-                for (int64_t jj = 0; jj < wc; ++jj) {
+                for (int64_t jj = 0; jj < split; ++jj) {
+                    ac[jj] = op_fma(bik, at[jj], ac[jj]);   // B[i][k] * A[j][k]
+                    ac[jj] = op_fma(aik, bt[jj], ac[jj]);   // A[i][k] * B[j][k]
+                }
+                for (int64_t jj = split; jj < wc; ++jj) {
                     ac[jj] = op_fma(aik, bt[jj], ac[jj]);   // A[i][k] * B[j][k]
                     ac[jj] = op_fma(bik, at[jj], ac[jj]);   // B[i][k] * A[j][k]
                 }
@@ -404,7 +412,10 @@ bool wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npart
         const T *bi = TWO ? B + i * m : nullptr, *bj = TWO ? B + j * m : nullptr;
         T acc = 0;
         for (int64_t k = 0; k < m; ++k) {
-            if (TWO) {
+            if (TWO && i > j) {                    // below the diagonal: the mirror's order
+                acc = op_fma(bi[k], aj[k], acc);   // B[i][k] * A[j][k]
+                acc = op_fma(ai[k], bj[k], acc);   // A[i][k] * B[j][k]
+            } else if (TWO) {
                 acc = op_fma(ai[k], bj[k], acc);   // A[i][k] * B[j][k]
                 acc = op_fma(bi[k], aj[k], acc);   // B[i][k] * A[j][k]
             } else {

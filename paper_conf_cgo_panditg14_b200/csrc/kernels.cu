@@ -21,6 +21,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <type_traits>
 
 #include "fcl_internal.h"
 
@@ -1056,11 +1057,19 @@ enum { G_SYRK = 0, G_SYR2K = 1, G_CORR = 2 };
 constexpr int GBM = 128, GBK = 16, GPAD = 4;
 
 // TN: outputs per thread along the tile's columns.  TN = 8: 256 threads, 8 x 8 outputs each,
-// two CTAs per SM.  TN = 4: 512 threads, 8 x 4 each, one CTA per SM -- for SYRK's upper-triangle
-// grid (136 tiles at N = 2048, one per SM), where 16 warps hide the k'-tile loads that 8 cannot.
+// two CTAs per SM.  TN = 4: 512 threads, 8 x 4 each, one CTA per SM -- for the SYRK / SYR2K
+// upper-triangle grids (136 tiles at N = 2048, one per SM), where 16 warps hide the k'-tile
+// loads that 8 cannot.
+//
+// SYR2K's canonical per-k order is symmetric: output (i, j) with i <= j
+// accumulates A_i[k]*B_j[k] then B_i[k]*A_j[k]; an output below the diagonal takes its mirror's
+// chain, B_i[k]*A_j[k] then A_i[k]*B_j[k].  So acc(i, j) == acc(j, i) bit for bit, and like SYRK
+// the kernel can run the upper-triangle tiles only and write each one's mirror block; a tile
+// below the diagonal (slices) is the same GEMM with A and B exchanged, and a diagonal tile
+// stores its upper half and that half's mirror.
 template <typename T, int OP, int TN = 8>
 struct GemmBody {
-    static_assert(TN == 8 || (TN == 4 && OP != G_SYR2K), "TN = 4: SYRK upper triangle, CORR symmat");
+    static_assert(TN == 8 || TN == 4, "TN = 4: the upper-triangle grids, CORR symmat");
     static constexpr int kThreads = TN == 8 ? 256 : 512;
 #ifndef FCL_GEMM_MINB
 #define FCL_GEMM_MINB 2
@@ -1086,7 +1095,7 @@ struct GemmBody {
     struct Smem { T s[2][2][GBK][GBM + GPAD]; };   // [stage][A|B][k'][m]
 
     __device__ static void tile_of(const Params &p, long long t, long long &bi, long long &bj) {
-        if (OP == G_CORR || (OP == G_SYRK && p.sym)) {  // upper triangle, row-major over (b1 <= b2)
+        if (OP == G_CORR || p.sym) {  // upper triangle, row-major over (b1 <= b2)
             long long b1 = 0, rem = t;
             while (rem >= p.ntile - b1) { rem -= p.ntile - b1; ++b1; }
             bi = b1; bj = b1 + rem;
@@ -1127,11 +1136,40 @@ struct GemmBody {
         const T4 v = ld_cached4(q);
         r[0] = v.x; r[1] = v.y; r[2] = v.z; r[3] = v.w;
     }
+    // KP consecutive k of row `row` of X (SYR2K operands): IN without bounds checks
+    template <bool IN, int KP>
+    __device__ static void loadk(const Params &p, const T *X, long long row, long long k, T *r) {
+        if (KP == 4) {
+            if (IN) ld4(X + row * p.ld + k, r);
+            else load4_k(p, X, row, k, r);
+        } else if (IN) {   // (k even, ld % 4 == 0: 8-byte aligned)
+            typedef typename std::conditional<sizeof(T) == 4 && std::is_same<T, float>::value, float2, int2>::type T2;
+            const T2 v = __ldg(reinterpret_cast<const T2 *>(X + row * p.ld + k));
+            r[0] = v.x; r[1] = v.y;
+        } else {
+#pragma unroll
+            for (int q = 0; q < KP; ++q) r[q] = (row < p.n && k + q < p.m) ? X[row * p.ld + k + q] : T(0);
+        }
+    }
     // One k'-tile into registers: 8 elements of each operand tile per thread.  IN: the tile and
     // the k'-range are interior (no bounds checks).
     template <bool IN>
-    __device__ static void gload(const Params &p, long long i0, long long j0, long long kt, T ra[LD], T rb[LD]) {
+    __device__ static void gload(const Params &p, long long i0, long long j0, long long kt, T ra[LD], T rb[LD], bool sw) {
         const int tid = threadIdx.x;
+        if (OP == G_SYR2K) {   // this k'-tile covers k in [kt*GBK/2, (kt+1)*GBK/2), KP of them per thread
+            constexpr int KP = LD / 2, TPR = (GBK / 2) / KP;
+            const int row = tid / TPR;
+            const long long k = kt * (GBK / 2) + (tid % TPR) * KP;
+            const T *PA = sw ? p.B : p.A, *PB = sw ? p.A : p.B;   // sw: a tile below the diagonal
+            T x[KP], y[KP];
+            loadk<IN, KP>(p, PA, i0 + row, k, x); loadk<IN, KP>(p, PB, i0 + row, k, y);
+#pragma unroll
+            for (int q = 0; q < KP; ++q) { ra[2 * q] = x[q]; ra[2 * q + 1] = y[q]; }   // A_i[k], B_i[k]
+            loadk<IN, KP>(p, PB, j0 + row, k, x); loadk<IN, KP>(p, PA, j0 + row, k, y);
+#pragma unroll
+            for (int q = 0; q < KP; ++q) { rb[2 * q] = x[q]; rb[2 * q + 1] = y[q]; }   // B_j[k], A_j[k]
+            return;
+        }
         if (IN) {
             if (OP == G_CORR) {
                 const int kk = tid / (GBM / LD), c = (tid % (GBM / LD)) * LD;
@@ -1144,16 +1182,6 @@ struct GemmBody {
                 const T *xa = p.A + (i0 + row) * p.ld + k, *xb = p.A + (j0 + row) * p.ld + k;
                 ld4(xa, ra); ld4(xb, rb);
                 if (LD == 8) { ld4(xa + 4, ra + 4); ld4(xb + 4, rb + 4); }
-            } else {
-                const int row = tid >> 1;
-                const long long k = kt * (GBK / 2) + (tid & 1) * 4;
-                T x[4], y[4];
-                ld4(p.A + (i0 + row) * p.ld + k, x); ld4(p.B + (i0 + row) * p.ld + k, y);
-#pragma unroll
-                for (int q = 0; q < 4; ++q) { ra[2 * q] = x[q]; ra[2 * q + 1] = y[q]; }
-                ld4(p.B + (j0 + row) * p.ld + k, x); ld4(p.A + (j0 + row) * p.ld + k, y);
-#pragma unroll
-                for (int q = 0; q < 4; ++q) { rb[2 * q] = x[q]; rb[2 * q + 1] = y[q]; }
             }
             return;
         }
@@ -1162,21 +1190,11 @@ struct GemmBody {
             const long long k = kt * GBK + kk;
             load4_row(p, p.A, k, i0 + c, ra); load4_row(p, p.A, k, j0 + c, rb);
             if (LD == 8) { load4_row(p, p.A, k, i0 + c + 4, ra + 4); load4_row(p, p.A, k, j0 + c + 4, rb + 4); }
-        } else if (OP == G_SYRK) {
+        } else {   // SYRK
             const int row = tid / (GBK / LD);
             const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
             load4_k(p, p.A, i0 + row, k, ra); load4_k(p, p.A, j0 + row, k, rb);
             if (LD == 8) { load4_k(p, p.A, i0 + row, k + 4, ra + 4); load4_k(p, p.A, j0 + row, k + 4, rb + 4); }
-        } else {   // SYR2K: this k'-tile covers k in [kt*GBK/2, (kt+1)*GBK/2)
-            const int row = tid >> 1;
-            const long long k = kt * (GBK / 2) + (tid & 1) * 4;
-            T x[4], y[4];
-            load4_k(p, p.A, i0 + row, k, x); load4_k(p, p.B, i0 + row, k, y);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) { ra[2 * q] = x[q]; ra[2 * q + 1] = y[q]; }   // A_i[k], B_i[k]
-            load4_k(p, p.B, j0 + row, k, x); load4_k(p, p.A, j0 + row, k, y);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) { rb[2 * q] = x[q]; rb[2 * q + 1] = y[q]; }   // B_j[k], A_j[k]
         }
     }
     __device__ static T4 mk4(T a, T b, T c, T d) { T4 v; v.x = a; v.y = b; v.z = c; v.w = d; return v; }
@@ -1268,12 +1286,13 @@ struct GemmBody {
 
     // The k'-loop (ascending k' per output, one fma per term).  Returns true on an abort.
     template <bool IN>
-    __device__ static bool mainloop(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][TN]) {
+    __device__ static bool mainloop(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][TN],
+                                    bool sw) {
         const int tx = threadIdx.x % TXN, ty = threadIdx.x / TXN;
         const long long kdim = (OP == G_SYR2K) ? 2 * p.m : p.m;   // K'
         const long long nkt = (kdim + GBK - 1) / GBK;
         T ra[LD], rb[LD];
-        gload<IN>(p, i0, j0, 0, ra, rb);
+        gload<IN>(p, i0, j0, 0, ra, rb, sw);
         sstore(sm, 0, ra, rb);
         __syncthreads();
         const long long per = tc.period();
@@ -1281,7 +1300,7 @@ struct GemmBody {
             const long long kend = (nkt - kb < per) ? nkt : kb + per;
             for (long long kt = kb; kt < kend; ++kt) {
                 const int st = (int)(kt & 1);
-                if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb);   // next k'-tile in flight
+                if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb, sw);   // next k'-tile in flight
                 T a[2][8], b[2][TN];
                 frag(sm, st, 0, tx, ty, a[0], b[0]);
 #pragma unroll
@@ -1323,7 +1342,8 @@ struct GemmBody {
                 done_async = true;
             }
         }
-        if (!done_async && (interior ? mainloop<true>(p, i0, j0, tc, sm, acc) : mainloop<false>(p, i0, j0, tc, sm, acc)))
+        const bool sw = OP == G_SYR2K && bi > bj;   // below the diagonal: the mirror's chain
+        if (!done_async && (interior ? mainloop<true>(p, i0, j0, tc, sm, acc, sw) : mainloop<false>(p, i0, j0, tc, sm, acc, sw)))
             return true;
         // epilogue: write-once stores, only of outputs whose work-group is below the mask
         const unsigned int wm = tc.wmask;
@@ -1334,7 +1354,10 @@ struct GemmBody {
                                                   : uj / (unsigned int)p.lws0 + (unsigned int)p.ngx * (ui / (unsigned int)p.lws1);
             return f < wm;
         };
-        if (OP == G_SYRK && p.sym && bi != bj) {
+        // SYR2K diagonal tile: only its upper half (i <= j) is in the canonical order; the lower
+        // half is that half's mirror
+        const bool diag2 = OP == G_SYR2K && bi == bj;
+        if (OP != G_CORR && ((p.sym && bi != bj) || diag2)) {
             // mirror block: C[j][i] from acc(i, j) (bit-identical to acc(j, i)); the four rows
             // r of a thread's half are four consecutive columns of the mirror row
 #pragma unroll
@@ -1345,7 +1368,7 @@ struct GemmBody {
 #pragma unroll
                 for (int half = 0; half < 2; ++half) {
                     const long long ib = i0 + half * 64 + ty * 4;
-                    if (p.vec4 && ib + 3 < p.n && keep(j, ib + 3)) {
+                    if (p.vec4 && ib + 3 < p.n && keep(j, ib + 3) && (!diag2 || ib + 3 < j)) {
                         T4 cv = *reinterpret_cast<T4 *>(crow + ib);
                         cv.x = op_fma(p.alpha, acc[half * 4 + 0][c], op_mul(p.beta, cv.x));
                         cv.y = op_fma(p.alpha, acc[half * 4 + 1][c], op_mul(p.beta, cv.y));
@@ -1356,7 +1379,8 @@ struct GemmBody {
 #pragma unroll
                         for (int r = 0; r < 4; ++r) {
                             const long long i = ib + r;
-                            if (i < p.n && keep(j, i)) crow[i] = op_fma(p.alpha, acc[half * 4 + r][c], op_mul(p.beta, crow[i]));
+                            if (i < p.n && keep(j, i) && (!diag2 || i < j))
+                                crow[i] = op_fma(p.alpha, acc[half * 4 + r][c], op_mul(p.beta, crow[i]));
                         }
                     }
                 }
@@ -1380,7 +1404,7 @@ struct GemmBody {
                 } else {
                     if (i >= p.n) continue;
                     T *crow = p.C + i * p.n;
-                    if (p.vec4 && jb + 3 < p.n && keep(i, jb + 3)) {
+                    if (p.vec4 && jb + 3 < p.n && keep(i, jb + 3) && (!diag2 || jb >= i)) {
                         T4 cv = *reinterpret_cast<T4 *>(crow + jb);
                         cv.x = op_fma(p.alpha, acc[r][half * 4 + 0], op_mul(p.beta, cv.x));
                         cv.y = op_fma(p.alpha, acc[r][half * 4 + 1], op_mul(p.beta, cv.y));
@@ -1391,7 +1415,8 @@ struct GemmBody {
 #pragma unroll
                         for (int c = 0; c < 4; ++c) {
                             const long long j = jb + c;
-                            if (j < p.n && keep(i, j)) crow[j] = op_fma(p.alpha, acc[r][half * 4 + c], op_mul(p.beta, crow[j]));
+                            if (j < p.n && keep(i, j) && (!diag2 || j >= i))
+                                crow[j] = op_fma(p.alpha, acc[r][half * 4 + c], op_mul(p.beta, crow[j]));
                         }
                     }
                 }
@@ -1535,7 +1560,7 @@ static typename GemmBody<T, OP, TN>::Params gemm_params(const KArgs &a, const Ge
     p.ngx = g.ng[0]; p.lws0 = g.lws[0]; p.lws1 = g.work_dim > 1 ? g.lws[1] : 1; p.lws = g.lws[0];
     p.vec4 = (p.ld % 4 == 0) && (p.n % 4 == 0) && is_aligned16(p.A) && is_aligned16(p.C) &&
              (OP != G_SYR2K || is_aligned16(p.B));
-    p.sym = (OP == G_SYRK && a.sym) ? 1 : 0;
+    p.sym = (OP != G_CORR && a.sym) ? 1 : 0;
     return p;
 }
 
@@ -1591,6 +1616,10 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
         if (a.integer) return f.template go<GemmBody<int32_t, G_SYRK>>(gemm_params<int32_t, G_SYRK>(a, g));
         return f.template go<GemmBody<float, G_SYRK>>(gemm_params<float, G_SYRK>(a, g));
     case K_SYR2K:
+        if (a.sym) {   // upper-triangle grid: one 512-thread CTA per SM
+            if (a.integer) return f.template go<GemmBody<int32_t, G_SYR2K, 4>>(gemm_params<int32_t, G_SYR2K, 4>(a, g));
+            return f.template go<GemmBody<float, G_SYR2K, 4>>(gemm_params<float, G_SYR2K, 4>(a, g));
+        }
         if (a.integer) return f.template go<GemmBody<int32_t, G_SYR2K>>(gemm_params<int32_t, G_SYR2K>(a, g));
         return f.template go<GemmBody<float, G_SYR2K>>(gemm_params<float, G_SYR2K>(a, g));
     case K_CORR_CORR:
@@ -1628,8 +1657,8 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
     }
     case K_SYRK: case K_SYR2K: {
         const long long nt = (a.n0 + GBM - 1) / GBM;
-        ts.ntasks = (a.kernel == K_SYRK && a.sym) ? nt * (nt + 1) / 2 : nt * nt;
-        ts.threads = (a.kernel == K_SYRK && a.sym) ? 512 : 256; break;
+        ts.ntasks = a.sym ? nt * (nt + 1) / 2 : nt * nt;
+        ts.threads = a.sym ? 512 : 256; break;
     }
     case K_CORR_CORR: {
         const long long nt = (a.n1 + GBM - 1) / GBM;
@@ -1655,7 +1684,7 @@ int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t) {
     case K_SYRK: case K_SYR2K: {
         const long long nt = (a.n0 + GBM - 1) / GBM;
         long long bi = t / nt, bj = t % nt;
-        if (a.kernel == K_SYRK && a.sym) {   // upper triangle; the key is the direct block's
+        if (a.sym) {   // upper triangle; the key is the direct block's
             long long rem = t;
             bi = 0;
             while (rem >= nt - bi) { rem -= nt - bi; ++bi; }
@@ -1694,7 +1723,7 @@ void gpu_task_wgs(const KArgs &a, const Geom &g, int64_t t, std::vector<int64_t>
     case K_SYRK: case K_SYR2K: {
         const long long nt = (a.n0 + GBM - 1) / GBM;
         long long bi = t / nt, bj = t % nt;
-        const bool sym = a.kernel == K_SYRK && a.sym;
+        const bool sym = a.sym;
         if (sym) {
             long long rem = t;
             bi = 0;
@@ -1886,6 +1915,7 @@ int gpu_preload_kernels() {
     bad |= preload_body<GemmBody<float, G_SYRK>>() | preload_body<GemmBody<int32_t, G_SYRK>>();
     bad |= preload_body<GemmBody<float, G_SYRK, 4>>() | preload_body<GemmBody<int32_t, G_SYRK, 4>>();
     bad |= preload_body<GemmBody<float, G_SYR2K>>() | preload_body<GemmBody<int32_t, G_SYR2K>>();
+    bad |= preload_body<GemmBody<float, G_SYR2K, 4>>() | preload_body<GemmBody<int32_t, G_SYR2K, 4>>();
     bad |= preload_body<GemmBody<float, G_CORR, FCL_CORR_TN>>();
     cudaFuncAttributes at;
     bad |= cudaFuncGetAttributes(&at, merge_kernel<1>) != cudaSuccess;

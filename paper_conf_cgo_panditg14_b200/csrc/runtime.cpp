@@ -2450,7 +2450,7 @@ static fcl_status build_launch(fcl_context ctx, fcl_kernel kernel, uint32_t work
         return set_err(ctx, FCL_INVALID_VALUE, "wg range must be aligned to %lld work-groups (fcl_slice_range)", (long long)al);
     // (the whole range only: a slice's mirror blocks would land in rows outside it and update
     // the device copy of C there -- a later slice on the same buffer would read them final)
-    a.sym = a.kernel == K_SYRK && lo == 0 && hi == g.n_wg && !ctx->no_sym;
+    a.sym = (a.kernel == K_SYRK || a.kernel == K_SYR2K) && lo == 0 && hi == g.n_wg && !ctx->no_sym;
     L.ctx = ctx; L.kd = kd; L.a = a; L.g = g; L.lo = lo; L.hi = hi; L.o = o;
     return FCL_SUCCESS;
 }

@@ -504,11 +504,14 @@ def test_executor_back_to_back_jobs_in_place(ctx):
             assert_bits(out[i], ref[i], f"syrk {n}x70 cpu-only")
 
 
-def test_syrk_slices_same_buffer(ctx):
-    """SYRK (C in place) run as consecutive slices on the SAME buffers, each slice cooperative:
-    every element of C is updated exactly once (a slice must not touch C's device copy outside
-    its rows -- the upper-triangle grid's mirror blocks would), and the result is the GPU-only one."""
-    P = W.make("syrk", 384, 96, seed=61)
+@pytest.mark.parametrize("kernel", ["syrk", "syr2k"])
+def test_syrk_slices_same_buffer(ctx, kernel):
+    """SYRK / SYR2K (C in place) run as consecutive slices on the SAME buffers, each slice
+    cooperative: every element of C is updated exactly once (a slice must not touch C's device
+    copy outside its rows -- the upper-triangle grid's mirror blocks would), and the result is the
+    GPU-only one (a slice runs every tile of its rows: SYR2K tiles below the diagonal take the
+    mirror's per-k order, diagonal tiles store their upper half and its mirror)."""
+    P = W.make(kernel, 384, 96, seed=61)
     ref, _ = H.run(ctx, P, mode="gpu")
     k = ctx.kernel(H.kernel_name(P))
     for nranks in (2, 3):
@@ -518,9 +521,27 @@ def test_syrk_slices_same_buffer(ctx):
             ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, bufs), mode="coop",
                                 wg_lo=lo, wg_hi=hi)
             ctx.finish()
-        out = bufs[1].read_array(np.float32)
-        assert_bits(out, ref[1], f"syrk {nranks} slices on one buffer")
-        dev = H.device_array(bufs[1], np.float32)
-        assert_bits(dev, ref[1], f"syrk {nranks} slices, device copy")
+        o = P.out_indices[0]
+        out = bufs[o].read_array(np.float32)
+        assert_bits(out, ref[o], f"{kernel} {nranks} slices on one buffer")
+        dev = H.device_array(bufs[o], np.float32)
+        assert_bits(dev, ref[o], f"{kernel} {nranks} slices, device copy")
         for b in bufs:
             b.release()
+
+
+@pytest.mark.parametrize("integer", [False, True])
+@pytest.mark.parametrize("kernel,n,m", [("syrk", 300, 77), ("syr2k", 300, 77), ("syr2k", 256, 64)])
+def test_symmetric_accumulators(ctx, kernel, n, m, integer):
+    """SYRK and SYR2K's canonical per-k order is symmetric: with a symmetric C
+    the result is symmetric bit for bit -- on the GPU (upper-triangle grid with mirrors, and the
+    full grid of a forced split), and on the host."""
+    P = W.make(kernel, n, m, integer=integer, seed=62)
+    o = P.out_indices[0]
+    C = P.bufs[o].reshape(n, n)
+    P.bufs[o] = np.ascontiguousarray(np.triu(C) + np.triu(C, 1).T).reshape(-1)
+    dt = np.int32 if integer else np.float32
+    for mode, opts in [("gpu", {}), ("cpu", {}), ("coop", {"forced_split": P.num_groups // 3})]:
+        out, _ = H.run(ctx, P, mode=mode, **opts)
+        r = out[o].reshape(n, n).view(np.uint32)
+        assert np.array_equal(r, r.T), f"{kernel} {mode} {opts}: not symmetric at {np.argwhere(r != r.T)[:3]}"

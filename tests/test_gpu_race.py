@@ -126,6 +126,7 @@ RACE_FULL = [
     # kernel, n0, n1, lws1d, gpu_delay_us: a slow GPU lets the host cover part of the range
     ("conv2d", 16384, 16384, None, 30),
     ("syrk", 2048, 2048, None, 40000),
+    ("syr2k", 2048, 2048, None, 80000),
     ("corr_reduce", 4096, 4096, None, 1000),
     ("gesummv", 4096, 4096, 64, 3000),
 ]
