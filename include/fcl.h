@@ -305,6 +305,24 @@ fcl_status fcl_merge(fcl_context ctx, fcl_buffer buf);
 fcl_status fcl_merge_raw(void *gpu, const void *cpu, const void *twin, size_t bytes,
                          uint32_t elem_size, void *stream);
 
+/* The caller changed [offset, offset+n) of buf's device copy outside the runtime -- the NCCL
+ * all-gather that brings other ranks' output slices into it ("the slices are
+ * concatenated ... when the kernel's output is needed whole").  The writes were queued on
+ * `stream` (cudaStream_t; NULL = the context's main stream): later work of the context is ordered
+ * after them.  The device copy becomes authoritative; the host mirror is refreshed on demand (a
+ * read, a host-side launch).  Waits for pending launches first.
+ * Errors: FCL_INVALID_MEM_OBJECT, FCL_INVALID_VALUE (range), FCL_CONTEXT_LOST. */
+fcl_status fcl_buffer_device_written(fcl_context ctx, fcl_buffer buf, size_t offset, size_t n, void *stream);
+
+/* Mirror the upper triangle of an n x n row-major matrix on the device into its lower
+ * triangle: a[j][i] = a[i][j] for every i < j (elem_size 4 or 8; the diagonal is untouched).
+ * The combine step of CORR's symmat across ranks: work-group j1 writes row j1 right of the
+ * diagonal and column j1 below it (PolyBench CORR, Table 2 / L22.s36), so a rank's slice is
+ * L-shaped; after the row slabs are all-gathered, the upper triangle is complete and the lower
+ * one follows from it.  `a` is a device pointer; asynchronous on `stream`.
+ * Errors: FCL_INVALID_VALUE, FCL_CUDA_ERROR. */
+fcl_status fcl_mirror_upper(void *a, size_t n, uint32_t elem_size, void *stream);
+
 /* Wait until every launch, merge and copy of the context has completed;
  * outputs are then coherent on host and device.  Reports deferred errors. */
 fcl_status fcl_finish(fcl_context ctx);

@@ -176,6 +176,8 @@ int gpu_launch_merge_dev(const DevMergeList &L, size_t max_bytes, int num_sms, v
 // pdl: launched with programmatic serialization behind plain grids, waiting in-kernel for them.
 int gpu_launch_copies(int n, void *const *dst, const void *const *src, const size_t *bytes, int num_sms,
                       void *stream, bool pdl = false);
+// a[j][i] = a[i][j] for i < j on an n x n row-major device matrix (multi-rank CORR combine).
+int gpu_launch_mirror_upper(void *a, long long n, int elem_size, int num_sms, void *stream);
 // One-thread kernel that stores `value` to `addr` (status publication fallback).
 int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream);
 const char *gpu_last_error_string();

@@ -115,33 +115,42 @@ struct TaskCtx {
     const CoopCtl *c;            // nullptr for plain launches (parameter space, no register copy)
     unsigned long long *s_st;    // shared, 16-byte aligned: status pair prefetched by thread 0
     long long *s_key;            // shared: key of the running task
-    int *s_flag;                 // shared broadcast slot (D2: the local 'completedatcpu'); w + 1 after an abort
+    int *s_flag;                 // shared, 2 slots (D2: the local 'completedatcpu'); w + 1 after an abort
+    int polls;                   // polls so far (uniform): slot polls & 1 is the next one's
     // The watermark this task was checked against: work-groups with flattened id >= wmask are
     // the host's, so a task spanning several work-groups (tiles) stores none of their outputs --
     // at a fixed split every output word is then written by exactly one device (north_star's
     // invariant, L16.s9 "non-overlapping parts").  0xFFFFFFFF: no mask (plain grids, first tasks).
     unsigned int wmask;
 
-    // In-task poll period in body iterations (a huge value when there is none): bodies run
-    // their inner loop in blocks of this many iterations and call check() between blocks, so
-    // the inner loop itself carries no polling code.
+    // In-task poll period in body iterations (a huge value when there is none).
     __device__ __forceinline__ long long period() const {
         return (c != nullptr && c->abort_period > 0) ? (long long)c->abort_period : (1ll << 62);
     }
-    // Called by ALL threads at a CTA-uniform point.
-    __device__ __forceinline__ bool check() {
-        if (c == nullptr || c->abort_period <= 0) return false;
+    // A poll in two halves around a barrier the body executes anyway (no barrier of its own):
+    // post() -- thread 0 takes the prefetched status and writes the verdict into this poll's
+    // slot -- before the barrier, verdict() after it (all threads).  Consecutive polls use
+    // alternate slots, so a poll never overwrites a verdict a slow thread has yet to read.
+    __device__ __forceinline__ void post() {
         if (threadIdx.x == 0) {
             const unsigned int w = decode_w(status_take(*c, s_st), *c);
             status_prefetch(*c, s_st);   // consumed at the next poll
-            *s_flag = ((unsigned long long)*s_key >= (unsigned long long)w) ? (int)(w + 1u) : 0;
+            s_flag[polls & 1] = ((unsigned long long)*s_key >= (unsigned long long)w) ? (int)(w + 1u) : 0;
         }
-        __syncthreads();
-        const int f = *s_flag;
-        __syncthreads();
+    }
+    __device__ __forceinline__ bool verdict() {
+        const int f = ((volatile int *)s_flag)[polls & 1];
+        ++polls;
         return f != 0;
     }
-    __device__ __forceinline__ unsigned int abort_w() const { return (unsigned int)(*s_flag - 1); }
+    // A complete poll (called by ALL threads at a CTA-uniform point).
+    __device__ __forceinline__ bool check() {
+        if (c == nullptr || c->abort_period <= 0) return false;
+        post();
+        __syncthreads();
+        return verdict();
+    }
+    __device__ __forceinline__ unsigned int abort_w() const { return (unsigned int)(s_flag[(polls - 1) & 1] - 1); }
 };
 
 // ------------------------------------------------------------------------------------------
@@ -358,7 +367,7 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     __shared__ long long s_task, s_key;
     __shared__ __align__(16) unsigned long long s_st[2];
     __shared__ unsigned int s_w;
-    __shared__ int s_flag;
+    __shared__ int s_flag[2];
     __shared__ __align__(16) typename Body::Smem smem;
 
     if (blockIdx.x == 0 && threadIdx.x == 0) {   // counters of the next launch (stream-ordered)
@@ -393,7 +402,7 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     }
     const bool claims = c.task_lo + (long long)gridDim.x < c.task_hi;
     TaskCtx tc;
-    tc.c = &c; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.s_st = s_st; tc.wmask = 0xFFFFFFFFu;
+    tc.c = &c; tc.s_flag = s_flag; tc.s_key = &s_key; tc.s_st = s_st; tc.wmask = 0xFFFFFFFFu; tc.polls = 0;
     // the status is needed only by in-task polls and by the check before a claimed task
     const bool need_status = claims || c.abort_period > 0;
     if (threadIdx.x == 0 && need_status) status_prefetch(c, s_st);
@@ -436,10 +445,10 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
                     __nanosleep(ns);
                     if (ns < 2048) ns *= 2;
                 }
-                s_flag = covered;
+                s_flag[0] = covered;
             }
             __syncthreads();
-            const int covered = s_flag;
+            const int covered = s_flag[0];
             __syncthreads();
             if (covered) break;
         }
@@ -551,7 +560,7 @@ __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.lau
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
 plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo, const SlotReset r, int pdl_wait) {
-    __shared__ int s_flag;
+    __shared__ int s_flag[2];
     if (pdl_wait) pdl_wait_prior();
     if (r.tstamp && blockIdx.x == 0 && threadIdx.x == 0) r.tstamp[0] = globaltimer();
     if (blockIdx.x == 0) {
@@ -572,7 +581,7 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
     __shared__ __align__(16) typename Body::Smem smem;
     __shared__ long long s_key;
     TaskCtx tc;
-    tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = &s_flag; tc.s_key = &s_key; tc.wmask = 0xFFFFFFFFu;
+    tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = s_flag; tc.s_key = &s_key; tc.wmask = 0xFFFFFFFFu; tc.polls = 0;
     Body::run(bp, task_lo + (long long)blockIdx.x, tc, smem);
     if (r.exec_cnt && threadIdx.x == 0) atomicAdd(r.exec_cnt + blockIdx.x, 1u);   // test hook
     if (r.tstamp) {
@@ -1161,13 +1170,10 @@ struct GemmBody {
             const int row = tid / TPR;
             const long long k = kt * (GBK / 2) + (tid % TPR) * KP;
             const T *PA = sw ? p.B : p.A, *PB = sw ? p.A : p.B;   // sw: a tile below the diagonal
-            T x[KP], y[KP];
-            loadk<IN, KP>(p, PA, i0 + row, k, x); loadk<IN, KP>(p, PB, i0 + row, k, y);
-#pragma unroll
-            for (int q = 0; q < KP; ++q) { ra[2 * q] = x[q]; ra[2 * q + 1] = y[q]; }   // A_i[k], B_i[k]
-            loadk<IN, KP>(p, PB, j0 + row, k, x); loadk<IN, KP>(p, PA, j0 + row, k, y);
-#pragma unroll
-            for (int q = 0; q < KP; ++q) { rb[2 * q] = x[q]; rb[2 * q + 1] = y[q]; }   // B_j[k], A_j[k]
+            // loaded straight into the staging registers in memory order (the interleave to
+            // k' = 2k, 2k + 1 happens in sstore: a register shuffle here would wait for the load)
+            loadk<IN, KP>(p, PA, i0 + row, k, ra); loadk<IN, KP>(p, PB, i0 + row, k, ra + KP);   // A_i[k..], B_i[k..]
+            loadk<IN, KP>(p, PB, j0 + row, k, rb); loadk<IN, KP>(p, PA, j0 + row, k, rb + KP);   // B_j[k..], A_j[k..]
             return;
         }
         if (IN) {
@@ -1207,6 +1213,14 @@ struct GemmBody {
             if (LD == 8) {
                 *reinterpret_cast<T4 *>(&sm.s[st][0][kk][c + 4]) = mk4(ra[4], ra[5], ra[6], ra[7]);
                 *reinterpret_cast<T4 *>(&sm.s[st][1][kk][c + 4]) = mk4(rb[4], rb[5], rb[6], rb[7]);
+            }
+        } else if (OP == G_SYR2K) {   // ra = [A_i k.., B_i k..] -> k' = 2q: A_i[k+q], 2q + 1: B_i[k+q]
+            constexpr int KP = LD / 2;
+            const int row = tid / (GBK / LD), kq = (tid % (GBK / LD)) * LD;
+#pragma unroll
+            for (int q = 0; q < KP; ++q) {
+                sm.s[st][0][kq + 2 * q][row] = ra[q]; sm.s[st][0][kq + 2 * q + 1][row] = ra[KP + q];
+                sm.s[st][1][kq + 2 * q][row] = rb[q]; sm.s[st][1][kq + 2 * q + 1][row] = rb[KP + q];
             }
         } else {
             const int row = tid / (GBK / LD), kq = (tid % (GBK / LD)) * LD;
@@ -1252,9 +1266,14 @@ struct GemmBody {
 #pragma unroll
         for (int q = 0; q < NSA - 1; ++q) issue(q);
         const long long per = 2 * tc.period();   // polls every `per` GBKA-tiles (= period GBK-tiles)
+        bool poll = false;   // a poll posted at the end of the previous tile, decided after the barrier
         for (long long kt = 0; kt < nkt; ++kt) {
             asm volatile("cp.async.wait_group %0;" ::"n"(NSA - 2) : "memory");
             __syncthreads();   // tile kt landed for every thread; stage (kt-1) % NSA is free
+            if (poll && tc.verdict()) {   // abort check (Fig 12)
+                asm volatile("cp.async.wait_all;" ::: "memory");
+                return true;
+            }
             issue(kt + NSA - 1);
             const int st = (int)(kt % NSA);
             T a[2][8], b[2][TN];
@@ -1275,10 +1294,8 @@ struct GemmBody {
 #pragma unroll
                     for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
             }
-            if ((kt + 1) % per == 0 && kt + 1 < nkt && tc.check()) {   // abort check (Fig 12)
-                asm volatile("cp.async.wait_all;" ::: "memory");
-                return true;
-            }
+            poll = per > 0 && (kt + 1) % per == 0 && kt + 1 < nkt && tc.c != nullptr && tc.c->abort_period > 0;
+            if (poll) tc.post();
         }
         asm volatile("cp.async.wait_all;" ::: "memory");
         return false;
@@ -1295,26 +1312,33 @@ struct GemmBody {
         gload<IN>(p, i0, j0, 0, ra, rb, sw);
         sstore(sm, 0, ra, rb);
         __syncthreads();
+        // abort check every abort_period k'-tiles (Fig 12), folded into the k'-tile's own barrier:
+        // one loop, no extra barrier (a plain grid has no polls at all: period() is constant)
         const long long per = tc.period();
-        for (long long kb = 0; kb < nkt; kb += per) {   // blocks of `per` k'-tiles, polls between them
-            const long long kend = (nkt - kb < per) ? nkt : kb + per;
-            for (long long kt = kb; kt < kend; ++kt) {
-                const int st = (int)(kt & 1);
-                if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb, sw);   // next k'-tile in flight
-                T a[2][8], b[2][TN];
-                frag(sm, st, 0, tx, ty, a[0], b[0]);
+        const bool polling = per < nkt;
+        long long left = per;
+        for (long long kt = 0; kt < nkt; ++kt) {
+            const int st = (int)(kt & 1);
+            if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb, sw);   // next k'-tile in flight
+            T a[2][8], b[2][TN];
+            frag(sm, st, 0, tx, ty, a[0], b[0]);
 #pragma unroll
-                for (int kk = 0; kk < GBK; ++kk) {
-                    if (kk + 1 < GBK) frag(sm, st, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
+            for (int kk = 0; kk < GBK; ++kk) {
+                if (kk + 1 < GBK) frag(sm, st, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
 #pragma unroll
-                    for (int r = 0; r < 8; ++r)
+                for (int r = 0; r < 8; ++r)
 #pragma unroll
-                        for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
-                }
-                if (kt + 1 < nkt) sstore(sm, st ^ 1, ra, rb);
-                __syncthreads();
+                    for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
             }
-            if (kend < nkt && tc.check()) return true;   // abort check every abort_period k'-tiles (Fig 12)
+            bool poll = false;
+            if (polling && --left == 0) {
+                left = per;
+                poll = kt + 1 < nkt;
+                if (poll) tc.post();
+            }
+            if (kt + 1 < nkt) sstore(sm, st ^ 1, ra, rb);
+            __syncthreads();
+            if (poll && tc.verdict()) return true;
         }
         return false;
     }
@@ -1879,6 +1903,43 @@ int gpu_launch_copies(int n, void *const *dst, const void *const *src, const siz
     return 1;
 }
 
+// a[j][i] = a[i][j] for i < j: 32 x 32 tiles of the upper triangle, transposed through shared
+// memory so that both the read of row block (bi) and the write of column block (bj) coalesce.
+template <typename T>
+__global__ void __launch_bounds__(256) mirror_upper_kernel(T *a, long long n) {
+    __shared__ T tile[32][33];
+    const long long nt = (n + 31) / 32;
+    for (long long t = blockIdx.x; t < nt * (nt + 1) / 2; t += gridDim.x) {
+        long long bi = 0, rem = t;   // upper-triangle tile (bi <= bj), row-major
+        while (rem >= nt - bi) { rem -= nt - bi; ++bi; }
+        const long long bj = bi + rem;
+        const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+        for (int r = ty; r < 32; r += 8) {
+            const long long i = bi * 32 + r, j = bj * 32 + tx;
+            if (i < n && j < n) tile[r][tx] = a[i * n + j];
+        }
+        __syncthreads();
+        for (int r = ty; r < 32; r += 8) {
+            const long long j = bj * 32 + r, i = bi * 32 + tx;   // destination row j, column i
+            if (i < n && j < n && i < j) a[j * n + i] = tile[tx][r];
+        }
+        __syncthreads();
+    }
+}
+
+int gpu_launch_mirror_upper(void *a, long long n, int elem_size, int num_sms, void *stream) {
+    if (n <= 1) return 0;
+    const long long nt = (n + 31) / 32;
+    long long grid = nt * (nt + 1) / 2;
+    if (grid > (long long)num_sms * 8) grid = (long long)num_sms * 8;
+    if (elem_size == 4) mirror_upper_kernel<uint32_t><<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>((uint32_t *)a, n);
+    else if (elem_size == 8) mirror_upper_kernel<unsigned long long><<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>((unsigned long long *)a, n);
+    else return -2;
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return seterr(e, "mirror_upper_kernel launch");
+    return 1;
+}
+
 int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream) {
     store64_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(addr, value);
     cudaError_t e = cudaGetLastError();
@@ -1925,6 +1986,8 @@ int gpu_preload_kernels() {
     bad |= cudaFuncGetAttributes(&at, merge_dev_kernel) != cudaSuccess;
     bad |= cudaFuncGetAttributes(&at, copies_kernel) != cudaSuccess;
     bad |= cudaFuncGetAttributes(&at, store64_kernel) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, mirror_upper_kernel<uint32_t>) != cudaSuccess;
+    bad |= cudaFuncGetAttributes(&at, mirror_upper_kernel<unsigned long long>) != cudaSuccess;
     if (bad) { cudaGetLastError(); return seterr(cudaErrorInvalidDeviceFunction, "kernel preload"); }
     return 0;
 }

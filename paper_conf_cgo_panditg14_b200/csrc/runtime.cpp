@@ -2586,6 +2586,12 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         fcl_buffer b = L.bufs[k];
         bool streamed = false;
         for (int q = 0; q < j->nstream; ++q) streamed |= j->sbuf[q] == k;
+        // A host copy left stale by a device-side update (fcl_buffer_device_written) is refreshed
+        // first: the host side reads (or, in place, updates) it (the queue is drained above).
+        if (!b->host_valid) {
+            s = make_valid(ctx, b, true, false, &info);
+            if (s != FCL_SUCCESS) break;
+        }
         // A device copy left stale by a CPU-only launch is refreshed first (lazy H2D; the
         // queue is drained above whenever a copy is stale).
         if (!b->dev_valid && !streamed) {
@@ -2671,6 +2677,37 @@ fcl_status fcl_merge_raw(void *gpu, const void *cpu, const void *twin, size_t by
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     if (gpu_launch_merge(gpu, cpu, twin, bytes, (int)elem_size, sms, stream) < 0) return FCL_CUDA_ERROR;
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_buffer_device_written(fcl_context ctx, fcl_buffer b, size_t offset, size_t n, void *stream) {
+    fcl_status s = check_ctx(ctx);
+    if (s != FCL_SUCCESS) return s;
+    if (!b || b->ctx != ctx) return FCL_INVALID_MEM_OBJECT;
+    if (offset > b->bytes || n > b->bytes - offset) return set_err(ctx, FCL_INVALID_VALUE, "range");
+    drain(ctx);
+    quiesce(ctx);
+    if (n == 0) return FCL_SUCCESS;
+    if (b->ret_lazy) {   // a registered lazy return would copy the old device words over the new
+        b->ret_lazy = false;
+        ctx->lazy.erase(std::remove(ctx->lazy.begin(), ctx->lazy.end(), b), ctx->lazy.end());
+    }
+    if (stream && (cudaStream_t)stream != ctx->main) {   // later work on main follows the writes
+        CK(ctx, cudaEventRecord(ctx->ev_mark, (cudaStream_t)stream));
+        CK(ctx, cudaStreamWaitEvent(ctx->main, ctx->ev_mark, 0));
+    }
+    ctx->main_fenced.store(1);
+    b->dev_valid = true;
+    b->host_valid = false;   // refreshed on demand (make_valid / fcl_read_buffer)
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_mirror_upper(void *a, size_t n, uint32_t elem_size, void *stream) {
+    if (!(elem_size == 4 || elem_size == 8) || (n > 1 && !a)) return FCL_INVALID_VALUE;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (gpu_launch_mirror_upper(a, (long long)n, (int)elem_size, sms, stream) < 0) return FCL_CUDA_ERROR;
     return FCL_SUCCESS;
 }
 

@@ -36,7 +36,7 @@ EXPORTED = [
     "fcl_get_kernel", "fcl_kernel_signature", "fcl_kernel_host_variants", "fcl_default_launch_opts",
     "fcl_enqueue_ndrange",
     "fcl_merge", "fcl_merge_raw", "fcl_finish", "fcl_get_launch_info", "fcl_get_counters", "fcl_slice_range",
-    "fcl_get_exec_counts",
+    "fcl_get_exec_counts", "fcl_buffer_device_written", "fcl_mirror_upper",
     "fcl_status_string", "fcl_last_error", "fcl_version",
 ]
 
@@ -124,6 +124,8 @@ def load() -> ctypes.CDLL:
         "fcl_get_launch_info": ([vp, ctypes.POINTER(LaunchInfo)], i32),
         "fcl_get_counters": ([vp, ctypes.POINTER(i64), i32], i32),
         "fcl_get_exec_counts": ([vp, i64, vp, vp, vp], i32),
+        "fcl_buffer_device_written": ([vp, vp, sz, sz, vp], i32),
+        "fcl_mirror_upper": ([vp, sz, ctypes.c_uint32, vp], i32),
         "fcl_slice_range": ([vp, ctypes.c_uint32, ctypes.POINTER(sz), ctypes.POINTER(sz), i32, i32,
                              ctypes.POINTER(i64), ctypes.POINTER(i64)], i32),
         "fcl_status_string": ([i32], ctypes.c_char_p),
@@ -205,6 +207,13 @@ class Buffer:
         out = np.empty(self.nbytes // np.dtype(dtype).itemsize if count is None else count, dtype)
         self.read(out.ctypes.data, out.nbytes)
         return out
+
+    def device_written(self, offset: int = 0, nbytes: Optional[int] = None, stream: int = 0):
+        """The device copy's [offset, offset+nbytes) was written outside the runtime (e.g. an
+        all-gather of other ranks' slices); the host mirror is refreshed on demand."""
+        n = self.nbytes - offset if nbytes is None else nbytes
+        _check(load().fcl_buffer_device_written(self.ctx.handle, self.handle, int(offset), int(n), stream or None),
+               "fcl_buffer_device_written", self.ctx.handle)
 
     def release(self):
         if self.handle:
@@ -407,3 +416,8 @@ def merge_raw(gpu_ptr: int, cpu_ptr: int, twin_ptr: int, nbytes: int, elem_size:
     """The Fig 9 diff-merge kernel on raw device pointers (asynchronous on `stream`)."""
     _check(load().fcl_merge_raw(gpu_ptr, cpu_ptr, twin_ptr, int(nbytes), int(elem_size), stream or None),
            "fcl_merge_raw")
+
+
+def mirror_upper(ptr: int, n: int, elem_size: int = 4, stream: int = 0):
+    """a[j][i] = a[i][j] for i < j on an n x n row-major device matrix (asynchronous on `stream`)."""
+    _check(load().fcl_mirror_upper(ptr, int(n), int(elem_size), stream or None), "fcl_mirror_upper")

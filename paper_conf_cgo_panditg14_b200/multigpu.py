@@ -1,4 +1,5 @@
-"""Multi-GPU slicing and all-gather glue (north_star; not in the paper, L22.s17).
+"""Multi-GPU slicing, exchange and the sharded runner (north_star; not in the paper,
+L22.s17).
 
 Each rank owns a contiguous, task-aligned flattened work-group range (``fcl_slice_range``),
 runs the cooperative FluidiCL path on it with its own host-thread pool
@@ -62,3 +63,98 @@ def gather_slices(local, counts: Sequence[int], group=None):
     out = torch.empty((world * mx,) + tail, dtype=local.dtype, device=local.device)
     dist.all_gather_into_tensor(out, pad, group=group)
     return torch.cat([out[r * mx: r * mx + counts[r]] for r in range(world)], dim=0)
+
+
+# ------------------------------------------------------------------------------------------
+# The sharded runner (BASELINE.json configs[3]): every rank runs the cooperative
+# path on its own task-aligned work-group slice with its own host pool, then the output slices
+# are exchanged so that every rank holds the whole output on its device.  The exchange is the
+# path's one collective: all_gather_into_tensor over NCCL (NVLink) straight into the fcl
+# buffers' device copies -- in place when the slices are even -- or, on the gloo backend (the
+# CPU-side tests, several ranks sharing one GPU), the same gather staged through host tensors.
+# ------------------------------------------------------------------------------------------
+class _DevView:
+    def __init__(self, ptr: int, nbytes: int, typestr: str, itemsize: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes // itemsize,), "typestr": typestr,
+                                         "data": (int(ptr), False), "version": 3, "strides": None}
+
+
+def device_tensor(buf, dtype=None):
+    """A torch tensor over an fcl buffer's device copy (no copy; the buffer must outlive it)."""
+    import torch
+    dtype = dtype or torch.float32
+    itemsize = torch.empty((), dtype=dtype).element_size()
+    typestr = {torch.float32: "<f4", torch.int32: "<i4", torch.float64: "<f8", torch.int64: "<i8"}[dtype]
+    return torch.as_tensor(_DevView(buf.device_ptr, buf.nbytes, typestr, itemsize), device="cuda")
+
+
+def exchange_rows(buf, nrows: int, ncols: int, spans: Sequence[Tuple[int, int]], group=None,
+                  dtype=None, mirror: bool = False):
+    """All-gather the row slabs spans[r] = [r0, r1) of the row-major nrows x ncols matrix held by
+    `buf` (rank r computed rows spans[r]); afterwards every rank's device copy holds all of them.
+    mirror: the matrix is CORR's symmat, whose slices are L-shaped (a work-group writes its row
+    right of the diagonal and its column below it): only the upper triangle of the gathered row
+    slabs is trusted, and fcl_mirror_upper rebuilds the lower one on the device."""
+    import torch
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    t = device_tensor(buf, dtype)[: nrows * ncols].view(nrows, ncols)
+    counts = [b - a for a, b in spans]
+    stream = torch.cuda.current_stream()
+    if world > 1:
+        r0, r1 = spans[rank]
+        contiguous = spans[0][0] == 0 and all(spans[k][1] == spans[k + 1][0] for k in range(world - 1))
+        if dist.get_backend(group) == "nccl":
+            if contiguous and len(set(counts)) == 1:
+                # in place: rank r's slab already sits at offset r * count of the output
+                dist.all_gather_into_tensor(t[: spans[-1][1]], t[r0:r1], group=group)
+            else:
+                full = gather_slices(t[r0:r1], counts, group)
+                t[spans[0][0]: spans[0][0] + full.shape[0]].copy_(full)
+        else:
+            full = gather_slices(t[r0:r1].cpu(), counts, group)
+            t[spans[0][0]: spans[0][0] + full.shape[0]].copy_(full.to(t.device, non_blocking=False))
+    if mirror:
+        fcl.mirror_upper(t.data_ptr(), nrows, t.element_size(), stream.cuda_stream)
+    # (the legacy default stream has handle 0, which the C-ABI reads as "the context's main
+    # stream": pass cudaStreamLegacy, 0x1, so that main is ordered after the writes)
+    buf.device_written(0, nrows * ncols * t.element_size(), stream.cuda_stream or 1)
+
+
+def run_slice(ctx, kernel: str, gws, lws, args, rank: int, world: int, **opts) -> Tuple[int, int]:
+    """Launch this rank's work-group slice of `kernel` (cooperative by default) and wait for it."""
+    lo, hi = ctx.slice_range(kernel, gws, lws, rank, world)
+    ctx.enqueue_ndrange(kernel, gws, lws, args, wg_lo=lo, wg_hi=hi, **opts)
+    ctx.finish()
+    return lo, hi
+
+
+def _spans(kernel: str, gws, lws, nrows: int, world: int):
+    return [row_span(lo, hi, gws, lws, nrows) for lo, hi in slice_ranges(kernel, gws, lws, world)]
+
+
+def conv2d_sharded(ctx, A, B, ni: int, nj: int, gws, lws, group=None, integer: bool = False, **opts):
+    """2DCONV (PolyBench/GPU) over ranks: row slabs of B, then the all-gather of B."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    name = f"conv2d_{'i32' if integer else 'f32'}"
+    run_slice(ctx, name, gws, lws, [A, B, ni, nj], rank, world, **opts)
+    import torch
+    exchange_rows(B, ni, nj, _spans(name, gws, lws, ni, world), group, torch.int32 if integer else torch.float32)
+
+
+def corr_sharded(ctx, data, mean, std, symmat, n: int, m: int, gws1, lws1, gws2, lws2, group=None,
+                 eps: float = 0.1, **opts):
+    """CORR's four kernels (Table 2) over ranks, each followed by the exchange of its output:
+    mean and std (column slices, 16 KiB at m = 4096), the reduced data (row slabs), symmat (row
+    slabs of the upper triangle + the device-side mirror)."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    run_slice(ctx, "corr_mean_f32", gws1, lws1, [data, mean, n, m], rank, world, **opts)
+    exchange_rows(mean, m, 1, _spans("corr_mean_f32", gws1, lws1, m, world), group)
+    run_slice(ctx, "corr_std_f32", gws1, lws1, [data, mean, std, n, m, eps], rank, world, **opts)
+    exchange_rows(std, m, 1, _spans("corr_std_f32", gws1, lws1, m, world), group)
+    run_slice(ctx, "corr_reduce_f32", gws2, lws2, [data, mean, std, n, m], rank, world, **opts)
+    exchange_rows(data, n, m, _spans("corr_reduce_f32", gws2, lws2, n, world), group)
+    run_slice(ctx, "corr_corr_f32", gws1, lws1, [data, symmat, n, m], rank, world, **opts)
+    exchange_rows(symmat, m, m, _spans("corr_corr_f32", gws1, lws1, m, world), group, mirror=True)
