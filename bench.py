@@ -500,12 +500,123 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
     ctx.release()
 
 
+# ---------------------------------------------------------------------------------- config 4
+CONV_N, CORR_N = 16384, 4096
+
+
+def conv2d_corr_bytes() -> dict:
+    """Algorithmic bytes of one config-4 step: 2DCONV reads A and writes B once; CORR mean/std read
+    the data once, reduce reads and writes it, symmat reads its operand once (its roofline is FP32
+    FFMA: its flops are M^2 N, reported separately)."""
+    f, n, m = 4, CORR_N, CORR_N
+    return {"conv2d": 2 * CONV_N * CONV_N * f, "corr_mean": n * m * f + m * f, "corr_std": n * m * f + 2 * m * f,
+            "corr_reduce": 2 * n * m * f + 2 * m * f, "corr_corr": n * m * f + m * m * f}
+
+
+def run_conv2d_corr(args, rank: int, world: int, local_rank: int):
+    """BASELINE.json configs[3]: 2DCONV 16384^2 and the CORR 4096^2 chain, the fixed problem sharded
+    over the N ranks (strong scaling): each rank runs the cooperative path on its work-group
+    slices with its own host pool, and every kernel's output is exchanged with an all-gather over
+    NCCL into the ranks' device copies.  One step = both kernels' chains with their
+    exchanges; the timed region covers the launches, the host sides and the collectives."""
+    import torch
+    import fcl_harness as H
+    import workloads as W
+    from paper_conf_cgo_panditg14_b200 import _build, fcl, multigpu
+    if rank == 0:
+        _build.build()
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    stream = torch.cuda.Stream(device=dev)
+    all_cores = sorted(os.sched_getaffinity(0))
+    lws_ranks = max(1, int(os.environ.get("LOCAL_WORLD_SIZE", world)))
+    per_rank = max(1, len(all_cores) // lws_ranks)
+    if lws_ranks > 1:
+        os.sched_setaffinity(0, all_cores[local_rank * per_rank:(local_rank + 1) * per_rank] or all_cores)
+    cores = len(os.sched_getaffinity(0))
+    host_threads = max(1, cores - 3)
+    ctx = fcl.Context(local_rank, n_host_threads=host_threads, streams=(stream.cuda_stream, None, None))
+    H.pin_caller()
+    P = W.make("conv2d", CONV_N, CONV_N, seed=11, out_init="zero")
+    A, B = H.create_buffers(ctx, P)
+    n = m = CORR_N
+    data0 = W.corr_chain_inputs(n, m, seed=12)
+    gws1, lws1 = W.geometry("corr_mean", n, m, lws1d=256)
+    gws2, lws2 = W.geometry("corr_reduce", n, m)
+    d = ctx.buffer_from_array(data0)
+    mean, std = ctx.buffer_from_array(np.zeros(m, np.float32)), ctx.buffer_from_array(np.zeros(m, np.float32))
+    sym = ctx.buffer_from_array(np.zeros(m * m, np.float32))
+    pristine = torch.from_numpy(data0).to(dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def reset():
+        # CORR's reduce works in place: both copies of the data back to the input (untimed)
+        d.write(data0.ctypes.data, blocking=True)
+        with torch.cuda.stream(stream):
+            flush.fill_(1.0)
+        stream.synchronize()
+
+    def step(mode):
+        with torch.cuda.stream(stream):
+            multigpu.conv2d_sharded(ctx, A, B, P.n0, P.n1, P.gws, P.lws, mode=mode)
+            multigpu.corr_sharded(ctx, d, mean, std, sym, n, m, gws1, lws1, gws2, lws2, mode=mode)
+
+    def timed(mode):
+        reset()
+        if dist is not None:
+            dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        step(mode)
+        e1.record(stream)
+        e1.synchronize()
+        t = e0.elapsed_time(e1)
+        if dist is not None:
+            x = torch.tensor([t], dtype=torch.float64, device=dev)
+            dist.all_reduce(x, op=dist.ReduceOp.MAX)
+            t = float(x.item())
+        return t
+
+    for _ in range(args.warmup):
+        timed("coop"); timed("gpu")
+    with ClockSampler(local_rank) as clk:
+        clk.wait_started()
+        ts = {"coop": [], "gpu": []}
+        for r in range(args.steps):
+            for mode in (("coop", "gpu") if r % 2 == 0 else ("gpu", "coop")):
+                ts[mode].append(timed(mode))
+    coop_ms, gpu_ms = statistics.mean(ts["coop"]), statistics.mean(ts["gpu"])
+    nbytes = sum(conv2d_corr_bytes().values())
+    del pristine
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(nbytes / (coop_ms * 1e-3) / 1e9, 2), "unit": "GB/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(coop_ms, 4), "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": "conv2d_corr", "conv2d_n": CONV_N, "corr_n": CORR_N, "mode": "coop",
+                           "parallelism": f"sharded{world} (work-group slices + NCCL all-gather)",
+                           "l2": "flushed before each step (256 MiB write)",
+                           "bytes_counted": "2DCONV 2 N^2 x 4 B; CORR mean/std/reduce data passes; symmat operand once"},
+                "coop_ms": round(coop_ms, 4), "gpu_only_ms": round(gpu_ms, 4),
+                "coop_vs_gpu_only": round(gpu_ms / coop_ms, 4), "clocks": clk.summary(), "host_cores": cores}
+        print(json.dumps(line), flush=True)
+    for b in (A, B, d, mean, std, sym):
+        b.release()
+    ctx.release()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="fcl", choices=["fcl", "reference"])
+    ap.add_argument("--workload", default="gesummv_bicg4096", choices=["gesummv_bicg4096", "conv2d_corr"],
+                    help="gesummv_bicg4096 (BASELINE configs[1], the headline; N > 1: replicas) or "
+                         "conv2d_corr (configs[3]: one problem sharded over the ranks + NCCL all-gather)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -519,7 +630,10 @@ def main():
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    run_fcl(args, rank, world, local_rank)
+    if args.workload == "conv2d_corr":
+        run_conv2d_corr(args, rank, world, local_rank)
+    else:
+        run_fcl(args, rank, world, local_rank)
     if world > 1:
         import torch.distributed as dist
         dist.barrier()

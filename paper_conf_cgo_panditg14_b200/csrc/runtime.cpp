@@ -2519,8 +2519,9 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
             const bool need_dev = L.o.mode != FCL_MODE_CPU_ONLY;
             s = make_valid(ctx, L.bufs[k], need_host, need_dev, &info, is_out);
             if (s != FCL_SUCCESS) return s;
-            if (L.o.mode == FCL_MODE_GPU_ONLY && is_out && !L.bufs[k]->host_valid) {
-                // partially returned outputs: the rest of the host copy must be current first
+            if (L.o.mode == FCL_MODE_GPU_ONLY && is_out && (L.acc[k] & 1) && !L.bufs[k]->host_valid) {
+                // partially returned in-place outputs: the rest of the host copy must be current
+                // first (a pure-OUT one stays stale on the host: the device copy is authoritative)
                 s = make_valid(ctx, L.bufs[k], true, true, &info);
                 if (s != FCL_SUCCESS) return s;
             }
@@ -2587,8 +2588,10 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         bool streamed = false;
         for (int q = 0; q < j->nstream; ++q) streamed |= j->sbuf[q] == k;
         // A host copy left stale by a device-side update (fcl_buffer_device_written) is refreshed
-        // first: the host side reads (or, in place, updates) it (the queue is drained above).
-        if (!b->host_valid) {
+        // first when the host side reads it (IN / INOUT; the queue is drained above).  A pure-OUT
+        // buffer stays stale on the host: the device copy is complete after the launch, and a
+        // read refreshes the host copy from it.
+        if (!b->host_valid && (L.acc[k] & 1)) {
             s = make_valid(ctx, b, true, false, &info);
             if (s != FCL_SUCCESS) break;
         }

@@ -88,6 +88,14 @@ def device_tensor(buf, dtype=None):
     return torch.as_tensor(_DevView(buf.device_ptr, buf.nbytes, typestr, itemsize), device="cuda")
 
 
+def rank_world(group=None) -> Tuple[int, int]:
+    """(rank, world size) of the process group, (0, 1) without one (a single GPU)."""
+    import torch.distributed as dist
+    if dist.is_available() and dist.is_initialized():
+        return dist.get_rank(group), dist.get_world_size(group)
+    return 0, 1
+
+
 def exchange_rows(buf, nrows: int, ncols: int, spans: Sequence[Tuple[int, int]], group=None,
                   dtype=None, mirror: bool = False):
     """All-gather the row slabs spans[r] = [r0, r1) of the row-major nrows x ncols matrix held by
@@ -97,7 +105,7 @@ def exchange_rows(buf, nrows: int, ncols: int, spans: Sequence[Tuple[int, int]],
     slabs is trusted, and fcl_mirror_upper rebuilds the lower one on the device."""
     import torch
     import torch.distributed as dist
-    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    rank, world = rank_world(group)
     t = device_tensor(buf, dtype)[: nrows * ncols].view(nrows, ncols)
     counts = [b - a for a, b in spans]
     stream = torch.cuda.current_stream()
@@ -135,8 +143,7 @@ def _spans(kernel: str, gws, lws, nrows: int, world: int):
 
 def conv2d_sharded(ctx, A, B, ni: int, nj: int, gws, lws, group=None, integer: bool = False, **opts):
     """2DCONV (PolyBench/GPU) over ranks: row slabs of B, then the all-gather of B."""
-    import torch.distributed as dist
-    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    rank, world = rank_world(group)
     name = f"conv2d_{'i32' if integer else 'f32'}"
     run_slice(ctx, name, gws, lws, [A, B, ni, nj], rank, world, **opts)
     import torch
@@ -148,8 +155,7 @@ def corr_sharded(ctx, data, mean, std, symmat, n: int, m: int, gws1, lws1, gws2,
     """CORR's four kernels (Table 2) over ranks, each followed by the exchange of its output:
     mean and std (column slices, 16 KiB at m = 4096), the reduced data (row slabs), symmat (row
     slabs of the upper triangle + the device-side mirror)."""
-    import torch.distributed as dist
-    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    rank, world = rank_world(group)
     run_slice(ctx, "corr_mean_f32", gws1, lws1, [data, mean, n, m], rank, world, **opts)
     exchange_rows(mean, m, 1, _spans("corr_mean_f32", gws1, lws1, m, world), group)
     run_slice(ctx, "corr_std_f32", gws1, lws1, [data, mean, std, n, m, eps], rank, world, **opts)
