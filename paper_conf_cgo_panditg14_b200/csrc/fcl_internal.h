@@ -14,10 +14,15 @@
 #include <cstddef>
 #include <cstdint>
 #include <vector>
+#include <atomic>
 
 typedef struct CUstream_st *cudaStream_t_fwd;
 
 namespace fcl {
+
+// The host executor's abort flag: set by the coordinator when the GPU has finished (L18.s19),
+// polled by the host bodies inside long loops (relaxed loads; a data race with a plain int).
+typedef std::atomic<int> AbortFlag;
 
 enum KernelId : int {
     K_ATAX_TMP = 0, K_ATAX_Y, K_BICG_S, K_BICG_Q, K_GESUMMV, K_SYRK, K_SYR2K,
@@ -188,13 +193,13 @@ const char *gpu_last_error_string();
 // storing an incomplete value (write-once).
 // Returns true when the part completed (every output stored), false when the abort flag stopped it.
 bool host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts,
-                  const volatile int *abort_flag);
+                  const AbortFlag *abort_flag);
 // Alternate host bodies (C26): how many a kernel has and their names ("cpu", "wi").
 int host_num_variants(int kernel);
 const char *host_variant_name(int kernel, int v);
 // Work-groups per executor claim (host_exec_range) and the range executor itself.
 int64_t host_batch(const KArgs &a, const Geom &g);
-bool host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *abort_flag);
+bool host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const AbortFlag *abort_flag);
 
 // Conservative contiguous byte span [*b0, *b1) of output buffer `buf_index` written by
 // work-groups [lo, hi) (superset of the exact footprint; the diff-merge tolerates it).

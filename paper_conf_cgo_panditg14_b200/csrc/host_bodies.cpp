@@ -28,7 +28,7 @@ inline uint32_t op_add(uint32_t a, uint32_t b) { return a + b; }
 inline float op_mul(float a, float b) { return a * b; }
 inline uint32_t op_mul(uint32_t a, uint32_t b) { return a * b; }
 
-inline bool aborted(const volatile int *f) { return f && *f; }
+inline bool aborted(const AbortFlag *f) { return f && f->load(std::memory_order_relaxed); }
 
 // [lo, hi) of `n` items for part `part` of `nparts` (contiguous, balanced).
 inline void part_range(int64_t n, int part, int nparts, int64_t &lo, int64_t &hi) {
@@ -42,7 +42,7 @@ inline void part_range(int64_t n, int part, int nparts, int64_t &lo, int64_t &hi
 // Returns false (and no value) when the abort flag is seen: it is polled every 1024 columns,
 // so an abandoned chunk stops within a fraction of a microsecond.
 template <typename T>
-bool rowdot(const T *Ar, const T *x, int64_t ncols, const volatile int *ab, T *res) {
+bool rowdot(const T *Ar, const T *x, int64_t ncols, const AbortFlag *ab, T *res) {
     T p[kRowPartitions];
     for (int q = 0; q < kRowPartitions; ++q) p[q] = 0;
     for (int64_t j0 = 0; j0 < ncols; j0 += kRowPartitions) {
@@ -61,7 +61,7 @@ bool rowdot(const T *Ar, const T *x, int64_t ncols, const volatile int *ab, T *r
 }
 
 template <typename T>
-bool wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t lws = g.lws[0];
     const bool ges = (a.kernel == K_GESUMMV);
     const int64_t nrows = a.n0, ncols = ges ? a.n0 : a.n1;
@@ -100,7 +100,7 @@ bool wg_rowdot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
 enum { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
 
 template <typename T, int MODE>
-bool wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_coldot(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t lws = g.lws[0];
     const int64_t nrows = a.n0, ncols = a.n1;
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, ncols);
@@ -160,7 +160,7 @@ inline Wg2D wg2d(const Geom &g, int64_t fgid, int64_t nrows, int64_t ncols) {
 // ---------------------------------------------------------------- CORR reduce (in place)
 // Rectangle [r0, r1) x [c0, c1) of the output (a work-group, or a batch of work-groups of one
 // work-group row: wide rows stream and vectorize).
-bool corr_reduce_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
+bool corr_reduce_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const AbortFlag *ab) {
     const int64_t n = a.n0, m = a.n1;
     float *d = (float *)a.host[0];
     const float *mean = (const float *)a.host[1], *sd = (const float *)a.host[2];
@@ -175,7 +175,7 @@ bool corr_reduce_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_
     return true;
 }
 
-bool wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     Wg2D w = wg2d(g, fgid, a.n0, a.n1);
     if (w.r0 >= w.r1 || w.c0 >= w.c1) return true;
     int64_t lo, hi;
@@ -186,7 +186,7 @@ bool wg_corr_reduce(const KArgs &a, const Geom &g, int64_t fgid, int part, int n
 // ---------------------------------------------------------------- 2DCONV
 // Rectangle [r0, r1) x [c0, c1) of the output, border excluded by the caller.
 template <typename T>
-bool conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const volatile int *ab) {
+bool conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1, const AbortFlag *ab) {
     const int64_t nj = a.n1;
     const T *A = (const T *)a.host[0];
     T *B = (T *)a.host[1];
@@ -218,7 +218,7 @@ bool conv2d_rect(const KArgs &a, int64_t r0, int64_t r1, int64_t c0, int64_t c1,
 }
 
 template <typename T>
-bool wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t ni = a.n0, nj = a.n1;
     Wg2D w = wg2d(g, fgid, ni, nj);
     const int64_t r0 = std::max<int64_t>(w.r0, 1), r1 = std::min<int64_t>(w.r1, ni - 1);
@@ -235,7 +235,7 @@ bool wg_conv2d(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts
 // B_i*A_j, for i > j the mirror's B_i*A_j then A_i*B_j -- so acc(i, j) == acc(j, i) bit for bit
 // (DESIGN.md §6.1).  Mirrors GemmBody in kernels.cu.
 template <typename T, bool TWO>
-bool wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t n = a.n0, m = a.n1;
     Wg2D w = wg2d(g, fgid, n, n);
     if (w.r0 >= w.r1 || w.c0 >= w.c1) return true;
@@ -305,7 +305,7 @@ bool wg_syrk(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, 
 // ---------------------------------------------------------------- CORR symmat
 // symmat[j1][j2] = symmat[j2][j1] = sum_i d[i][j1] * d[i][j2] (j2 > j1, ascending i, fma
 // chain); symmat[j1][j1] = 1.  Work-items j1 processed in blocks of 8 for row reuse.
-bool wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t n = a.n0, m = a.n1;
     const int64_t lws = g.lws[0];
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, m);
@@ -356,7 +356,7 @@ bool wg_corr_corr(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
 
 // col-dot: work-item j walks its column, partition by partition
 template <typename T, int MODE>
-bool wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t lws = g.lws[0];
     const int64_t nrows = a.n0, ncols = a.n1;
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, ncols);
@@ -393,7 +393,7 @@ bool wg_coldot_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npa
 
 // SYRK / SYR2K: work-item (i, j) runs its k-chain
 template <typename T, bool TWO>
-bool wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t n = a.n0, m = a.n1;
     Wg2D w = wg2d(g, fgid, n, n);
     if (w.r0 >= w.r1 || w.c0 >= w.c1) return true;
@@ -428,7 +428,7 @@ bool wg_syrk_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int npart
 }
 
 // CORR symmat: work-item j1 computes its row, each j2 > j1 down the two columns
-bool wg_corr_corr_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *ab) {
+bool wg_corr_corr_wi(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *ab) {
     const int64_t n = a.n0, m = a.n1;
     const int64_t lws = g.lws[0];
     const int64_t c0 = fgid * lws, c1 = std::min<int64_t>(c0 + lws, m);
@@ -467,7 +467,7 @@ const char *host_variant_name(int kernel, int v) {
     return v == 0 ? "cpu" : "wi";
 }
 
-bool host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const volatile int *abort_flag) {
+bool host_exec_wg(const KArgs &a, const Geom &g, int64_t fgid, int part, int nparts, const AbortFlag *abort_flag) {
     if (a.host_variant == 1 && host_num_variants(a.kernel) > 1) {
         switch (a.kernel) {
         case K_ATAX_Y: case K_BICG_S:
@@ -519,7 +519,7 @@ int64_t host_batch(const KArgs &a, const Geom &g) {
 
 // Work-groups [f_lo, f_hi) (any order is valid: every work-group writes only its own outputs).
 // Returns true when every one of them completed (false: the abort flag stopped the run).
-bool host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const volatile int *ab) {
+bool host_exec_range(const KArgs &a, const Geom &g, int64_t f_lo, int64_t f_hi, const AbortFlag *ab) {
     if ((a.kernel == K_CONV2D || a.kernel == K_CORR_REDUCE) && g.work_dim == 2) {
         const int64_t ngx = g.ng[0];
         for (int64_t f = f_lo; f < f_hi;) {   // one segment per work-group row

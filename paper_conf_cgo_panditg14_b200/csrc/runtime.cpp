@@ -153,14 +153,16 @@ struct Executor {
     Geom g{};
     int64_t lo = 0, hi = 0;
     int nparts = 1;
-    int64_t total = 0;
-    int active = 0;
+    // read by workers before their claim is validated (a worker still looping on the previous
+    // job): atomics, relaxed -- the compare-and-swap on `next` decides
+    std::atomic<int64_t> total{0};
+    std::atomic<int> active{0};
     // claim word: (job generation << 40) | next item.  Claims use compare-and-swap so a
     // worker still looping on a finished job can never consume an item of the next one.
     std::atomic<uint64_t> next{0};
     std::atomic<int64_t> done{0};
     int64_t batch = 1;   // work-groups per claim (host_batch), 1 when work-groups are split
-    volatile int abort_flag = 0;
+    AbortFlag abort_flag{0};
     int64_t spin_ns = 2 * 1000 * 1000;    // spin 2 ms after a job before sleeping
 
     void start(int nthreads, bool pin) {
@@ -210,14 +212,14 @@ struct Executor {
             }
             if (stop.load()) return;
             seen = gen.load(std::memory_order_acquire);
-            if (idx >= active) continue;
+            if (idx >= active.load(std::memory_order_relaxed)) continue;
             for (;;) {
                 uint64_t v = next.load(std::memory_order_acquire);
                 if ((v >> 40) != (seen & 0xFFFFFFu)) break;
                 const int64_t it = (int64_t)(v & ((1ull << 40) - 1));
-                if (it >= total) break;
+                if (it >= total.load(std::memory_order_relaxed)) break;
                 if (!next.compare_exchange_weak(v, v + 1, std::memory_order_acq_rel)) continue;
-                if (!abort_flag) {
+                if (!abort_flag.load(std::memory_order_relaxed)) {
                     if (batch == 1) {
                         const int64_t fgid = hi - 1 - it / nparts;   // descending (L14.s36)
                         const bool ok = host_exec_wg(a, g, fgid, (int)(it % nparts), nparts, &abort_flag);
@@ -251,8 +253,8 @@ struct Executor {
         next.store(((g1 & 0xFFFFFFu) << 40) | ((1ull << 40) - 1), std::memory_order_seq_cst);
         a = a_; g = g_; lo = lo_; hi = hi_; nparts = parts;
         batch = parts > 1 ? 1 : std::max<int64_t>(1, host_batch(a_, g_));
-        total = parts > 1 ? (hi_ - lo_) * parts : (hi_ - lo_ + batch - 1) / batch;
-        active = std::max(1, std::min(nact, T));
+        total.store(parts > 1 ? (hi_ - lo_) * parts : (hi_ - lo_ + batch - 1) / batch, std::memory_order_relaxed);
+        active.store(std::max(1, std::min(nact, T)), std::memory_order_relaxed);
         done.store(0, std::memory_order_relaxed);
         next.store((g1 & 0xFFFFFFu) << 40, std::memory_order_release);
         gen.store(g1, std::memory_order_release);
@@ -261,7 +263,7 @@ struct Executor {
             cv.notify_all();
         }
     }
-    bool finished() const { return done.load(std::memory_order_acquire) >= total; }
+    bool finished() const { return done.load(std::memory_order_acquire) >= total.load(std::memory_order_relaxed); }
     void wait() {
         while (!finished()) _mm_pause();
     }
