@@ -133,6 +133,13 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer buf, size_t offset, size
 fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer buf, size_t offset, size_t n,
                            void *dst, int32_t blocking);
 
+/* Buffer versions (C18, L20.s1-9): the kernel ID (a per-context launch counter, from 1) of the
+ * last launch that writes the buffer, and of the data its host and device copies hold once the
+ * work queued for them has landed -- after fcl_finish both equal `expected` unless a copy is
+ * stale by design (the device copy after a CPU-only launch until a GPU launch needs it, the host
+ * copy after fcl_buffer_device_written until it is read).  Any out pointer may be NULL. */
+fcl_status fcl_buffer_versions(fcl_buffer buf, uint64_t *expected, uint64_t *host, uint64_t *device);
+
 /* Query a buffer's pointers and sizes (any out pointer may be NULL). */
 fcl_status fcl_buffer_info(fcl_buffer buf, void **host_ptr, void **device_ptr, size_t *bytes,
                            uint32_t *elem_size);
@@ -343,7 +350,9 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info);
 #define FCL_COUNT_CPU_ONLY   5  /* CPU_ONLY-mode launches */
 #define FCL_COUNT_H2D_BYTES  6  /* bytes copied host -> device (writes, refreshes, staged chunks) */
 #define FCL_COUNT_D2H_BYTES  7  /* bytes copied device -> host (returns, reads) */
-#define FCL_COUNT_N          8
+#define FCL_COUNT_LAUNCH_DRAINS 8  /* launches that had to wait for pending host sides first (the
+                                      hazards buffer versions do not order) */
+#define FCL_COUNT_N          9
 fcl_status fcl_get_counters(fcl_context ctx, int64_t *counts, int32_t n);
 
 /* Per-work-group execution counts of the most recent launch made with opts.record_exec_counts

@@ -322,9 +322,17 @@ struct fcl_buffer_st {
     bool merge_pending;
     void *twin, *stage;
     size_t m_b0, m_b1, r_b0, r_b1;   // merge span, return (D2H) span
+    // Buffer versions (C18, L20.s1-9): the kernel ID of the last launch that writes the buffer
+    // (expected), and of the data its host and device copies hold once everything queued for
+    // them has landed (host_ver / dev_ver).  host_seq: the host-only job (a queued CPU-only
+    // launch) that last writes its host copy -- while it is pending, a GPU-side reader waits for
+    // the copy's transfer on the device (a stream memory wait), not on the host.
+    uint64_t ver_expected, ver_host, ver_dev;
+    uint64_t host_seq;
 };
 
 typedef CUresult (*PFN_writeValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+typedef CUresult (*PFN_waitValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 
 namespace {
 
@@ -345,6 +353,15 @@ struct Launch {
 // One cooperative launch in flight: phase A (GPU side, calling thread) then phase B (host
 // side, coordinator thread).
 struct Job {
+    // JOB_COOP: a cooperative launch's host side (phase B); JOB_CPU: a CPU-only launch, run by the
+    // coordinator in queue order; JOB_XFER: host->device copies of buffers a pending JOB_CPU
+    // writes, published by a ticket a later GPU launch waits for on the device
+    enum { JOB_COOP = 0, JOB_CPU = 1, JOB_XFER = 2 };
+    int kind = JOB_COOP;
+    uint64_t host_seq = 0;     // JOB_CPU: its host-job sequence number
+    uint64_t ticket = 0;       // JOB_XFER: the value stored to the transfer word after the copies
+    int nx = 0;
+    fcl_buffer xb[6] = {};     // JOB_XFER: the buffers
     Launch L;
     uint32_t epoch = 0;
     int slot = 0;
@@ -381,7 +398,11 @@ struct fcl_context_st {
     int num_sms = 148;
     cudaStream_t main = nullptr, hd = nullptr, dh = nullptr;
     bool own_main = false, own_hd = false, own_dh = false;
-    cudaStream_t xs = nullptr;   // exit-signal memops of lite launches (never carries data)
+    // JOB_XFER copies and their tickets.  Not hd: phase A queues waits for main positions on hd
+    // (forced splits, staging) that can lie behind a launch's wait for a ticket -- a transfer on
+    // hd would then wait for itself.  xt only ever waits for main positions before that wait.
+    cudaStream_t xt = nullptr;
+    std::atomic<int> xt_used{0};
     // Return-race pieces (DESIGN.md §6.4 item 8) go on their own stream: on dh they would queue
     // behind a later launch's return that waits for its (long) kernel, and stop returning while
     // that kernel runs.  A later return of the same buffer waits for the race's d2h_ev.
@@ -426,6 +447,15 @@ struct fcl_context_st {
     cudaEvent_t main_tail = nullptr;             // ev_k1 of the last cooperative dispatcher
     uint32_t epoch = 0;
     PFN_writeValue64 write64 = nullptr;
+    PFN_waitValue64 wait64 = nullptr;
+    // Buffer versions (C18/C21): launch ids (the paper's kernel IDs), host-only jobs and transfers
+    uint64_t kid = 0;                            // kernel ID of the latest launch
+    uint64_t host_seq = 0;                       // host-only jobs queued
+    std::atomic<uint64_t> host_done_seq{0};      // host-only jobs completed (in queue order)
+    uint64_t xfer_seq = 0;                       // transfer tickets issued
+    unsigned long long *d_xfer = nullptr;        // device word: the last ticket whose copies landed
+    bool no_version_wait = false;                // FCL_NO_VERSION_WAIT=1: skip the device-side wait
+                                                 // (test hook: shows the stale read it prevents)
     bool stats = false;                          // count executed GPU tasks, time merges (FCL_STATS=1)
     size_t eager_return_bytes = 8u << 20;        // outputs up to this size return right behind the merge
     // Lazy return: small outputs of free-running and GPU-only launches are not
@@ -689,6 +719,7 @@ fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_d
         CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->main));
         ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)b->bytes;
         b->dev_valid = true;
+        b->ver_dev = b->ver_host;
         if (info) info->h2d_bytes += (int64_t)b->bytes;
     }
     if (need_host && !b->host_valid) {
@@ -696,6 +727,7 @@ fcl_status make_valid(fcl_context ctx, fcl_buffer b, bool need_host, bool need_d
         ctx->counts[FCL_COUNT_D2H_BYTES] += (int64_t)b->bytes;
         CK(ctx, cudaStreamSynchronize(ctx->main));
         b->host_valid = true;
+        b->ver_host = b->ver_dev;
         if (info) info->d2h_bytes += (int64_t)b->bytes;
     }
     return FCL_SUCCESS;
@@ -1050,6 +1082,9 @@ Job *job_alloc(fcl_context ctx) {
     }
     j->status = FCL_SUCCESS;
     j->done.store(0);
+    j->kind = Job::JOB_COOP;
+    j->host_seq = j->ticket = 0;
+    j->nx = 0;
     j->have_k = j->have_m = j->wm_pending = false;
     j->gpu_launched = j->dev_merge = j->eager = j->forced = j->twin_alias = j->lite = j->exact_spans = false;
     j->lazy = false;
@@ -1536,6 +1571,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     if (race) {
         ctx->tr.add("race_begin", j.epoch);
         info.race = 1;
+        quiesce(ctx);   // an earlier launch's abandoned chunk may still read a host copy written below
         ctx->dr_used.store(1, std::memory_order_relaxed);
         CK(ctx, cudaStreamWaitEvent(ctx->dr, j.ev_k1, 0));
         for (int q = 0; q < L.nout; ++q) {   // behind any earlier return of the same buffers
@@ -1651,6 +1687,7 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
                 // watermark >= the lowest one published, so returning the device copy (merged
                 // by the fused tail) below the host's own published watermark is complete --
                 // no device read of the GPU's watermark on this path.
+                quiesce(ctx);   // (an earlier launch's abandoned chunk may still read these host copies)
                 st = enqueue_d2h(ctx, L, L.lo, info.published_watermark, info, j.ev_k1);
             }
             j.wm_pending = !j.lite;   // info.gpu_watermark resolved lazily by fcl_get_launch_info
@@ -1694,11 +1731,46 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
             }
         } else {
             CK(ctx, cudaEventRecord(j.ev_ret, ctx->main));   // after the host-side merges
+            quiesce(ctx);
             st = enqueue_d2h(ctx, L, L.lo, merge_lo, info, j.ev_ret);
         }
     }
     job_release_buffers(ctx, j, staged_any);
     return st;
+}
+
+fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info);
+
+// A CPU-only launch in queue order (C22: the host side of every earlier launch has run): its
+// inputs' host copies must hold the expected versions -- every return copy of an earlier launch
+// has landed (the paper's CPU scheduler waits "until the most recent data arrives from the
+// GPU", L20.s7) -- then the executor runs the whole range.
+fcl_status cpu_job(fcl_context ctx, Job &j) {
+    Launch &L = j.L;
+    for (int k = 0; k < L.a.nbuf; ++k) {
+        fcl_buffer b = L.bufs[k];
+        if (d2h_busy(ctx, b)) {
+            CK(ctx, cudaEventSynchronize(b->d2h_ev));
+        }
+    }
+    if (L.o.host_delay_us > 0) std::this_thread::sleep_for(std::chrono::microseconds(L.o.host_delay_us));
+    return run_cpu_only(ctx, L, j.info);
+}
+
+// Host->device copies of the host copies a pending CPU-only job produced, ordered after the GPU
+// work queued before the launch that needs them (xt waits for that main-stream position), then
+// the ticket: the launch's grid waits on the device until the ticket has landed (C18: "the GPU
+// ... discarding stale data", here: never reading it).
+fcl_status xfer_job(fcl_context ctx, Job &j) {
+    ctx->xt_used.store(1, std::memory_order_relaxed);
+    CK(ctx, cudaStreamWaitEvent(ctx->xt, j.ev_start, 0));
+    for (int q = 0; q < j.nx; ++q) {
+        fcl_buffer b = j.xb[q];
+        CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->xt));
+        ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)b->bytes;
+        j.info.h2d_bytes += (int64_t)b->bytes;
+    }
+    return stream_store(ctx, ctx->d_xfer, (unsigned long long)j.ticket, ctx->xt, true, &j.info);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1737,8 +1809,11 @@ void coordinator(fcl_context ctx) {
         }
         fcl_status st = FCL_SUCCESS;
         ctx->tr.add("phaseB_begin", j->epoch);
-        if (ctx->sticky.load() == FCL_SUCCESS) st = coop_phase_b(ctx, *j);
-        else st = ctx->sticky.load();
+        if (ctx->sticky.load() != FCL_SUCCESS) st = ctx->sticky.load();
+        else if (j->kind == Job::JOB_CPU) st = cpu_job(ctx, *j);
+        else if (j->kind == Job::JOB_XFER) st = xfer_job(ctx, *j);
+        else st = coop_phase_b(ctx, *j);
+        if (j->kind == Job::JOB_CPU) ctx->host_done_seq.store(j->host_seq, std::memory_order_release);
         ctx->tr.add("phaseB_end", j->epoch);
         {
             std::lock_guard<std::mutex> lk(ctx->q_mu);
@@ -1776,16 +1851,39 @@ void drain(fcl_context ctx) {
 // on main, and the new launch's host side runs after the pending one's (FIFO) and waits for
 // the buffer's return copy before reading the host copy.  So a dependent kernel is not held
 // back by the host side of the one before it (e.g. a return race still in progress).
+//
+// Buffer versions make more of these safe without waiting (C18, L20.s1-9):
+//  * RAW on a pending CPU-only job: its host side runs after the job (queue order), and a GPU
+//    read waits on the device for the transfer of the job's result (JOB_XFER);
+//  * WAR, when the pending launch (free-running, or a CPU-only job) only reads the buffer, does
+//    not stream it to the device, and the new launch is cooperative and updates the buffer in
+//    place (INOUT): its device writes follow the pending grid on main, and every write to the
+//    host copy happens in its own host side -- after the pending one's (queue order), and after
+//    any chunk of it that is still stopping (phase B quiesces before returning data).
 bool conflicts_with_pending(fcl_context ctx, const Launch &L) {
     std::lock_guard<std::mutex> lk(ctx->q_mu);
     for (Job *p : ctx->queue) {
-        const bool free_running = p->dev_merge || p->lite;
+        if (p->kind == Job::JOB_XFER) {   // reads host copies, writes device copies of xb
+            for (int a = 0; a < L.a.nbuf; ++a)
+                for (int q = 0; q < p->nx; ++q)
+                    if (L.bufs[a] == p->xb[q] && (L.acc[a] & 2)) return true;
+            continue;
+        }
+        const bool cpu_job = p->kind == Job::JOB_CPU;
+        const bool free_running = !cpu_job && (p->dev_merge || p->lite);
         for (int a = 0; a < L.a.nbuf; ++a)
             for (int b = 0; b < p->L.a.nbuf; ++b) {
                 if (L.bufs[a] != p->L.bufs[b]) continue;
                 const bool we_write = (L.acc[a] & 2) != 0, they_write = (p->L.acc[b] & 2) != 0;
-                if (we_write) return true;                        // WAR / WAW
-                if (they_write && !free_running) return true;     // RAW on a host-decided merge
+                if (we_write) {
+                    bool streamed = false;
+                    for (int q = 0; q < p->nstream; ++q) streamed |= p->sbuf[q] == b;
+                    const bool war_ok = !they_write && (free_running || cpu_job) && !streamed &&
+                                        L.o.mode == FCL_MODE_COOP && L.acc[a] == 3;
+                    if (!war_ok) return true;                     // WAR / WAW
+                    continue;
+                }
+                if (they_write && !free_running && !cpu_job) return true;   // RAW on a host-decided merge
             }
     }
     return false;
@@ -1820,6 +1918,8 @@ fcl_status run_gpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
 }
 
 fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
+    info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
+    info.gpu_watermark = L.hi;
     Executor &ex = ctx->ex;
     const int nact = L.o.n_host_threads > 0 ? L.o.n_host_threads : ex.T;
     const int64_t nwg = L.hi - L.lo;
@@ -1867,8 +1967,7 @@ fcl_status run_cpu_only(fcl_context ctx, Launch &L, fcl_launch_info &info) {
     info.n_c11_chunks = 0;   // (CPU-only: profiling allocations, then the rest in one job)
     info.cpu_did_all = 1;
     info.published_watermark = L.lo;
-    for (int q = 0; q < L.nout; ++q) L.bufs[L.out_idx[q]]->dev_valid = false;   // lazy H2D on next GPU use
-    return FCL_SUCCESS;
+    return FCL_SUCCESS;   // (the outputs' device copies were marked stale at enqueue: program order)
 }
 
 }  // namespace
@@ -1971,7 +2070,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if ((e = mk(d.main_stream, &ctx->main, &ctx->own_main)) != cudaSuccess) return fail(e, "main stream");
     if ((e = mk(d.hd_stream, &ctx->hd, &ctx->own_hd)) != cudaSuccess) return fail(e, "hd stream");
     if ((e = mk(d.dh_stream, &ctx->dh, &ctx->own_dh)) != cudaSuccess) return fail(e, "dh stream");
-    if ((e = cudaStreamCreateWithFlags(&ctx->xs, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "exit-signal stream");
+    if ((e = cudaStreamCreateWithFlags(&ctx->xt, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "transfer stream");
     if ((e = cudaStreamCreateWithFlags(&ctx->dr, cudaStreamNonBlocking)) != cudaSuccess) return fail(e, "race stream");
     // status words (one per launch slot), GPU-exit word, pinned copy of the wm word
     void *hp = nullptr, *dp = nullptr;
@@ -2028,7 +2127,20 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
         else
             cudaGetLastError();
     }
-    if (getenv("FCL_NO_MEMOPS")) ctx->write64 = nullptr;
+    {
+        void *fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuStreamWaitValue64", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess && fn)
+            ctx->wait64 = (PFN_waitValue64)fn;
+        else
+            cudaGetLastError();
+    }
+    if (getenv("FCL_NO_MEMOPS")) { ctx->write64 = nullptr; ctx->wait64 = nullptr; }
+    ctx->no_version_wait = getenv("FCL_NO_VERSION_WAIT") && atoi(getenv("FCL_NO_VERSION_WAIT")) != 0;
+    if ((e = cudaMalloc(&dp, 8)) != cudaSuccess) return fail(e, "transfer word");
+    cudaMemset(dp, 0, 8);
+    ctx->d_xfer = (unsigned long long *)dp;
     if (getenv("FCL_EAGER_RETURN_BYTES")) ctx->eager_return_bytes = (size_t)atoll(getenv("FCL_EAGER_RETURN_BYTES"));
     ctx->stats = getenv("FCL_STATS") && atoi(getenv("FCL_STATS")) != 0;
     ctx->tr.on = getenv("FCL_TRACE") && atoi(getenv("FCL_TRACE")) != 0;
@@ -2115,10 +2227,11 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->rec.d_cnt) cudaFree(ctx->rec.d_cnt);
     if (ctx->rec.d_w) cudaFree(ctx->rec.d_w);
     if (ctx->darrival) cudaFree(ctx->darrival);
+    if (ctx->d_xfer) cudaFree(ctx->d_xfer);
     if (ctx->own_main) cudaStreamDestroy(ctx->main);
     if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
     if (ctx->own_dh) cudaStreamDestroy(ctx->dh);
-    if (ctx->xs) cudaStreamDestroy(ctx->xs);
+    if (ctx->xt) cudaStreamDestroy(ctx->xt);
     if (ctx->dr) cudaStreamDestroy(ctx->dr);
     delete ctx;
     return FCL_SUCCESS;
@@ -2204,6 +2317,7 @@ fcl_status fcl_release_buffer(fcl_buffer b) {
     cudaStreamSynchronize(ctx->hd);
     cudaStreamSynchronize(ctx->dh);
     cudaStreamSynchronize(ctx->dr);
+    cudaStreamSynchronize(ctx->xt);
     if (b->merge_pending) {
         if (b->twin) pool_put(ctx, b->twin, false);
         if (b->stage) pool_put(ctx, b->stage, false);
@@ -2233,11 +2347,13 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
     // overwriting the pinned mirror: no queued copy may still read its old contents (main, and
     // the pieces of a streamed launch on hd)
     if (src != h) CK(ctx, cudaStreamSynchronize(ctx->main));
+    if (src != h && ctx->xt_used.load()) CK(ctx, cudaStreamSynchronize(ctx->xt));   // transfers read mirrors
     if (ctx->stream_pending) {
         CK(ctx, cudaEventSynchronize(ctx->ev_stream_done));
         ctx->stream_pending = false;
     }
     if (src != h) std::memcpy(h, src, n);
+    b->ver_expected = b->ver_host = ++ctx->kid;   // a write is a new version of the buffer
     if (!blocking && n == b->bytes) {
         // a non-blocking write of the whole buffer refreshes the device copy lazily, when a
         // launch first needs it on the GPU -- never, if the data is consumed on the host alone
@@ -2246,6 +2362,7 @@ fcl_status fcl_write_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t
         b->dev_valid = false;
         return FCL_SUCCESS;
     }
+    b->ver_dev = b->ver_host;
     CK(ctx, cudaMemcpyAsync((char *)b->dev + offset, h, n, cudaMemcpyHostToDevice, ctx->main));
     ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)n;
     b->host_valid = b->dev_valid = true;
@@ -2270,9 +2387,17 @@ fcl_status fcl_read_buffer(fcl_context ctx, fcl_buffer b, size_t offset, size_t 
     }
     CK(ctx, cudaStreamSynchronize(ctx->main));
     CK(ctx, cudaMemcpy((char *)b->host + offset, (char *)b->dev + offset, n, cudaMemcpyDeviceToHost));
-    if (n == b->bytes) b->host_valid = true;
+    if (n == b->bytes) { b->host_valid = true; b->ver_host = b->ver_dev; }
     const char *h = (const char *)b->host + offset;
     if (dst != h) std::memcpy(dst, h, n);
+    return FCL_SUCCESS;
+}
+
+fcl_status fcl_buffer_versions(fcl_buffer b, uint64_t *expected, uint64_t *host, uint64_t *device) {
+    if (!b) return FCL_INVALID_MEM_OBJECT;
+    if (expected) *expected = b->ver_expected;
+    if (host) *host = b->host_valid ? b->ver_host : 0;
+    if (device) *device = b->dev_valid ? b->ver_dev : 0;
     return FCL_SUCCESS;
 }
 
@@ -2492,18 +2617,114 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         else if (selected == FCL_SELECTED_CPU) L.o.mode = FCL_MODE_CPU_ONLY;
     }
     const bool coop = L.o.mode == FCL_MODE_COOP;
+    const bool cpu_only = L.o.mode == FCL_MODE_CPU_ONLY;
     ctx->tr.add("enq_begin", ctx->epoch + 1);
-    // The single-device modes and any launch that conflicts with a pending one wait for the
-    // pending launches' host sides first (the cross-launch hazards the paper's version
-    // tracking resolves, L20.s1-9; here conservatively by draining).
-    bool host_needed = false;
-    for (int k = 0; k < L.a.nbuf; ++k) host_needed |= !L.bufs[k]->host_valid || !L.bufs[k]->dev_valid;
-    // A launch redirected to the GPU alone (device selection) is ordered like a cooperative one:
-    // on main behind every pending grid, waiting only for host sides it conflicts with.
-    const bool gpu_sel = selected == FCL_SELECTED_GPU;
-    if ((!coop && !gpu_sel) || host_needed || L.o.blocking || conflicts_with_pending(ctx, L)) drain(ctx);
-    if ((!coop && !gpu_sel) || conflicts_with_quiescing(ctx, L)) quiesce(ctx);
+    // Buffer versions (C18, L20.s1-9) and location tracking (C22, L20.s31-33) order launches
+    // without waiting for the pending host sides:
+    //  * a host-side reader (a cooperative launch's chunks, a CPU-only launch -- both run by the
+    //    coordinator in queue order) finds every earlier host-side writer done, and waits for
+    //    the return copies of earlier GPU work on its inputs;
+    //  * a GPU-side reader of a buffer a pending CPU-only launch writes waits ON THE DEVICE for a
+    //    transfer the coordinator issues after that launch (JOB_XFER + a stream memory wait);
+    //  * the remaining hazards (conflicts_with_pending, a host copy written on the device by the
+    //    caller, streamed inputs) still wait for the queue -- counted in FCL_COUNT_LAUNCH_DRAINS.
+    const uint64_t host_done = ctx->host_done_seq.load(std::memory_order_acquire);
+    bool need_drain = L.o.blocking || conflicts_with_pending(ctx, L);
+    int nxfer = 0;
+    fcl_buffer xfer[6];
+    for (int k = 0; k < L.a.nbuf; ++k) {
+        fcl_buffer b = L.bufs[k];
+        if (cpu_only) {
+            need_drain |= !b->host_valid;   // device-written: refreshed synchronously below
+            continue;
+        }
+        if (!b->dev_valid) {
+            // a pending host-only job writes it: transfer after that job, wait on the device
+            if (b->host_seq > host_done && ctx->write64 && ctx->wait64 && !need_drain) xfer[nxfer++] = b;
+            else if (b->host_seq > host_done) need_drain = true;
+            // (otherwise the host copy is final: refreshed on main below -- except for a launch
+            // that streams its stale rows, which starts on an empty queue)
+            else if (coop && ctx->stream_on && (L.a.kernel == K_GESUMMV || L.a.kernel == K_ATAX_TMP || L.a.kernel == K_BICG_Q))
+                need_drain = true;
+        }
+        if (!b->host_valid && coop && (L.acc[k] & 1)) need_drain = true;
+    }
+    if (need_drain) nxfer = 0;   // (drained: the host copies are final, make_valid refreshes)
+    if (need_drain) {
+        if (ctx->q_len.load(std::memory_order_acquire) > 0) ctx->counts[FCL_COUNT_LAUNCH_DRAINS] += 1;
+        drain(ctx);
+    }
+    if (conflicts_with_quiescing(ctx, L) || (cpu_only && need_drain)) quiesce(ctx);
     if (ctx->sticky.load() != FCL_SUCCESS) return ctx->sticky.load();
+    const uint64_t kid = ++ctx->kid;
+    if (nxfer > 0) {
+        // the host copies of a pending CPU-only launch go to the device after it, on hd behind
+        // the GPU work queued so far (which may still read the old device copies); this launch's
+        // GPU work waits on main until the ticket has landed
+        Job *t = job_alloc(ctx);
+        if (!t) return set_err(ctx, FCL_OUT_OF_RESOURCES, "job allocation");
+        t->kind = Job::JOB_XFER;
+        t->ticket = ++ctx->xfer_seq;
+        t->nx = nxfer;
+        for (int q = 0; q < nxfer; ++q) t->xb[q] = xfer[q];
+        CK(ctx, cudaEventRecord(t->ev_start, ctx->main));
+        {
+            std::lock_guard<std::mutex> lk(ctx->q_mu);
+            ctx->queue.push_back(t);
+            ctx->q_len.fetch_add(1, std::memory_order_release);
+        }
+        if (ctx->coord_sleeping.load()) ctx->q_cv.notify_all();
+        if (!ctx->no_version_wait) {
+            const CUresult r = ctx->wait64((CUstream)ctx->main, (CUdeviceptr)ctx->d_xfer, (cuuint64_t)t->ticket,
+                                           CU_STREAM_WAIT_VALUE_GEQ);
+            if (r != CUDA_SUCCESS) return set_err(ctx, FCL_CUDA_ERROR, "cuStreamWaitValue64 failed (%d)", (int)r);
+        }
+        ctx->main_fenced.store(1);
+        for (int q = 0; q < nxfer; ++q) { xfer[q]->dev_valid = true; xfer[q]->ver_dev = xfer[q]->ver_host; }
+    }
+    for (int k = 0; k < L.a.nbuf; ++k)   // (the versions this launch produces)
+        if (L.acc[k] & 2) L.bufs[k]->ver_expected = kid;
+
+    if (cpu_only && !need_drain) {
+        // A CPU-only launch runs in queue order on the coordinator (JOB_CPU).  The host copies it
+        // reads must not be overwritten by a lazy return flushed later: flush them now (the job
+        // waits for their copies).  Its outputs' device copies are stale from here on.
+        for (int k = 0; k < L.a.nbuf; ++k)
+            if (L.bufs[k]->ret_lazy) {
+                s = flush_returns(ctx, false);
+                if (s != FCL_SUCCESS) return s;
+                break;
+            }
+        Job *j = job_alloc(ctx);
+        if (!j) return set_err(ctx, FCL_OUT_OF_RESOURCES, "job allocation");
+        j->kind = Job::JOB_CPU;
+        j->L = L;
+        j->host_seq = ++ctx->host_seq;
+        j->epoch = (uint32_t)kid;
+        fcl_launch_info &info = j->info;
+        info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
+        info.gpu_watermark = info.published_watermark = L.hi;
+        info.selected = selected;
+        for (int k = 0; k < L.a.nbuf; ++k)
+            if (L.acc[k] & 2) {
+                fcl_buffer b = L.bufs[k];
+                b->dev_valid = false;   // lazy H2D (or a JOB_XFER) on the next GPU use
+                b->host_seq = j->host_seq;
+                b->ver_host = kid;      // (once the job has run: queue order)
+            }
+        ctx->counts[selected == FCL_SELECTED_CPU ? FCL_COUNT_SEL_CPU : FCL_COUNT_CPU_ONLY] += 1;
+        info.t_call_ms = now_ms() - t_call;
+        if (info_out) *info_out = info;
+        {
+            std::lock_guard<std::mutex> lk(ctx->q_mu);
+            if (ctx->last && ctx->last != j && ctx->last->done.load()) ctx->free_jobs.push_back(ctx->last);
+            ctx->last = j;
+            ctx->queue.push_back(j);
+            ctx->q_len.fetch_add(1, std::memory_order_release);
+        }
+        if (ctx->coord_sleeping.load()) ctx->q_cv.notify_all();
+        return FCL_SUCCESS;
+    }
 
     if (!coop) {
         ctx->main_tail = nullptr;   // later launches record their own main position
@@ -2517,18 +2738,23 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
             // GPU-only: the host copy of an output is only rewritten by the return copy (which
             // is ordered behind earlier ones on dh), so it need not be current; CPU-only reads
             // and writes host copies
-            const bool need_host = L.o.mode == FCL_MODE_CPU_ONLY;
-            const bool need_dev = L.o.mode != FCL_MODE_CPU_ONLY;
+            const bool need_host = cpu_only;
+            const bool need_dev = !cpu_only;
             s = make_valid(ctx, L.bufs[k], need_host, need_dev, &info, is_out);
             if (s != FCL_SUCCESS) return s;
-            if (L.o.mode == FCL_MODE_GPU_ONLY && is_out && (L.acc[k] & 1) && !L.bufs[k]->host_valid) {
+            if (!cpu_only && is_out && (L.acc[k] & 1) && !L.bufs[k]->host_valid) {
                 // partially returned in-place outputs: the rest of the host copy must be current
                 // first (a pure-OUT one stays stale on the host: the device copy is authoritative)
                 s = make_valid(ctx, L.bufs[k], true, true, &info);
                 if (s != FCL_SUCCESS) return s;
             }
         }
+        if (cpu_only)
+            for (int k = 0; k < L.a.nbuf; ++k)
+                if (L.acc[k] & 2) { L.bufs[k]->dev_valid = false; L.bufs[k]->ver_host = kid; }
         s = (L.o.mode == FCL_MODE_GPU_ONLY) ? run_gpu_only(ctx, L, info) : run_cpu_only(ctx, L, info);
+        for (int k = 0; k < L.a.nbuf && !cpu_only; ++k)
+            if (L.acc[k] & 2) { L.bufs[k]->ver_dev = kid; L.bufs[k]->ver_host = kid; }
         info.selected = selected;
         ctx->counts[selected == FCL_SELECTED_GPU ? FCL_COUNT_SEL_GPU
                     : selected == FCL_SELECTED_CPU ? FCL_COUNT_SEL_CPU
@@ -2542,6 +2768,8 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         if (info_out) *info_out = info;
         return s;
     }
+    for (int k = 0; k < L.a.nbuf; ++k)
+        if (L.acc[k] & 2) { L.bufs[k]->ver_dev = kid; L.bufs[k]->ver_host = kid; }
 
     // lazy returns of buffers whose host copy this launch's host side reads (or that a
     // host-decided merge may change) are queued first; phase B waits for them
@@ -2704,6 +2932,7 @@ fcl_status fcl_buffer_device_written(fcl_context ctx, fcl_buffer b, size_t offse
     ctx->main_fenced.store(1);
     b->dev_valid = true;
     b->host_valid = false;   // refreshed on demand (make_valid / fcl_read_buffer)
+    b->ver_expected = b->ver_dev = ++ctx->kid;
     return FCL_SUCCESS;
 }
 
@@ -2764,6 +2993,7 @@ fcl_status fcl_finish(fcl_context ctx) {
     ctx->pdl_chain_grids = 0;
     ctx->tr.add("finish_main", ctx->epoch);
     if (ctx->hd_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->hd));
+    if (ctx->xt_used.exchange(0)) CK(ctx, cudaStreamSynchronize(ctx->xt));
     ctx->tr.add("finish_hd", ctx->epoch);
     // An abandoned chunk of a free-running launch may still be stopping: it only writes words
     // identical to the returned ones, so every host copy is already coherent.  Whatever could

@@ -36,7 +36,7 @@ EXPORTED = [
     "fcl_get_kernel", "fcl_kernel_signature", "fcl_kernel_host_variants", "fcl_default_launch_opts",
     "fcl_enqueue_ndrange",
     "fcl_merge", "fcl_merge_raw", "fcl_finish", "fcl_get_launch_info", "fcl_get_counters", "fcl_slice_range",
-    "fcl_get_exec_counts", "fcl_buffer_device_written", "fcl_mirror_upper",
+    "fcl_get_exec_counts", "fcl_buffer_device_written", "fcl_mirror_upper", "fcl_buffer_versions",
     "fcl_status_string", "fcl_last_error", "fcl_version",
 ]
 
@@ -126,6 +126,8 @@ def load() -> ctypes.CDLL:
         "fcl_get_exec_counts": ([vp, i64, vp, vp, vp], i32),
         "fcl_buffer_device_written": ([vp, vp, sz, sz, vp], i32),
         "fcl_mirror_upper": ([vp, sz, ctypes.c_uint32, vp], i32),
+        "fcl_buffer_versions": ([vp, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64),
+                                 ctypes.POINTER(ctypes.c_uint64)], i32),
         "fcl_slice_range": ([vp, ctypes.c_uint32, ctypes.POINTER(sz), ctypes.POINTER(sz), i32, i32,
                              ctypes.POINTER(i64), ctypes.POINTER(i64)], i32),
         "fcl_status_string": ([i32], ctypes.c_char_p),
@@ -214,6 +216,13 @@ class Buffer:
         n = self.nbytes - offset if nbytes is None else nbytes
         _check(load().fcl_buffer_device_written(self.ctx.handle, self.handle, int(offset), int(n), stream or None),
                "fcl_buffer_device_written", self.ctx.handle)
+
+    def versions(self) -> tuple:
+        """(expected, host, device) buffer versions (fcl_buffer_versions; 0 = that copy is stale)."""
+        e, h, d = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint64()
+        _check(load().fcl_buffer_versions(self.handle, ctypes.byref(e), ctypes.byref(h), ctypes.byref(d)),
+               "fcl_buffer_versions")
+        return e.value, h.value, d.value
 
     def release(self):
         if self.handle:
@@ -344,7 +353,8 @@ class Context:
         _check(load().fcl_get_launch_info(self.handle, ctypes.byref(info)), "fcl_get_launch_info", self.handle)
         return info.as_dict()
 
-    COUNTERS = ("coop", "probe", "sel_gpu", "sel_cpu", "gpu_only", "cpu_only", "h2d_bytes", "d2h_bytes")
+    COUNTERS = ("coop", "probe", "sel_gpu", "sel_cpu", "gpu_only", "cpu_only", "h2d_bytes", "d2h_bytes",
+                "launch_drains")
 
     def counters(self) -> dict:
         """Cumulative launch counters (fcl_get_counters): how COOP launches ran under device selection."""
