@@ -138,6 +138,48 @@ int main() {
         std::printf("done %s\n", p.kernel);
         std::fflush(stdout);
     }
+    {   // a chain across devices without fcl_finish in between (queued CPU-only jobs, transfers
+        // with device-side waits, GPU-only launches ordered like cooperative ones)
+        const int64_t n = 512;
+        std::vector<float> A = rnd(n * n, 9), x = rnd(n, 10), zero(n);
+        fcl_kernel k1, k2;
+        CHECK(fcl_get_kernel(ctx, "atax_tmp_f32", &k1));
+        CHECK(fcl_get_kernel(ctx, "atax_y_f32", &k2));
+        size_t gws[3] = {(size_t)n, 1, 1}, lws[3] = {64, 1, 1};
+        std::vector<float> want;
+        const int modes[4][2] = {{FCL_MODE_GPU_ONLY, FCL_MODE_GPU_ONLY}, {FCL_MODE_CPU_ONLY, FCL_MODE_GPU_ONLY},
+                                 {FCL_MODE_GPU_ONLY, FCL_MODE_CPU_ONLY}, {FCL_MODE_CPU_ONLY, FCL_MODE_COOP}};
+        for (auto &md : modes) {
+            fcl_buffer bA, bx, bt, by;
+            CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, A.size() * 4, 4, A.data(), &bA));
+            CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, n * 4, 4, x.data(), &bx));
+            CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, n * 4, 4, zero.data(), &bt));
+            CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, n * 4, 4, zero.data(), &by));
+            fcl_arg a1[5] = {}, a2[5] = {};
+            a1[0].kind = a1[1].kind = a1[2].kind = FCL_ARG_BUFFER;
+            a1[0].buffer = bA; a1[1].buffer = bx; a1[2].buffer = bt;
+            a1[0].access = a1[1].access = FCL_ACCESS_IN; a1[2].access = FCL_ACCESS_OUT;
+            a1[3].kind = a1[4].kind = FCL_ARG_INT; a1[3].i = a1[4].i = n;
+            std::memcpy(a2, a1, sizeof a1);
+            a2[1].buffer = bt; a2[2].buffer = by;
+            fcl_launch_opts o;
+            CHECK(fcl_default_launch_opts(&o));
+            o.select = FCL_SELECT_OFF;
+            o.mode = md[0];
+            o.host_delay_us = 2000;
+            CHECK(fcl_enqueue_ndrange(ctx, k1, 1, gws, lws, a1, 5, &o, nullptr));
+            o.mode = md[1];
+            o.host_delay_us = 0;
+            CHECK(fcl_enqueue_ndrange(ctx, k2, 1, gws, lws, a2, 5, &o, nullptr));
+            CHECK(fcl_finish(ctx));
+            std::vector<float> y(n);
+            CHECK(fcl_read_buffer(ctx, by, 0, n * 4, y.data(), 1));
+            if (want.empty()) want = y;
+            else if (std::memcmp(want.data(), y.data(), n * 4) != 0) { std::fprintf(stderr, "MISMATCH chain\n"); ++bad; }
+            for (auto b : {bA, bx, bt, by}) CHECK(fcl_release_buffer(b));
+        }
+        std::printf("done chain\n");
+    }
     CHECK(fcl_release_context(ctx));
     std::printf(bad ? "tsan driver: %d MISMATCHES\n" : "tsan driver ok\n", bad);
     return bad ? 1 : 0;
