@@ -184,7 +184,9 @@ int gpu_launch_copies(int n, void *const *dst, const void *const *src, const siz
 // a[j][i] = a[i][j] for i < j on an n x n row-major device matrix (multi-rank CORR combine).
 int gpu_launch_mirror_upper(void *a, long long n, int elem_size, int num_sms, void *stream);
 // One-thread kernel that stores `value` to `addr` (status publication fallback).
-int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream);
+// stamp (nullable): %globaltimer right after the store (exit-drain measurement, FCL_TEST_PUBLISH_ZERO_US).
+int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream,
+                       unsigned long long *stamp = nullptr);
 const char *gpu_last_error_string();
 
 // ---- Host side (host_bodies.cpp) ----

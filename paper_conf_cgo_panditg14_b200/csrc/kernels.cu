@@ -621,8 +621,9 @@ __global__ void __launch_bounds__(256) copies_kernel(const CopyList L, int pdl_w
     }
 }
 
-__global__ void store64_kernel(unsigned long long *addr, unsigned long long v) {
+__global__ void store64_kernel(unsigned long long *addr, unsigned long long v, unsigned long long *stamp) {
     asm volatile("st.release.sys.global.b64 [%0], %1;" ::"l"(addr), "l"(v) : "memory");
+    if (stamp) *stamp = globaltimer();   // (measurement: when the store became visible)
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1940,8 +1941,8 @@ int gpu_launch_mirror_upper(void *a, long long n, int elem_size, int num_sms, vo
     return 1;
 }
 
-int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream) {
-    store64_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(addr, value);
+int gpu_launch_store64(unsigned long long *addr, unsigned long long value, void *stream, unsigned long long *stamp) {
+    store64_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(addr, value, stamp);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return seterr(e, "store64_kernel launch");
     return 1;

@@ -454,6 +454,12 @@ struct fcl_context_st {
     std::atomic<uint64_t> host_done_seq{0};      // host-only jobs completed (in queue order)
     uint64_t xfer_seq = 0;                       // transfer tickets issued
     unsigned long long *d_xfer = nullptr;        // device word: the last ticket whose copies landed
+    // Exit-drain measurement (FCL_TEST_PUBLISH_ZERO_US, with FCL_STATS=1): the host side
+    // of a free-running dispatcher launch computes nothing, publishes W = wg_lo this many us after
+    // it starts, with a store kernel that stamps %globaltimer, and no merge runs -- the outputs are
+    // INCOMPLETE; only for scripts/exit_drain.py.  dpub: the stamps, one per slot.
+    int64_t test_publish_zero_us = 0;
+    unsigned long long *dpub = nullptr;
     bool no_version_wait = false;                // FCL_NO_VERSION_WAIT=1: skip the device-side wait
                                                  // (test hook: shows the stale read it prevents)
     bool stats = false;                          // count executed GPU tasks, time merges (FCL_STATS=1)
@@ -1281,6 +1287,7 @@ fcl_status coop_phase_a(fcl_context ctx, Job &j) {
     M.epoch = j.epoch;
     M.hi = L.hi;
     c.fused = ctx->unfused ? 0 : 1;
+    if (ctx->test_publish_zero_us > 0) M.n = 0;   // (exit-drain measurement: no merge, see the context)
     if (c.fused) c.mg = M;   // mg.n == 0 (forced / deferred): barrier + exit signal only
     c.mg.tstamp = ctx->stats ? ctx->dstamp + 4 * j.slot + 2 : nullptr;
 
@@ -1394,6 +1401,20 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
         exited_before = gpu_exited();
     }
 
+    if (ctx->test_publish_zero_us > 0 && j.dev_merge && !exited_before) {
+        // exit-drain measurement: publish W = lo after the given time, compute nothing
+        std::this_thread::sleep_for(std::chrono::microseconds(ctx->test_publish_zero_us));
+        ctx->hd_used.store(1, std::memory_order_relaxed);
+        CK(ctx, cudaStreamWaitEvent(ctx->hd, j.main_before, 0));
+        if (gpu_launch_store64(ctx->status_dptr + j.slot, ((unsigned long long)j.epoch << 32) | (uint32_t)L.lo, ctx->hd,
+                               ctx->dpub + j.slot) < 0)
+            return set_err(ctx, FCL_CUDA_ERROR, "%s", gpu_last_error_string());
+        while (!exit_word_seen()) _mm_pause();
+        info.published_watermark = L.lo;
+        j.wm_pending = true;
+        job_release_buffers(ctx, j, true);
+        return FCL_SUCCESS;
+    }
     auto start_chunk = [&]() {
         int64_t size = ceil_pct(pct, nwg);
         const int64_t min_units = L.o.cpu_wg_split ? 1 : nact;   // L18.s31 without C23
@@ -2138,6 +2159,12 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     }
     if (getenv("FCL_NO_MEMOPS")) { ctx->write64 = nullptr; ctx->wait64 = nullptr; }
     ctx->no_version_wait = getenv("FCL_NO_VERSION_WAIT") && atoi(getenv("FCL_NO_VERSION_WAIT")) != 0;
+    if (getenv("FCL_TEST_PUBLISH_ZERO_US") && getenv("FCL_STATS") && atoi(getenv("FCL_STATS")) != 0) {
+        ctx->test_publish_zero_us = atoll(getenv("FCL_TEST_PUBLISH_ZERO_US"));
+        if ((e = cudaMalloc(&dp, 8 * fcl_context_st::kSlots)) != cudaSuccess) return fail(e, "publish stamps");
+        cudaMemset(dp, 0, 8 * fcl_context_st::kSlots);
+        ctx->dpub = (unsigned long long *)dp;
+    }
     if ((e = cudaMalloc(&dp, 8)) != cudaSuccess) return fail(e, "transfer word");
     cudaMemset(dp, 0, 8);
     ctx->d_xfer = (unsigned long long *)dp;
@@ -2228,6 +2255,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->rec.d_w) cudaFree(ctx->rec.d_w);
     if (ctx->darrival) cudaFree(ctx->darrival);
     if (ctx->d_xfer) cudaFree(ctx->d_xfer);
+    if (ctx->dpub) cudaFree(ctx->dpub);
     if (ctx->own_main) cudaStreamDestroy(ctx->main);
     if (ctx->own_hd) cudaStreamDestroy(ctx->hd);
     if (ctx->own_dh) cudaStreamDestroy(ctx->dh);
@@ -3007,6 +3035,11 @@ fcl_status fcl_finish(fcl_context ctx) {
             std::lock_guard<std::mutex> lk(ctx->tr.mu);
             for (int k = 0; k < fcl_context_st::kSlots; ++k) {
                 static const char *names[4] = {"gpu_disp_start_ns", "gpu_disp_end_ns", "gpu_merge_start_ns", "gpu_merge_end_ns"};
+                if (ctx->dpub) {
+                    unsigned long long pst = 0;
+                    if (cudaMemcpy(&pst, ctx->dpub + k, 8, cudaMemcpyDeviceToHost) == cudaSuccess && pst)
+                        ctx->tr.recs.push_back({(double)(pst % 1000000000000ull) * 1e-6, "gpu_publish_ns", (uint32_t)k});
+                }
                 for (int q = 0; q < 4; ++q)
                     if (st[4 * k + q] && st[4 * k + q] != ~0ull)
                         ctx->tr.recs.push_back({(double)(st[4 * k + q] % 1000000000000ull) * 1e-6, names[q], (uint32_t)k});
