@@ -1266,7 +1266,10 @@ struct GemmBody {
         };
 #pragma unroll
         for (int q = 0; q < NSA - 1; ++q) issue(q);
-        const long long per = 2 * tc.period();   // polls every `per` GBKA-tiles (= period GBK-tiles)
+        // polls every `per` GBKA-tiles (= period GBK-tiles): a countdown, no division per tile
+        const bool polling = tc.c != nullptr && tc.c->abort_period > 0;
+        const long long per = polling ? 2 * (long long)tc.c->abort_period : 1;
+        long long left = per;
         bool poll = false;   // a poll posted at the end of the previous tile, decided after the barrier
         for (long long kt = 0; kt < nkt; ++kt) {
             asm volatile("cp.async.wait_group %0;" ::"n"(NSA - 2) : "memory");
@@ -1295,8 +1298,12 @@ struct GemmBody {
 #pragma unroll
                     for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
             }
-            poll = per > 0 && (kt + 1) % per == 0 && kt + 1 < nkt && tc.c != nullptr && tc.c->abort_period > 0;
-            if (poll) tc.post();
+            poll = false;
+            if (polling && --left == 0) {
+                left = per;
+                poll = kt + 1 < nkt;
+                if (poll) tc.post();
+            }
         }
         asm volatile("cp.async.wait_all;" ::: "memory");
         return false;
@@ -1318,6 +1325,20 @@ struct GemmBody {
         const long long per = tc.period();
         const bool polling = per < nkt;
         long long left = per;
+#ifndef FCL_GEMM_UNROLL2
+#define FCL_GEMM_UNROLL2 1
+#endif
+        if (FCL_GEMM_UNROLL2 && TN == 4) {   // (TN = 8: 128 registers already, unrolling spills)
+            // two k'-tiles per iteration: the shared-memory stage of each is a compile-time
+            // constant (no per-tile stage arithmetic on the fragment addresses)
+            long long kt = 0;
+            for (; kt + 1 < nkt; kt += 2) {
+                if (ktile<IN, 0>(p, i0, j0, kt, nkt, tx, ty, sm, acc, ra, rb, sw, tc, polling, per, left)) return true;
+                if (ktile<IN, 1>(p, i0, j0, kt + 1, nkt, tx, ty, sm, acc, ra, rb, sw, tc, polling, per, left)) return true;
+            }
+            if (kt < nkt && ktile<IN, 0>(p, i0, j0, kt, nkt, tx, ty, sm, acc, ra, rb, sw, tc, polling, per, left)) return true;
+            return false;
+        }
         for (long long kt = 0; kt < nkt; ++kt) {
             const int st = (int)(kt & 1);
             if (kt + 1 < nkt) gload<IN>(p, i0, j0, kt + 1, ra, rb, sw);   // next k'-tile in flight
@@ -1342,6 +1363,35 @@ struct GemmBody {
             if (poll && tc.verdict()) return true;
         }
         return false;
+    }
+
+    // One k'-tile out of shared-memory stage ST (the next one's loads in flight, stored to the
+    // other stage before the barrier; a poll folded into that barrier).  Returns true on an abort.
+    template <bool IN, int ST>
+    __device__ __forceinline__ static bool ktile(const Params &p, long long i0, long long j0, long long kt, long long nkt,
+                                                 int tx, int ty, Smem &sm, T (&acc)[8][TN], T (&ra)[LD], T (&rb)[LD],
+                                                 bool sw, TaskCtx &tc, bool polling, long long per, long long &left) {
+        const bool more = kt + 1 < nkt;
+        if (more) gload<IN>(p, i0, j0, kt + 1, ra, rb, sw);   // next k'-tile in flight
+        T a[2][8], b[2][TN];
+        frag(sm, ST, 0, tx, ty, a[0], b[0]);
+#pragma unroll
+        for (int kk = 0; kk < GBK; ++kk) {
+            if (kk + 1 < GBK) frag(sm, ST, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
+#pragma unroll
+            for (int r = 0; r < 8; ++r)
+#pragma unroll
+                for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+        }
+        bool poll = false;
+        if (polling && --left == 0) {
+            left = per;
+            poll = more;
+            if (poll) tc.post();
+        }
+        if (more) sstore(sm, ST ^ 1, ra, rb);
+        __syncthreads();
+        return poll && tc.verdict();
     }
 
     __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &sm) {
