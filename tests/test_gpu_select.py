@@ -159,14 +159,17 @@ def test_lazy_write_refresh_and_host_alone(ctx):
         b.release()
 
 
-@pytest.mark.parametrize("kernel,integer,lws", [("gesummv", False, 64), ("gesummv", True, 64),
-                                                ("atax_tmp", False, 32), ("bicg_q", False, 128)])
-def test_streamed_inputs(ctx, kernel, integer, lws):
+@pytest.mark.parametrize("kernel,integer,lws,n1", [("gesummv", False, 64, 2048), ("gesummv", True, 64, 2048),
+                                                   ("atax_tmp", False, 32, 2048), ("bicg_q", False, 128, 2048),
+                                                   ("atax_tmp", False, 32, 2045), ("bicg_q", True, 64, 2047)])
+def test_streamed_inputs(ctx, kernel, integer, lws, n1):
     """Stale input matrices (a non-blocking whole-buffer write) of a row-dot kernel stream to the
     GPU in row pieces while the host computes from the top; GPU work-groups
     wait for their rows or for the host to cover them.  The result is the GPU-only one bit for
-    bit, with the host slowed down (the GPU then takes most pieces) and at full speed."""
-    P = W.make(kernel, 2048, 2048, integer=integer, seed=33, lws1d=lws)
+    bit, with the host slowed down (the GPU then takes most pieces) and at full speed.  Rows that
+    are not a multiple of 16 bytes (n1 % 4 != 0, the scalar path) put piece boundaries inside
+    cache lines: the streamed rows are read through L2 only, never from a stale L1 line."""
+    P = W.make(kernel, 2048, n1, integer=integer, seed=33, lws1d=lws)
     ref, _ = H.run(ctx, P, mode="gpu")
     for kw in (dict(host_delay_us=300), dict()):
         bufs = H.create_buffers(ctx, P)
