@@ -108,3 +108,42 @@ def test_sharded_conv2d_and_corr_two_ranks(mode):
     bad = [(r, m) for r, msgs in results for m, ok in msgs if not ok]
     assert not bad, bad
     assert all(len(msgs) == 10 for _, msgs in results), results
+
+
+def test_mirror_upper_and_device_written():
+    """The exchange's building blocks: fcl_mirror_upper copies the upper triangle onto the lower
+    one (ragged n, both element sizes), leaving the diagonal and the upper triangle untouched;
+    fcl_buffer_device_written makes a device-side update the authoritative copy -- a read and a
+    cooperative launch whose host side reads the buffer both see it."""
+    import torch
+    import fcl_harness as H
+    import workloads as W
+    from paper_conf_cgo_panditg14_b200 import _build, fcl, multigpu
+    _build.build()
+    for n, dt in ((300, torch.float32), (129, torch.float64), (1, torch.float32), (64, torch.float32)):
+        a = torch.randn(n, n, dtype=dt, device="cuda")
+        want = torch.triu(a) + torch.triu(a, 1).T
+        fcl.mirror_upper(a.data_ptr(), n, a.element_size())
+        torch.cuda.synchronize()
+        assert torch.equal(a, want), (n, dt)
+    ctx = fcl.Context(0, n_host_threads=4)
+    try:
+        P = W.make("atax_tmp", 512, 512, seed=83, lws1d=64)
+        A, x, tmp = H.create_buffers(ctx, P)
+        x2 = (P.bufs[1] * 3.0 - 1.0).astype(np.float32)
+        dev = multigpu.device_tensor(x)
+        dev.copy_(torch.from_numpy(x2).cuda())
+        x.device_written(0, x.nbytes, torch.cuda.current_stream().cuda_stream or 1)
+        assert x.versions()[1] == 0 and x.versions()[2] > 0          # host copy stale, device current
+        assert np.array_equal(x.read_array(np.float32), x2)
+        x.device_written(0, x.nbytes, torch.cuda.current_stream().cuda_stream or 1)
+        ref = x2.copy()
+        ctx.enqueue_ndrange("atax_tmp_f32", P.gws, P.lws, [A, x, tmp, 512, 512], mode="coop", forced_split=3)
+        ctx.finish()
+        got = tmp.read_array(np.float32)
+        A2 = P.bufs[0].reshape(512, 512).astype(np.float64)
+        assert np.allclose(got, A2 @ ref.astype(np.float64), rtol=1e-5, atol=1e-4)
+        for b in (A, x, tmp):
+            b.release()
+    finally:
+        ctx.release()
