@@ -460,7 +460,8 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
             t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
         // a task that may span work-groups the host covers stores only those below w (the
         // watermark acted on: the merge domain starts at or below it)
-        tc.wmask = (Body::kMasks && checked) ? w : 0xFFFFFFFFu;
+        // (w == the range end: nothing covered, no mask -- the stores then skip the per-row work-group test)
+        tc.wmask = (Body::kMasks && checked && w < c.w_default) ? w : 0xFFFFFFFFu;
         if (Body::kMasks && checked && w < rec_w && threadIdx.x == 0) {
             record_wm(c, w);
             rec_w = w;
