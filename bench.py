@@ -475,6 +475,11 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
             "selection": selection,
             "ideal_coop_ms": round(ideal_ms, 4), "frac_of_ideal": round(ideal_ms / coop_ms, 4),
             "coop_vs_best_single": round(min(gpu_ms, cpu_ms) / coop_ms, 4),
+            # (medians of the same interleaved steps: GPU-only and COOP-with-selection run the same
+            # grids, so at 20 steps their means differ by the odd slow step of either)
+            "median_ms": {"coop": round(statistics.median(coop_ts), 4), "gpu_only": round(statistics.median(gpu_ts), 4),
+                          "coop_always": round(statistics.median(always_ts), 4)},
+            "coop_vs_best_single_median": round(min(statistics.median(gpu_ts), cpu_ms) / statistics.median(coop_ts), 4),
             "wall_ms_per_step": round(t_wall * 1e3 / args.steps, 4),
             "roofline": {"kernel": gesummv_kernel, "bound": "hbm",
                          "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
