@@ -70,16 +70,25 @@ typedef struct fcl_kernel_st  *fcl_kernel;
 
 typedef struct {
     int32_t device;          /* CUDA device ordinal */
-    int32_t n_host_threads;  /* host executor threads; 0 = (cores in affinity mask) - 2: one core
-                                is the coordinator's, one is left to the calling thread */
+    int32_t n_host_threads;  /* host executor threads; 0 = (cores of the affinity mask on the GPU's
+                                NUMA node, or all of the mask if fewer than 3) - 2: one core is
+                                the coordinator's, one is left to the calling thread */
     int32_t pin_threads;     /* 1 = pin executor threads to cores of the affinity mask */
     int32_t status_location; /* FCL_STATUS_DEVICE (default) | FCL_STATUS_HOST_MAPPED */
     void   *main_stream;     /* optional cudaStream_t for kernels/merge; NULL = own stream */
     void   *hd_stream;       /* optional cudaStream_t for CPU->GPU staging (L20.s10-12) */
     void   *dh_stream;       /* optional cudaStream_t for GPU->CPU results   (L20.s10-12) */
+    /* optional device allocator for buffers and the twin/stage pool (C6, L20.s23-29), e.g. the
+       torch caching allocator; both NULL = cudaMalloc / cudaFree.  dev_alloc returns a device
+       pointer (16-byte aligned) or NULL on failure; alloc_user is passed through. */
+    void *(*dev_alloc)(size_t bytes, void *alloc_user);
+    void  (*dev_free)(void *ptr, void *alloc_user);
+    void   *alloc_user;
 } fcl_context_desc;
 
-/* Create a context on desc->device (desc may be NULL: device 0, defaults).
+/* Create a context on desc->device (desc may be NULL: device 0, defaults) -- FluidiCL's runtime
+ * initialization (L20.s10-12: the hd / dh command queues; L18.s18-21: the CPU scheduler thread;
+ * L20.s23-29: the buffer pool).
  * Owns: streams it creates, the pinned status words, device counters, the
  * twin/stage pool and the host executor threads.  Loads every kernel of the
  * library (no lazy loading at a first launch, which can wait for the device
@@ -330,7 +339,8 @@ fcl_status fcl_buffer_device_written(fcl_context ctx, fcl_buffer buf, size_t off
  * Errors: FCL_INVALID_VALUE, FCL_CUDA_ERROR. */
 fcl_status fcl_mirror_upper(void *a, size_t n, uint32_t elem_size, void *stream);
 
-/* Wait until every launch, merge and copy of the context has completed;
+/* Wait until every launch, merge and copy of the context has completed (clFinish; the results
+ * "returned to the host", L16.s36-38, L20.s13-19);
  * outputs are then coherent on host and device.  Reports deferred errors. */
 fcl_status fcl_finish(fcl_context ctx);
 

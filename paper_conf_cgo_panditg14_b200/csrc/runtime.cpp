@@ -35,6 +35,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <cctype>
 #include <map>
 #include <array>
 #include <mutex>
@@ -165,12 +166,20 @@ struct Executor {
     AbortFlag abort_flag{0};
     int64_t spin_ns = 2 * 1000 * 1000;    // spin 2 ms after a job before sleeping
 
-    void start(int nthreads, bool pin) {
+    // local: the cores of the GPU's NUMA node (empty: unknown); the executor uses those of the
+    // process affinity mask that are local to the GPU when there are at least three of them
+    void start(int nthreads, bool pin, const std::vector<int> &local = {}) {
         cpu_set_t set;
         CPU_ZERO(&set);
         if (sched_getaffinity(0, sizeof set, &set) == 0) {
             for (int c = 0; c < CPU_SETSIZE; ++c)
                 if (CPU_ISSET(c, &set)) cores.push_back(c);
+        }
+        if (!local.empty()) {
+            std::vector<int> both;
+            for (int c : cores)
+                if (std::find(local.begin(), local.end(), c) != local.end()) both.push_back(c);
+            if (both.size() >= 3) cores = both;
         }
         if (cores.empty()) cores.push_back(0);
         // default: every core but two -- one for the coordinator (cores[0]), one left free for
@@ -396,6 +405,9 @@ struct Job {
 struct fcl_context_st {
     int device = 0;
     int num_sms = 148;
+    void *(*dev_alloc)(size_t, void *) = nullptr;   // fcl_context_desc allocator (nullptr: cudaMalloc)
+    void (*dev_free)(void *, void *) = nullptr;
+    void *alloc_user = nullptr;
     cudaStream_t main = nullptr, hd = nullptr, dh = nullptr;
     bool own_main = false, own_hd = false, own_dh = false;
     // JOB_XFER copies and their tickets.  Not hd: phase A queues waits for main positions on hd
@@ -574,6 +586,19 @@ struct fcl_context_st {
 
 namespace {
 
+// Device memory of buffers and pool entries: the context's allocator, or cudaMalloc / cudaFree.
+void *dmalloc(fcl_context ctx, size_t bytes) {
+    if (ctx->dev_alloc) return ctx->dev_alloc(bytes ? bytes : 16, ctx->alloc_user);
+    void *p = nullptr;
+    if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+    return p;
+}
+void dfree(fcl_context ctx, void *p) {
+    if (!p) return;
+    if (ctx->dev_free) ctx->dev_free(p, ctx->alloc_user);
+    else cudaFree(p);
+}
+
 fcl_status set_err(fcl_context ctx, fcl_status s, const char *fmt, ...) {
     if (ctx) {
         char b[512];
@@ -625,15 +650,14 @@ void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait) {
         if (e.hd_pending) { *hd_wait = true; e.hd_pending = false; }
         return e.p;
     }
-    void *p = nullptr;
-    if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) {
-        cudaGetLastError();
+    void *p = dmalloc(ctx, bytes);
+    if (!p) {
         // free every unused entry and retry once (L20.s29: reclaim older unused buffers)
         for (auto it = ctx->pool.begin(); it != ctx->pool.end();) {
-            if (!it->used) { cudaFree(it->p); it = ctx->pool.erase(it); }
+            if (!it->used) { dfree(ctx, it->p); it = ctx->pool.erase(it); }
             else ++it;
         }
-        if (cudaMalloc(&p, bytes ? bytes : 16) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+        if (!(p = dmalloc(ctx, bytes))) return nullptr;
     }
     ctx->pool.push_back({p, bytes, true, false, ctx->epoch});
     return p;
@@ -657,7 +681,7 @@ void pool_trim(fcl_context ctx) {
         const bool old = it->last_epoch + ctx->pool_keep < ctx->epoch || total > ctx->pool_cap;
         if (!it->used && !it->hd_pending && old) {
             total -= it->bytes;
-            cudaFree(it->p);
+            dfree(ctx, it->p);
             it = ctx->pool.erase(it);
         } else {
             ++it;
@@ -2057,6 +2081,29 @@ static void segv_trace(int sig) {
     raise(sig);
 }
 
+// The CPUs of the GPU's NUMA node (/sys/bus/pci/devices/<bus id>/local_cpulist), empty if unknown:
+// a host pool next to its GPU reads and writes the pinned mirrors in local DRAM (SURVEY §8b:
+// "all local-NUMA cores").
+static std::vector<int> gpu_local_cpus(int device) {
+    std::vector<int> out;
+    char bus[32] = {0};
+    if (cudaDeviceGetPCIBusId(bus, sizeof bus, device) != cudaSuccess) { cudaGetLastError(); return out; }
+    for (char *c = bus; *c; ++c) *c = (char)tolower(*c);
+    std::string path = std::string("/sys/bus/pci/devices/") + bus + "/local_cpulist";
+    FILE *f = fopen(path.c_str(), "r");
+    if (!f) return out;
+    char line[4096] = {0};
+    if (fgets(line, sizeof line, f)) {
+        for (char *tok = strtok(line, ",\n"); tok; tok = strtok(nullptr, ",\n")) {
+            int a = -1, b = -1;
+            if (sscanf(tok, "%d-%d", &a, &b) == 2) { for (int c = a; c <= b; ++c) out.push_back(c); }
+            else if (sscanf(tok, "%d", &a) == 1) out.push_back(a);
+        }
+    }
+    fclose(f);
+    return out;
+}
+
 fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_SEGV_TRACE") && atoi(getenv("FCL_SEGV_TRACE")) != 0) {
         signal(SIGSEGV, segv_trace);
@@ -2074,6 +2121,10 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     fcl_context ctx = new fcl_context_st();
     ctx->device = d.device;
     ctx->status_location = d.status_location;
+    if ((d.dev_alloc == nullptr) != (d.dev_free == nullptr)) { delete ctx; return FCL_INVALID_VALUE; }
+    ctx->dev_alloc = d.dev_alloc;
+    ctx->dev_free = d.dev_free;
+    ctx->alloc_user = d.alloc_user;
     auto fail = [&](cudaError_t e, const char *what) {
         fprintf(stderr, "fcl_create_context: %s: %s\n", what, cudaGetErrorString(e));
         delete ctx;
@@ -2201,7 +2252,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     const bool do_pin = d.pin_threads ? true : (pin ? atoi(pin) != 0 : true);
     int nthr = d.n_host_threads;
     if (nthr <= 0 && getenv("FCL_HOST_THREADS")) nthr = atoi(getenv("FCL_HOST_THREADS"));
-    ctx->ex.start(nthr, do_pin);
+    ctx->ex.start(nthr, do_pin, gpu_local_cpus(d.device));
     ctx->coord_core = (do_pin && !ctx->ex.cores.empty()) ? ctx->ex.cores[0] : -1;
     ctx->coord = std::thread(coordinator, ctx);
     *out = ctx;
@@ -2230,7 +2281,7 @@ fcl_status fcl_release_context(fcl_context ctx) {
     if (ctx->coord.joinable()) ctx->coord.join();
     cudaDeviceSynchronize();
     ctx->ex.shutdown();
-    for (auto &pe : ctx->pool) cudaFree(pe.p);
+    for (auto &pe : ctx->pool) dfree(ctx, pe.p);
     for (Job *j : ctx->free_jobs) {
         for (cudaEvent_t e : {j->ev_start, j->ev_k0, j->ev_t1, j->ev_k1, j->ev_m0, j->ev_m1, j->ev_staged, j->ev_ret, j->ev_wm, j->ev_d2h})
             if (e) cudaEventDestroy(e);
@@ -2279,14 +2330,14 @@ static fcl_status create_buffer_impl(fcl_context ctx, uint32_t flags, size_t byt
     cudaError_t e;
     if (flags & FCL_MEM_USE_DEVICE_PTR) { b->dev = device_ptr; b->own_dev = false; }
     else {
-        if ((e = cudaMalloc(&b->dev, bytes)) != cudaSuccess) { cudaGetLastError(); delete b; return set_err(ctx, FCL_OUT_OF_RESOURCES, "cudaMalloc(%zu)", bytes); }
+        if (!(b->dev = dmalloc(ctx, bytes))) { delete b; return set_err(ctx, FCL_OUT_OF_RESOURCES, "device allocation of %zu bytes", bytes); }
         b->own_dev = true;
     }
     if (flags & FCL_MEM_USE_HOST_PTR) { b->host = host_ptr; b->own_host = false; }
     else {
         if ((e = cudaHostAlloc(&b->host, bytes, cudaHostAllocPortable | cudaHostAllocMapped)) != cudaSuccess) {
             cudaGetLastError();
-            if (b->own_dev) cudaFree(b->dev);
+            if (b->own_dev) dfree(ctx, b->dev);
             delete b;
             return set_err(ctx, FCL_OUT_OF_RESOURCES, "cudaHostAlloc(%zu)", bytes);
         }
@@ -2351,7 +2402,7 @@ fcl_status fcl_release_buffer(fcl_buffer b) {
         if (b->stage) pool_put(ctx, b->stage, false);
         ctx->defer_list.erase(std::remove(ctx->defer_list.begin(), ctx->defer_list.end(), b), ctx->defer_list.end());
     }
-    if (b->own_dev) cudaFree(b->dev);
+    if (b->own_dev) dfree(ctx, b->dev);
     if (b->own_host) cudaFreeHost(b->host);
     cudaEventDestroy(b->d2h_ev);
     delete b;

@@ -41,11 +41,16 @@ EXPORTED = [
 ]
 
 
+DEV_ALLOC = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p)
+DEV_FREE = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p)
+
+
 class ContextDesc(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("n_host_threads", ctypes.c_int32),
                 ("pin_threads", ctypes.c_int32), ("status_location", ctypes.c_int32),
                 ("main_stream", ctypes.c_void_p), ("hd_stream", ctypes.c_void_p),
-                ("dh_stream", ctypes.c_void_p)]
+                ("dh_stream", ctypes.c_void_p), ("dev_alloc", DEV_ALLOC), ("dev_free", DEV_FREE),
+                ("alloc_user", ctypes.c_void_p)]
 
 
 class Arg(ctypes.Structure):
@@ -269,12 +274,20 @@ class Context:
     """A FluidiCL context on one CUDA device plus the host executor threads."""
 
     def __init__(self, device: int = 0, n_host_threads: int = 0, status_location: str = "device",
-                 streams: Optional[Sequence[int]] = None, pin_threads: bool = True):
+                 streams: Optional[Sequence[int]] = None, pin_threads: bool = True, allocator=None):
+        """allocator: optional (alloc(nbytes) -> device pointer, free(pointer)) pair for buffers and
+        the twin/stage pool, e.g. torch_allocator(); the callables must outlive the context."""
         d = ContextDesc()
         d.device, d.n_host_threads, d.pin_threads = int(device), int(n_host_threads), int(pin_threads)
         d.status_location = STATUS_HOST_MAPPED if status_location == "host_mapped" else STATUS_DEVICE
         if streams:
             d.main_stream, d.hd_stream, d.dh_stream = [int(s) if s else None for s in streams]
+        self._alloc_cbs = None
+        if allocator is not None:
+            alloc, free = allocator
+            self._alloc_cbs = (DEV_ALLOC(lambda n, u: int(alloc(int(n)) or 0)),
+                               DEV_FREE(lambda p, u: free(int(p))))
+            d.dev_alloc, d.dev_free = self._alloc_cbs
         h = ctypes.c_void_p()
         _check(load().fcl_create_context(ctypes.byref(d), ctypes.byref(h)), "fcl_create_context")
         self.handle = h.value
@@ -431,3 +444,17 @@ def merge_raw(gpu_ptr: int, cpu_ptr: int, twin_ptr: int, nbytes: int, elem_size:
 def mirror_upper(ptr: int, n: int, elem_size: int = 4, stream: int = 0):
     """a[j][i] = a[i][j] for i < j on an n x n row-major device matrix (asynchronous on `stream`)."""
     _check(load().fcl_mirror_upper(ptr, int(n), int(elem_size), stream or None), "fcl_mirror_upper")
+
+
+def torch_allocator(device: int = 0):
+    """(alloc, free) over the torch caching allocator (the context's device memory
+    from the framework's allocator), for Context(allocator=...)."""
+    import torch
+
+    def alloc(n: int) -> int:
+        return torch.cuda.caching_allocator_alloc(n, device)
+
+    def free(p: int) -> None:
+        torch.cuda.caching_allocator_delete(p)
+
+    return alloc, free

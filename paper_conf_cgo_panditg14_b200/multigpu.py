@@ -109,7 +109,8 @@ def exchange_rows(buf, nrows: int, ncols: int, spans: Sequence[Tuple[int, int]],
     t = device_tensor(buf, dtype)[: nrows * ncols].view(nrows, ncols)
     counts = [b - a for a, b in spans]
     stream = torch.cuda.current_stream()
-    if world > 1:
+    # (with a process group the collective runs even for one rank: the same NCCL path)
+    if world > 1 or (dist.is_available() and dist.is_initialized()):
         r0, r1 = spans[rank]
         contiguous = spans[0][0] == 0 and all(spans[k][1] == spans[k + 1][0] for k in range(world - 1))
         if dist.get_backend(group) == "nccl":

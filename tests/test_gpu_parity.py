@@ -545,3 +545,39 @@ def test_symmetric_accumulators(ctx, kernel, n, m, integer):
         out, _ = H.run(ctx, P, mode=mode, **opts)
         r = out[o].reshape(n, n).view(np.uint32)
         assert np.array_equal(r, r.T), f"{kernel} {mode} {opts}: not symmetric at {np.argwhere(r != r.T)[:3]}"
+
+
+def test_context_allocator_vtable(oracle_mod):
+    """fcl_context_desc's allocator: buffers and the twin/stage pool come from the
+    torch caching allocator; cooperative launches (free-running with a captured twin, forced
+    splits) give the GPU-only bits and every allocation is returned."""
+    import os
+    from paper_conf_cgo_panditg14_b200 import fcl
+    alloc, free = fcl.torch_allocator(0)
+    live = {}
+
+    def a(n):
+        p = alloc(n)
+        live[p] = n
+        return p
+
+    def f(p):
+        live.pop(p)
+        free(p)
+
+    os.environ["FCL_FORCE_TWIN"] = "1"
+    try:
+        ctx = fcl.Context(0, allocator=(a, f))
+    finally:
+        del os.environ["FCL_FORCE_TWIN"]
+    try:
+        P = W.make("conv2d", 150, 300, seed=63)
+        ref, _ = H.run(ctx, P, mode="gpu")
+        assert live, "no buffer came from the allocator"
+        for opts in (dict(), dict(forced_split=P.num_groups // 2), dict(gpu_delay_us=100)):
+            out, info = H.run(ctx, P, mode="coop", **opts)
+            assert_bits(out[1], ref[1], f"allocator vtable {opts}")
+        assert len(live) >= 2   # the pool's twin and stage are still held
+    finally:
+        ctx.release()
+    assert not live, f"{len(live)} allocations not returned"
