@@ -554,11 +554,12 @@ def test_context_allocator_vtable(oracle_mod):
     import os
     from paper_conf_cgo_panditg14_b200 import fcl
     alloc, free = fcl.torch_allocator(0)
-    live = {}
+    live, made = {}, [0]
 
     def a(n):
         p = alloc(n)
         live[p] = n
+        made[0] += 1
         return p
 
     def f(p):
@@ -573,7 +574,7 @@ def test_context_allocator_vtable(oracle_mod):
     try:
         P = W.make("conv2d", 150, 300, seed=63)
         ref, _ = H.run(ctx, P, mode="gpu")
-        assert live, "no buffer came from the allocator"
+        assert made[0] >= 2, "no buffer came from the allocator"
         for opts in (dict(), dict(forced_split=P.num_groups // 2), dict(gpu_delay_us=100)):
             out, info = H.run(ctx, P, mode="coop", **opts)
             assert_bits(out[1], ref[1], f"allocator vtable {opts}")
