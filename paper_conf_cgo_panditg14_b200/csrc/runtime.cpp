@@ -1808,10 +1808,17 @@ fcl_status cpu_job(fcl_context ctx, Job &j) {
 // ... discarding stale data", here: never reading it).
 fcl_status xfer_job(fcl_context ctx, Job &j) {
     ctx->xt_used.store(1, std::memory_order_relaxed);
-    CK(ctx, cudaStreamWaitEvent(ctx->xt, j.ev_start, 0));
+    auto fail = [&](cudaError_t e, const char *what) {   // (the waiting grid must still be released)
+        const fcl_status st = cuda_fail(ctx, e, what);
+        stream_store(ctx, ctx->d_xfer, (unsigned long long)j.ticket, ctx->xt, false);
+        return st;
+    };
+    cudaError_t e = cudaStreamWaitEvent(ctx->xt, j.ev_start, 0);
+    if (e != cudaSuccess) return fail(e, "transfer wait");
     for (int q = 0; q < j.nx; ++q) {
         fcl_buffer b = j.xb[q];
-        CK(ctx, cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->xt));
+        e = cudaMemcpyAsync(b->dev, b->host, b->bytes, cudaMemcpyHostToDevice, ctx->xt);
+        if (e != cudaSuccess) return fail(e, "transfer copy");
         ctx->counts[FCL_COUNT_H2D_BYTES] += (int64_t)b->bytes;
         j.info.h2d_bytes += (int64_t)b->bytes;
     }
@@ -1854,7 +1861,12 @@ void coordinator(fcl_context ctx) {
         }
         fcl_status st = FCL_SUCCESS;
         ctx->tr.add("phaseB_begin", j->epoch);
-        if (ctx->sticky.load() != FCL_SUCCESS) st = ctx->sticky.load();
+        if (ctx->sticky.load() != FCL_SUCCESS) {
+            st = ctx->sticky.load();
+            // a GPU launch waits on the device for this ticket: store it anyway (the context is
+            // lost; the grid must still be able to finish so that the caller's sync returns)
+            if (j->kind == Job::JOB_XFER) stream_store(ctx, ctx->d_xfer, (unsigned long long)j->ticket, ctx->xt, false);
+        }
         else if (j->kind == Job::JOB_CPU) st = cpu_job(ctx, *j);
         else if (j->kind == Job::JOB_XFER) st = xfer_job(ctx, *j);
         else st = coop_phase_b(ctx, *j);

@@ -261,3 +261,26 @@ def test_runtime_chunk_sizes_follow_c11(ctx, oracle_mod, init, step):
         assert_bits(out[q], ref[q], f"gesummv C11 run buf{q}")
     for b in bufs:
         b.release()
+
+
+@pytest.mark.parametrize("kernel,lws2d", [("conv2d", (32, 8)), ("syrk", (32, 8)), ("corr_reduce", (16, 4))])
+def test_exactly_once_inside_a_slice(ctx, kernel, lws2d):
+    """A multi-GPU slice [lo, hi) split at s (forced): [lo, s) on the GPU only, [s, hi) once on the
+    host only, and nothing outside the slice on either device."""
+    P = W.make(kernel, 300 if kernel != "syrk" else 256, 200 if kernel != "syrk" else 64, seed=7, lws2d=lws2d)
+    n = P.num_groups
+    k = ctx.kernel(H.kernel_name(P))
+    lo, hi = ctx.slice_range(k, P.gws, P.lws, 1, 3)
+    assert 0 < lo < hi < n
+    for s in sorted({lo, lo + 1, (lo + hi) // 2, hi - 1, hi}):
+        bufs = H.create_buffers(ctx, P)
+        H.run(ctx, P, mode="coop", bufs=bufs, wg_lo=lo, wg_hi=hi, forced_split=s, record_exec_counts=1)
+        c = ctx.exec_counts(n)
+        f = np.arange(n)
+        inside = (f >= lo) & (f < hi)
+        assert np.all(c["gpu_done"][~inside] == 0) and np.all(c["cpu_done"][~inside] == 0), (kernel, s)
+        g, h = inside & (f < s), inside & (f >= s)
+        assert np.all(c["gpu_done"][g] == c["gpu_frags"][g]) and np.all(c["gpu_frags"][g] > 0), (kernel, s)
+        assert np.all(c["cpu_done"][g] == 0) and np.all(c["gpu_done"][h] == 0) and np.all(c["cpu_done"][h] == 1), (kernel, s)
+        for b in bufs:
+            b.release()
