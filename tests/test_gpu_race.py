@@ -267,7 +267,7 @@ def test_runtime_chunk_sizes_follow_c11(ctx, oracle_mod, init, step):
 def test_exactly_once_inside_a_slice(ctx, kernel, lws2d):
     """A multi-GPU slice [lo, hi) split at s (forced): [lo, s) on the GPU only, [s, hi) once on the
     host only, and nothing outside the slice on either device."""
-    P = W.make(kernel, 300 if kernel != "syrk" else 256, 200 if kernel != "syrk" else 64, seed=7, lws2d=lws2d)
+    P = W.make(kernel, 300 if kernel != "syrk" else 512, 200 if kernel != "syrk" else 64, seed=7, lws2d=lws2d)
     n = P.num_groups
     k = ctx.kernel(H.kernel_name(P))
     lo, hi = ctx.slice_range(k, P.gws, P.lws, 1, 3)
