@@ -908,10 +908,22 @@ struct CorrReduceBody {
 // columns (float4) of 8 rows; its 10 input rows are loaded up front (memory-level parallelism),
 // the left/right halo columns come from the neighbouring lanes by shuffle (edge lanes load
 // them), and each output row is one 16-byte store (masked at the image border).
+// The 2DCONV task tile: FCL_CONV_TILE_COLS x FCL_CONV_TILE_ROWS outputs, one warp per 128 x 8
+// block.  Default 128 x 8 -- one warp per CTA: the body has no barrier, so a warp-sized CTA lets
+// the persistent dispatcher hand out tasks without a CTA barrier between them (256 x 32 tiles
+// with 8 warps spent 1.25 barrier stalls per issue waiting for the slowest warp of each task).
+#ifndef FCL_CONV_TILE_COLS
+#define FCL_CONV_TILE_COLS 128
+#endif
+#ifndef FCL_CONV_TILE_ROWS
+#define FCL_CONV_TILE_ROWS 8
+#endif
 template <typename T>
 struct Conv2DBody {
-    static constexpr int kThreads = 256;
-    static constexpr int kMinBlocks = 2;   // 10 x 16 B of loads in flight per thread needs the registers
+    static constexpr int kWarpsX = FCL_CONV_TILE_COLS / 128;   // 128-column warp blocks across a tile
+    static constexpr int kThreads = 32 * kWarpsX * (FCL_CONV_TILE_ROWS / 8);
+    // 10 x 16 B of loads in flight per thread needs the registers: 2 CTAs of 8 warps, or 16 of one
+    static constexpr int kMinBlocks = 512 / kThreads;
     static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = false;
     struct Params { const T *A; T *B; Tile2D tl; T c[9]; int vec4; };   // c[a*3+b]: row offset a-1, col offset b-1
@@ -980,10 +992,10 @@ struct Conv2DBody {
         const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
         const long long ni = tl.nrows, nj = tl.ncols;
         const unsigned int wm = tc.wmask;
-        if (p.vec4 && tcols == 256 && trows == 32) {
+        if (p.vec4 && tcols == FCL_CONV_TILE_COLS && trows == FCL_CONV_TILE_ROWS) {
             const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-            const int cg = warp & 1;                 // which 128-column half of the tile
-            const int rg = warp >> 1;                // which 8-row group
+            const int cg = warp % kWarpsX;           // which 128-column block of the tile
+            const int rg = warp / kWarpsX;           // which 8-row group
             const long long j = c0 + cg * 128 + lane * 4;   // first of this thread's 4 columns
             const long long ib = r0 + rg * 8;        // first output row of the group
             const long long wj0 = c0 + cg * 128;     // the warp's first column (warp-uniform test)
@@ -1586,6 +1598,12 @@ static void tile_shape(const Geom &g, int want_cols, int want_rows, int &tw, int
     tw = (int)(want_cols / g.lws[0]); if (tw < 1) tw = 1;
     th = (int)(want_rows / g.lws[1]); if (th < 1) th = 1;
 }
+// Task tile (in work-groups) of the 2-D tiled kernels: 2DCONV's warp-sized tile, CORR-reduce's
+// 256 x 32.
+static void tile_shape_of(const KArgs &a, const Geom &g, int &tw, int &th) {
+    if (a.kernel == K_CONV2D) tile_shape(g, FCL_CONV_TILE_COLS, FCL_CONV_TILE_ROWS, tw, th);
+    else tile_shape(g, 256, 32, tw, th);
+}
 
 template <typename T, int NMAT>
 static typename RowDotBody<T, NMAT>::Params rowdot_params(const KArgs &a, const Geom &g) {
@@ -1666,7 +1684,7 @@ static int with_body(const KArgs &a, const Geom &g, F &&f) {
         return f.template go<CorrReduceBody>(p);
     }
     case K_CONV2D: {
-        int tw, th; tile_shape(g, 256, 32, tw, th);
+        int tw, th; tile_shape_of(a, g, tw, th);
         if (a.integer) {
             Conv2DBody<int32_t>::Params p;
             p.A = (const int32_t *)a.dev[0]; p.B = (int32_t *)a.dev[1];
@@ -1727,7 +1745,7 @@ TaskSpace gpu_task_space(const KArgs &a, const Geom &g) {
         ts.threads = 256; break;
     }
     case K_CORR_REDUCE: case K_CONV2D: {
-        int tw, th; tile_shape(g, 256, 32, tw, th);
+        int tw, th; tile_shape_of(a, g, tw, th);
         const long long ntx = (g.ng[0] + tw - 1) / tw, nty = (g.ng[1] + th - 1) / th;
         ts.ntasks = ntx * nty; ts.threads = 256; break;
     }
@@ -1753,7 +1771,7 @@ int64_t gpu_task_key(const KArgs &a, const Geom &g, int64_t t) {
         return (t * CB) / g.lws[0];
     }
     case K_CORR_REDUCE: case K_CONV2D: {
-        int tw, th; tile_shape(g, 256, 32, tw, th);
+        int tw, th; tile_shape_of(a, g, tw, th);
         const long long ntx = (g.ng[0] + tw - 1) / tw;
         return (t % ntx) * tw + g.ng[0] * ((t / ntx) * th);
     }
@@ -1791,7 +1809,7 @@ void gpu_task_wgs(const KArgs &a, const Geom &g, int64_t t, std::vector<int64_t>
         out.push_back(gpu_task_key(a, g, t));   // a task is part of one work-group
         break;
     case K_CORR_REDUCE: case K_CONV2D: {
-        int tw, th; tile_shape(g, 256, 32, tw, th);
+        int tw, th; tile_shape_of(a, g, tw, th);
         const long long ntx = (g.ng[0] + tw - 1) / tw, tx = t % ntx, ty = t / ntx;
         rect(tx * tw, tx * tw + tw, ty * th, ty * th + th);
         break;
@@ -1845,7 +1863,7 @@ bool gpu_geometry_ok(const KArgs &a, const Geom &g, const char **why) {
 int64_t gpu_slice_align(const KArgs &a, const Geom &g) {
     switch (a.kernel) {
     case K_CORR_REDUCE: case K_CONV2D: {
-        int tw, th; tile_shape(g, 256, 32, tw, th);
+        int tw, th; tile_shape_of(a, g, tw, th);
         return g.ng[0] * th;                       // whole tile rows
     }
     case K_SYRK: case K_SYR2K: return g.ng[0] * (GBM / g.lws[1]);
