@@ -361,8 +361,11 @@ __device__ __forceinline__ void record_wm(const CoopCtl &c, unsigned int w) {
     atomicMax(c.wm_out, ((unsigned long long)c.epoch << 32) | (unsigned long long)(0xFFFFFFFFu - w));
 }
 
+// (a body may ask for a lower occupancy target in the dispatcher, whose loop state costs registers)
+template <class Body> struct CoopMinBlocks { static constexpr int value = Body::kMinBlocks; };
+
 template <class Body>
-__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+__global__ void __launch_bounds__(Body::kThreads, CoopMinBlocks<Body>::value)
 coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename Body::Params bp) {
     __shared__ long long s_task, s_key;
     __shared__ __align__(16) unsigned long long s_st[2];
@@ -764,7 +767,10 @@ enum { COL_DOT = 0, COL_SUM = 1, COL_SQDEV = 2 };
 template <typename T, int MODE>
 struct ColDotBody {
     static constexpr int kThreads = 256;
-    static constexpr int kMinBlocks = 2;
+#ifndef FCL_COLDOT_MINB
+#define FCL_COLDOT_MINB 2
+#endif
+    static constexpr int kMinBlocks = FCL_COLDOT_MINB;
     static constexpr bool kMasks = false;   // a task is part of one work-group
     static constexpr bool kLateClaim = false;
     static constexpr int U = 16;
@@ -923,7 +929,10 @@ struct Conv2DBody {
     static constexpr int kWarpsX = FCL_CONV_TILE_COLS / 128;   // 128-column warp blocks across a tile
     static constexpr int kThreads = 32 * kWarpsX * (FCL_CONV_TILE_ROWS / 8);
     // 10 x 16 B of loads in flight per thread needs the registers: 2 CTAs of 8 warps, or 16 of one
-    static constexpr int kMinBlocks = 512 / kThreads;
+    // plain grid: 20 warps per SM at 96 registers (0.337 -> 0.316 ms at 16384^2); the dispatcher
+    // keeps 16 (its loop state does not fit 96 registers without spilling: 0.74 ms)
+    static constexpr int kMinBlocks = 20 * 32 / kThreads;
+    static constexpr int kMinBlocksCoop = 16 * 32 / kThreads;
     static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = false;
     struct Params { const T *A; T *B; Tile2D tl; T c[9]; int vec4; };   // c[a*3+b]: row offset a-1, col offset b-1
@@ -1067,6 +1076,7 @@ struct Conv2DBody {
         return false;
     }
 };
+template <typename T> struct CoopMinBlocks<Conv2DBody<T>> { static constexpr int value = Conv2DBody<T>::kMinBlocksCoop; };
 
 // ------------------------------------------------------------------------------------------
 // GEMM-like bodies on CUDA cores (fp32 FFMA / int32 IMAD; no tensor cores: fp32 parity, see
