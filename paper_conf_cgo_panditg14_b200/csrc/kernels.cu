@@ -646,7 +646,13 @@ struct RowDotBody {
     // GESUMMV: 4 blocks of loads in flight at 72 registers = 7 CTAs per SM (1036 >= 1024 tasks,
     // still one wave at N = 4096; 0.74 vs 0.71 of HBM with 2 blocks, scripts/ubench_dots.cu).
     static constexpr int kThreads = 128;
-    static constexpr int kMinBlocks = (NMAT == 2) ? 7 : 8;
+#ifndef FCL_ROWDOT_MINB2
+#define FCL_ROWDOT_MINB2 7
+#endif
+#ifndef FCL_ROWDOT_MINB1
+#define FCL_ROWDOT_MINB1 8
+#endif
+    static constexpr int kMinBlocks = (NMAT == 2) ? FCL_ROWDOT_MINB2 : FCL_ROWDOT_MINB1;
     static constexpr bool kMasks = false;   // a task is part of one work-group
     static constexpr bool kLateClaim = false;
     static constexpr int kWarps = kThreads / 32;
