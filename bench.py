@@ -312,6 +312,11 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
         torch.cuda.synchronize()
         gc.collect()
         gc.disable()   # as timeit does: no cyclic collection inside the timed region
+        # one untimed step of every mode right before the timed ones: the first step after the
+        # collection above runs cold (host caches, the pool of worker threads asleep) and would
+        # otherwise always land on the first mode of the rotation
+        for m in ("coop", "gpu", "coop_always"):
+            one_step(m)
         c0 = ctx.counters()
         t_wall0 = time.perf_counter()
         # the timed COOP steps, each followed by a GPU-only step and a COOP step without device
