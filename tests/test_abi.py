@@ -109,14 +109,14 @@ def _slice(lib, name, gws, lws, r, n):
 
 @pytest.mark.parametrize("nranks", [1, 2, 3, 4, 8])
 def test_slice_ranges_partition_and_align(lib, nranks):
-    # 2DCONV 16384^2, lws 32x8: 512 x 2048 work-groups, tiles of 8 x 4 work-groups
+    # 2DCONV 16384^2, lws 32x8: 512 x 2048 work-groups, tiles of 4 x 1 work-groups (128 x 8 outputs)
     gws, lws = (16384, 16384), (32, 8)
     n_wg = 512 * 2048
     prev = 0
     for r in range(nranks):
         lo, hi = _slice(lib, "conv2d_f32", gws, lws, r, nranks)
         assert lo == prev and hi >= lo
-        assert lo % (512 * 4) == 0
+        assert lo % 512 == 0   # whole tile rows
         prev = hi
     assert prev == n_wg
     # 1-D kernels slice at any work-group

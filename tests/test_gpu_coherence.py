@@ -150,3 +150,50 @@ def test_without_the_version_wait_the_gpu_reads_stale_data(monkeypatch):
             b.release()
     finally:
         c.release()
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_chains_across_devices(ctx, seed):
+    """Random chains of dependent launches (RAW / WAR / WAW through four shared vectors) with every
+    launch on a random device (cooperative with random host / GPU delays, GPU-only, CPU-only,
+    device selection), no fcl_finish in between and the occasional read in the middle: every host
+    and device copy ends bit-identical to the same chain run one launch at a time on the GPU.
+    Integer kernels (exact wraparound), so values never overflow into inf."""
+    rng = np.random.default_rng(1000 + seed)
+    n = 384
+    A = rng.integers(-8, 9, size=n * n, dtype=np.int32)
+    vecs0 = [rng.integers(-8, 9, size=n, dtype=np.int32) for _ in range(4)]
+    gws, lws = (n,), (64,)
+    kernels = ["atax_tmp_i32", "atax_y_i32", "bicg_s_i32", "bicg_q_i32"]
+    ops = []
+    for _ in range(14):
+        i, j = rng.choice(4, size=2, replace=False)
+        ops.append((kernels[rng.integers(4)], int(i), int(j)))
+
+    def run(modes):
+        bA = ctx.buffer_from_array(A)
+        bv = [ctx.buffer_from_array(v) for v in vecs0]
+        for k, (name, i, j) in enumerate(ops):
+            m = modes[k]
+            opts = dict(m[1])
+            ctx.enqueue_ndrange(name, gws, lws, [bA, bv[i], bv[j], n, n], mode=m[0], **opts)
+            if modes is REF:
+                ctx.finish()
+            elif m[2]:   # a read in the middle of the chain
+                bv[j].read_array(np.int32)
+        ctx.finish()
+        out = [b.read_array(np.int32) for b in bv] + [H.device_array(b, np.int32) if b.versions()[2] else None for b in bv]
+        for b in [bA] + bv:
+            b.release()
+        return out
+
+    REF = [("gpu", {}, False)] * len(ops)
+    choices = [("coop", {}), ("coop", {"host_delay_us": 100}), ("coop", {"gpu_delay_us": 200}), ("gpu", {}),
+               ("cpu", {}), ("cpu", {"host_delay_us": 300}), ("coop", {"select": 1}), ("coop", {"forced_split": 3})]
+    modes = [choices[rng.integers(len(choices))] + (bool(rng.random() < 0.15),) for _ in ops]
+    want = run(REF)
+    got = run(modes)
+    for q in range(4):
+        _same(got[q], want[q], f"seed {seed} vector {q} host ({modes})")
+        if got[4 + q] is not None:
+            _same(got[4 + q], want[q], f"seed {seed} vector {q} device")
