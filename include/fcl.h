@@ -221,7 +221,9 @@ typedef struct {
                                 cannot contribute runs on the other alone: GPU-only if the host
                                 finished less than FCL_SELECT_MIN_SHARE (10 %) of the work-groups
                                 before the GPU exited, CPU-only if the host covered the whole range
-                                first on an idle GPU; the FCL_SELECT_PERIOD-th (16) launch after a
+                                first on an idle GPU, or at least FCL_SELECT_STREAM_SHARE (75 %) of a
+                                launch whose stale inputs were streamed over PCIe;
+                                the FCL_SELECT_PERIOD-th (16) launch after a
                                 probe probes cooperatively again, a period that doubles (up to 16x)
                                 while probes keep confirming the choice.  Forced splits, deferred
                                 merges and fault injection are never redirected. */

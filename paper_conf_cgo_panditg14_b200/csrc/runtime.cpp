@@ -500,6 +500,8 @@ struct fcl_context_st {
     std::atomic<int64_t> counts[FCL_COUNT_N] = {};   // fcl_get_counters (launch counts, bytes moved)
     int select_period = 16;                      // FCL_SELECT_PERIOD: every n-th launch of a shape probes
     double select_min_share = 0.10;              // FCL_SELECT_MIN_SHARE: host share a probe must reach
+    double select_stream_share = 0.75;           // FCL_SELECT_STREAM_SHARE: host share of a streamed probe
+                                                 // above which the host runs the shape alone
     uint32_t pool_keep = 256;                    // FCL_POOL_KEEP: launches an unused pool buffer survives
     size_t pool_cap = 16ull << 30;               // FCL_POOL_CAP_MB: unused buffers beyond this are freed
     unsigned long long test_gpu_delay_ns = 0;    // FCL_TEST_GPU_DELAY_US: lite grids start late (test hook)
@@ -1051,6 +1053,13 @@ void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
     // reduce: 7 % of the work-groups, 0.39 vs 0.26 ms GPU-only).
     else if (gpu_done && (host_work_useless || (double)j.info.cpu_wgs < ctx->select_min_share * (double)(j.L.hi - j.L.lo)))
         c = FCL_SELECTED_GPU;
+    // A launch whose inputs crossed PCIe while it ran (streamed) and of which the
+    // host still covered most of the range: the GPU's part was bounded by the link, not by its
+    // compute, and it held the link that the launches after it need for their own stale inputs.
+    // The host alone costs at most 1/share of the cooperative time and leaves the link to them
+    // (bench.py's e2e step: GESUMMV on the host while BICG's matrix crosses, 2.5 -> 1.4 ms).
+    else if (gpu_done && j.stream && (double)j.info.cpu_wgs >= ctx->select_stream_share * (double)(j.L.hi - j.L.lo))
+        c = FCL_SELECTED_CPU;
     std::lock_guard<std::mutex> lk(ctx->sel_mu);
     auto &e = ctx->sel[j.sel_key];
     // a probe that confirms the standing single-device choice backs the next one off; any change
@@ -2243,6 +2252,7 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_SELECT")) ctx->select_on = atoi(getenv("FCL_SELECT")) != 0;
     if (getenv("FCL_TEST_GPU_DELAY_US")) ctx->test_gpu_delay_ns = 1000ull * (unsigned long long)atoll(getenv("FCL_TEST_GPU_DELAY_US"));
     if (getenv("FCL_SELECT_MIN_SHARE")) ctx->select_min_share = atof(getenv("FCL_SELECT_MIN_SHARE"));
+    if (getenv("FCL_SELECT_STREAM_SHARE")) ctx->select_stream_share = atof(getenv("FCL_SELECT_STREAM_SHARE"));
     if (getenv("FCL_SELECT_PERIOD")) ctx->select_period = std::max(0, atoi(getenv("FCL_SELECT_PERIOD")));
     if (getenv("FCL_LAZY_BYTES")) ctx->lazy_max_bytes = (size_t)atoll(getenv("FCL_LAZY_BYTES"));
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;

@@ -186,6 +186,54 @@ def test_streamed_inputs(ctx, kernel, integer, lws, n1):
             b.release()
 
 
+def test_streamed_probe_with_host_majority_moves_to_the_host(monkeypatch):
+    """A streamed probe (stale inputs crossing PCIe while the launch runs) of which the host covered
+    at least FCL_SELECT_STREAM_SHARE of the range sends the next launches of that shape to the
+    host alone: no bytes cross PCIe for them.  The share is set to 0 here (any streamed probe the
+    GPU finished qualifies, FCL_SELECT_MIN_SHARE 0 so that the GPU-alone rule cannot take it
+    first); the same shape with resident inputs is not streamed and stays cooperative.  Every
+    result is the GPU-only one bit for bit."""
+    from paper_conf_cgo_panditg14_b200 import fcl
+    monkeypatch.setenv("FCL_SELECT_STREAM_SHARE", "0")
+    monkeypatch.setenv("FCL_SELECT_MIN_SHARE", "0")
+    c2 = fcl.Context(0)
+    try:
+        # the bench's size: the link delivers a third of the rows while the host computes the rest
+        P = W.make("gesummv", 4096, seed=34, lws1d=64)
+        ref, _ = H.run(c2, P, mode="gpu")
+        bufs = H.create_buffers(c2, P)
+        ins = [bufs[k] for k in range(len(P.bufs)) if k not in P.out_indices]
+        seen = []
+        for i in range(4):
+            for b in ins:
+                b.write(b.host_ptr, blocking=False)
+            c0 = c2.counters()
+            out, info = H.run(c2, P, mode="coop", bufs=bufs, select=1)
+            moved = c2.counters()["h2d_bytes"] - c0["h2d_bytes"]
+            seen.append((info["probe"], info["selected"], info["streamed_wgs"] > 0, moved))
+            for k in P.out_indices:
+                assert_bits(out[k], ref[k], f"launch {i}")
+        assert seen[0][0] == 1 and seen[0][2], seen
+        assert all(s[:2] == (0, SEL_CPU) and s[3] == 0 for s in seen[1:]), seen
+        # resident inputs (blocking writes refresh the device copies): another key, nothing to
+        # stream, so the probe's outcome is the ordinary one -- not the host alone (a lite grid
+        # computes everything: the GPU alone)
+        for b in ins:
+            b.write(b.host_ptr)
+        infos = []
+        for i in range(2):
+            out, info = H.run(c2, P, mode="coop", bufs=bufs, select=1)
+            infos.append(info)
+            for k in P.out_indices:
+                assert_bits(out[k], ref[k], f"resident launch {i}")
+        assert infos[0]["probe"] == 1 and infos[0]["streamed_wgs"] == 0, infos[0]
+        assert infos[1]["selected"] != SEL_CPU and infos[1]["gpu_path"] != PATH_NONE, infos[1]
+        for b in bufs:
+            b.release()
+    finally:
+        c2.release()
+
+
 def test_e2e_loop_selection_and_streaming(ctx):
     """The bench's e2e loop at a reduced size: every step writes the inputs (non-blocking, device
     copies stale), runs GESUMMV + BICG s/q as COOP launches with device selection, reads the
