@@ -10,7 +10,9 @@ pinned host mirrors when the timed region starts; L2 is flushed between steps.
 Reported value: algorithmic GB/s of the step (bytes the kernels must move: every matrix
 read once per kernel, vectors read/written) / device-timed step duration, summed over ranks.
 Multi-GPU (torchrun): each rank runs an independent problem of the same size ("replicas",
-weak scaling, no data-path collective); the max step time over ranks is used.
+weak scaling, no data-path collective); the max step time over ranks is used.  Every line also
+carries `sharded_conv2d_corr`: BASELINE configs[3] (2DCONV 16384^2 + CORR 4096^2) sharded over
+the same N ranks with NCCL all-gathers (strong scaling), so a 1/2/4/8-GPU run records both.
 
 Also reported: GPU-only / CPU-only step times (the paper's two baselines, Fig 13), the merge
 kernel's HBM bandwidth on a 1 GiB diff-merge, the dispatcher's roofline, the oracle timed
@@ -466,6 +468,13 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
                         "sample": f"one full step (GESUMMV + BICG s/q, N={N}) in the serial fp64 C oracle: "
                                   f"{t_or * 1e3:.0f} ms"}
 
+    # BASELINE configs[3] at the same N, sharded over the ranks (strong scaling; the headline
+    # `value` above is configs[1], one independent problem per rank): so that every line of a
+    # 1/2/4/8-GPU scaling run also carries the sharded 2DCONV + CORR step with its NCCL exchanges
+    sharded = None
+    if os.environ.get("FCL_BENCH_SHARDED", "1") != "0":
+        sharded = conv2d_corr_measure(max(2, min(args.steps, 10)), args.warmup, ctx, world, dev, stream, dist)
+
     if rank == 0:
         value = step_bytes * world / (coop_ms * 1e-3) / 1e9
         line = {
@@ -503,6 +512,7 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
                     "gpu_only_ms_per_step": round(e2e_gpu_ms, 4),
                     "gpu_only_value": round(step_bytes * world / (e2e_gpu_ms * 1e-3) / 1e9, 3)},
             "gpu_launches": int(round(launches_per_step * args.steps)),
+            "sharded_conv2d_corr": sharded,
             "clocks": clk.summary(),
             "host_cores": cores,
         }
@@ -524,15 +534,10 @@ def conv2d_corr_bytes() -> dict:
 
 
 def run_conv2d_corr(args, rank: int, world: int, local_rank: int):
-    """BASELINE.json configs[3]: 2DCONV 16384^2 and the CORR 4096^2 chain, the fixed problem sharded
-    over the N ranks (strong scaling): each rank runs the cooperative path on its work-group
-    slices with its own host pool, and every kernel's output is exchanged with an all-gather over
-    NCCL into the ranks' device copies (SURVEY §8e).  One step = both kernels' chains with their
-    exchanges; the timed region covers the launches, the host sides and the collectives."""
+    """BASELINE.json configs[3] on its own (`--workload conv2d_corr`): see conv2d_corr_measure."""
     import torch
     import fcl_harness as H
-    import workloads as W
-    from paper_conf_cgo_panditg14_b200 import _build, fcl, multigpu
+    from paper_conf_cgo_panditg14_b200 import _build, fcl
     if rank == 0:
         _build.build()
     dist = None
@@ -551,6 +556,30 @@ def run_conv2d_corr(args, rank: int, world: int, local_rank: int):
     host_threads = max(1, cores - 3)
     ctx = fcl.Context(local_rank, n_host_threads=host_threads, streams=(stream.cuda_stream, None, None))
     H.pin_caller()
+    with ClockSampler(local_rank) as clk:
+        clk.wait_started()
+        res = conv2d_corr_measure(args.steps, args.warmup, ctx, world, dev, stream, dist)
+    if rank == 0:
+        line = {"metric": METRIC, "value": res["value"], "unit": "GB/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["coop_ms"], "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": res["config"], "coop_ms": res["coop_ms"], "gpu_only_ms": res["gpu_only_ms"],
+                "coop_vs_gpu_only": res["coop_vs_gpu_only"], "clocks": clk.summary(), "host_cores": cores}
+        print(json.dumps(line), flush=True)
+    ctx.release()
+
+
+def conv2d_corr_measure(steps: int, warmup: int, ctx, world: int, dev, stream, dist) -> dict:
+    """BASELINE.json configs[3]: 2DCONV 16384^2 and the CORR 4096^2 chain, the fixed problem sharded
+    over the N ranks (strong scaling): each rank runs the cooperative path on its work-group
+    slices with its own host pool, and every kernel's output is exchanged with an all-gather over
+    NCCL into the ranks' device copies (SURVEY §8e).  One step = both kernels' chains with their
+    exchanges; the timed region covers the launches, the host sides and the collectives (CUDA
+    events on the launching stream, max over ranks).  COOP and GPU-only steps alternate."""
+    import torch
+    import fcl_harness as H
+    import workloads as W
+    from paper_conf_cgo_panditg14_b200 import multigpu
     P = W.make("conv2d", CONV_N, CONV_N, seed=11, out_init="zero")
     A, B = H.create_buffers(ctx, P)
     n = m = CORR_N
@@ -560,7 +589,6 @@ def run_conv2d_corr(args, rank: int, world: int, local_rank: int):
     d = ctx.buffer_from_array(data0)
     mean, std = ctx.buffer_from_array(np.zeros(m, np.float32)), ctx.buffer_from_array(np.zeros(m, np.float32))
     sym = ctx.buffer_from_array(np.zeros(m * m, np.float32))
-    pristine = torch.from_numpy(data0).to(dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
 
     def reset():
@@ -591,31 +619,24 @@ def run_conv2d_corr(args, rank: int, world: int, local_rank: int):
             t = float(x.item())
         return t
 
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         timed("coop"); timed("gpu")
-    with ClockSampler(local_rank) as clk:
-        clk.wait_started()
-        ts = {"coop": [], "gpu": []}
-        for r in range(args.steps):
-            for mode in (("coop", "gpu") if r % 2 == 0 else ("gpu", "coop")):
-                ts[mode].append(timed(mode))
+    ts = {"coop": [], "gpu": []}
+    for r in range(steps):
+        for mode in (("coop", "gpu") if r % 2 == 0 else ("gpu", "coop")):
+            ts[mode].append(timed(mode))
     coop_ms, gpu_ms = statistics.mean(ts["coop"]), statistics.mean(ts["gpu"])
     nbytes = sum(conv2d_corr_bytes().values())
-    del pristine
-    if rank == 0:
-        line = {"metric": METRIC, "value": round(nbytes / (coop_ms * 1e-3) / 1e9, 2), "unit": "GB/s", "n_gpus": world,
-                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(coop_ms, 4), "higher_is_better": True,
-                "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-                "config": {"workload": "conv2d_corr", "conv2d_n": CONV_N, "corr_n": CORR_N, "mode": "coop",
-                           "parallelism": f"sharded{world} (work-group slices + NCCL all-gather)",
-                           "l2": "flushed before each step (256 MiB write)",
-                           "bytes_counted": "2DCONV 2 N^2 x 4 B; CORR mean/std/reduce data passes; symmat operand once"},
-                "coop_ms": round(coop_ms, 4), "gpu_only_ms": round(gpu_ms, 4),
-                "coop_vs_gpu_only": round(gpu_ms / coop_ms, 4), "clocks": clk.summary(), "host_cores": cores}
-        print(json.dumps(line), flush=True)
     for b in (A, B, d, mean, std, sym):
         b.release()
-    ctx.release()
+    del flush
+    return {"value": round(nbytes / (coop_ms * 1e-3) / 1e9, 2), "unit": "GB/s", "steps": steps,
+            "coop_ms": round(coop_ms, 4), "gpu_only_ms": round(gpu_ms, 4),
+            "coop_vs_gpu_only": round(gpu_ms / coop_ms, 4), "scaling": "strong",
+            "config": {"workload": "conv2d_corr", "conv2d_n": CONV_N, "corr_n": CORR_N, "mode": "coop",
+                       "parallelism": f"sharded{world} (work-group slices + NCCL all-gather)",
+                       "l2": "flushed before each step (256 MiB write)",
+                       "bytes_counted": "2DCONV 2 N^2 x 4 B; CORR mean/std/reduce data passes; symmat operand once"}}
 
 
 def main():
