@@ -1131,7 +1131,30 @@ struct GemmBody {
         int vec4;
         int sym;          // SYRK: upper-triangle tiles, each also writes its mirror (KArgs::sym)
     };
-    struct Smem { T s[2][2][GBK][GBM + GPAD]; };   // [stage][A|B][k'][m]
+    // CORR's operand is K-major already (data[k][col]): interior tiles stream it with cp.async
+    // straight into shared memory, NSA stages of GBKA k-rows (NSA - 1 tiles in flight, no register
+    // staging), sharing the bytes of the register-staged path's stages.  16 k-rows x 2 stages:
+    // half the barriers of 8 x 4 (1.448 against 1.565 ms at 4096, scripts/ab_corr.sh; 8 x 3,
+    // 8 x 5 and unpadded rows no better; in dynamic shared memory 32 x 2 ran 1.444, 16 x 3 1.516,
+    // 32 x 3 1.481, 64 x 2 1.665 ms -- not worth leaving static shared memory).
+#ifndef FCL_CORR_GBKA
+#define FCL_CORR_GBKA 16
+#endif
+#ifndef FCL_CORR_NSA
+#define FCL_CORR_NSA 2
+#endif
+#ifndef FCL_CORR_APAD
+#define FCL_CORR_APAD 4
+#endif
+    static constexpr int GBKA = FCL_CORR_GBKA, NSA = FCL_CORR_NSA, APAD = FCL_CORR_APAD;
+    struct SmemBase { T s[2][2][GBK][GBM + GPAD]; };   // [stage][A|B][k'][m]
+    struct SmemCorr {
+        union {
+            T s[2][2][GBK][GBM + GPAD];
+            T a[NSA][2][GBKA][GBM + APAD];   // mainloop_async's stages
+        };
+    };
+    typedef typename std::conditional<OP == G_CORR && TN == 8, SmemCorr, SmemBase>::type Smem;
 
     __device__ static void tile_of(const Params &p, long long t, long long &bi, long long &bj) {
         if (OP == G_CORR || p.sym) {  // upper triangle, row-major over (b1 <= b2)
@@ -1269,27 +1292,23 @@ struct GemmBody {
         }
     }
 
-    // CORR's operand is K-major already (data[k][col]): interior tiles stream it with cp.async
-    // straight into shared memory, NSA stages of GBKA k-rows (three tiles in flight, no register
-    // staging), in the same bytes as Smem.
-    static constexpr int GBKA = 8, NSA = 4;
-    struct SmemA { T s[NSA][2][GBKA][GBM + GPAD]; };
     __device__ static void cp_async16(void *dst, const void *src) {
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
     }
     __device__ static bool mainloop_async(const Params &p, long long i0, long long j0, TaskCtx &tc, Smem &sm, T (&acc)[8][TN]) {
-        static_assert(sizeof(SmemA) <= sizeof(Smem), "async stages must fit the static smem");
-        static_assert(kThreads == 256 && TN == 8, "one 16-byte copy per operand and thread");
-        SmemA &sa = *reinterpret_cast<SmemA *>(&sm);
+        static_assert(kThreads == 256 && TN == 8 && GBKA % 8 == 0, "GBKA / 8 16-byte copies per operand and thread");
         const int tid = threadIdx.x, tx = tid % TXN, ty = tid / TXN;
         const int lr = tid >> 5, lc = (tid & 31) * 4;
         const long long nkt = p.m / GBKA;
         auto issue = [&](long long kt) {
             if (kt < nkt) {
                 const int st = (int)(kt % NSA);
-                const T *row = p.A + (kt * GBKA + lr) * p.ld;
-                cp_async16(&sa.s[st][0][lr][lc], row + i0 + lc);
-                cp_async16(&sa.s[st][1][lr][lc], row + j0 + lc);
+#pragma unroll
+                for (int q = 0; q < GBKA / 8; ++q) {
+                    const T *row = p.A + (kt * GBKA + lr + 8 * q) * p.ld;
+                    cp_async16(&sm.a[st][0][lr + 8 * q][lc], row + i0 + lc);
+                    cp_async16(&sm.a[st][1][lr + 8 * q][lc], row + j0 + lc);
+                }
             }
             asm volatile("cp.async.commit_group;" ::: "memory");
         };
@@ -1297,7 +1316,7 @@ struct GemmBody {
         for (int q = 0; q < NSA - 1; ++q) issue(q);
         // polls every `per` GBKA-tiles (= period GBK-tiles): a countdown, no division per tile
         const bool polling = tc.c != nullptr && tc.c->abort_period > 0;
-        const long long per = polling ? 2 * (long long)tc.c->abort_period : 1;
+        const long long per = polling ? ((long long)tc.c->abort_period * GBK + GBKA - 1) / GBKA : 1;
         long long left = per;
         bool poll = false;   // a poll posted at the end of the previous tile, decided after the barrier
         for (long long kt = 0; kt < nkt; ++kt) {
@@ -1311,10 +1330,10 @@ struct GemmBody {
             const int st = (int)(kt % NSA);
             T a[2][8], b[2][TN];
             auto fr = [&](int kk, T *fa, T *fb) {
-                const T4 a0 = *reinterpret_cast<const T4 *>(&sa.s[st][0][kk][ty * 4]);
-                const T4 a1 = *reinterpret_cast<const T4 *>(&sa.s[st][0][kk][64 + ty * 4]);
-                const T4 b0 = *reinterpret_cast<const T4 *>(&sa.s[st][1][kk][tx * 4]);
-                const T4 b1 = *reinterpret_cast<const T4 *>(&sa.s[st][1][kk][64 + tx * 4]);
+                const T4 a0 = *reinterpret_cast<const T4 *>(&sm.a[st][0][kk][ty * 4]);
+                const T4 a1 = *reinterpret_cast<const T4 *>(&sm.a[st][0][kk][64 + ty * 4]);
+                const T4 b0 = *reinterpret_cast<const T4 *>(&sm.a[st][1][kk][tx * 4]);
+                const T4 b1 = *reinterpret_cast<const T4 *>(&sm.a[st][1][kk][64 + tx * 4]);
                 fa[0] = a0.x; fa[1] = a0.y; fa[2] = a0.z; fa[3] = a0.w; fa[4] = a1.x; fa[5] = a1.y; fa[6] = a1.z; fa[7] = a1.w;
                 fb[0] = b0.x; fb[1] = b0.y; fb[2] = b0.z; fb[3] = b0.w; fb[4] = b1.x; fb[5] = b1.y; fb[6] = b1.z; fb[7] = b1.w;
             };
