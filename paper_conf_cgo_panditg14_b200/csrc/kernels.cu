@@ -364,6 +364,21 @@ __device__ __forceinline__ void record_wm(const CoopCtl &c, unsigned int w) {
 // (a body may ask for a lower occupancy target in the dispatcher, whose loop state costs registers)
 template <class Body> struct CoopMinBlocks { static constexpr int value = Body::kMinBlocks; };
 
+// A body's shared memory: static (the default), or dynamic for a body whose stages exceed the
+// 48 KB of static shared memory (Body::kDynSmem; the launch passes sizeof(Smem) and the kernels
+// get the attribute once, ensure_smem).
+template <class Body, class = void> struct DynSmem { static constexpr bool value = false; };
+template <class Body> struct DynSmem<Body, std::void_t<decltype(Body::kDynSmem)>> { static constexpr bool value = Body::kDynSmem; };
+template <class Body> struct SmemHolder {
+    typedef typename std::conditional<DynSmem<Body>::value, int, typename Body::Smem>::type type;
+};
+extern __shared__ __align__(16) unsigned char fcl_dyn_smem[];
+template <class Body>
+__device__ __forceinline__ typename Body::Smem &body_smem(typename SmemHolder<Body>::type &st) {
+    if constexpr (DynSmem<Body>::value) return *reinterpret_cast<typename Body::Smem *>(fcl_dyn_smem);
+    else return st;
+}
+
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, CoopMinBlocks<Body>::value)
 coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename Body::Params bp) {
@@ -371,7 +386,8 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     __shared__ __align__(16) unsigned long long s_st[2];
     __shared__ unsigned int s_w;
     __shared__ int s_flag[2];
-    __shared__ __align__(16) typename Body::Smem smem;
+    __shared__ __align__(16) typename SmemHolder<Body>::type smem_st;
+    typename Body::Smem &smem = body_smem<Body>(smem_st);
 
     if (blockIdx.x == 0 && threadIdx.x == 0) {   // counters of the next launch (stream-ordered)
         *c.claim_next = 0ull;
@@ -582,7 +598,8 @@ plain_kernel(const __grid_constant__ typename Body::Params bp, long long task_lo
         const unsigned long long t0 = globaltimer();
         while (globaltimer() - t0 < r.delay_ns) __nanosleep(1000);
     }
-    __shared__ __align__(16) typename Body::Smem smem;
+    __shared__ __align__(16) typename SmemHolder<Body>::type smem_st;
+    typename Body::Smem &smem = body_smem<Body>(smem_st);
     __shared__ long long s_key;
     TaskCtx tc;
     tc.c = nullptr; tc.s_st = nullptr; tc.s_flag = s_flag; tc.s_key = &s_key; tc.wmask = 0xFFFFFFFFu; tc.polls = 0;
@@ -1110,6 +1127,17 @@ template <typename T, int OP, int TN = 8>
 struct GemmBody {
     static_assert(TN == 8 || TN == 4, "TN = 4: the upper-triangle grids, CORR symmat");
     static constexpr int kThreads = TN == 8 ? 256 : 512;
+    // k'-tile (k' rows per barrier).  SYR2K's upper-triangle grid: 32 -- half the barriers, its
+    // 67 KB of stages in dynamic shared memory (0.515 -> 0.475 ms at 2048, 0.90 -> 0.97 of FP32
+    // FFMA); SYRK runs slower with 32 (0.237 -> 0.248 ms) and keeps 16 (scripts/ab_build.sh,
+    // profiles/r02_ab_gemm_gbk.txt).
+#ifndef FCL_GEMM_GBK_SYR2K
+#define FCL_GEMM_GBK_SYR2K 32
+#endif
+#ifndef FCL_GEMM_GBK_SYRK
+#define FCL_GEMM_GBK_SYRK 16
+#endif
+    static constexpr int GBK = TN != 4 ? ::fcl::GBK : (OP == G_SYR2K ? FCL_GEMM_GBK_SYR2K : FCL_GEMM_GBK_SYRK);
 #ifndef FCL_GEMM_MINB
 #define FCL_GEMM_MINB 2
 #endif
@@ -1155,6 +1183,7 @@ struct GemmBody {
         };
     };
     typedef typename std::conditional<OP == G_CORR && TN == 8, SmemCorr, SmemBase>::type Smem;
+    static constexpr bool kDynSmem = sizeof(Smem) > 40960;
 
     __device__ static void tile_of(const Params &p, long long t, long long &bi, long long &bj) {
         if (OP == G_CORR || p.sym) {  // upper triangle, row-major over (b1 <= b2)
@@ -1568,11 +1597,30 @@ static int largest_pow2_divisor_le(long long v, int cap) {
 }
 
 template <class Body>
+static size_t dyn_smem_bytes() { return DynSmem<Body>::value ? sizeof(typename Body::Smem) : 0; }
+
+// the dynamic shared memory attribute of both kernels of a body, once per process
+template <class Body>
+static void ensure_smem() {
+    static const bool once = [] {
+        const size_t b = dyn_smem_bytes<Body>();
+        if (b > 0) {
+            cudaFuncSetAttribute((const void *)coop_kernel<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)b);
+            cudaFuncSetAttribute((const void *)plain_kernel<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)b);
+            cudaGetLastError();
+        }
+        return true;
+    }();
+    (void)once;
+}
+
+template <class Body>
 static int occupancy_grid(int num_sms) {
     static int per_sm = 0;   // cached per body type
     if (per_sm == 0) {
         int v = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, coop_kernel<Body>, Body::kThreads, 0) != cudaSuccess || v < 1)
+        ensure_smem<Body>();
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, coop_kernel<Body>, Body::kThreads, dyn_smem_bytes<Body>()) != cudaSuccess || v < 1)
             v = 1;
         cudaGetLastError();
         per_sm = v;
@@ -1585,6 +1633,8 @@ static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long l
                        int num_sms, cudaStream_t s, const SlotReset *reset = nullptr, int pdl = PDL_OFF) {
     const long long n = task_hi - task_lo;
     if (n <= 0) return 0;
+    ensure_smem<Body>();
+    const size_t smem = dyn_smem_bytes<Body>();
     if (c) {
         long long grid = occupancy_grid<Body>(num_sms);
         if (grid > n) grid = n;
@@ -1595,11 +1645,11 @@ static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long l
             typename Body::Params pp = bp;
             void *args[] = {(void *)&cc, (void *)&pp};
             cudaError_t e = cudaLaunchCooperativeKernel((const void *)coop_kernel<Body>, dim3((unsigned)grid),
-                                                        dim3(Body::kThreads), args, 0, s);
+                                                        dim3(Body::kThreads), args, smem, s);
             if (e != cudaSuccess) return seterr(e, "coop_kernel cooperative launch");
             return (int)grid;
         }
-        coop_kernel<Body><<<(unsigned)grid, Body::kThreads, 0, s>>>(*c, bp);
+        coop_kernel<Body><<<(unsigned)grid, Body::kThreads, smem, s>>>(*c, bp);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return seterr(e, "coop_kernel launch");
         return (int)grid;
@@ -1609,6 +1659,7 @@ static int launch_body(const typename Body::Params &bp, const CoopCtl *c, long l
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)n);
     cfg.blockDim = dim3(Body::kThreads);
+    cfg.dynamicSmemBytes = smem;
     cfg.stream = s;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
