@@ -953,9 +953,14 @@ struct Conv2DBody {
     static constexpr int kThreads = 32 * kWarpsX * (FCL_CONV_TILE_ROWS / 8);
     // 10 x 16 B of loads in flight per thread needs the registers: 2 CTAs of 8 warps, or 16 of one
     // plain grid: 20 warps per SM at 96 registers (0.337 -> 0.316 ms at 16384^2); the dispatcher
-    // keeps 16 (its loop state does not fit 96 registers without spilling: 0.74 ms)
+    // keeps 16 (its loop state does not fit 96 registers without spilling: 0.74 ms with the
+    // 256 x 32 tiles; with 128 x 8 tiles 17-20 warps spill 38-70 bytes and run within 2 %,
+    // profiles/r02_ab_conv2d_coop_warps.txt)
     static constexpr int kMinBlocks = 20 * 32 / kThreads;
-    static constexpr int kMinBlocksCoop = 16 * 32 / kThreads;
+#ifndef FCL_CONV_COOP_WARPS
+#define FCL_CONV_COOP_WARPS 16
+#endif
+    static constexpr int kMinBlocksCoop = FCL_CONV_COOP_WARPS * 32 / kThreads;
     static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = false;
     struct Params { const T *A; T *B; Tile2D tl; T c[9]; int vec4; };   // c[a*3+b]: row offset a-1, col offset b-1
