@@ -226,7 +226,14 @@ typedef struct {
                                 the FCL_SELECT_PERIOD-th (16) launch after a
                                 probe probes cooperatively again, a period that doubles (up to 16x)
                                 while probes keep confirming the choice.  Forced splits, deferred
-                                merges and fault injection are never redirected. */
+                                merges and fault injection are never redirected.  Sequence
+                                selection on top (FCL_SEQ_SELECT=0 turns it off): the eligible
+                                launches between two fcl_finish calls are timed as a whole, first
+                                enqueue to the end of fcl_finish, per signature; when the probes'
+                                host rates predict the host alone faster (or, with no rate, the
+                                sequence is small), three sequences now and then run on the host
+                                alone, and the better of each kind's last four wins
+                                (info.seq_host). */
     int32_t gpu_delay_us;        /* fault injection: in a COOP launch every GPU task starts this many us
                                     late (a slow GPU, so that the host covers part of the range in a
                                     free-running race); such a launch runs the persistent dispatcher */
@@ -285,6 +292,9 @@ typedef struct {
                                     0 = abandoned.  The first n_c11_chunks are the C11 chunks, timed
                                     exactly as the heuristic saw them (L18.s23-32) */
     int32_t n_c11_chunks;        /* chunks sized by C11; the rest of n_chunks are return-race chunks */
+    int32_t seq_host;            /* 1 = run on the host alone by sequence selection: the launches
+                                    between two fcl_finish calls, timed as a whole, ran faster on
+                                    the host alone than with per-launch selection */
 } fcl_launch_info;
 
 /* info.selected */
@@ -364,7 +374,10 @@ fcl_status fcl_get_launch_info(fcl_context ctx, fcl_launch_info *info);
 #define FCL_COUNT_D2H_BYTES  7  /* bytes copied device -> host (returns, reads) */
 #define FCL_COUNT_LAUNCH_DRAINS 8  /* launches that had to wait for pending host sides first (the
                                       hazards buffer versions do not order) */
-#define FCL_COUNT_N          9
+#define FCL_COUNT_SEQ_HOST   9  /* COOP launches run on the host alone by sequence selection (also
+                                      counted in FCL_COUNT_SEL_CPU) */
+#define FCL_COUNT_SEQ_TRIALS 10 /* sequence-selection trials started */
+#define FCL_COUNT_N          11
 fcl_status fcl_get_counters(fcl_context ctx, int64_t *counts, int32_t n);
 
 /* Per-work-group execution counts of the most recent launch made with opts.record_exec_counts

@@ -493,9 +493,36 @@ struct fcl_context_st {
     // next_probe: the launch index of the next probe; period: launches between probes, which
     // doubles (up to 16x select_period) each time a probe confirms the standing choice and
     // falls back to select_period when it changes
-    struct SelectEnt { int64_t launches = 0; int choice = FCL_SELECTED_COOP; int64_t next_probe = 0; int64_t period = 0; };
+    // host_ms_per_wg: the host's best rate in the last probe (min over its completed C11 chunks of
+    // chunk time / chunk size; -1 = it completed none)
+    struct SelectEnt { int64_t launches = 0; int choice = FCL_SELECTED_COOP; int64_t next_probe = 0; int64_t period = 0;
+                       double host_ms_per_wg = -1; };
     std::mutex sel_mu;
     std::map<std::array<int64_t, 9>, SelectEnt> sel;
+    // Sequence selection (last item): the selection-eligible COOP launches
+    // between two fcl_finish calls form a sequence.  Per signature (the launches' keys without the
+    // stale bit, in order) the wall times from the first enqueue to the end of fcl_finish of the
+    // default per-launch selection and of the host alone (last four of each), the standing
+    // choice, and the trial schedule.
+    typedef std::array<int64_t, 8> SeqKey;
+    struct SeqEnt {
+        std::vector<SeqKey> keys;
+        double t_run[2][4] = {}; int n_run[2] = {0, 0};   // [0] default selection, [1] host alone
+        double est_host = -1;                             // Σ host-alone estimates (ms); -1 unknown
+        double work = 0;                                  // Σ multiply-adds of its launches
+        int choice = 0, trial = 0, trial_kind = 0;        // trial: sequences left in the running trial
+        int64_t seqs = 0, next_trial = 1, period = 16, loss_period = 32;
+    };
+    std::map<uint64_t, SeqEnt> seq_tab;
+    std::map<SeqKey, uint64_t> seq_first;   // a signature's first key -> the signature
+    struct SeqCur {
+        std::vector<SeqKey> keys; uint64_t h = 0; double t0 = 0; double est = 0, work = 0;
+        bool ok = true;       // every launch eligible, the plan (if any) followed
+        int run = -1;         // what this sequence runs: -1 no plan, 0 default, 1 host alone
+        bool trial = false; uint64_t plan = 0;
+    } seq;
+    bool seq_on = true;                          // FCL_SEQ_SELECT=0: per-launch selection only
+    bool seq_debug = false;                      // FCL_SEQ_DEBUG=1: one stderr line per recorded sequence
     bool select_on = true;                       // FCL_SELECT=0: off unless a launch asks for it
     std::atomic<int64_t> counts[FCL_COUNT_N] = {};   // fcl_get_counters (launch counts, bytes moved)
     int select_period = 16;                      // FCL_SELECT_PERIOD: every n-th launch of a shape probes
@@ -1071,6 +1098,171 @@ void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
     if (c == FCL_SELECTED_GPU && j.info.cpu_wgs == 0) e.period = 16 * base;
     e.choice = c;
     e.next_probe = e.launches + e.period - 1;
+    double best = -1;
+    for (int q = 0; q < std::min<int32_t>(j.info.n_c11_chunks, 64); ++q)
+        if (j.info.chunk_ms[q] > 0 && j.info.chunk_sizes[q] > 0) {
+            const double r = j.info.chunk_ms[q] / (double)j.info.chunk_sizes[q];
+            if (best < 0 || r < best) best = r;
+        }
+    e.host_ms_per_wg = best;
+}
+
+// ---- sequence selection (last item) ----
+// Per-launch selection sees one launch's race, not what the caller waits for: a chain of small
+// kernels whose GPU grids each win their race can still finish later on the GPU than on the
+// host alone, once launch latencies, the return of the results and the synchronisation are
+// counted (ATAX 256: 32 us GPU-alone, 26 us host-alone).  So the runtime also times whole
+// sequences -- the eligible COOP launches from one fcl_finish to the next, first enqueue to the
+// end of fcl_finish -- and, per signature, runs now and then the other way: the host alone for
+// three sequences, when the probes' host rates predict it faster than the default (or, where no
+// probe's host completed a chunk, when the sequence is small), or the default selection for one,
+// when the host alone is the standing choice.  The better of each kind's last four wins.  A sequence whose launches
+// do not follow the planned signature stops the plan (the launches already run on the host are
+// correct either way: every host body reproduces the GPU's bits).
+fcl_context_st::SeqKey seq_key(const Launch &L) {
+    const auto k = select_key(L);
+    fcl_context_st::SeqKey s;
+    for (int q = 0; q < 8; ++q) s[q] = k[q];
+    return s;
+}
+
+// The best of the last (up to) four sequences of a kind: the first run of a signature on the
+// host alone pays for waking the workers and touching the host copies (0.4 ms against 0.025 ms
+// warm for ATAX 256), and one such outlier must not decide.
+double seq_best(const double *t, int n) {
+    double v = 0;
+    for (int q = 0; q < std::min(n, 4); ++q) v = (q == 0 || t[q] < v) ? t[q] : v;
+    return v;
+}
+
+// Multiply-adds of a launch's range (the order of magnitude of its host work; a probe whose
+// host completed no chunk gives no rate, and then only small launches are worth a trial).
+double host_madds(const Launch &L) {
+    const double n0 = (double)L.a.n0, n1 = (double)L.a.n1;
+    double m;
+    switch (L.a.kernel) {
+    case K_GESUMMV: m = 2 * n0 * n0; break;
+    case K_SYRK: m = n0 * n0 * n1; break;
+    case K_SYR2K: m = 2 * n0 * n0 * n1; break;
+    case K_CORR_CORR: m = 0.5 * n1 * n1 * n0; break;
+    case K_CONV2D: m = 9 * n0 * n1; break;
+    default: m = n0 * n1; break;
+    }
+    const double nwg = (double)(L.g.ng[0] * L.g.ng[1] * L.g.ng[2]);
+    return nwg > 0 ? m * (double)(L.hi - L.lo) / nwg : m;
+}
+
+// Called for every launch before device selection; returns true if it runs on the host alone.
+bool seq_launch(fcl_context ctx, const Launch &L, bool eligible) {
+    auto &c = ctx->seq;
+    if (!ctx->seq_on) return false;
+    if (!eligible) { c.ok = false; c.run = -1; return false; }
+    if (!c.ok || c.keys.size() >= 64) { c.ok = false; c.run = -1; return false; }
+    const fcl_context_st::SeqKey k = seq_key(L);
+    std::lock_guard<std::mutex> lk(ctx->sel_mu);
+    if (c.keys.empty()) {
+        c.t0 = now_ms();
+        c.h = 1469598103934665603ull;
+        c.est = 0;
+        c.work = 0;
+        c.run = -1;
+        c.trial = false;
+        auto f = ctx->seq_first.find(k);
+        if (f != ctx->seq_first.end()) {
+            auto t = ctx->seq_tab.find(f->second);
+            if (t != ctx->seq_tab.end()) {
+                const auto &e = t->second;
+                c.run = e.trial > 0 ? e.trial_kind : e.choice;
+                c.trial = e.trial > 0;
+                c.plan = f->second;
+            }
+        }
+    }
+    const size_t pos = c.keys.size();
+    c.keys.push_back(k);
+    for (int64_t v : k) c.h = (c.h ^ (uint64_t)v) * 1099511628211ull;   // FNV-1a over the keys
+    c.work += host_madds(L);
+    {
+        const auto se = ctx->sel.find(select_key(L));
+        const double r = se == ctx->sel.end() ? -1.0 : se->second.host_ms_per_wg;
+        c.est = (c.est < 0 || r < 0) ? -1.0 : c.est + r * (double)(L.hi - L.lo);
+    }
+    if (c.run == 1) {
+        const auto t = ctx->seq_tab.find(c.plan);
+        if (t != ctx->seq_tab.end() && pos < t->second.keys.size() && t->second.keys[pos] == k) return true;
+        c.ok = false;   // off the planned signature: the rest runs by per-launch selection
+        c.run = -1;
+    }
+    return false;
+}
+
+// Called at the end of a successful fcl_finish.
+void seq_end(fcl_context ctx) {
+    auto &c = ctx->seq;
+    if (!ctx->seq_on) return;
+    const bool record = c.ok && !c.keys.empty();
+    if (record) {
+        const double wall = now_ms() - c.t0;
+        std::lock_guard<std::mutex> lk(ctx->sel_mu);
+        auto &e = ctx->seq_tab[c.h];
+        if (e.keys.empty()) {
+            e.keys = c.keys;
+            ctx->seq_first[c.keys[0]] = c.h;
+        }
+        const int kind = c.run == 1 ? 1 : 0;
+        // a sequence run as the other kind than planned (none: the first of its signature)
+        double *ring = e.t_run[kind];
+        for (int q = 3; q > 0; --q) ring[q] = ring[q - 1];
+        ring[0] = wall;
+        e.n_run[kind] = std::min(4, e.n_run[kind] + 1);
+        if (kind == 0) e.est_host = c.est;
+        e.work = c.work;
+        e.seqs += 1;
+        if (ctx->seq_debug)
+            fprintf(stderr, "[fcl seq] sig %016llx n %zu run %d trial %d wall %.4f est %.4f work %.3g choice %d seqs %lld next %lld\n",
+                    (unsigned long long)c.h, c.keys.size(), c.run, (int)c.trial, wall, c.est, c.work, e.choice, (long long)e.seqs,
+                    (long long)e.next_trial);
+        // a host trial whose two best sequences are both far slower than the default ends at once
+        if (c.trial && e.trial > 0 && kind == 1 && e.n_run[0] > 0 && e.n_run[1] >= 2 &&
+            std::max(e.t_run[1][0], e.t_run[1][1]) > 4.0 * seq_best(e.t_run[0], e.n_run[0]))
+            e.trial = 1;
+        if (c.trial && e.trial > 0) {
+            if (--e.trial == 0) {
+                const double d = seq_best(e.t_run[0], e.n_run[0]), h = seq_best(e.t_run[1], e.n_run[1]);
+                const int win = (e.n_run[1] > 0 && e.n_run[0] > 0 && h < d) ? 1 : 0;
+                if (win == e.choice && win == 0) {
+                    e.loss_period = std::min<int64_t>(4096, e.loss_period * 8);
+                    e.next_trial = e.seqs + e.loss_period;
+                } else if (win == e.choice) {
+                    e.period = std::min<int64_t>(256, e.period * 2);
+                    e.next_trial = e.seqs + e.period;
+                } else {
+                    e.choice = win;
+                    e.period = 16;
+                    e.next_trial = e.seqs + e.period;
+                }
+            }
+        } else if (e.trial == 0 && e.seqs >= e.next_trial) {
+            const int other = 1 - e.choice;
+            const double d = seq_best(e.t_run[0], e.n_run[0]);
+            // the host alone is tried when the probes' best host rates predict it faster (2DCONV:
+            // 21 ms predicted against 14.6 cooperative -- no trial), or -- no rate (the host
+            // completed no chunk before the GPU was done) -- when the sequence is small (at most
+            // 2^20 multiply-adds: well under a millisecond on the host)
+            const bool worth = e.est_host >= 0 ? e.est_host <= d : e.work <= (double)(1 << 20);
+            if (other == 1 && !worth) {
+                e.next_trial = e.seqs + e.loss_period;   // the host cannot come close: do not try
+            } else {
+                e.trial = other == 1 ? 3 : 1;   // (a default re-check is one sequence: its last four stand)
+                e.trial_kind = other;
+                ctx->counts[FCL_COUNT_SEQ_TRIALS] += 1;
+            }
+        }
+    }
+    c.keys.clear();
+    c.ok = true;
+    c.run = -1;
+    c.trial = false;
 }
 
 unsigned long long *plain_stamp(fcl_context ctx) {
@@ -2253,6 +2445,8 @@ fcl_status fcl_create_context(const fcl_context_desc *desc, fcl_context *out) {
     if (getenv("FCL_TEST_GPU_DELAY_US")) ctx->test_gpu_delay_ns = 1000ull * (unsigned long long)atoll(getenv("FCL_TEST_GPU_DELAY_US"));
     if (getenv("FCL_SELECT_MIN_SHARE")) ctx->select_min_share = atof(getenv("FCL_SELECT_MIN_SHARE"));
     if (getenv("FCL_SELECT_STREAM_SHARE")) ctx->select_stream_share = atof(getenv("FCL_SELECT_STREAM_SHARE"));
+    if (getenv("FCL_SEQ_DEBUG")) ctx->seq_debug = atoi(getenv("FCL_SEQ_DEBUG")) != 0;
+    if (getenv("FCL_SEQ_SELECT")) ctx->seq_on = atoi(getenv("FCL_SEQ_SELECT")) != 0;
     if (getenv("FCL_SELECT_PERIOD")) ctx->select_period = std::max(0, atoi(getenv("FCL_SELECT_PERIOD")));
     if (getenv("FCL_LAZY_BYTES")) ctx->lazy_max_bytes = (size_t)atoll(getenv("FCL_LAZY_BYTES"));
     ctx->force_twin = getenv("FCL_FORCE_TWIN") && atoi(getenv("FCL_FORCE_TWIN")) != 0;
@@ -2712,10 +2906,19 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
     }
     int selected = FCL_SELECTED_COOP;
     bool probe = false;
-    if (select_eligible(ctx, L)) {
-        selected = select_device(ctx, L, &probe);
-        if (selected == FCL_SELECTED_GPU) L.o.mode = FCL_MODE_GPU_ONLY;
-        else if (selected == FCL_SELECTED_CPU) L.o.mode = FCL_MODE_CPU_ONLY;
+    int seq_host = 0;
+    {
+        const bool eligible = select_eligible(ctx, L);
+        if (seq_launch(ctx, L, eligible)) {   // sequence selection: the host alone (§6.6)
+            selected = FCL_SELECTED_CPU;
+            L.o.mode = FCL_MODE_CPU_ONLY;
+            seq_host = 1;
+            ctx->counts[FCL_COUNT_SEQ_HOST] += 1;
+        } else if (eligible) {
+            selected = select_device(ctx, L, &probe);
+            if (selected == FCL_SELECTED_GPU) L.o.mode = FCL_MODE_GPU_ONLY;
+            else if (selected == FCL_SELECTED_CPU) L.o.mode = FCL_MODE_CPU_ONLY;
+        }
     }
     const bool coop = L.o.mode == FCL_MODE_COOP;
     const bool cpu_only = L.o.mode == FCL_MODE_CPU_ONLY;
@@ -2806,6 +3009,7 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         info.n_wg = L.hi - L.lo; info.wg_lo = L.lo; info.wg_hi = L.hi;
         info.gpu_watermark = info.published_watermark = L.hi;
         info.selected = selected;
+        info.seq_host = seq_host;
         for (int k = 0; k < L.a.nbuf; ++k)
             if (L.acc[k] & 2) {
                 fcl_buffer b = L.bufs[k];
@@ -2857,6 +3061,7 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         for (int k = 0; k < L.a.nbuf && !cpu_only; ++k)
             if (L.acc[k] & 2) { L.bufs[k]->ver_dev = kid; L.bufs[k]->ver_host = kid; }
         info.selected = selected;
+        info.seq_host = seq_host;
         ctx->counts[selected == FCL_SELECTED_GPU ? FCL_COUNT_SEL_GPU
                     : selected == FCL_SELECTED_CPU ? FCL_COUNT_SEL_CPU
                     : L.o.mode == FCL_MODE_GPU_ONLY ? FCL_COUNT_GPU_ONLY : FCL_COUNT_CPU_ONLY] += 1;
@@ -3101,6 +3306,7 @@ fcl_status fcl_finish(fcl_context ctx) {
     // change what it reads or writes (buffer I/O, a conflicting or host-side launch, release)
     // waits for it (quiesce); fcl_finish does not.
     CK(ctx, cudaGetLastError());
+    seq_end(ctx);
     ctx->tr.add("finish_end", ctx->epoch);
     if (ctx->tr.on && ctx->stats) {
         unsigned long long st[4 * fcl_context_st::kSlots];

@@ -84,7 +84,7 @@ class LaunchInfo(ctypes.Structure):
                 ("host_variant", ctypes.c_int32), ("n_host_variants", ctypes.c_int32),
                 ("profile_ms_per_wg", ctypes.c_double * 4), ("selected", ctypes.c_int32), ("probe", ctypes.c_int32),
                 ("streamed_wgs", ctypes.c_int64), ("chunk_ms", ctypes.c_double * 64),
-                ("n_c11_chunks", ctypes.c_int32)]
+                ("n_c11_chunks", ctypes.c_int32), ("seq_host", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("chunk_sizes", "profile_ms_per_wg", "chunk_ms")}
@@ -367,7 +367,7 @@ class Context:
         return info.as_dict()
 
     COUNTERS = ("coop", "probe", "sel_gpu", "sel_cpu", "gpu_only", "cpu_only", "h2d_bytes", "d2h_bytes",
-                "launch_drains")
+                "launch_drains", "seq_host", "seq_trials")
 
     def counters(self) -> dict:
         """Cumulative launch counters (fcl_get_counters): how COOP launches ran under device selection."""

@@ -300,3 +300,59 @@ def test_first_launch_of_a_kernel_behind_a_streamed_grid(tmp_path):
     env = dict(os.environ, FCL_SELECT="0")
     r = subprocess.run([sys.executable, str(script), root], capture_output=True, text=True, timeout=120, env=env)
     assert r.returncode == 0 and "ok" in r.stdout, (r.stdout[-2000:], r.stderr[-2000:])
+
+
+def _atax_chain(ctx, seed=0):
+    """BASELINE configs[0]: ATAX N=256, 16 work-groups per kernel; kernel 2 reads kernel 1's tmp."""
+    P1 = W.make("atax_tmp", 256, 256, seed=seed, lws1d=16, out_init="zero")
+    P2 = W.make("atax_y", 256, 256, seed=seed + 1, lws1d=16, out_init="zero")
+    b1, b2 = H.create_buffers(ctx, P1), H.create_buffers(ctx, P2)
+    b2[0].release(); b2[0] = b1[0]   # A
+    b2[1].release(); b2[1] = b1[2]   # tmp
+    return (P1, b1), (P2, b2)
+
+
+def test_sequence_selection_atax_chain(ctx):
+    """Sequence selection (last item): the two ATAX launches between fcl_finish
+    calls are timed as one sequence; the probes' host rates put the host alone within 2x, so a
+    trial of two sequences runs every launch on the host alone (info.seq_host) and the faster
+    median wins.  Whatever each sequence ran, y and tmp equal the GPU-only chain bit for bit."""
+    (P1, b1), (P2, b2) = _atax_chain(ctx, seed=61)
+    launches = [(P1, b1), (P2, b2)]
+
+    def step(mode, select):
+        for P, b in launches:
+            ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, select=select)
+        ctx.finish()
+        return (b1[2].read_array(np.float32).copy(), b2[2].read_array(np.float32).copy())
+
+    ref = step("gpu", 0)
+    c0 = ctx.counters()
+    for i in range(80):
+        got = step("coop", 1)
+        assert_bits(got[0], ref[0], f"tmp, sequence {i}")
+        assert_bits(got[1], ref[1], f"y, sequence {i}")
+    c1 = ctx.counters()
+    d = {k: c1[k] - c0[k] for k in c1}
+    assert d["seq_trials"] >= 1, d
+    assert d["seq_host"] >= 4 and d["seq_host"] % 2 == 0, d   # whole sequences: both launches
+    assert d["seq_host"] <= d["sel_cpu"], d
+    for bl in (b1, b2):
+        for k, b in enumerate(bl):
+            if not (bl is b2 and k in (0, 1)):
+                b.release()
+
+
+def test_sequence_selection_never_tries_a_hopeless_host(ctx):
+    """GESUMMV 4096: the GPU finishes before the host's first chunk, so the host rate is unknown
+    and no trial ever runs the host alone (it would cost ~40x the GPU's time)."""
+    P = W.make("gesummv", 4096, seed=62, lws1d=256)
+    b = H.create_buffers(ctx, P)
+    c0 = ctx.counters()
+    for i in range(40):
+        ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode="coop", select=1)
+        ctx.finish()
+    c1 = ctx.counters()
+    assert c1["seq_host"] == c0["seq_host"] and c1["seq_trials"] == c0["seq_trials"], (c0, c1)
+    for x in b:
+        x.release()
