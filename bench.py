@@ -387,6 +387,25 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
             ceil_ts.append(e0.elapsed_time(e1))
     del ra, rb
     read_ceiling_gbs = 2 * N * N * 4 / (statistics.median(ceil_ts) * 1e-3) / 1e9
+    # ... and torch's own read of the same bytes, GESUMMV's traffic pattern: one reduction over
+    # 2 x 64 MiB (134 MB read, nothing written back) -- a reference point, not a ceiling (the
+    # GESUMMV grid reads faster).  At this size a copy looks faster than a read: its 67 MB of
+    # writes land in the 126 MB L2 and drain after the timed region.  The read ceiling of this
+    # size, event-timed, is in profiles/r02_ubench_gesummv.txt (26.6 us, GESUMMV's pattern at it).
+    ro_ts = []
+    rr = torch.ones(2 * N * N, dtype=torch.float32, device=dev)
+    for r in range(8):
+        with torch.cuda.stream(stream):
+            flush.fill_(1.0); sweep.sum()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            rr.sum()
+            e1.record(stream)
+        e1.synchronize()
+        if r >= 2:
+            ro_ts.append(e0.elapsed_time(e1))
+    del rr
+    readonly_ceiling_gbs = 2 * N * N * 4 / (statistics.median(ro_ts) * 1e-3) / 1e9
     launches_per_step = statistics.mean(
         sum(i["gpu_launches"] for i in infos[j:j + 3]) for j in range(0, len(infos) - 2, 3))
 
@@ -502,7 +521,10 @@ def run_fcl(args, rank: int, world: int, local_rank: int):
                          "peak_source": peaks["source"],
                          "size_ceiling": {"what": "torch copy of 64 MiB (134 MB moved, as MEASURED_PEAKS but at this size), CUDA events, L2 flushed",
                                           "gbs": round(read_ceiling_gbs, 1),
-                                          "achieved_over_ceiling": round(achieved / read_ceiling_gbs, 4)}},
+                                          "achieved_over_ceiling": round(achieved / read_ceiling_gbs, 4),
+                                          "torch_read": {"what": "torch sum over 2 x 64 MiB (134 MB read, one launch), CUDA events, L2 flushed; a reference point, not a ceiling",
+                                                         "gbs": round(readonly_ceiling_gbs, 1),
+                                                         "achieved_over": round(achieved / readonly_ceiling_gbs, 4)}}},
             "merge": merge,
             "cpu_baseline": cpu_baseline,
             "e2e": {"value": round(step_bytes * world / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GB/s",
