@@ -39,6 +39,50 @@ __device__ __forceinline__ int32_t op_add(int32_t a, int32_t b) { return (int32_
 __device__ __forceinline__ float op_mul(float a, float b) { return __fmul_rn(a, b); }
 __device__ __forceinline__ int32_t op_mul(int32_t a, int32_t b) { return (int32_t)((uint32_t)a * (uint32_t)b); }
 
+// Packed fp32 fma (sm_100a FFMA2, PTX fma.rn.f32x2): two independent IEEE fp32 fmas with
+// round-to-nearest in one instruction -- each lane's result is bit-identical to op_fma's.  Used
+// by the GEMM bodies' register outer product, which is issue-bound with scalar FFMA.
+__device__ __forceinline__ float2 op_fma2(float2 a, float2 b, float2 c) {
+    unsigned long long r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;"
+        : "=l"(r)
+        : "l"(*reinterpret_cast<const unsigned long long *>(&a)), "l"(*reinterpret_cast<const unsigned long long *>(&b)),
+          "l"(*reinterpret_cast<const unsigned long long *>(&c)));
+    return *reinterpret_cast<const float2 *>(&r);
+}
+
+// acc[r][c] = fma(a[r], b[c], acc[r][c]) for every r < 8, c < TN (one k step of a register tile;
+// every output one fma, so the per-output k-chain is unchanged)
+#ifndef FCL_GEMM_FFMA2
+#define FCL_GEMM_FFMA2 1
+#endif
+template <int TN>
+__device__ __forceinline__ void outer(float (&acc)[8][TN], const float *a, const float *b) {
+    if (FCL_GEMM_FFMA2) {
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            const float2 ar = make_float2(a[r], a[r]);
+#pragma unroll
+            for (int c = 0; c < TN; c += 2) {
+                const float2 v = op_fma2(ar, make_float2(b[c], b[c + 1]), make_float2(acc[r][c], acc[r][c + 1]));
+                acc[r][c] = v.x; acc[r][c + 1] = v.y;
+            }
+        }
+    } else {
+#pragma unroll
+        for (int r = 0; r < 8; ++r)
+#pragma unroll
+            for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[r], b[c], acc[r][c]);
+    }
+}
+template <int TN>
+__device__ __forceinline__ void outer(int32_t (&acc)[8][TN], const int32_t *a, const int32_t *b) {
+#pragma unroll
+    for (int r = 0; r < 8; ++r)
+#pragma unroll
+        for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[r], b[c], acc[r][c]);
+}
+
 template <typename T> struct V4;
 template <> struct V4<float> { typedef float4 type; };
 template <> struct V4<int32_t> { typedef int4 type; };
@@ -1375,10 +1419,7 @@ struct GemmBody {
 #pragma unroll
             for (int kk = 0; kk < GBKA; ++kk) {
                 if (kk + 1 < GBKA) fr(kk + 1, a[(kk + 1) & 1], b[(kk + 1) & 1]);
-#pragma unroll
-                for (int r = 0; r < 8; ++r)
-#pragma unroll
-                    for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+                outer<TN>(acc, a[kk & 1], b[kk & 1]);
             }
             poll = false;
             if (polling && --left == 0) {
@@ -1429,10 +1470,7 @@ struct GemmBody {
 #pragma unroll
             for (int kk = 0; kk < GBK; ++kk) {
                 if (kk + 1 < GBK) frag(sm, st, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
-#pragma unroll
-                for (int r = 0; r < 8; ++r)
-#pragma unroll
-                    for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+                outer<TN>(acc, a[kk & 1], b[kk & 1]);
             }
             bool poll = false;
             if (polling && --left == 0) {
@@ -1460,10 +1498,7 @@ struct GemmBody {
 #pragma unroll
         for (int kk = 0; kk < GBK; ++kk) {
             if (kk + 1 < GBK) frag(sm, ST, kk + 1, tx, ty, a[(kk + 1) & 1], b[(kk + 1) & 1]);
-#pragma unroll
-            for (int r = 0; r < 8; ++r)
-#pragma unroll
-                for (int c = 0; c < TN; ++c) acc[r][c] = op_fma(a[kk & 1][r], b[kk & 1][c], acc[r][c]);
+            outer<TN>(acc, a[kk & 1], b[kk & 1]);
         }
         bool poll = false;
         if (polling && --left == 0) {
