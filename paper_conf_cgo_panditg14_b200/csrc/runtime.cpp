@@ -318,13 +318,18 @@ struct fcl_buffer_st {
     void *host;
     bool own_dev, own_host;
     bool host_valid, dev_valid;
-    bool d2h_pending;
-    bool d2h_on_main;      // the pending return copy is queued on main (a lazy return): later
-                           // grids on main are ordered behind it without a cross-stream wait
-    bool d2h_on_race;      // ... queued on the race stream (a later return on dh waits for it)
+    // The return-copy state below is written by the API thread (queueing a return) and read,
+    // for the buffers of its job, by the coordinator's phase B while later launches are being
+    // enqueued: atomics (relaxed -- the order that matters comes from the job queue and events)
+    std::atomic<bool> d2h_pending{false};
+    std::atomic<bool> d2h_on_main{false};   // the pending return copy is queued on main (a lazy
+                                            // return): later grids on main are ordered behind it
+                                            // without a cross-stream wait
+    std::atomic<bool> d2h_on_race{false};   // ... queued on the race stream (a later return on dh
+                                            // waits for it)
     bool ret_lazy;         // a lazy return of [ret_b0, ret_b1) is registered, not yet queued
     size_t ret_b0, ret_b1;
-    uint64_t d2h_gen;      // ctx->finish_gen when the pending return was queued
+    std::atomic<uint64_t> d2h_gen{0};   // ctx->finish_gen when the pending return was queued
     void *host_dptr;       // device-visible address of the (mapped) host mirror, nullptr = none
     cudaEvent_t d2h_ev;    // completion of the buffer's pending return copy (recorded on dh)
     // deferred merge state (opts.defer_merge)
@@ -1590,7 +1595,9 @@ fcl_status coop_phase_b(fcl_context ctx, Job &j) {
     // host copies of every argument must be current (pending returns of earlier launches)
     for (int k = 0; k < L.a.nbuf; ++k) {
         fcl_buffer b = L.bufs[k];
-        if (d2h_busy(ctx, b) && !((j.eager || j.lazy) && (L.acc[k] & 2))) {
+        // (the outputs of an eager / lazy launch are excluded before their state is read: the
+        // API thread may be queueing their lazy return for a later launch right now)
+        if (!((j.eager || j.lazy) && (L.acc[k] & 2)) && d2h_busy(ctx, b)) {
             CK(ctx, cudaEventSynchronize(b->d2h_ev));
         }
     }

@@ -180,6 +180,44 @@ int main() {
         }
         std::printf("done chain\n");
     }
+    {   // sequence selection: the ATAX 256 chain with device selection on, 60
+        // sequences -- host-alone trials, probes on the coordinator, buffer versions between them
+        const int64_t n = 256;
+        const size_t gws[3] = {256, 1, 1}, lws[3] = {16, 1, 1};
+        std::vector<float> A = rnd(n * n, 91), x = rnd(n, 92), zero(n, 0.f), want;
+        fcl_kernel k1, k2;
+        CHECK(fcl_get_kernel(ctx, "atax_tmp_f32", &k1));
+        CHECK(fcl_get_kernel(ctx, "atax_y_f32", &k2));
+        fcl_buffer bA, bx, bt, by;
+        CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, A.size() * 4, 4, A.data(), &bA));
+        CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, n * 4, 4, x.data(), &bx));
+        CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, n * 4, 4, zero.data(), &bt));
+        CHECK(fcl_create_buffer(ctx, FCL_MEM_READ_WRITE, n * 4, 4, zero.data(), &by));
+        fcl_arg a1[5] = {}, a2[5] = {};
+        a1[0].kind = a1[1].kind = a1[2].kind = FCL_ARG_BUFFER;
+        a1[0].buffer = bA; a1[1].buffer = bx; a1[2].buffer = bt;
+        a1[0].access = a1[1].access = FCL_ACCESS_IN; a1[2].access = FCL_ACCESS_OUT;
+        a1[3].kind = a1[4].kind = FCL_ARG_INT; a1[3].i = a1[4].i = n;
+        std::memcpy(a2, a1, sizeof a1);
+        a2[1].buffer = bt; a2[2].buffer = by;
+        fcl_launch_opts o;
+        CHECK(fcl_default_launch_opts(&o));
+        o.select = FCL_SELECT_ON;
+        for (int q = 0; q < 60; ++q) {
+            CHECK(fcl_enqueue_ndrange(ctx, k1, 1, gws, lws, a1, 5, &o, nullptr));
+            CHECK(fcl_enqueue_ndrange(ctx, k2, 1, gws, lws, a2, 5, &o, nullptr));
+            CHECK(fcl_finish(ctx));
+            std::vector<float> y(n);
+            CHECK(fcl_read_buffer(ctx, by, 0, n * 4, y.data(), 1));
+            if (want.empty()) want = y;
+            else if (std::memcmp(want.data(), y.data(), n * 4) != 0) { std::fprintf(stderr, "MISMATCH sequence %d\n", q); ++bad; }
+        }
+        int64_t cnt[FCL_COUNT_N];
+        CHECK(fcl_get_counters(ctx, cnt, FCL_COUNT_N));
+        std::printf("done sequences (seq_host %lld, seq_trials %lld)\n", (long long)cnt[FCL_COUNT_SEQ_HOST],
+                    (long long)cnt[FCL_COUNT_SEQ_TRIALS]);
+        for (auto b : {bA, bx, bt, by}) CHECK(fcl_release_buffer(b));
+    }
     CHECK(fcl_release_context(ctx));
     std::printf(bad ? "tsan driver: %d MISMATCHES\n" : "tsan driver ok\n", bad);
     return bad ? 1 : 0;

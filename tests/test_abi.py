@@ -77,6 +77,17 @@ def test_struct_layouts_match_header(tmp_path):
             assert got[(cname, fname)] == getattr(py, fname).offset, (cname, fname)
 
 
+def test_counter_names_match_header():
+    """fcl.Context.counters() names the FCL_COUNT_* entries in the header's order, all of them."""
+    inc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include", "fcl.h")
+    text = open(inc).read()
+    idx = {m.group(1): int(m.group(2)) for m in re.finditer(r"#define FCL_COUNT_([A-Z_0-9]+)\s+(\d+)", text)}
+    n = idx.pop("N")
+    assert sorted(idx.values()) == list(range(n))
+    names = [k.lower() for k, _ in sorted(idx.items(), key=lambda kv: kv[1])]
+    assert list(fcl.Context.COUNTERS) == names
+
+
 def test_kernel_table_and_signatures(lib):
     names = ["atax_tmp", "atax_y", "bicg_s", "bicg_q", "gesummv", "syrk", "syr2k", "conv2d"]
     for n in names:
