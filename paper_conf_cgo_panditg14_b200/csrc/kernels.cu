@@ -423,6 +423,11 @@ __device__ __forceinline__ typename Body::Smem &body_smem(typename SmemHolder<Bo
     else return st;
 }
 
+// Tasks claimed per atomic on the claim counter by bodies that claim ahead (A/B knob; 1 = the
+// paper's one work-group claim at a time, Fig 8)
+#ifndef FCL_CLAIM_BATCH
+#define FCL_CLAIM_BATCH 1
+#endif
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, CoopMinBlocks<Body>::value)
 coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename Body::Params bp) {
@@ -469,6 +474,7 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
     // the status is needed only by in-task polls and by the check before a claimed task
     const bool need_status = claims || c.abort_period > 0;
     if (threadIdx.x == 0 && need_status) status_prefetch(c, s_st);
+    long long b_next = 0, b_end = 0;   // thread 0: claimed batch (FCL_CLAIM_BATCH > 1)
     bool marked = false;   // thread 0: this CTA recorded a watermark (skip or abort)
     unsigned int rec_w = c.w_default;   // thread 0: lowest mask watermark recorded so far
     for (;;) {
@@ -519,8 +525,17 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
         // claim the next task while this one runs (no claim at all when the grid already
         // covers every task: no contention on the counter)
         long long t_next = c.task_hi;
-        if (!Body::kLateClaim && threadIdx.x == 0 && claims)
-            t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
+        if (!Body::kLateClaim && threadIdx.x == 0 && claims) {
+            if (FCL_CLAIM_BATCH == 1) {
+                t_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, 1ull);
+            } else {   // B ascending tasks per atomic (thread 0's batch: [b_next, b_end))
+                if (b_next >= b_end) {
+                    b_next = c.task_lo + (long long)gridDim.x + (long long)atomicAdd(c.claim, (unsigned long long)FCL_CLAIM_BATCH);
+                    b_end = b_next + FCL_CLAIM_BATCH;
+                }
+                t_next = b_next++;
+            }
+        }
         // a task that may span work-groups the host covers stores only those below w (the
         // watermark acted on: the merge domain starts at or below it)
         // (w == the range end: nothing covered, no mask -- the stores then skip the per-row work-group test)
