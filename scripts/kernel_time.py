@@ -29,6 +29,9 @@ def main():
     stream = torch.cuda.Stream()
     ctx = fcl.Context(0, streams=(stream.cuda_stream, None, None))
     flush = torch.empty(256 << 18, dtype=torch.float32, device="cuda")
+    # bench.py's flush: a write sweep, then a read sweep (L2 left full of clean lines, so the
+    # timed kernel pays no write-backs of the flush)
+    sweep = torch.ones(256 << 18, dtype=torch.float32, device="cuda")
     for spec in sys.argv[1:]:
         k, n0, n1, lws = spec.split(":")
         P = W.make(k, int(n0), int(n1), seed=0, lws1d=int(lws), out_init="zero")
@@ -37,7 +40,7 @@ def main():
         ts = []
         for r in range(20):
             with torch.cuda.stream(stream):
-                flush.fill_(float(r))
+                flush.fill_(float(r)); sweep.sum()
             L()
             ctx.finish()
             if r >= 5:
