@@ -505,8 +505,8 @@ struct fcl_context_st {
     std::mutex sel_mu;
     std::map<std::array<int64_t, 9>, SelectEnt> sel;
     // Sequence selection (last item): the selection-eligible COOP launches
-    // between two fcl_finish calls form a sequence.  Per signature (the launches' keys without the
-    // stale bit, in order) the wall times from the first enqueue to the end of fcl_finish of the
+    // between two fcl_finish calls form a sequence.  Per signature (the launches' keys in order,
+    // the stale bit counting only inputs no earlier launch of the sequence wrote: seq_key) the wall times from the first enqueue to the end of fcl_finish of the
     // default per-launch selection and of the host alone (last four of each), the standing
     // choice, and the trial schedule.
     typedef std::array<int64_t, 8> SeqKey;
@@ -522,6 +522,7 @@ struct fcl_context_st {
     std::map<SeqKey, uint64_t> seq_first;   // a signature's first key -> the signature
     struct SeqCur {
         std::vector<SeqKey> keys; uint64_t h = 0; double t0 = 0; double est = 0, work = 0;
+        std::vector<const void *> written;   // buffers written by the sequence's launches so far
         bool ok = true;       // every launch eligible, the plan (if any) followed
         int run = -1;         // what this sequence runs: -1 no plan, 0 default, 1 host alone
         bool trial = false; uint64_t plan = 0;
@@ -1124,10 +1125,20 @@ void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
 // when the host alone is the standing choice.  The better of each kind's last four wins.  A sequence whose launches
 // do not follow the planned signature stops the plan (the launches already run on the host are
 // correct either way: every host body reproduces the GPU's bits).
-fcl_context_st::SeqKey seq_key(const Launch &L) {
+// The selection key with its stale-input bit counting only inputs that no earlier launch of the
+// sequence wrote: a sequence whose first kernel ran on the host leaves the second one's input
+// stale on the device, and that must not change the signature, while inputs the caller wrote
+// (the e2e loop's non-blocking writes) do.
+fcl_context_st::SeqKey seq_key(const Launch &L, const std::vector<const void *> &written) {
     const auto k = select_key(L);
     fcl_context_st::SeqKey s;
     for (int q = 0; q < 8; ++q) s[q] = k[q];
+    int64_t stale = 0;
+    for (int b = 0; b < L.a.nbuf; ++b)
+        if ((L.acc[b] & 1) && !L.bufs[b]->dev_valid &&
+            std::find(written.begin(), written.end(), (const void *)L.bufs[b]) == written.end())
+            stale = 1;
+    s[7] = s[7] * 2 + stale;   // (s[7]: the range end, folded with the bit)
     return s;
 }
 
@@ -1163,7 +1174,10 @@ bool seq_launch(fcl_context ctx, const Launch &L, bool eligible) {
     if (!ctx->seq_on) return false;
     if (!eligible) { c.ok = false; c.run = -1; return false; }
     if (!c.ok || c.keys.size() >= 64) { c.ok = false; c.run = -1; return false; }
-    const fcl_context_st::SeqKey k = seq_key(L);
+    if (c.keys.empty()) c.written.clear();
+    const fcl_context_st::SeqKey k = seq_key(L, c.written);
+    for (int b = 0; b < L.a.nbuf; ++b)
+        if (L.acc[b] & 2) c.written.push_back(L.bufs[b]);
     std::lock_guard<std::mutex> lk(ctx->sel_mu);
     if (c.keys.empty()) {
         c.t0 = now_ms();
