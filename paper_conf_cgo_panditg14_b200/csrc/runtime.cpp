@@ -3187,7 +3187,10 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
         ctx->q_len.fetch_add(1, std::memory_order_release);
     }
     if (ctx->coord_sleeping.load()) ctx->q_cv.notify_all();
-    pool_trim(ctx);
+    // (no pool_trim here: cudaFree synchronises the device, and with this job queued the device
+    // may be waiting for the coordinator -- a streamed grid for its input pieces, a stream wait
+    // for a transfer ticket -- while the coordinator's own CUDA calls wait behind the cudaFree;
+    // that deadlock hit the 5 s stream guard.  fcl_finish trims, with nothing in flight.)
     if (L.o.blocking) {
         drain(ctx);
         s = j->status;
@@ -3327,6 +3330,10 @@ fcl_status fcl_finish(fcl_context ctx) {
     // change what it reads or writes (buffer I/O, a conflicting or host-side launch, release)
     // waits for it (quiesce); fcl_finish does not.
     CK(ctx, cudaGetLastError());
+    // "At the end of each kernel execution, older unused buffers are freed" (L20.s29): here, where
+    // every queued launch is done and the device idle, so cudaFree's synchronisation costs nothing
+    // and cannot wait for work that waits for the host
+    if (ctx->q_len.load(std::memory_order_acquire) == 0) pool_trim(ctx);
     seq_end(ctx);
     ctx->tr.add("finish_end", ctx->epoch);
     if (ctx->tr.on && ctx->stats) {
