@@ -356,3 +356,41 @@ def test_sequence_selection_never_tries_a_hopeless_host(ctx):
     assert c1["seq_host"] == c0["seq_host"] and c1["seq_trials"] == c0["seq_trials"], (c0, c1)
     for x in b:
         x.release()
+
+
+def test_sequence_plan_broken_midway(ctx):
+    """A sequence that starts like a signature whose plan is "host alone" but then launches a
+    different kernel: the first launch runs on the host by the plan, the plan stops at the
+    mismatch, the rest runs by per-launch selection -- and every result is still the GPU-only
+    one bit for bit (sequences alternate between the two shapes, 60 times)."""
+    (P1, b1), (P2, b2) = _atax_chain(ctx, seed=71)
+    Q = W.make("gesummv", 256, seed=72, lws1d=16, out_init="zero")
+    bq = H.create_buffers(ctx, Q)
+
+    def launch(P, b, mode, select):
+        ctx.enqueue_ndrange(H.kernel_name(P), P.gws, P.lws, H.make_args(ctx, P, b), mode=mode, select=select)
+
+    def seq(kind, mode, select):
+        launch(P1, b1, mode, select)
+        if kind == "a":
+            launch(P2, b2, mode, select)
+        else:
+            launch(Q, bq, mode, select)
+        ctx.finish()
+        out = [b1[2].read_array(np.float32).copy()]
+        out.append(b2[2].read_array(np.float32).copy() if kind == "a" else bq[4].read_array(np.float32).copy())
+        return out
+
+    ref = {k: seq(k, "gpu", 0) for k in ("a", "b")}
+    c0 = ctx.counters()
+    for i in range(60):
+        k = "a" if i % 3 else "b"
+        got = seq(k, "coop", 1)
+        for g, r in zip(got, ref[k]):
+            assert_bits(g, r, f"sequence {i} ({k})")
+    c1 = ctx.counters()
+    assert c1["seq_trials"] > c0["seq_trials"], (c0, c1)
+    for bl in (b1, b2, bq):
+        for k, b in enumerate(bl):
+            if not (bl is b2 and k in (0, 1)):
+                b.release()
