@@ -1350,6 +1350,18 @@ struct GemmBody {
         }
     }
     __device__ static T4 mk4(T a, T b, T c, T d) { T4 v; v.x = a; v.y = b; v.z = c; v.w = d; return v; }
+    // Shared-memory column swizzle of the K-major stages (SYRK / SYR2K): sstore transposes, a warp
+    // writing RW = 32 / G consecutive rows at G k-offsets LD apart -- which, with rows of GBM + GPAD
+    // = 132 floats (4 banks per k), fall on the same banks (2- to 4-way conflicts; ncu r02h: 13.4 M
+    // for SYR2K 2048).  Column c of k-row k lives at c ^ swz(k): each k-group moves to its own RW
+    // banks, and the xor (a multiple of 4 below 32) keeps every float4 of frag() contiguous.
+#ifndef FCL_GEMM_SWIZZLE
+#define FCL_GEMM_SWIZZLE 1
+#endif
+    static constexpr int SG = GBK / LD;   // threads per k-row group in sstore
+    __device__ static int swz(int k) {
+        return (FCL_GEMM_SWIZZLE && OP != G_CORR) ? ((k / LD) % SG) * (32 / SG) : 0;
+    }
     __device__ static void sstore(Smem &sm, int st, const T ra[LD], const T rb[LD]) {
         const int tid = threadIdx.x;
         if (OP == G_CORR) {
@@ -1364,23 +1376,26 @@ struct GemmBody {
             constexpr int KP = LD / 2;
             const int row = tid / (GBK / LD), kq = (tid % (GBK / LD)) * LD;
 #pragma unroll
-            for (int q = 0; q < KP; ++q) {
-                sm.s[st][0][kq + 2 * q][row] = ra[q]; sm.s[st][0][kq + 2 * q + 1][row] = ra[KP + q];
-                sm.s[st][1][kq + 2 * q][row] = rb[q]; sm.s[st][1][kq + 2 * q + 1][row] = rb[KP + q];
+            for (int q = 0; q < KP; ++q) {   // (k' = kq .. kq + LD - 1: one swizzle for the thread)
+                const int c = row ^ swz(kq);
+                sm.s[st][0][kq + 2 * q][c] = ra[q]; sm.s[st][0][kq + 2 * q + 1][c] = ra[KP + q];
+                sm.s[st][1][kq + 2 * q][c] = rb[q]; sm.s[st][1][kq + 2 * q + 1][c] = rb[KP + q];
             }
         } else {
             const int row = tid / (GBK / LD), kq = (tid % (GBK / LD)) * LD;
+            const int c = row ^ swz(kq);
 #pragma unroll
-            for (int q = 0; q < LD; ++q) { sm.s[st][0][kq + q][row] = ra[q]; sm.s[st][1][kq + q][row] = rb[q]; }
+            for (int q = 0; q < LD; ++q) { sm.s[st][0][kq + q][c] = ra[q]; sm.s[st][1][kq + q][c] = rb[q]; }
         }
     }
     __device__ static void frag(const Smem &sm, int st, int kk, int tx, int ty, T a[8], T b[TN]) {
-        const T4 a0 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][ty * 4]);
-        const T4 a1 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][64 + ty * 4]);
+        const int x = swz(kk);
+        const T4 a0 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][(ty * 4) ^ x]);
+        const T4 a1 = *reinterpret_cast<const T4 *>(&sm.s[st][0][kk][(64 + ty * 4) ^ x]);
         a[0] = a0.x; a[1] = a0.y; a[2] = a0.z; a[3] = a0.w; a[4] = a1.x; a[5] = a1.y; a[6] = a1.z; a[7] = a1.w;
 #pragma unroll
         for (int h = 0; h < NB; ++h) {
-            const T4 bv = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][h * 64 + tx * 4]);
+            const T4 bv = *reinterpret_cast<const T4 *>(&sm.s[st][1][kk][(h * 64 + tx * 4) ^ x]);
             b[4 * h] = bv.x; b[4 * h + 1] = bv.y; b[4 * h + 2] = bv.z; b[4 * h + 3] = bv.w;
         }
     }
