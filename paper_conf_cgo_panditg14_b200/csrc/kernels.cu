@@ -1191,17 +1191,18 @@ template <typename T, int OP, int TN = 8>
 struct GemmBody {
     static_assert(TN == 8 || TN == 4, "TN = 4: the upper-triangle grids, CORR symmat");
     static constexpr int kThreads = TN == 8 ? 256 : 512;
-    // k'-tile (k' rows per barrier).  SYR2K's upper-triangle grid: 32 -- half the barriers, its
-    // 67 KB of stages in dynamic shared memory (0.515 -> 0.475 ms at 2048, 0.90 -> 0.97 of FP32
-    // FFMA); SYRK runs slower with 32 (0.237 -> 0.248 ms) and keeps 16 (scripts/ab_build.sh,
-    // profiles/r02_ab_gemm_gbk.txt).
+    // k'-tile (k' rows per barrier) of the upper-triangle grids.  SYR2K: 64 (its 135 KB of stages
+    // in dynamic shared memory, one CTA per SM), 0.449 -> 0.415 ms at 2048 against 32 with the FFMA2
+    // loop and swizzled stages; SYRK keeps 16 (64: 0.229, 32: 0.215, 16: 0.216 ms)
+    // (profiles/r02_ab_gemm_gbk64.txt; before FFMA2: profiles/r02_ab_gemm_gbk.txt).
 #ifndef FCL_GEMM_GBK_SYR2K
-#define FCL_GEMM_GBK_SYR2K 32
+#define FCL_GEMM_GBK_SYR2K 64
 #endif
 #ifndef FCL_GEMM_GBK_SYRK
 #define FCL_GEMM_GBK_SYRK 16
 #endif
-    static constexpr int GBK = TN != 4 ? ::fcl::GBK : (OP == G_SYR2K ? FCL_GEMM_GBK_SYR2K : FCL_GEMM_GBK_SYRK);
+    static constexpr int GBK = TN != 4 ? ::fcl::GBK
+                               : (OP == G_SYR2K ? FCL_GEMM_GBK_SYR2K : OP == G_SYRK ? FCL_GEMM_GBK_SYRK : ::fcl::GBK);
 #ifndef FCL_GEMM_MINB
 #define FCL_GEMM_MINB 2
 #endif
@@ -1209,6 +1210,7 @@ struct GemmBody {
     static constexpr int TXN = GBM / TN;                 // threads along the columns
     static constexpr int NB = TN / 4;                    // float4 column groups per thread
     static constexpr int LD = GBM * GBK / kThreads;      // elements of each operand a thread loads per k'-tile
+    static_assert(LD % 4 == 0 && GBK % LD == 0, "gload / sstore: whole float4 loads, whole k-row groups");
     static constexpr bool kMasks = true;   // a task may span work-groups: stores masked by TaskCtx::wmask
     static constexpr bool kLateClaim = true;   // tasks of ~0.1-1 ms: an exposed claim costs nothing
     typedef typename V4<T>::type T4;
@@ -1294,9 +1296,12 @@ struct GemmBody {
     // KP consecutive k of row `row` of X (SYR2K operands): IN without bounds checks
     template <bool IN, int KP>
     __device__ static void loadk(const Params &p, const T *X, long long row, long long k, T *r) {
-        if (KP == 4) {
-            if (IN) ld4(X + row * p.ld + k, r);
-            else load4_k(p, X, row, k, r);
+        if (KP % 4 == 0) {   // (k a multiple of KP: 16-byte aligned when IN)
+#pragma unroll
+            for (int u = 0; u < KP / 4; ++u) {
+                if (IN) ld4(X + row * p.ld + k + 4 * u, r + 4 * u);
+                else load4_k(p, X, row, k + 4 * u, r + 4 * u);
+            }
         } else if (IN) {   // (k even, ld % 4 == 0: 8-byte aligned)
             typedef typename std::conditional<sizeof(T) == 4 && std::is_same<T, float>::value, float2, int2>::type T2;
             const T2 v = __ldg(reinterpret_cast<const T2 *>(X + row * p.ld + k));
@@ -1332,8 +1337,8 @@ struct GemmBody {
                 const int row = tid / (GBK / LD);
                 const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
                 const T *xa = p.A + (i0 + row) * p.ld + k, *xb = p.A + (j0 + row) * p.ld + k;
-                ld4(xa, ra); ld4(xb, rb);
-                if (LD == 8) { ld4(xa + 4, ra + 4); ld4(xb + 4, rb + 4); }
+#pragma unroll
+                for (int u = 0; u < LD / 4; ++u) { ld4(xa + 4 * u, ra + 4 * u); ld4(xb + 4 * u, rb + 4 * u); }
             }
             return;
         }
@@ -1345,8 +1350,10 @@ struct GemmBody {
         } else {   // SYRK
             const int row = tid / (GBK / LD);
             const long long k = kt * GBK + (tid % (GBK / LD)) * LD;
-            load4_k(p, p.A, i0 + row, k, ra); load4_k(p, p.A, j0 + row, k, rb);
-            if (LD == 8) { load4_k(p, p.A, i0 + row, k + 4, ra + 4); load4_k(p, p.A, j0 + row, k + 4, rb + 4); }
+#pragma unroll
+            for (int u = 0; u < LD / 4; ++u) {
+                load4_k(p, p.A, i0 + row, k + 4 * u, ra + 4 * u); load4_k(p, p.A, j0 + row, k + 4 * u, rb + 4 * u);
+            }
         }
     }
     __device__ static T4 mk4(T a, T b, T c, T d) { T4 v; v.x = a; v.y = b; v.z = c; v.w = d; return v; }
