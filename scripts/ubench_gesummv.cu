@@ -52,6 +52,32 @@ __global__ void __launch_bounds__(128, MINB) rows(const float *A, const float *B
     if (lane == 0) { tmp[i] = va; y[i] = __fadd_rn(__fmul_rn(alpha, va), __fmul_rn(beta, vb)); }
 }
 
+// rows_u4 with the row length a runtime argument (as in the library body)
+template <int U, int MINB>
+__global__ void __launch_bounds__(128, MINB) rows_rt(const float *A, const float *B, const float *x, float *tmp, float *y, float alpha, float beta, long long ncols) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const long long i = (long long)blockIdx.x * 4 + warp;
+    const float *pa = A + i * ncols + 4 * lane, *pb = B + i * ncols + 4 * lane, *px = x + 4 * lane;
+    float a0 = 0, a1 = 0, a2 = 0, a3 = 0, b0 = 0, b1 = 0, b2 = 0, b3 = 0;
+    const long long nfull = ncols / 128;
+    for (long long k = 0; k + U <= nfull; k += U, pa += U * 128, pb += U * 128, px += U * 128) {
+        float4 av[U], bv[U], xv[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) { av[u] = ldnc(pa + u * 128); bv[u] = ldnc(pb + u * 128); }
+#pragma unroll
+        for (int u = 0; u < U; ++u) xv[u] = __ldg(reinterpret_cast<const float4 *>(px + u * 128));
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            a0 = __fmaf_rn(av[u].x, xv[u].x, a0); a1 = __fmaf_rn(av[u].y, xv[u].y, a1);
+            a2 = __fmaf_rn(av[u].z, xv[u].z, a2); a3 = __fmaf_rn(av[u].w, xv[u].w, a3);
+            b0 = __fmaf_rn(bv[u].x, xv[u].x, b0); b1 = __fmaf_rn(bv[u].y, xv[u].y, b1);
+            b2 = __fmaf_rn(bv[u].z, xv[u].z, b2); b3 = __fmaf_rn(bv[u].w, xv[u].w, b3);
+        }
+    }
+    const float va = fold(a0, a1, a2, a3), vb = fold(b0, b1, b2, b3);
+    if (lane == 0) { tmp[i] = va; y[i] = __fadd_rn(__fmul_rn(alpha, va), __fmul_rn(beta, vb)); }
+}
+
 __device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(unsigned long long *b, unsigned cnt) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(cnt) : "memory");
@@ -188,6 +214,8 @@ int main() {
     for (int rep = 0; rep < 2; ++rep) {
         run("rows_u4", [&] { rows<4, 7><<<N / 4, 128>>>(A, B, x, tmp, y, alpha, beta); }, true);
         run("rows_u8", [&] { rows<8, 4><<<N / 4, 128>>>(A, B, x, tmp, y, alpha, beta); }, true);
+        run("rows_rt_u4", [&] { rows_rt<4, 7><<<N / 4, 128>>>(A, B, x, tmp, y, alpha, beta, (long long)N); }, true);
+        run("rows_rt_u8m6", [&] { rows_rt<8, 6><<<N / 4, 128>>>(A, B, x, tmp, y, alpha, beta, (long long)N); }, true);
         run("bulk_s2_b4", [&] { bulk<2, 4, 6><<<N / 4, 128, 4 * 2 * 2 * 512 * 4>>>(A, B, x, tmp, y, alpha, beta); }, true);
         run("bulk_s3_b4", [&] { bulk<3, 4, 4><<<N / 4, 128, 4 * 3 * 2 * 512 * 4>>>(A, B, x, tmp, y, alpha, beta); }, true);
         run("bulk_s4_b2", [&] { bulk<4, 2, 6><<<N / 4, 128, 4 * 4 * 2 * 256 * 4>>>(A, B, x, tmp, y, alpha, beta); }, true);
