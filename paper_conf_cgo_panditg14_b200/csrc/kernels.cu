@@ -423,6 +423,10 @@ __device__ __forceinline__ typename Body::Smem &body_smem(typename SmemHolder<Bo
     else return st;
 }
 
+// Masked bodies get a second, unmasked copy in the dispatcher (A/B knob)
+#ifndef FCL_UNMASKED_COPY
+#define FCL_UNMASKED_COPY 1
+#endif
 // Tasks claimed per atomic on the claim counter by bodies that claim ahead (A/B knob; 1 = the
 // paper's one work-group claim at a time, Fig 8)
 #ifndef FCL_CLAIM_BATCH
@@ -545,7 +549,17 @@ coop_kernel(const __grid_constant__ CoopCtl c, const __grid_constant__ typename 
             rec_w = w;
             marked = true;
         }
-        const bool aborted = Body::run(bp, t, tc, smem);
+        // (a task with nothing covered -- the common case -- runs a copy of the body in which the
+        // mask is the constant "keep everything": no per-row work-group tests or their branches)
+        bool aborted;
+        if (FCL_UNMASKED_COPY && Body::kMasks && tc.wmask == 0xFFFFFFFFu) {
+            TaskCtx t2 = tc;
+            t2.wmask = 0xFFFFFFFFu;
+            aborted = Body::run(bp, t, t2, smem);
+            tc.polls = t2.polls;
+        } else {
+            aborted = Body::run(bp, t, tc, smem);
+        }
         if (aborted) {
             if (threadIdx.x == 0) { record_wm(c, tc.abort_w()); marked = true; }
             break;
