@@ -961,8 +961,17 @@ struct Tile2D {
     long long ngx, lws0, lws1;
     int tw, th;              // tile size in work-groups
     long long ntx;           // tiles per tile-row
+    // task t -> (tile column, tile row).  32-bit division: task ids are below the flattened
+    // work-group count, < 2^32 (checked at launch) -- a 64-bit one is a called subroutine of ~70
+    // instructions, run for every task by the body and again by the dispatcher's key
+    __device__ __host__ void split(long long t, long long &tx, long long &ty) const {
+        const unsigned int ut = (unsigned int)t, un = (unsigned int)ntx;
+        tx = (long long)(ut % un);
+        ty = (long long)(ut / un);
+    }
     __device__ __host__ long long key(long long t) const {
-        const long long tx = t % ntx, ty = t / ntx;
+        long long tx, ty;
+        split(t, tx, ty);
         return tx * tw + ngx * (ty * th);
     }
     // work-group of output element (i, j), Fig 5 flattening
@@ -987,7 +996,8 @@ struct CorrReduceBody {
     __device__ static long long key(const Params &p, long long t) { return p.tl.key(t); }
     __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &) {
         const Tile2D &tl = p.tl;
-        const long long tx = t % tl.ntx, ty = t / tl.ntx;
+        long long tx, ty;
+        tl.split(t, tx, ty);
         const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
         const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
         const unsigned int wm = tc.wmask;
@@ -1097,7 +1107,8 @@ struct Conv2DBody {
 
     __device__ static bool run(const Params &p, long long t, TaskCtx &tc, Smem &) {
         const Tile2D &tl = p.tl;
-        const long long tx = t % tl.ntx, ty = t / tl.ntx;
+        long long tx, ty;
+        tl.split(t, tx, ty);
         const long long c0 = tx * tl.tw * tl.lws0, r0 = ty * tl.th * tl.lws1;
         const int tcols = (int)(tl.tw * tl.lws0), trows = (int)(tl.th * tl.lws1);
         const long long ni = tl.nrows, nj = tl.ncols;

@@ -527,6 +527,11 @@ struct fcl_context_st {
         int run = -1;         // what this sequence runs: -1 no plan, 0 default, 1 host alone
         bool trial = false; uint64_t plan = 0;
     } seq;
+    // Streamed launches (§6.7) queued or in phase B: their grids wait for pieces the coordinator
+    // issues, so the API thread must not allocate device or pinned memory meanwhile -- an
+    // allocation is an implicit synchronisation point, after which the pieces could not run
+    // before the grid that waits for them (a deadlock the 5 s stream guard turned into a trap)
+    std::atomic<int> stream_jobs{0};
     bool seq_on = true;                          // FCL_SEQ_SELECT=0: per-launch selection only
     bool seq_debug = false;                      // FCL_SEQ_DEBUG=1: one stderr line per recorded sequence
     bool select_on = true;                       // FCL_SELECT=0: off unless a launch asks for it
@@ -668,8 +673,10 @@ bool d2h_busy(fcl_context ctx, fcl_buffer b) {
 
 // ---- pool ----
 // Returns the buffer and whether main must wait for ctx->ev_hd_release before writing it.
-void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait) {
-    std::lock_guard<std::mutex> lk(ctx->pool_mu);
+void drain(fcl_context ctx);
+void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait, bool drained = false);
+void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait, bool drained) {
+    std::unique_lock<std::mutex> lk(ctx->pool_mu);
     int best = -1;
     for (size_t k = 0; k < ctx->pool.size(); ++k) {
         const PoolEnt &e = ctx->pool[k];
@@ -684,6 +691,12 @@ void *pool_get(fcl_context ctx, size_t bytes, bool *hd_wait) {
         e.last_epoch = ctx->epoch;
         if (e.hd_pending) { *hd_wait = true; e.hd_pending = false; }
         return e.p;
+    }
+    if (!drained && ctx->stream_jobs.load(std::memory_order_acquire) > 0) {
+        // (pool_mu released: the coordinator returns buffers under it while it drains)
+        lk.unlock();
+        drain(ctx);
+        return pool_get(ctx, bytes, hd_wait, true);
     }
     void *p = dmalloc(ctx, bytes);
     if (!p) {
@@ -2091,7 +2104,10 @@ void coordinator(fcl_context ctx) {
         }
         else if (j->kind == Job::JOB_CPU) st = cpu_job(ctx, *j);
         else if (j->kind == Job::JOB_XFER) st = xfer_job(ctx, *j);
-        else st = coop_phase_b(ctx, *j);
+        else {
+            st = coop_phase_b(ctx, *j);
+            if (j->stream) ctx->stream_jobs.fetch_sub(1, std::memory_order_acq_rel);
+        }
         if (j->kind == Job::JOB_CPU) ctx->host_done_seq.store(j->host_seq, std::memory_order_release);
         ctx->tr.add("phaseB_end", j->epoch);
         {
@@ -2562,6 +2578,7 @@ static fcl_status create_buffer_impl(fcl_context ctx, uint32_t flags, size_t byt
         return set_err(ctx, FCL_INVALID_VALUE, "elem_size %u invalid for %zu bytes", elem_size, bytes);
     if ((flags & FCL_MEM_USE_HOST_PTR) && !host_ptr) return set_err(ctx, FCL_INVALID_VALUE, "USE_HOST_PTR without host_ptr");
     if ((flags & FCL_MEM_USE_DEVICE_PTR) && !device_ptr) return set_err(ctx, FCL_INVALID_VALUE, "USE_DEVICE_PTR without device_ptr");
+    if (ctx->stream_jobs.load(std::memory_order_acquire) > 0) drain(ctx);   // (allocations below: see stream_jobs)
     fcl_buffer b = new fcl_buffer_st();
     b->ctx = ctx; b->bytes = bytes; b->elem_size = elem_size; b->flags = flags;
     cudaError_t e;
@@ -3138,6 +3155,7 @@ fcl_status fcl_enqueue_ndrange(fcl_context ctx, fcl_kernel kernel, uint32_t work
                 j->sbuf[j->nstream++] = k;
         }
         j->stream = j->nstream > 0;
+        if (j->stream) ctx->stream_jobs.fetch_add(1, std::memory_order_acq_rel);
         j->L.a.streamed = j->stream;
     }
     for (int k = 0; k < L.a.nbuf; ++k) {
