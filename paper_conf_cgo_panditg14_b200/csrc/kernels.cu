@@ -961,13 +961,22 @@ struct Tile2D {
     long long ngx, lws0, lws1;
     int tw, th;              // tile size in work-groups
     long long ntx;           // tiles per tile-row
-    // task t -> (tile column, tile row).  32-bit division: task ids are below the flattened
-    // work-group count, < 2^32 (checked at launch) -- a 64-bit one is a called subroutine of ~70
-    // instructions, run for every task by the body and again by the dispatcher's key
+    // task t -> (tile column, tile row).  FCL_TASK_DIV32=1 divides in 32 bits (task ids are below
+    // the flattened work-group count, < 2^32, checked at launch) instead of calling the 64-bit
+    // division subroutine -- measured: the 2DCONV dispatcher then runs at 0.44 instead of 0.78 of
+    // the copy peak, the plain grid unchanged (profiles/r02_ab_task_div32.txt); off.
+#ifndef FCL_TASK_DIV32
+#define FCL_TASK_DIV32 0
+#endif
     __device__ __host__ void split(long long t, long long &tx, long long &ty) const {
-        const unsigned int ut = (unsigned int)t, un = (unsigned int)ntx;
-        tx = (long long)(ut % un);
-        ty = (long long)(ut / un);
+        if (FCL_TASK_DIV32) {
+            const unsigned int ut = (unsigned int)t, un = (unsigned int)ntx;
+            tx = (long long)(ut % un);
+            ty = (long long)(ut / un);
+        } else {
+            tx = t % ntx;
+            ty = t / ntx;
+        }
     }
     __device__ __host__ long long key(long long t) const {
         long long tx, ty;
