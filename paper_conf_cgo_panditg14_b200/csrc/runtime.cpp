@@ -516,7 +516,7 @@ struct fcl_context_st {
         double est_host = -1;                             // Σ host-alone estimates (ms); -1 unknown
         double work = 0;                                  // Σ multiply-adds of its launches
         int choice = 0, trial = 0, trial_kind = 0;        // trial: sequences left in the running trial
-        int64_t seqs = 0, next_trial = 1, period = 16, loss_period = 32;
+        int64_t seqs = 0, next_trial = 1, period = 64, loss_period = 32;
     };
     std::map<uint64_t, SeqEnt> seq_tab;
     std::map<SeqKey, uint64_t> seq_first;   // a signature's first key -> the signature
@@ -526,6 +526,7 @@ struct fcl_context_st {
         bool ok = true;       // every launch eligible, the plan (if any) followed
         int run = -1;         // what this sequence runs: -1 no plan, 0 default, 1 host alone
         bool trial = false; uint64_t plan = 0;
+        const std::vector<SeqKey> *plan_keys = nullptr;   // the planned signature's keys
     } seq;
     // Streamed launches (§6.7) queued or in phase B: their grids wait for pieces the coordinator
     // issues, so the API thread must not allocate device or pinned memory meanwhile -- an
@@ -1142,8 +1143,7 @@ void select_update(fcl_context ctx, const Job &j, bool gpu_done) {
 // sequence wrote: a sequence whose first kernel ran on the host leaves the second one's input
 // stale on the device, and that must not change the signature, while inputs the caller wrote
 // (the e2e loop's non-blocking writes) do.
-fcl_context_st::SeqKey seq_key(const Launch &L, const std::vector<const void *> &written) {
-    const auto k = select_key(L);
+fcl_context_st::SeqKey seq_key(const Launch &L, const std::array<int64_t, 9> &k, const std::vector<const void *> &written) {
     fcl_context_st::SeqKey s;
     for (int q = 0; q < 8; ++q) s[q] = k[q];
     int64_t stale = 0;
@@ -1188,9 +1188,22 @@ bool seq_launch(fcl_context ctx, const Launch &L, bool eligible) {
     if (!eligible) { c.ok = false; c.run = -1; return false; }
     if (!c.ok || c.keys.size() >= 64) { c.ok = false; c.run = -1; return false; }
     if (c.keys.empty()) c.written.clear();
-    const fcl_context_st::SeqKey k = seq_key(L, c.written);
+    const auto k9 = select_key(L);
+    const fcl_context_st::SeqKey k = seq_key(L, k9, c.written);
     for (int b = 0; b < L.a.nbuf; ++b)
         if (L.acc[b] & 2) c.written.push_back(L.bufs[b]);
+    const size_t pos = c.keys.size();
+    // a host plan past its first launch needs none of the shared tables: follow the plan's keys
+    // (std::map nodes never move, and entries are never erased)
+    if (c.run == 1 && pos > 0 && c.plan_keys) {
+        c.keys.push_back(k);
+        for (int64_t v : k) c.h = (c.h ^ (uint64_t)v) * 1099511628211ull;
+        c.work += host_madds(L);
+        if (pos < c.plan_keys->size() && (*c.plan_keys)[pos] == k) return true;
+        c.ok = false;   // off the planned signature: the rest runs by per-launch selection
+        c.run = -1;
+        return false;
+    }
     std::lock_guard<std::mutex> lk(ctx->sel_mu);
     if (c.keys.empty()) {
         c.t0 = now_ms();
@@ -1199,6 +1212,7 @@ bool seq_launch(fcl_context ctx, const Launch &L, bool eligible) {
         c.work = 0;
         c.run = -1;
         c.trial = false;
+        c.plan_keys = nullptr;
         auto f = ctx->seq_first.find(k);
         if (f != ctx->seq_first.end()) {
             auto t = ctx->seq_tab.find(f->second);
@@ -1207,21 +1221,20 @@ bool seq_launch(fcl_context ctx, const Launch &L, bool eligible) {
                 c.run = e.trial > 0 ? e.trial_kind : e.choice;
                 c.trial = e.trial > 0;
                 c.plan = f->second;
+                c.plan_keys = &e.keys;
             }
         }
     }
-    const size_t pos = c.keys.size();
     c.keys.push_back(k);
     for (int64_t v : k) c.h = (c.h ^ (uint64_t)v) * 1099511628211ull;   // FNV-1a over the keys
     c.work += host_madds(L);
-    {
-        const auto se = ctx->sel.find(select_key(L));
+    if (c.run != 1) {   // (the host-alone estimate is recorded for default sequences only)
+        const auto se = ctx->sel.find(k9);
         const double r = se == ctx->sel.end() ? -1.0 : se->second.host_ms_per_wg;
         c.est = (c.est < 0 || r < 0) ? -1.0 : c.est + r * (double)(L.hi - L.lo);
     }
     if (c.run == 1) {
-        const auto t = ctx->seq_tab.find(c.plan);
-        if (t != ctx->seq_tab.end() && pos < t->second.keys.size() && t->second.keys[pos] == k) return true;
+        if (c.plan_keys && pos < c.plan_keys->size() && (*c.plan_keys)[pos] == k) return true;
         c.ok = false;   // off the planned signature: the rest runs by per-launch selection
         c.run = -1;
     }
@@ -1266,11 +1279,13 @@ void seq_end(fcl_context ctx) {
                     e.loss_period = std::min<int64_t>(4096, e.loss_period * 8);
                     e.next_trial = e.seqs + e.loss_period;
                 } else if (win == e.choice) {
-                    e.period = std::min<int64_t>(256, e.period * 2);
+                    e.period = std::min<int64_t>(1024, e.period * 2);
                     e.next_trial = e.seqs + e.period;
                 } else {
+                    // a new choice is re-checked after 64 sequences, then 128, ... 1024 while it
+                    // holds (each re-check costs one sequence run the other way)
                     e.choice = win;
-                    e.period = 16;
+                    e.period = 64;
                     e.next_trial = e.seqs + e.period;
                 }
             }

@@ -389,7 +389,9 @@ def test_sequence_plan_broken_midway(ctx):
         for g, r in zip(got, ref[k]):
             assert_bits(g, r, f"sequence {i} ({k})")
     c1 = ctx.counters()
-    assert c1["seq_trials"] > c0["seq_trials"], (c0, c1)
+    # host plans ran (this test's trial, or the standing choice of the ATAX signature an earlier
+    # test of the module established: sequence keys are shapes, not buffers)
+    assert c1["seq_host"] > c0["seq_host"] or c1["seq_trials"] > c0["seq_trials"], (c0, c1)
     for bl in (b1, b2, bq):
         for k, b in enumerate(bl):
             if not (bl is b2 and k in (0, 1)):
