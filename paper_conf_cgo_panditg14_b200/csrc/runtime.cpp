@@ -517,6 +517,7 @@ struct fcl_context_st {
         double work = 0;                                  // Σ multiply-adds of its launches
         int choice = 0, trial = 0, trial_kind = 0;        // trial: sequences left in the running trial
         int64_t seqs = 0, next_trial = 1, period = 64, loss_period = 32;
+        int64_t inert = 0;   // sequences still to run untracked (a signature no trial is worth)
     };
     std::map<uint64_t, SeqEnt> seq_tab;
     std::map<SeqKey, uint64_t> seq_first;   // a signature's first key -> the signature
@@ -1216,6 +1217,14 @@ bool seq_launch(fcl_context ctx, const Launch &L, bool eligible) {
         auto f = ctx->seq_first.find(k);
         if (f != ctx->seq_first.end()) {
             auto t = ctx->seq_tab.find(f->second);
+            if (t != ctx->seq_tab.end() && t->second.inert > 0) {
+                // nothing to decide for this signature for a while: run it untracked (no
+                // bookkeeping on its launches or at its fcl_finish)
+                t->second.inert -= 1;
+                c.ok = false;
+                c.keys.push_back(k);
+                return false;
+            }
             if (t != ctx->seq_tab.end()) {
                 const auto &e = t->second;
                 c.run = e.trial > 0 ? e.trial_kind : e.choice;
@@ -1304,6 +1313,13 @@ void seq_end(fcl_context ctx) {
                 e.trial_kind = other;
                 ctx->counts[FCL_COUNT_SEQ_TRIALS] += 1;
             }
+        }
+        // a default signature whose host alone is not worth a trial (no rate and not small, or a
+        // predicted loss) runs its next 255 sequences untracked
+        if (e.trial == 0 && e.choice == 0 && kind == 0) {
+            const double d = seq_best(e.t_run[0], e.n_run[0]);
+            const bool worth = e.est_host >= 0 ? e.est_host <= d : e.work <= (double)(1 << 20);
+            if (!worth) e.inert = 255;
         }
     }
     c.keys.clear();
